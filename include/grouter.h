@@ -1,0 +1,237 @@
+/*
+ * grouter.h -- C ABI of the B200-native GROUTER data-passing hot path.
+ *
+ * What this library is (PAPER.md = marker text of Wu et al., EuroSys '26):
+ *   L165 §4.2.1  Put() stores an intermediate object locally and returns a
+ *                globally unique id; Get(id) retrieves it and picks the
+ *                transfer method from the consumer's placement.
+ *   L167 §4.2.2  same GPU -> zero copy (share the address); other GPU ->
+ *                allocate on the consumer GPU and copy over NVLink; host ->
+ *                stage over parallel PCIe links, then map.
+ *   L178-L182    host<->GPU traffic striped over route GPUs' PCIe links,
+ *                forwarded over NVLink; payloads cut in 2 MB chunks under a
+ *                precomputed plan; in-order delivery.
+ *   L193-L229    per-function bandwidth shares; batches of 5 chunks.
+ *   L248-L262    elastic GPU pool (2 MiB pages here), 50%-of-free cap,
+ *                queue-aware migration to pinned host memory.
+ *   L260         data no longer needed is removed promptly.
+ *   L394 §7      every access is authenticated by function id + workflow id.
+ * Readings of silent/ambiguous points (R1-R31) are listed in DESIGN.md.
+ *
+ * Conventions (all calls):
+ *   - Every call returns a grouter_status; on error outputs are untouched
+ *     and no C++ exception crosses the ABI.  CUDA failures -> GROUTER_ECUDA
+ *     (sticky; grouter_last_error() has the text).
+ *   - "stream" arguments are a cudaStream_t (CUstream) of the caller's
+ *     device passed as void*.  Device callers are stream-ordered: a put reads
+ *     `src` after prior work on the stream, and the stream cannot overwrite
+ *     `src` before the library's copy completes; a get returns at once and
+ *     work enqueued on the stream afterwards sees the data.  A NULL stream
+ *     means a host caller: the call blocks until the bytes are in place.
+ *   - Ownership: the caller owns put `src` and get_into `dst`; the library
+ *     owns object pages, leases, staging rings and the host store.  A lease
+ *     stays valid until grouter_release(); a zero-copy lease aliases the
+ *     object and must not be written.
+ *   - n == 0 is valid: empty plan, get returns ptr = NULL, n = 0, GROUTER_OK.
+ *   - All calls are thread-safe.
+ */
+#ifndef GROUTER_H
+#define GROUTER_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GROUTER_MAX_GPUS 16
+#define GROUTER_MAX_PATHS 8
+#define GROUTER_HOST (-1)          /* location / device of a CPU function  */
+#define GROUTER_NOHINT (-2)        /* put: no placement hint               */
+#define GROUTER_UNLIMITED UINT64_MAX
+
+/* flags for grouter_config.flags */
+#define GROUTER_REPLAY        0x1u /* dispatch only at grouter_flush() (deterministic log) */
+#define GROUTER_NO_MULTIPATH  0x2u /* host->GPU uses the direct PCIe link only (ablation)  */
+#define GROUTER_PLAN_ONLY     0x4u /* no CUDA at all: planner/introspection only            */
+#define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
+#define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
+
+typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
+typedef struct grouter_ctx grouter_ctx;
+
+typedef enum {
+  GROUTER_OK = 0,
+  GROUTER_EINVAL = 1,  /* bad argument, unknown device, dst_cap < n, unknown lease */
+  GROUTER_ENOENT = 2,  /* unknown, freed, consumed or unsealed object            */
+  GROUTER_EPERM = 3,   /* workflow mismatch (L394)                               */
+  GROUTER_ENOMEM = 4,  /* pool/lease/alloc cannot fit after eviction; host full  */
+  GROUTER_EBUSY = 5,   /* free of an unsealed object; no completion slot free    */
+  GROUTER_ECUDA = 6,   /* CUDA error (sticky)                                    */
+  GROUTER_ESTATE = 7   /* wrong object state (e.g. seal twice)                   */
+} grouter_status;
+
+/* A serverless function: its workflow, its id, and its resident device
+ * (a logical GPU index 0..n_gpus-1, or GROUTER_HOST for a CPU function).
+ * Placement is given explicitly by the caller (L110: virtualised device ids
+ * make it unobservable from inside a container). */
+typedef struct {
+  uint32_t workflow_id;
+  uint32_t function_id;
+  int32_t device;
+} grouter_fn;
+
+/* One chunk of a transfer plan (L182).  path = index into the route set
+ * R(dst) for host->GPU plans (0 = direct link of dst), 0 otherwise;
+ * route_gpu = GPU whose link/engine moves the chunk. */
+typedef struct {
+  uint64_t offset;
+  uint64_t bytes;
+  int32_t path;
+  int32_t route_gpu;
+} grouter_chunk;
+
+/* Node calibration (the topology matrix of Alg. 1) plus knobs.
+ * Fill with grouter_config_default(), then override. */
+typedef struct {
+  uint32_t n_gpus;                                   /* logical GPUs            */
+  int32_t device_map[GROUTER_MAX_GPUS];              /* logical -> CUDA ordinal */
+  uint64_t nvl_Bps;                                  /* NVLink B/s per direction*/
+  uint64_t h2d_Bps[GROUTER_MAX_GPUS];                /* solo pinned H2D, B/s    */
+  uint64_t h2d_alpha_ps[GROUTER_MAX_GPUS];           /* per-chunk CE cost, ps   */
+  uint64_t h2d_phi_ps[GROUTER_MAX_GPUS];             /* first-chunk latency, ps */
+  uint64_t relay_phi_ps;                             /* extra fill of a relay   */
+  uint64_t h2d_pair_Bps[GROUTER_MAX_GPUS][GROUTER_MAX_GPUS]; /* concurrent sums */
+  int32_t uplink_group[GROUTER_MAX_GPUS];            /* explicit group id or -1 */
+  uint8_t p2p[GROUTER_MAX_GPUS][GROUTER_MAX_GPUS];   /* peer access matrix      */
+  uint64_t chunk_bytes;        /* C, default 2 MiB (L182, R1)                 */
+  uint32_t batch_chunks;       /* default 5 (L229)                            */
+  uint64_t granule;            /* split granule g, default 4096               */
+  uint64_t pool_floor_bytes;   /* trim floor, default 300 MiB (L256, R13)     */
+  uint32_t pool_cap_permille;  /* auto cap = permille of free, default 500 (L262) */
+  uint64_t pool_cap_bytes[GROUTER_MAX_GPUS]; /* explicit cap; 0 = auto         */
+  uint64_t host_store_bytes;   /* pinned host store H, default 1 GiB          */
+  uint64_t round_bytes;        /* SM-copy dispatch horizon, default 64 MiB    */
+  uint32_t copy_ctas_per_sm;   /* SM copy kernel CTAs per SM, default 2       */
+  uint32_t flags;              /* GROUTER_* flags                              */
+} grouter_config;
+
+typedef struct {
+  uint64_t used[GROUTER_MAX_GPUS];       /* sum of charges (objects + leases)   */
+  uint64_t cap[GROUTER_MAX_GPUS];        /* current cap                         */
+  uint64_t mapped[GROUTER_MAX_GPUS];     /* physical bytes mapped in the pool   */
+  uint64_t host_used, host_cap;
+  uint64_t spill_count, spill_bytes;     /* migrations to host (L258)           */
+  uint64_t xfer_count;                   /* transfers planned                   */
+  uint64_t link_bytes[3][GROUTER_MAX_GPUS]; /* [0]=SM copy egress, [1]=H2D, [2]=D2H */
+  uint64_t kernel_launches;              /* copy/forward kernels launched       */
+  uint64_t rounds;                       /* dispatch rounds                     */
+} grouter_stats_t;
+
+/* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
+ * server).  server_kind: 0 = SM copy egress of server_dev, 1 = H2D engine of
+ * route GPU server_dev, 2 = D2H engine of server_dev.  Chunk ids are
+ * (xfer << 32 | chunk index) where xfer numbers transfers from 1 in call order. */
+typedef struct {
+  int32_t server_kind;
+  int32_t server_dev;
+  uint32_t tenant;
+  uint32_t n_chunks;
+  uint64_t chunk_ids[8];
+  uint64_t bytes;
+} grouter_dispatch;
+
+/* ------------------------------------------------------------ lifecycle */
+void grouter_config_default(grouter_config *cfg);
+/* Creates the context: per-GPU pools (VMM reservations), host store, streams,
+ * route sets R(d) (precomputed, L271).  cfg is copied. */
+grouter_status grouter_init(const grouter_config *cfg, grouter_ctx **out);
+/* Waits for all library work, releases every resource. */
+grouter_status grouter_finalize(grouter_ctx *ctx);
+
+/* ------------------------------------------------------------ data path */
+/* Put by copy (L165).  fn->device GPU: stored on that GPU (locality, hint
+ * ignored).  CPU fn: stored on `hint` GPU if given (eager striped H2D, R23),
+ * else in the pinned host store.  If the home GPU cannot fit even after
+ * eviction the object goes to the host store (R16).  `consumers` = k: the
+ * object is freed after k completed gets (0 = explicit free only). */
+grouter_status grouter_put(grouter_ctx *ctx, const grouter_fn *fn, const void *src, uint64_t n,
+                           int32_t hint, uint32_t consumers, void *stream, grouter_oid *out);
+/* Zero-copy put, step 1: library-owned, page-aligned buffer on fn->device
+ * (or the host store for a CPU fn).  ENOMEM if it cannot fit. */
+grouter_status grouter_alloc(grouter_ctx *ctx, const grouter_fn *fn, uint64_t n, int32_t hint,
+                             uint32_t consumers, void **buf, grouter_oid *out);
+/* Zero-copy put, step 2: the object becomes visible once prior work on
+ * `stream` (which wrote the buffer) completes.  ESTATE if already sealed. */
+grouter_status grouter_seal(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *stream);
+/* Get (L165, L167): read-only lease on fn->device.  Same location -> the
+ * object's own address (zero copy, pins the object).  Otherwise a copy lease
+ * (D2D over NVLink, striped H2D, or D2H for a CPU fn).  *ptr/*n out. */
+grouter_status grouter_get(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *stream,
+                           const void **ptr, uint64_t *n);
+/* Get into caller memory `dst` (device memory of fn->device, or host memory
+ * for a CPU fn); always copies.  EINVAL if dst_cap < n. *n_out may be NULL. */
+grouter_status grouter_get_into(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *dst,
+                                uint64_t dst_cap, void *stream, uint64_t *n_out);
+/* Drops a lease (ptr as returned by grouter_get).  Stream-ordered: pages are
+ * reused only after prior work on `stream` completes (NULL: now). */
+grouter_status grouter_release(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid,
+                               const void *ptr, void *stream);
+/* Frees an object (L260); later gets fail with ENOENT.  Pages are reclaimed
+ * once zero-copy pins drain.  EBUSY if unsealed. */
+grouter_status grouter_free(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid);
+
+/* ------------------------------------------------------------ control */
+/* Tenant (workflow) bandwidth weight, >= 1 (north star; L193-L197). */
+grouter_status grouter_set_tenant_weight(grouter_ctx *ctx, uint32_t workflow_id, uint32_t weight);
+/* Queue position of the object's next consumer (D8; L258 queue-aware eviction). */
+grouter_status grouter_set_next_use(grouter_ctx *ctx, grouter_oid oid, uint64_t queue_pos);
+/* Pool cap of a GPU (GROUTER_UNLIMITED = no cap); evicts at once until used <= cap
+ * (L262).  ENOMEM if unevictable data keeps the pool above the cap. */
+grouter_status grouter_set_pool_limit(grouter_ctx *ctx, int32_t device, uint64_t bytes);
+/* Replay mode: dispatch every queued chunk (stride order); no-op otherwise. */
+grouter_status grouter_flush(grouter_ctx *ctx);
+/* Blocks until all library work issued so far has completed. */
+grouter_status grouter_sync(grouter_ctx *ctx);
+
+/* ------------------------------------------------------------ introspection */
+/* Transfer plan (L182) for n bytes from src_loc (GPU or GROUTER_HOST) to
+ * dst_dev (GPU or GROUTER_HOST).  *n_out = chunk count even if cap is short
+ * (then EINVAL and nothing written). */
+grouter_status grouter_plan(grouter_ctx *ctx, int32_t src_loc, int32_t dst_dev, uint64_t n,
+                            grouter_chunk *out, uint64_t cap, uint64_t *n_out);
+/* Route set R(dst) (L178, precomputed at init, L271). */
+grouter_status grouter_route_set(grouter_ctx *ctx, int32_t dst_dev, int32_t *out, uint32_t cap,
+                                 uint32_t *n_out);
+/* Current location of an object: GPU index or GROUTER_HOST. */
+grouter_status grouter_where(grouter_ctx *ctx, grouter_oid oid, int32_t *loc);
+grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
+/* Takes (and clears) the objects spilled since the last call, in order. */
+grouter_status grouter_victims(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
+/* Takes (and clears) up to cap dispatch records, oldest first. */
+grouter_status grouter_dispatch_log(grouter_ctx *ctx, grouter_dispatch *out, uint64_t cap,
+                                    uint64_t *n_out);
+
+/* ------------------------------------------------------------ stride scheduler
+ * The tenant-share scheduler used by every server (L229 batches, stride
+ * order), exposed standalone for host-side tests; needs no GPU. */
+typedef struct grouter_sched grouter_sched;
+grouter_status grouter_sched_new(uint32_t batch_chunks, grouter_sched **out);
+grouter_status grouter_sched_set_weight(grouter_sched *s, uint32_t tenant, uint32_t weight);
+grouter_status grouter_sched_enqueue(grouter_sched *s, uint32_t tenant, uint64_t chunk_id,
+                                     uint64_t bytes);
+/* Next batch: *tenant, up to 8 ids, *n, *bytes, tenant's pass after it.
+ * ENOENT when nothing is backlogged. */
+grouter_status grouter_sched_dispatch(grouter_sched *s, uint32_t *tenant, uint64_t *ids,
+                                      uint32_t *n, uint64_t *bytes, uint64_t *pass_after);
+void grouter_sched_free(grouter_sched *s);
+
+const char *grouter_strerror(grouter_status st);
+/* Text of the last error seen by this thread (thread-local). */
+const char *grouter_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GROUTER_H */

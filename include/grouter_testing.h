@@ -1,0 +1,43 @@
+/*
+ * grouter_testing.h -- test-infrastructure kernels.
+ *
+ * Not part of the data path.  These implement, on the device, the
+ * SplitMix64 counter-mode payload generator of SURVEY §8(c) O11 (the same
+ * input recipe synth/payload.py implements on the host) so large payloads
+ * can be produced and verified in HBM, plus an exactly-once probe that runs
+ * the PRODUCTION copy kernel over a chunk list while counting every 16-byte
+ * destination granule it writes.
+ *
+ * All functions take device pointers (or host-mapped pinned pointers), are
+ * stream-ordered on `stream` (a cudaStream_t as void*), and return
+ * grouter_status (ECUDA on CUDA failure, EINVAL on bad arguments).
+ */
+#ifndef GROUTER_TESTING_H
+#define GROUTER_TESTING_H
+
+#include "grouter.h"
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* dst[i] = byte (offset + i) of stream `seed`, i in [0, n). */
+grouter_status grouter_test_fill(void *dst, uint64_t n, uint64_t seed, uint64_t offset,
+                                 void *stream);
+/* Counts bytes of src[0, n) that differ from stream `seed` at `offset`.
+ * Blocking: synchronizes `stream`; *mismatches and *first_bad (UINT64_MAX if
+ * none) are host outputs. */
+grouter_status grouter_test_verify(const void *src, uint64_t n, uint64_t seed, uint64_t offset,
+                                   void *stream, uint64_t *mismatches, uint64_t *first_bad);
+/* Runs the production SM copy kernel over `n_chunks` chunks
+ * (dst_base + chunk.offset <- src_base + chunk.offset, chunk.bytes) on the
+ * current device.  If counts != NULL (device array of ceil((max_end)/16)
+ * uint32), every 16-byte destination granule touched is counted (exactly-once
+ * probe, invariant I1).  tma != 0 selects the cp.async.bulk variant. */
+grouter_status grouter_test_copy(void *dst_base, const void *src_base, const grouter_chunk *chunks,
+                                 uint32_t n_chunks, uint32_t *counts, int tma, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GROUTER_TESTING_H */

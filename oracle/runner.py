@@ -103,6 +103,13 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
             rec["dispatched"] = out["dispatched"]
         else:
             raise ValueError(k)
+        if st == 0 and k in ("put", "get", "get_into") and op["fn"]["dev"] == HOST:
+            # a CPU caller blocks until its bytes are in place; in replay mode
+            # that dispatches everything queued (R31)
+            victims = list(orc.victims)
+            _, fl = orc.flush()
+            orc.victims = victims
+            rec["dispatched"] = fl["dispatched"]
         rec["status"] = STATUS[st]
         rec["victims"] = list(orc.victims)
         rec["used"] = list(orc.used)

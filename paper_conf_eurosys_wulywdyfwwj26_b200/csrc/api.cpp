@@ -1,0 +1,731 @@
+// api.cpp -- the C ABI of include/grouter.h: object table, placement,
+// authentication, refcounted lifetimes, queue-aware eviction.
+//
+// PAPER.md L165 (locality-aware Put, Get dispatch, one transfer per get),
+// L167 (zero copy on the same GPU; allocate on the consumer GPU + NVLink;
+// host data staged over parallel PCIe), L173 (id -> address/location table),
+// L248-L262 (elastic pool, 50% cap, queue-aware migration, prompt removal),
+// L394 (authentication by function id + workflow id).  Readings R14-R24 in
+// DESIGN.md.  Byte movement is delegated to engine.cpp.
+#include <algorithm>
+#include <cstring>
+
+#include "../../include/grouter.h"
+#include "ctx.h"
+
+using namespace gr;
+
+namespace {
+
+struct Guard {
+  grouter_ctx *c;
+  std::unique_lock<std::mutex> lk;
+  explicit Guard(grouter_ctx *c_) : c(c_), lk(c_->mu) {}
+};
+
+grouter_status fail(grouter_status st, const char *msg) {
+  set_error(msg);
+  return st;
+}
+
+#define API_TRY try {
+#define API_CATCH(ctx)                                                        \
+  }                                                                           \
+  catch (const gr::Error &e) {                                                \
+    gr::set_error(e.what());                                                  \
+    if (e.st == GROUTER_ECUDA && (ctx)) (ctx)->sticky_error = true;           \
+    return e.st;                                                              \
+  }                                                                           \
+  catch (const std::exception &e) {                                           \
+    gr::set_error(e.what());                                                  \
+    return GROUTER_EINVAL;                                                    \
+  }
+
+bool valid_gpu(const grouter_ctx *c, int d) { return d >= 0 && d < (int)c->cfg.n_gpus; }
+bool valid_loc(const grouter_ctx *c, int d) { return d == GROUTER_HOST || valid_gpu(c, d); }
+
+int phys_of(grouter_ctx *c, int logical) { return c->dev[logical].phys; }
+
+bool dead(const Obj &o) { return o.state == OBJ_CONSUMED || o.state == OBJ_FREED; }
+
+Obj *lookup_live(grouter_ctx *c, grouter_oid oid) {
+  auto it = c->objects.find(oid);
+  if (it == c->objects.end() || dead(it->second)) return nullptr;
+  return &it->second;
+}
+
+// Storage of a consumed/freed object goes back to its pool once no zero-copy
+// lease pins it ("promptly removes intermediate data", L260).
+void release_storage_if_dead(grouter_ctx *c, Obj &o) {
+  if (!dead(o) || o.pins) return;
+  const uint64_t ch = charge(o.n);
+  Fences f = std::move(o.readers);
+  for (auto &w : o.ready) f.push_back(w);
+  if (o.loc == GROUTER_HOST) {
+    c->host_used -= ch;
+    host_free(c, o.ptr, ch, std::move(f));
+  } else {
+    c->dev[o.loc].used -= ch;
+    dev_free(c, o.loc, o.ptr, ch, std::move(f));
+  }
+  c->objects.erase(o.oid);
+}
+
+void consume(grouter_ctx *c, Obj &o) {
+  if (o.consumers_left > 0 && --o.consumers_left == 0) {
+    o.state = OBJ_CONSUMED;
+    release_storage_if_dead(c, o);
+  }
+}
+
+// Eviction order (L258 queue-aware; R15 tie-breaks): objects without a
+// next-use hint first, then the TAIL of the request queue (largest
+// next_use), then least recently accessed, then lower oid.
+std::vector<Obj *> candidates(grouter_ctx *c, int d) {
+  std::vector<Obj *> v;
+  for (auto &kv : c->objects) {
+    Obj &o = kv.second;
+    if (o.loc == d && o.state == OBJ_SEALED && o.pins == 0 && o.n > 0) v.push_back(&o);
+  }
+  std::sort(v.begin(), v.end(), [](const Obj *a, const Obj *b) {
+    if (a->has_next_use != b->has_next_use) return !a->has_next_use;
+    if (a->has_next_use && a->next_use != b->next_use) return a->next_use > b->next_use;
+    if (a->last_access != b->last_access) return a->last_access < b->last_access;
+    return a->oid < b->oid;
+  });
+  return v;
+}
+
+// Migrates a victim to the pinned host store.
+void spill(grouter_ctx *c, Obj &o) {
+  const uint64_t ch = charge(o.n);
+  uint8_t *h = host_alloc(c, ch);
+  const int d = o.loc;
+  spill_copy(c, o, h);            // D2H + device pages to quarantine
+  o.loc = GROUTER_HOST;
+  o.ptr = h;
+  c->dev[d].used -= ch;
+  c->host_used += ch;
+  c->victims.push_back(o.oid);
+}
+
+// reserve(d, ch): admit if it fits under the cap; else evict in victim order
+// until it fits -- all or nothing (no eviction when it cannot fit, or when
+// the host store cannot take the victims).
+bool reserve(grouter_ctx *c, int d, uint64_t ch) {
+  LogicalDev &D = c->dev[d];
+  if (D.cap == GROUTER_UNLIMITED || D.used + ch <= D.cap) {
+    D.used += ch;
+    return true;
+  }
+  const uint64_t need = D.used + ch - D.cap;
+  uint64_t freed = 0;
+  std::vector<Obj *> picked;
+  for (Obj *o : candidates(c, d)) {
+    picked.push_back(o);
+    freed += charge(o->n);
+    if (freed >= need) break;
+  }
+  if (freed < need || c->host_used + freed > c->host_cap) return false;
+  for (Obj *o : picked) spill(c, *o);
+  D.used += ch;
+  return true;
+}
+
+bool host_reserve(grouter_ctx *c, uint64_t ch) {
+  if (c->host_used + ch > c->host_cap) return false;
+  c->host_used += ch;
+  return true;
+}
+
+// Physical storage for a reservation already charged; undoes the charge on failure.
+uint8_t *storage(grouter_ctx *c, int loc, uint64_t ch) {
+  if (!ch) return nullptr;
+  try {
+    return loc == GROUTER_HOST ? host_alloc(c, ch) : dev_alloc(c, loc, ch);
+  } catch (...) {
+    if (loc == GROUTER_HOST) c->host_used -= ch;
+    else c->dev[loc].used -= ch;
+    throw;
+  }
+}
+
+bool is_pageable(const void *p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return true;
+  }
+  return a.type == cudaMemoryTypeUnregistered;
+}
+
+// Blocking completion for host callers: in replay mode the call flushes
+// (R31), otherwise everything queued is dispatched so the wait
+// cannot depend on the daemon (we hold the lock).
+void block_on(grouter_ctx *c, const Fences &f) {
+  if (c->replay) flush_all(c);
+  else pump(c, true);
+  host_wait(f);
+}
+
+int server_kind_for(int src, int dst) {
+  if (src == GROUTER_HOST) return SK_H2D;
+  if (dst == GROUTER_HOST) return SK_D2H;
+  return SK_COPY;
+}
+
+// Plans, enqueues and starts one transfer; returns it.
+XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc, uint64_t n,
+                       const uint8_t *src, uint8_t *dst, Fences deps, bool pageable_src) {
+  std::vector<grouter_chunk> plan;
+  c->planner.plan(src_loc, dst_loc, n, plan);
+  XferRef x = new_xfer(c, tenant, plan);
+  x->deps = std::move(deps);
+  x->pageable_src = pageable_src;
+  enqueue_plan(c, x, plan, server_kind_for(src_loc, dst_loc), (uint64_t)(uintptr_t)src,
+               (uint64_t)(uintptr_t)dst, dst_loc);
+  pump(c, false);  // inline dispatch when the server has room (no-op in replay mode)
+  return x;
+}
+
+bool check_ready(grouter_ctx *c) {
+  if (c->sticky_error) {
+    set_error("sticky CUDA error; see the first failure");
+    return false;
+  }
+  return true;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *grouter_strerror(grouter_status st) {
+  static const char *s[] = {"GROUTER_OK",     "GROUTER_EINVAL", "GROUTER_ENOENT", "GROUTER_EPERM",
+                            "GROUTER_ENOMEM", "GROUTER_EBUSY",  "GROUTER_ECUDA",  "GROUTER_ESTATE"};
+  return ((unsigned)st < 8) ? s[st] : "GROUTER_?";
+}
+
+const char *grouter_last_error(void) { return gr::last_error(); }
+
+void grouter_config_default(grouter_config *cfg) {
+  if (!cfg) return;
+  std::memset(cfg, 0, sizeof(*cfg));
+  for (int i = 0; i < GROUTER_MAX_GPUS; ++i) {
+    cfg->device_map[i] = i;
+    cfg->h2d_Bps[i] = 55000000000ull;
+    cfg->h2d_alpha_ps[i] = 4000000ull;
+    cfg->h2d_phi_ps[i] = 10000000ull;
+    cfg->uplink_group[i] = i;  // uncalibrated: every GPU its own uplink
+    for (int j = 0; j < GROUTER_MAX_GPUS; ++j) cfg->p2p[i][j] = 1;
+  }
+  cfg->nvl_Bps = 900000000000ull;
+  cfg->relay_phi_ps = 20000000ull;
+  cfg->chunk_bytes = 2ull << 20;
+  cfg->batch_chunks = 5;
+  cfg->granule = 4096;
+  cfg->pool_floor_bytes = 300ull << 20;
+  cfg->pool_cap_permille = 500;
+  cfg->host_store_bytes = 1ull << 30;
+  cfg->round_bytes = 64ull << 20;
+  cfg->copy_ctas_per_sm = 4;
+}
+
+grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
+  if (!cfg_in || !out) return fail(GROUTER_EINVAL, "null argument");
+  grouter_config cfg = *cfg_in;
+  if (cfg.granule < 16 || cfg.chunk_bytes < cfg.granule || cfg.chunk_bytes % cfg.granule ||
+      cfg.batch_chunks < 1 || cfg.batch_chunks > 8)
+    return fail(GROUTER_EINVAL, "bad chunk/granule/batch configuration");
+  if (!(cfg.flags & GROUTER_PLAN_ONLY) && cfg.n_gpus == 0) {
+    int nd = 0;
+    if (cudaGetDeviceCount(&nd) != cudaSuccess || nd == 0)
+      return fail(GROUTER_ECUDA, "no CUDA device (the data path has no CPU fallback)");
+    cfg.n_gpus = (uint32_t)std::min(nd, GROUTER_MAX_GPUS);
+  }
+  if (cfg.n_gpus == 0 || cfg.n_gpus > GROUTER_MAX_GPUS) return fail(GROUTER_EINVAL, "bad n_gpus");
+  if (cfg.copy_ctas_per_sm == 0) cfg.copy_ctas_per_sm = 4;
+  if (cfg.round_bytes == 0) cfg.round_bytes = 64ull << 20;
+  auto *c = new grouter_ctx();
+  c->cfg = cfg;
+  c->replay = (cfg.flags & GROUTER_REPLAY) != 0;
+  c->plan_only = (cfg.flags & GROUTER_PLAN_ONLY) != 0;
+  c->planner.build(cfg);
+  c->dev.resize(cfg.n_gpus);
+  if (c->plan_only) {
+    *out = c;
+    return GROUTER_OK;
+  }
+  try {
+    int prev = 0;
+    cudaGetDevice(&prev);
+    engine_init(c);
+    cudaSetDevice(prev);
+  } catch (const gr::Error &e) {
+    set_error(e.what());
+    grouter_status st = e.st;
+    try {
+      engine_shutdown(c);
+    } catch (...) {
+    }
+    delete c;
+    return st;
+  }
+  *out = c;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_finalize(grouter_ctx *c) {
+  if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  if (!c->plan_only) {
+    API_TRY
+    engine_shutdown(c);
+    API_CATCH(c)
+  }
+  delete c;
+  return GROUTER_OK;
+}
+
+// ------------------------------------------------------------------ put / alloc / seal
+grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src, uint64_t n,
+                           int32_t hint, uint32_t consumers, void *stream, grouter_oid *out) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->seq++;
+  c->victims.clear();
+  API_TRY
+  if (!check_ready(c)) return GROUTER_ECUDA;
+  if (!fn || !out || !valid_loc(c, fn->device) ||
+      !(hint == GROUTER_NOHINT || hint == GROUTER_HOST || valid_gpu(c, hint)) || (!src && n))
+    return fail(GROUTER_EINVAL, "put: bad argument");
+  const int from = fn->device;
+  const bool blocking = !stream || from == GROUTER_HOST;
+  int home = from != GROUTER_HOST ? from : (hint >= 0 ? hint : GROUTER_HOST);  // L165, R23
+  const uint64_t ch = charge(n);
+  if (home != GROUTER_HOST && !reserve(c, home, ch)) home = GROUTER_HOST;    // R16
+  if (home == GROUTER_HOST && !host_reserve(c, ch)) return fail(GROUTER_ENOMEM, "host store full");
+  uint8_t *ptr = storage(c, home, ch);
+  Obj o;
+  o.oid = c->next_oid++;
+  o.wf = fn->workflow_id;
+  o.fid = fn->function_id;
+  o.n = n;
+  o.loc = home;
+  o.ptr = ptr;
+  o.state = OBJ_SEALED;
+  o.consumers_left = consumers;
+  o.last_access = c->seq;
+  Fences done;
+  if (n) {
+    if (from == GROUTER_HOST && home == GROUTER_HOST) {
+      std::memcpy(ptr, src, n);  // cFn -> host store: plain memcpy
+    } else {
+      Fences deps;
+      if (!blocking) deps.push_back({record(c, (cudaStream_t)stream, phys_of(c, from)), nullptr, 0, c->epoch});
+      bool pageable = from == GROUTER_HOST && is_pageable(src);
+      XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr,
+                                 std::move(deps), pageable);
+      x->add_done_fences(done);
+      o.ready = done;
+      if (!blocking) stream_wait(c, (cudaStream_t)stream, phys_of(c, from), done);
+    }
+  }
+  *out = o.oid;
+  c->objects.emplace(o.oid, std::move(o));
+  if (blocking && (c->replay || !done.empty())) block_on(c, done);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, int32_t hint,
+                             uint32_t consumers, void **buf, grouter_oid *out) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->seq++;
+  c->victims.clear();
+  API_TRY
+  if (!check_ready(c)) return GROUTER_ECUDA;
+  if (!fn || !buf || !out || !valid_loc(c, fn->device) ||
+      !(hint == GROUTER_NOHINT || hint == GROUTER_HOST || valid_gpu(c, hint)))
+    return fail(GROUTER_EINVAL, "alloc: bad argument");
+  const int home = fn->device;
+  const uint64_t ch = charge(n);
+  if (home != GROUTER_HOST ? !reserve(c, home, ch) : !host_reserve(c, ch))
+    return fail(GROUTER_ENOMEM, "alloc: does not fit after eviction");
+  uint8_t *ptr = storage(c, home, ch);
+  Obj o;
+  o.oid = c->next_oid++;
+  o.wf = fn->workflow_id;
+  o.fid = fn->function_id;
+  o.n = n;
+  o.loc = home;
+  o.ptr = ptr;
+  o.state = OBJ_OPEN;
+  o.consumers_left = consumers;
+  o.last_access = c->seq;
+  *buf = ptr;
+  *out = o.oid;
+  c->objects.emplace(o.oid, std::move(o));
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_seal(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *stream) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->seq++;
+  c->victims.clear();
+  API_TRY
+  if (!fn) return fail(GROUTER_EINVAL, "seal: null fn");
+  auto it = c->objects.find(oid);
+  if (it == c->objects.end() || dead(it->second)) return fail(GROUTER_ENOENT, "seal: unknown oid");
+  Obj &o = it->second;
+  if (o.wf != fn->workflow_id) return fail(GROUTER_EPERM, "seal: workflow mismatch");
+  if (o.state != OBJ_OPEN) return fail(GROUTER_ESTATE, "seal: not open");
+  o.state = OBJ_SEALED;
+  o.last_access = c->seq;
+  if (stream && o.loc != GROUTER_HOST)
+    o.ready.push_back({record(c, (cudaStream_t)stream, phys_of(c, o.loc)), nullptr, 0, c->epoch});
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+// ------------------------------------------------------------------ get / get_into
+static grouter_status get_common(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, Obj **out) {
+  if (!fn || !valid_loc(c, fn->device)) return fail(GROUTER_EINVAL, "get: bad function");
+  auto it = c->objects.find(oid);
+  if (it == c->objects.end() || dead(it->second)) return fail(GROUTER_ENOENT, "get: unknown oid");
+  if (it->second.wf != fn->workflow_id) return fail(GROUTER_EPERM, "get: workflow mismatch (L394)");
+  if (it->second.state == OBJ_OPEN) return fail(GROUTER_ENOENT, "get: object not sealed");
+  *out = &it->second;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *stream,
+                           const void **ptr, uint64_t *n_out) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->seq++;
+  c->victims.clear();
+  API_TRY
+  if (!check_ready(c)) return GROUTER_ECUDA;
+  if (!ptr || !n_out) return fail(GROUTER_EINVAL, "get: null output");
+  Obj *op = nullptr;
+  grouter_status st = get_common(c, fn, oid, &op);
+  if (st) return st;
+  Obj &o = *op;
+  const int d = fn->device;
+  const bool blocking = !stream || d == GROUTER_HOST;
+  const uint64_t n = o.n;
+  Fences wait;
+  const void *result = nullptr;
+  if (n == 0) {
+    result = nullptr;
+  } else if (o.loc == d) {  // zero copy: share the address (L167 (1))
+    o.pins++;
+    result = o.ptr;
+    wait = o.ready;
+  } else {
+    const uint64_t ch = charge(n);
+    if (d == GROUTER_HOST ? !host_reserve(c, ch) : !reserve(c, d, ch))
+      return fail(GROUTER_ENOMEM, "get: lease does not fit after eviction");
+    uint8_t *lease = storage(c, d, ch);
+    XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false);
+    Fences done;
+    x->add_done_fences(done);
+    for (auto &w : done) o.readers.push_back(w);
+    Lease L{oid, o.wf, d, lease, n, done};
+    c->leases[(uintptr_t)lease] = std::move(L);
+    result = lease;
+    wait = done;
+  }
+  o.last_access = c->seq;
+  *ptr = result;
+  *n_out = n;
+  consume(c, o);  // may release the object's storage (quarantined behind `wait`)
+  if (blocking) block_on(c, wait);
+  else stream_wait(c, (cudaStream_t)stream, phys_of(c, d), wait);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *dst,
+                                uint64_t dst_cap, void *stream, uint64_t *n_out) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->seq++;
+  c->victims.clear();
+  API_TRY
+  if (!check_ready(c)) return GROUTER_ECUDA;
+  Obj *op = nullptr;
+  grouter_status st = get_common(c, fn, oid, &op);
+  if (st) return st;
+  Obj &o = *op;
+  const uint64_t n = o.n;
+  if (dst_cap < n || (!dst && n)) return fail(GROUTER_EINVAL, "get_into: dst too small");
+  const int d = fn->device;
+  const bool blocking = !stream || d == GROUTER_HOST;
+  Fences wait;
+  if (n) {
+    if (o.loc == GROUTER_HOST && d == GROUTER_HOST) {
+      if (c->replay) flush_all(c);
+      else pump(c, true);
+      host_wait(o.ready);
+      std::memcpy(dst, o.ptr, n);
+    } else {
+      Fences deps = o.ready;
+      if (!blocking)  // the copy must not overwrite dst before prior work on the stream
+        deps.push_back({record(c, (cudaStream_t)stream, phys_of(c, d)), nullptr, 0, c->epoch});
+      XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, (uint8_t *)dst,
+                                 std::move(deps), false);
+      x->add_done_fences(wait);
+      for (auto &w : wait) o.readers.push_back(w);
+    }
+  }
+  o.last_access = c->seq;
+  if (n_out) *n_out = n;
+  consume(c, o);
+  if (blocking) block_on(c, wait);
+  else stream_wait(c, (cudaStream_t)stream, phys_of(c, d), wait);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+// ------------------------------------------------------------------ release / free
+grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid,
+                               const void *ptr, void *stream) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (!fn || !ptr) return fail(GROUTER_EINVAL, "release: bad argument");
+  const bool dev_stream = stream && fn->device != GROUTER_HOST && valid_gpu(c, fn->device);
+  auto it = c->objects.find(oid);
+  if (it != c->objects.end() && it->second.ptr == ptr && it->second.pins > 0) {
+    Obj &o = it->second;  // zero-copy lease: drop the pin
+    if (o.wf != fn->workflow_id) return fail(GROUTER_EPERM, "release: workflow mismatch");
+    o.pins--;
+    if (dev_stream)
+      o.readers.push_back({record(c, (cudaStream_t)stream, phys_of(c, fn->device)), nullptr, 0, c->epoch});
+    release_storage_if_dead(c, o);
+    return GROUTER_OK;
+  }
+  auto lt = c->leases.find((uintptr_t)ptr);
+  if (lt == c->leases.end() || lt->second.oid != oid) return fail(GROUTER_EINVAL, "release: unknown lease");
+  Lease &L = lt->second;
+  if (L.wf != fn->workflow_id) return fail(GROUTER_EPERM, "release: workflow mismatch");
+  Fences f = std::move(L.fill);
+  if (dev_stream) f.push_back({record(c, (cudaStream_t)stream, phys_of(c, fn->device)), nullptr, 0, c->epoch});
+  const uint64_t ch = charge(L.n);
+  if (L.dev == GROUTER_HOST) {
+    c->host_used -= ch;
+    host_free(c, L.ptr, ch, std::move(f));
+  } else {
+    c->dev[L.dev].used -= ch;
+    dev_free(c, L.dev, L.ptr, ch, std::move(f));
+  }
+  c->leases.erase(lt);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_free(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (!fn) return fail(GROUTER_EINVAL, "free: null fn");
+  Obj *o = lookup_live(c, oid);
+  if (!o) return fail(GROUTER_ENOENT, "free: unknown oid");
+  if (o->wf != fn->workflow_id) return fail(GROUTER_EPERM, "free: workflow mismatch");
+  if (o->state == OBJ_OPEN) return fail(GROUTER_EBUSY, "free: object not sealed");
+  o->state = OBJ_FREED;
+  release_storage_if_dead(c, *o);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+// ------------------------------------------------------------------ control
+grouter_status grouter_set_tenant_weight(grouter_ctx *c, uint32_t wf, uint32_t w) {
+  if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  Guard g(c);
+  c->victims.clear();
+  if (w < 1) return fail(GROUTER_EINVAL, "weight must be >= 1");
+  c->weights[wf] = w;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_set_next_use(grouter_ctx *c, grouter_oid oid, uint64_t pos) {
+  if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  Guard g(c);
+  c->victims.clear();
+  Obj *o = lookup_live(c, oid);
+  if (!o) return fail(GROUTER_ENOENT, "set_next_use: unknown oid");
+  o->has_next_use = true;
+  o->next_use = pos;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_set_pool_limit(grouter_ctx *c, int32_t d, uint64_t bytes) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (!valid_gpu(c, d)) return fail(GROUTER_EINVAL, "set_pool_limit: bad device");
+  LogicalDev &D = c->dev[d];
+  D.cap = bytes;
+  if (bytes != GROUTER_UNLIMITED)
+    for (Obj *o : candidates(c, d)) {  // migrate until under the new cap (L262)
+      if (D.used <= D.cap) break;
+      if (c->host_used + charge(o->n) > c->host_cap) break;
+      spill(c, *o);
+    }
+  return (bytes == GROUTER_UNLIMITED || D.used <= D.cap) ? GROUTER_OK
+                                                         : fail(GROUTER_ENOMEM, "pool above cap");
+  API_CATCH(c)
+}
+
+grouter_status grouter_flush(grouter_ctx *c) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (c->replay) flush_all(c);
+  else pump(c, true);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_sync(grouter_ctx *c) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  API_TRY
+  if (!c->replay) pump(c, true);
+  for (auto &d : c->dev) {
+    DeviceGuard dg(d.phys);
+    for (Server *s : {&d.copy, &d.h2d, &d.d2h}) {
+      if (s->stream) GR_CUDA(cudaStreamSynchronize(s->stream));
+      if (s->fwd_stream) GR_CUDA(cudaStreamSynchronize(s->fwd_stream));
+    }
+  }
+  return c->sticky_error ? GROUTER_ECUDA : GROUTER_OK;
+  API_CATCH(c)
+}
+
+// ------------------------------------------------------------------ introspection
+grouter_status grouter_plan(grouter_ctx *c, int32_t src, int32_t dst, uint64_t n, grouter_chunk *out,
+                            uint64_t cap, uint64_t *n_out) {
+  if (!c || !n_out) return fail(GROUTER_EINVAL, "null argument");
+  if (!valid_loc(c, src) || !valid_loc(c, dst)) return fail(GROUTER_EINVAL, "plan: bad location");
+  std::vector<grouter_chunk> plan;
+  c->planner.plan(src, dst, n, plan);
+  *n_out = plan.size();
+  if (plan.size() > cap || (!out && !plan.empty())) return fail(GROUTER_EINVAL, "plan: cap too small");
+  if (!plan.empty()) std::memcpy(out, plan.data(), plan.size() * sizeof(grouter_chunk));
+  return GROUTER_OK;
+}
+
+grouter_status grouter_route_set(grouter_ctx *c, int32_t d, int32_t *out, uint32_t cap, uint32_t *n_out) {
+  if (!c || !n_out) return fail(GROUTER_EINVAL, "null argument");
+  if (!valid_gpu(c, d)) return fail(GROUTER_EINVAL, "route_set: bad device");
+  const auto &R = c->planner.routes[d];
+  *n_out = (uint32_t)R.size();
+  if (R.size() > cap || !out) return fail(GROUTER_EINVAL, "route_set: cap too small");
+  for (size_t i = 0; i < R.size(); ++i) out[i] = R[i];
+  return GROUTER_OK;
+}
+
+grouter_status grouter_where(grouter_ctx *c, grouter_oid oid, int32_t *loc) {
+  if (!c || !loc) return fail(GROUTER_EINVAL, "null argument");
+  Guard g(c);
+  auto it = c->objects.find(oid);
+  if (it == c->objects.end()) return fail(GROUTER_ENOENT, "where: unknown oid");
+  *loc = it->second.loc;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
+  if (!c || !out) return fail(GROUTER_EINVAL, "null argument");
+  Guard g(c);
+  *out = c->stats;
+  for (size_t i = 0; i < c->dev.size(); ++i) {
+    out->used[i] = c->dev[i].used;
+    out->cap[i] = c->dev[i].cap;
+    out->mapped[i] = c->dev[i].pool.mapped;
+  }
+  out->host_used = c->host_used;
+  out->host_cap = c->host_cap;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_victims(grouter_ctx *c, grouter_oid *out, uint64_t cap, uint64_t *n_out) {
+  if (!c || !n_out) return fail(GROUTER_EINVAL, "null argument");
+  Guard g(c);
+  *n_out = c->victims.size();
+  if (c->victims.size() > cap || (!out && !c->victims.empty()))
+    return fail(GROUTER_EINVAL, "victims: cap too small");
+  for (size_t i = 0; i < c->victims.size(); ++i) out[i] = c->victims[i];
+  c->victims.clear();
+  return GROUTER_OK;
+}
+
+grouter_status grouter_dispatch_log(grouter_ctx *c, grouter_dispatch *out, uint64_t cap, uint64_t *n_out) {
+  if (!c || !n_out) return fail(GROUTER_EINVAL, "null argument");
+  Guard g(c);
+  uint64_t k = 0;
+  while (k < cap && !c->dlog.empty() && out) {
+    out[k++] = c->dlog.front();
+    c->dlog.pop_front();
+  }
+  *n_out = k;
+  return GROUTER_OK;
+}
+
+// ------------------------------------------------------------------ standalone scheduler
+struct grouter_sched {
+  struct Item {
+    uint64_t id, bytes;
+  };
+  gr::Stride<Item> s;
+  std::map<uint32_t, uint32_t> w;
+};
+
+grouter_status grouter_sched_new(uint32_t batch, grouter_sched **out) {
+  if (!out || batch < 1 || batch > 8) return fail(GROUTER_EINVAL, "sched_new: bad argument");
+  *out = new grouter_sched();
+  (*out)->s.batch = batch;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_sched_set_weight(grouter_sched *s, uint32_t t, uint32_t w) {
+  if (!s || w < 1) return fail(GROUTER_EINVAL, "sched_set_weight: bad argument");
+  s->w[t] = w;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_sched_enqueue(grouter_sched *s, uint32_t t, uint64_t id, uint64_t bytes) {
+  if (!s) return fail(GROUTER_EINVAL, "null sched");
+  s->s.enqueue(t, {id, bytes});
+  return GROUTER_OK;
+}
+
+grouter_status grouter_sched_dispatch(grouter_sched *s, uint32_t *tenant, uint64_t *ids, uint32_t *n,
+                                      uint64_t *bytes, uint64_t *pass_after) {
+  if (!s || !tenant || !ids || !n || !bytes || !pass_after) return fail(GROUTER_EINVAL, "null argument");
+  std::vector<grouter_sched::Item> b;
+  uint32_t t = s->s.dispatch(
+      [&](uint32_t x) {
+        auto it = s->w.find(x);
+        return it == s->w.end() ? 1u : it->second;
+      },
+      b, bytes, pass_after);
+  if (t == UINT32_MAX) return GROUTER_ENOENT;
+  *tenant = t;
+  *n = (uint32_t)b.size();
+  for (size_t i = 0; i < b.size(); ++i) ids[i] = b[i].id;
+  return GROUTER_OK;
+}
+
+void grouter_sched_free(grouter_sched *s) { delete s; }
+
+}  // extern "C"

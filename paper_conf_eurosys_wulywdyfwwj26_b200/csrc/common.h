@@ -1,0 +1,122 @@
+// common.h -- internal helpers shared by the libgrouter translation units.
+//
+// The library links cudart statically and reaches the driver API through
+// cudaGetDriverEntryPoint, so libgrouter.so loads (and exports its symbols)
+// on a machine without libcuda.so.1; nothing touches CUDA before
+// grouter_init().
+#pragma once
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/grouter.h"
+
+namespace gr {
+
+constexpr uint64_t kPage = 2ull << 20;   // R14: 2 MiB pool pages (= VMM granularity)
+
+inline uint64_t charge(uint64_t n) { return (n + kPage - 1) / kPage * kPage; }
+inline uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// thread-local last error text (grouter_last_error)
+void set_error(const std::string &msg);
+const char *last_error();
+
+// An internal failure that maps to a status at the ABI boundary.
+struct Error : std::runtime_error {
+  grouter_status st;
+  Error(grouter_status s, const std::string &m) : std::runtime_error(m), st(s) {}
+};
+
+#define GR_CUDA(call)                                                                   \
+  do {                                                                                  \
+    cudaError_t e_ = (call);                                                            \
+    if (e_ != cudaSuccess)                                                              \
+      throw ::gr::Error(GROUTER_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+
+#define GR_CU(call)                                                                     \
+  do {                                                                                  \
+    CUresult r_ = (call);                                                               \
+    if (r_ != CUDA_SUCCESS)                                                             \
+      throw ::gr::Error(GROUTER_ECUDA, std::string(#call) + ": CUresult " + std::to_string((int)r_)); \
+  } while (0)
+
+// Driver entry points (resolved once, lazily, through the runtime).
+struct Driver {
+  CUresult (*memCreate)(CUmemGenericAllocationHandle *, size_t, const CUmemAllocationProp *,
+                        unsigned long long);
+  CUresult (*memRelease)(CUmemGenericAllocationHandle);
+  CUresult (*memAddressReserve)(CUdeviceptr *, size_t, size_t, CUdeviceptr, unsigned long long);
+  CUresult (*memAddressFree)(CUdeviceptr, size_t);
+  CUresult (*memMap)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long);
+  CUresult (*memUnmap)(CUdeviceptr, size_t);
+  CUresult (*memSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc *, size_t);
+  CUresult (*memGetAllocationGranularity)(size_t *, const CUmemAllocationProp *,
+                                          CUmemAllocationGranularity_flags);
+  CUresult (*streamWaitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+  CUresult (*streamWriteValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+};
+const Driver &drv();
+
+// Saves/restores the caller's current device around library work.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  void set(int dev) {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (cur != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+// A pooled CUDA event; returns itself to its pool when the last reference drops.
+struct EventPool;
+struct Event {
+  cudaEvent_t ev = nullptr;
+  int phys = -1;
+  EventPool *pool = nullptr;
+};
+using EventRef = std::shared_ptr<Event>;
+
+struct EventPool {
+  int phys = -1;
+  std::mutex mu;
+  std::vector<Event *> free_list;
+  EventRef get();                  // caller must have `phys` current
+  ~EventPool();
+};
+
+// Something the library can wait for: a CUDA event, or a completion word
+// (host-mapped u32) reaching a target value (wrap-safe compare, the same
+// rule as CU_STREAM_WAIT_VALUE_GEQ).  `epoch` = replay epoch of creation.
+struct Waitable {
+  EventRef ev;
+  volatile uint32_t *word = nullptr;
+  uint32_t target = 0;
+  uint64_t epoch = 0;
+  bool done() const {
+    if (word) return (int32_t)(*word - target) >= 0;
+    if (ev) return cudaEventQuery(ev->ev) == cudaSuccess;
+    return true;
+  }
+};
+using Fences = std::vector<Waitable>;
+
+}  // namespace gr

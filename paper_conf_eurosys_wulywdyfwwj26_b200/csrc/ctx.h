@@ -1,0 +1,215 @@
+// ctx.h -- the libgrouter runtime: pools, servers, transfers, object table.
+//
+// Layering: api.cpp (the C ABI, object table, auth, refcounts,
+// eviction: PAPER.md L165-L173, L248-L262, L394) sits on engine.cpp (per-GPU
+// servers, stride scheduling, dispatch rounds, completion words: L182,
+// L193-L229, L269-L271) which drives the sm_100a kernels of kernels.cu and
+// the copy engines; pool.cpp holds the VMM device pools, the pinned host
+// store and the staging rings (L229, L248-L256, L269).
+#pragma once
+
+#include <array>
+#include <atomic>
+#include <condition_variable>
+#include <deque>
+#include <map>
+#include <memory>
+#include <set>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "common.h"
+#include "plan.h"
+#include "stride.h"
+
+namespace gr {
+
+// ------------------------------------------------------------------ pages
+struct Quarantined {
+  uint64_t off, len;
+  Fences fences;
+};
+
+// Page-granular first-fit allocator over offsets, with a quarantine of
+// freed runs that in-flight GPU work may still touch.
+struct PageHeap {
+  std::map<uint64_t, uint64_t> free_runs;  // offset -> length
+  std::vector<Quarantined> quarantine;
+  bool take(uint64_t len, uint64_t *off);
+  void give(uint64_t off, uint64_t len);
+  void reclaim();                           // returns quarantined runs whose fences are done
+  uint64_t free_bytes() const;
+  uint64_t tail_free(uint64_t end) const;   // length of the free run ending at `end`
+};
+
+struct DevicePool {
+  int logical = -1, phys = -1;
+  CUdeviceptr base = 0;
+  uint64_t va_size = 0, mapped = 0;
+  struct Seg {
+    uint64_t off, size;
+    CUmemGenericAllocationHandle h;
+  };
+  std::vector<Seg> segs;
+  PageHeap heap;
+  std::vector<int> access;  // physical devices that may access the pages
+  void init(int logical, int phys, uint64_t va, const std::vector<int> &access, uint64_t prewarm);
+  void grow(uint64_t need);
+  void trim(uint64_t keep);
+  void destroy();
+};
+
+struct HostStore {
+  uint8_t *base = nullptr;
+  uint64_t size = 0;
+  PageHeap heap;
+};
+
+// ------------------------------------------------------------------ transfers
+enum ServerKind { SK_COPY = 0, SK_H2D = 1, SK_D2H = 2 };
+
+struct Xfer {
+  uint64_t id = 0;
+  uint32_t tenant = 0;
+  uint32_t slot = 0;
+  volatile uint32_t *words = nullptr;       // host-mapped completion words of the slot
+  uint32_t target[GROUTER_MAX_PATHS] = {};  // final word value per path
+  uint32_t total[GROUTER_MAX_PATHS] = {};   // chunks per path
+  uint32_t issued[GROUTER_MAX_PATHS] = {};  // chunks dispatched so far per path
+  // absolute word value once the first `issued` chunks of `path` are done
+  uint32_t value_after(uint32_t path) const { return target[path] - total[path] + issued[path]; }
+  uint32_t npath = 0;
+  Fences deps;                              // must complete before the first chunk moves
+  uint64_t deps_waited = 0;                 // bitmask of servers that already waited
+  uint64_t epoch = 0;
+  bool pageable_src = false;
+  void add_done_fences(Fences &f) const;    // "all chunks complete"
+  bool done() const;
+};
+using XferRef = std::shared_ptr<Xfer>;
+
+struct ChunkItem {
+  XferRef x;
+  uint32_t idx;       // chunk index in the plan
+  uint32_t path;
+  uint64_t src, dst;  // absolute addresses (device VA or host)
+  uint64_t bytes;
+  int dst_logical;    // destination device (H2D: relay if != server device)
+};
+
+struct Server {
+  int kind = 0, logical = -1, phys = -1;
+  Stride<ChunkItem> sched;
+  cudaStream_t stream = nullptr;      // SM-copy stream / CE stream
+  cudaStream_t fwd_stream = nullptr;  // H2D: relay forward kernel stream
+  uint32_t *scratch = nullptr;        // device scratch of the copy kernel on `stream`
+  uint32_t *fwd_scratch = nullptr;    // ... on `fwd_stream`
+  std::deque<EventRef> inflight;
+  // H2D relay staging ring on this GPU (device memory)
+  uint8_t *staging = nullptr;
+  uint32_t n_slots = 0, next_slot = 0;
+  uint64_t slot_bytes = 0;
+  std::vector<EventRef> slot_free;
+  uint64_t id_bit() const { return 1ull << (kind * GROUTER_MAX_GPUS + logical); }
+};
+
+// ------------------------------------------------------------------ objects
+enum ObjState { OBJ_OPEN, OBJ_SEALED, OBJ_CONSUMED, OBJ_FREED };
+
+struct Obj {
+  grouter_oid oid = 0;
+  uint32_t wf = 0, fid = 0;
+  uint64_t n = 0;
+  int loc = GROUTER_HOST;
+  uint8_t *ptr = nullptr;          // device VA or host-store address
+  ObjState state = OBJ_OPEN;
+  uint32_t consumers_left = 0;
+  uint32_t pins = 0;
+  uint64_t last_access = 0;
+  bool has_next_use = false;
+  uint64_t next_use = 0;
+  Fences ready;                    // the bytes are in place once these complete
+  Fences readers;                  // in-flight library reads of the bytes
+};
+
+struct Lease {
+  grouter_oid oid;
+  uint32_t wf;
+  int dev;
+  uint8_t *ptr;
+  uint64_t n;
+  Fences fill;                     // the copy into the lease
+};
+
+struct LogicalDev {
+  int phys = -1;
+  DevicePool pool;
+  uint64_t used = 0, cap = GROUTER_UNLIMITED;
+  Server copy, h2d, d2h;
+};
+
+struct PhysDev {
+  int ordinal = -1;
+  int sm_count = 148;
+  EventPool events;
+};
+
+}  // namespace gr
+
+struct grouter_ctx {
+  grouter_config cfg;
+  gr::Planner planner;
+  bool plan_only = false, replay = false;
+  std::mutex mu;                                       // the big lock
+  std::vector<gr::LogicalDev> dev;
+  std::map<int, std::unique_ptr<gr::PhysDev>> phys;
+  gr::HostStore host;
+  uint64_t host_used = 0, host_cap = 0;
+  // completion slots (host-mapped pinned memory)
+  uint32_t *words = nullptr;
+  uint32_t n_slots = 0, next_slot = 0;
+  std::vector<std::array<uint32_t, GROUTER_MAX_PATHS>> slot_final;
+  // pageable-source bounce ring (the circular pinned buffer of L229)
+  uint8_t *bounce = nullptr;
+  uint32_t bounce_slots = 0, bounce_next = 0;
+  std::vector<gr::EventRef> bounce_ev;
+  // object table (L173)
+  std::unordered_map<grouter_oid, gr::Obj> objects;
+  std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
+  std::unordered_map<uint32_t, uint32_t> weights;
+  uint64_t seq = 0, next_oid = 1, xfer_seq = 0;
+  uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
+  std::vector<grouter_oid> victims;
+  std::deque<grouter_dispatch> dlog;
+  grouter_stats_t stats{};
+  // background I/O + dispatch thread (L269, L271)
+  std::thread daemon;
+  std::condition_variable cv;
+  bool stop = false;
+  std::atomic<bool> sticky_error{false};
+};
+
+namespace gr {
+// engine.cpp
+void engine_init(grouter_ctx *c);
+void engine_shutdown(grouter_ctx *c);
+XferRef new_xfer(grouter_ctx *c, uint32_t tenant, const std::vector<grouter_chunk> &plan);
+// Enqueue every chunk of a planned transfer to its server.  src_base/dst_base
+// are the absolute base addresses; kind = server kind for single-path plans,
+// SK_H2D for host->GPU plans.
+void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_chunk> &plan,
+                  int kind, uint64_t src_base, uint64_t dst_base, int dst_logical);
+void pump(grouter_ctx *c, bool force_all);            // dispatch rounds (caller holds mu)
+void flush_all(grouter_ctx *c);                        // replay flush
+void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);
+EventRef record(grouter_ctx *c, cudaStream_t s, int phys);
+void host_wait(const Fences &f, double timeout_s = 120.0);
+bool grounded(const grouter_ctx *c, const Fences &f);
+void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst);  // D2H of a victim (unscheduled)
+// pool.cpp
+uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len);   // may grow the pool
+void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f);
+uint8_t *host_alloc(grouter_ctx *c, uint64_t len);
+void host_free(grouter_ctx *c, uint8_t *p, uint64_t len, Fences &&f);
+}  // namespace gr

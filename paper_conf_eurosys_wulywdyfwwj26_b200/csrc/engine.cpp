@@ -1,0 +1,572 @@
+// engine.cpp -- per-GPU servers: stride-ordered dispatch rounds, copy
+// engines, SM copy/forward kernels, completion words, the daemon thread.
+//
+// chunks are "pipelined across GPU streams, with
+// synchronization primitives ensuring in-order delivery".  L229: batches of
+// 5 chunks so new functions preempt at batch boundaries; a circular pinned
+// buffer is reused across batches.  L269-L271: one daemon per GPU with
+// several streams for the different directions, plus an I/O thread that
+// reclaims memory; fixed PCIe routes generated at init.
+//
+// B200 design:
+//  * A transfer owns a completion SLOT of <= 8 u32 words in pinned,
+//    host-mapped memory, one per path.  Producers publish ABSOLUTE values
+//    (the host knows how many of the transfer's path-p chunks each round
+//    carries): SM kernels with st.release.sys from the round's last CTA, copy
+//    engines with cuStreamWriteValue32 after their memcpys.  Consumers wait
+//    with cuStreamWaitValue32(GEQ) on their own stream, or poll from the
+//    host -- no host round trip on the data path, no partial visibility.
+//  * Each server (SM-copy egress of a GPU, H2D engine of a route GPU, D2H
+//    engine) owns a Stride scheduler; a ROUND = consecutive batches in
+//    stride order up to a byte horizon, executed by ONE kernel launch (SM
+//    copy) or one memcpy burst (CE).  <= 2 rounds in flight per server in
+//    real-time mode; replay mode dispatches only at grouter_flush().
+//  * Host->GPU relay: CE copies a chunk into a staging slot on route GPU r,
+//    an event hands the slot to r's forward stream, the forward round kernel
+//    pushes it over NVLink into the lease on d and publishes the word; the
+//    slot is reused after the forward round's event.
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <thread>
+
+#include "ctx.h"
+#include "kernels.h"
+
+namespace gr {
+
+static const uint32_t kSlots = 4096;
+static const uint32_t kBounceSlots = 16;
+
+// ------------------------------------------------------------------ waits
+bool grounded(const grouter_ctx *c, const Fences &f) {
+  if (!c->replay) return true;
+  for (auto &w : f)
+    if (w.epoch >= c->epoch && !w.done()) return false;
+  return true;
+}
+
+void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f) {
+  (void)c;
+  (void)phys;
+  for (auto &w : f) {
+    if (w.done()) continue;  // fast path: already satisfied, no GPU wait
+    if (w.word) {
+      GR_CU(drv().streamWaitValue32((CUstream)s, (CUdeviceptr)(uintptr_t)w.word, w.target,
+                                    CU_STREAM_WAIT_VALUE_GEQ));
+    } else if (w.ev) {
+      GR_CUDA(cudaStreamWaitEvent(s, w.ev->ev, 0));
+    }
+  }
+}
+
+EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
+  EventRef e = c->phys.at(phys)->events.get();
+  GR_CUDA(cudaEventRecord(e->ev, s));
+  return e;
+}
+
+void host_wait(const Fences &f, double timeout_s) {
+  auto t0 = std::chrono::steady_clock::now();
+  for (auto &w : f) {
+    if (w.ev && !w.word) {
+      GR_CUDA(cudaEventSynchronize(w.ev->ev));
+      continue;
+    }
+    uint32_t spins = 0;
+    while (!w.done()) {
+      if (++spins > 64) std::this_thread::yield();
+      if ((spins & 1023) == 0) {
+        double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        if (dt > timeout_s) throw Error(GROUTER_ECUDA, "timeout waiting for a transfer");
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ transfers
+void Xfer::add_done_fences(Fences &f) const {
+  for (uint32_t p = 0; p < npath; ++p) {
+    if (!total[p]) continue;
+    Waitable w;
+    w.word = &words[p];
+    w.target = target[p];
+    w.epoch = epoch;
+    f.push_back(w);
+  }
+}
+
+bool Xfer::done() const {
+  for (uint32_t p = 0; p < npath; ++p)
+    if (total[p] && (int32_t)(words[p] - target[p]) < 0) return false;
+  return true;
+}
+
+XferRef new_xfer(grouter_ctx *c, uint32_t tenant, const std::vector<grouter_chunk> &plan) {
+  auto x = std::make_shared<Xfer>();
+  x->id = ++c->xfer_seq;
+  x->tenant = tenant;
+  x->epoch = c->epoch;
+  uint32_t np = 1;
+  for (auto &ch : plan) {
+    x->total[ch.path]++;
+    np = std::max<uint32_t>(np, (uint32_t)ch.path + 1);
+  }
+  x->npath = np;
+  // a slot is reusable once its previous transfer has completed
+  for (uint32_t tries = 0; tries < c->n_slots; ++tries) {
+    uint32_t s = c->next_slot;
+    c->next_slot = (c->next_slot + 1) % c->n_slots;
+    volatile uint32_t *w = c->words + (uint64_t)s * GROUTER_MAX_PATHS;
+    bool free_ = true;
+    for (int p = 0; p < GROUTER_MAX_PATHS; ++p)
+      if ((int32_t)(w[p] - c->slot_final[s][p]) < 0) free_ = false;
+    if (!free_) continue;
+    x->slot = s;
+    x->words = w;
+    for (uint32_t p = 0; p < np; ++p) {
+      x->target[p] = c->slot_final[s][p] + x->total[p];
+      c->slot_final[s][p] = x->target[p];
+    }
+    c->stats.xfer_count++;
+    return x;
+  }
+  throw Error(GROUTER_EBUSY, "no free completion slot (too many transfers in flight)");
+}
+
+static Server &server_of(grouter_ctx *c, int kind, int logical) {
+  LogicalDev &d = c->dev[logical];
+  return kind == SK_COPY ? d.copy : kind == SK_H2D ? d.h2d : d.d2h;
+}
+
+void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_chunk> &plan, int kind,
+                  uint64_t src_base, uint64_t dst_base, int dst_logical) {
+  for (uint32_t i = 0; i < plan.size(); ++i) {
+    const grouter_chunk &ch = plan[i];
+    ChunkItem it;
+    it.x = x;
+    it.idx = i;
+    it.path = (uint32_t)ch.path;
+    it.src = src_base + ch.offset;
+    it.dst = dst_base + ch.offset;
+    it.bytes = ch.bytes;
+    it.dst_logical = dst_logical;
+    server_of(c, kind, ch.route_gpu).sched.enqueue(x->tenant, it);
+  }
+}
+
+// ------------------------------------------------------------------ rounds
+static uint32_t weight_of(grouter_ctx *c, uint32_t t) {
+  auto it = c->weights.find(t);
+  return it == c->weights.end() ? 1u : it->second;
+}
+
+static void log_batch(grouter_ctx *c, const Server &s, uint32_t tenant,
+                      const std::vector<ChunkItem> &b, uint64_t bytes) {
+  if (!(c->replay || (c->cfg.flags & GROUTER_LOG))) return;
+  grouter_dispatch d{};
+  d.server_kind = s.kind;
+  d.server_dev = s.logical;
+  d.tenant = tenant;
+  d.n_chunks = (uint32_t)b.size();
+  for (size_t i = 0; i < b.size() && i < 8; ++i) d.chunk_ids[i] = (b[i].x->id << 32) | b[i].idx;
+  d.bytes = bytes;
+  c->dlog.push_back(d);
+  if (c->dlog.size() > (1u << 20)) c->dlog.pop_front();
+}
+
+// Pops whole batches (stride order) for one round.
+static void take_round(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes,
+                       uint32_t max_chunks, std::vector<ChunkItem> &round) {
+  round.clear();
+  std::vector<ChunkItem> b;
+  uint64_t bytes = 0;
+  uint32_t nb = 0, npub = 0;
+  const uint32_t batch = s.sched.batch;
+  while (!s.sched.empty() && nb < max_batches && bytes < max_bytes &&
+         round.size() + batch <= max_chunks && npub + batch <= (uint32_t)kMaxPublish) {
+    uint64_t bb = 0;
+    uint32_t t = s.sched.dispatch([&](uint32_t tn) { return weight_of(c, tn); }, b, &bb);
+    if (t == UINT32_MAX) break;
+    log_batch(c, s, t, b, bb);
+    round.insert(round.end(), b.begin(), b.end());
+    bytes += bb;
+    npub += (uint32_t)b.size();
+    ++nb;
+  }
+  c->stats.rounds++;
+}
+
+static void wait_deps(grouter_ctx *c, Server &s, cudaStream_t st, const std::vector<ChunkItem> &items) {
+  for (auto &it : items) {
+    Xfer &x = *it.x;
+    if (x.deps_waited & s.id_bit()) continue;
+    x.deps_waited |= s.id_bit();
+    stream_wait(c, st, s.phys, x.deps);
+  }
+}
+
+// Marks the items as issued and returns the distinct (xfer, path) pairs with
+// their absolute word values after these items complete.
+struct Pub {
+  Xfer *x;
+  uint32_t path;
+};
+static std::vector<Pub> issue(const std::vector<ChunkItem> &items) {
+  std::vector<Pub> pubs;
+  for (auto &it : items) {
+    Xfer *x = it.x.get();
+    x->issued[it.path]++;
+    bool found = false;
+    for (auto &p : pubs) found |= (p.x == x && p.path == it.path);
+    if (!found) pubs.push_back({x, it.path});
+  }
+  return pubs;
+}
+
+static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *scratch,
+                         const std::vector<ChunkItem> &items, const uint64_t *src_override) {
+  auto p = std::make_unique<CopyParams>();
+  p->n_chunks = (uint32_t)items.size();
+  p->scratch = scratch;
+  p->tile_log2 = 16;
+  uint64_t t = 0;
+  for (size_t i = 0; i < items.size(); ++i) {
+    p->chunk[i] = {src_override ? src_override[i] : items[i].src, items[i].dst, items[i].bytes};
+    p->tile_prefix[i] = t;
+    t += (items[i].bytes + (1ull << p->tile_log2) - 1) >> p->tile_log2;
+  }
+  p->tile_prefix[items.size()] = t;
+  std::vector<Pub> pubs = issue(items);
+  p->n_pub = (uint32_t)pubs.size();
+  for (size_t i = 0; i < pubs.size(); ++i) {
+    p->pub[i].word = (uint64_t)(uintptr_t)&pubs[i].x->words[pubs[i].path];
+    p->pub[i].value = pubs[i].x->value_after(pubs[i].path);
+  }
+  PhysDev &pd = *c->phys.at(s.phys);
+  int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm,
+                      (c->cfg.flags & GROUTER_COPY_TMA) != 0, st);
+  if (e != 0)
+    throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
+  c->stats.kernel_launches++;
+}
+
+// SM-copy server: one kernel launch per round (D2D push over NVLink, or a
+// same-GPU HBM copy).
+static void round_copy(grouter_ctx *c, Server &s) {
+  std::vector<ChunkItem> items;
+  take_round(c, s, UINT32_MAX, c->cfg.round_bytes, (uint32_t)kMaxRoundChunks, items);
+  if (items.empty()) return;
+  DeviceGuard g(s.phys);
+  wait_deps(c, s, s.stream, items);
+  launch_round(c, s, s.stream, s.scratch, items, nullptr);
+  for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
+  s.inflight.push_back(record(c, s.stream, s.phys));
+}
+
+// Copies a pageable host chunk into the circular pinned buffer (L229) and
+// returns the pinned address to DMA from.
+static uint64_t bounce(grouter_ctx *c, cudaStream_t st, int phys, uint64_t src, uint64_t bytes) {
+  uint32_t k = c->bounce_next;
+  c->bounce_next = (k + 1) % c->bounce_slots;
+  if (c->bounce_ev[k]) GR_CUDA(cudaEventSynchronize(c->bounce_ev[k]->ev));
+  uint8_t *slot = c->bounce + (uint64_t)k * c->cfg.chunk_bytes;
+  std::memcpy(slot, (const void *)src, bytes);
+  (void)st;
+  (void)phys;
+  return (uint64_t)slot;
+}
+
+// H2D server of route GPU r: CE copies of up to two batches (L229); chunks
+// for r itself land in the lease, relayed chunks go through r's staging
+// ring and one forward round kernel on r pushes them to their destination.
+static void round_h2d(grouter_ctx *c, Server &s) {
+  std::vector<ChunkItem> items;
+  take_round(c, s, 2, UINT64_MAX, (uint32_t)kMaxRoundChunks, items);
+  if (items.empty()) return;
+  DeviceGuard g(s.phys);
+  wait_deps(c, s, s.stream, items);
+  std::vector<ChunkItem> direct, relay;
+  std::vector<uint64_t> slot_src;
+  std::vector<uint32_t> slots_used;
+  for (auto &it : items) {
+    uint64_t src = it.src;
+    if (it.x->pageable_src) {
+      src = bounce(c, s.stream, s.phys, it.src, it.bytes);
+    }
+    if (it.dst_logical == s.logical) {
+      GR_CUDA(cudaMemcpyAsync((void *)it.dst, (const void *)src, it.bytes, cudaMemcpyHostToDevice,
+                              s.stream));
+      direct.push_back(it);
+    } else {
+      uint32_t k = s.next_slot;
+      s.next_slot = (k + 1) % s.n_slots;
+      if (s.slot_free[k]) GR_CUDA(cudaStreamWaitEvent(s.stream, s.slot_free[k]->ev, 0));
+      uint8_t *slot = s.staging + (uint64_t)k * s.slot_bytes;
+      GR_CUDA(cudaMemcpyAsync(slot, (const void *)src, it.bytes, cudaMemcpyHostToDevice, s.stream));
+      relay.push_back(it);
+      slot_src.push_back((uint64_t)slot);
+      slots_used.push_back(k);
+    }
+    if (it.x->pageable_src) c->bounce_ev[(c->bounce_next + c->bounce_slots - 1) % c->bounce_slots] =
+        record(c, s.stream, s.phys);
+    c->stats.link_bytes[1][s.logical] += it.bytes;
+  }
+  for (auto &p : issue(direct))
+    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
+                                   p.x->value_after(p.path), 0));
+  if (!relay.empty()) {
+    EventRef ce = record(c, s.stream, s.phys);
+    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
+    launch_round(c, s, s.fwd_stream, s.fwd_scratch, relay, slot_src.data());
+    EventRef fwd = record(c, s.fwd_stream, s.phys);
+    for (uint32_t k : slots_used) s.slot_free[k] = fwd;
+    s.inflight.push_back(fwd);
+  } else {
+    s.inflight.push_back(record(c, s.stream, s.phys));
+  }
+}
+
+// D2H server: CE copies device -> host (host store, host leases, caller
+// host buffers).
+static void round_d2h(grouter_ctx *c, Server &s) {
+  std::vector<ChunkItem> items;
+  take_round(c, s, 2, UINT64_MAX, (uint32_t)kMaxRoundChunks, items);
+  if (items.empty()) return;
+  DeviceGuard g(s.phys);
+  wait_deps(c, s, s.stream, items);
+  for (auto &it : items) {
+    GR_CUDA(cudaMemcpyAsync((void *)it.dst, (const void *)it.src, it.bytes, cudaMemcpyDeviceToHost,
+                            s.stream));
+    c->stats.link_bytes[2][s.logical] += it.bytes;
+  }
+  for (auto &p : issue(items))
+    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
+                                   p.x->value_after(p.path), 0));
+  s.inflight.push_back(record(c, s.stream, s.phys));
+}
+
+static void retire(Server &s) {
+  while (!s.inflight.empty() && cudaEventQuery(s.inflight.front()->ev) == cudaSuccess)
+    s.inflight.pop_front();
+}
+
+static void pump_server(grouter_ctx *c, Server &s, bool force) {
+  if (!s.stream) return;
+  retire(s);
+  while (!s.sched.empty() && (force || s.inflight.size() < 2)) {
+    if (s.kind == SK_COPY) round_copy(c, s);
+    else if (s.kind == SK_H2D) round_h2d(c, s);
+    else round_d2h(c, s);
+  }
+}
+
+void pump(grouter_ctx *c, bool force_all) {
+  if (c->replay && !force_all) return;
+  for (auto &d : c->dev) {
+    pump_server(c, d.copy, force_all);
+    pump_server(c, d.h2d, force_all);
+    pump_server(c, d.d2h, force_all);
+  }
+  bool backlog = false;
+  for (auto &d : c->dev) backlog |= !d.copy.sched.empty() || !d.h2d.sched.empty() || !d.d2h.sched.empty();
+  if (backlog) c->cv.notify_one();
+}
+
+void flush_all(grouter_ctx *c) {
+  pump(c, true);
+  c->epoch++;   // everything created before is now dispatched (grounded)
+}
+
+// Unscheduled D2H of an eviction victim (L258-L262; the per-GPU I/O path of L269).
+void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
+  Server &s = c->dev[o.loc].d2h;
+  DeviceGuard g(s.phys);
+  stream_wait(c, s.stream, s.phys, o.ready);
+  if (o.n)
+    GR_CUDA(cudaMemcpyAsync(host_dst, o.ptr, o.n, cudaMemcpyDeviceToHost, s.stream));
+  Waitable w;
+  w.ev = record(c, s.stream, s.phys);
+  w.epoch = c->epoch;
+  Fences old = std::move(o.readers);
+  for (auto &f : o.ready) old.push_back(f);
+  old.push_back(w);
+  dev_free(c, o.loc, o.ptr, charge(o.n), std::move(old));
+  o.ready.clear();
+  o.ready.push_back(w);
+  o.readers.clear();
+  c->stats.spill_count++;
+  c->stats.spill_bytes += o.n;
+  c->stats.link_bytes[2][o.loc] += o.n;
+}
+
+// ------------------------------------------------------------------ lifecycle
+static void daemon_main(grouter_ctx *c) {
+  std::unique_lock<std::mutex> lk(c->mu);
+  auto last_trim = std::chrono::steady_clock::now();
+  while (!c->stop) {
+    bool backlog = false, busy = false;
+    try {
+      if (!c->replay) {
+        for (auto &d : c->dev) {
+          pump_server(c, d.copy, false);
+          pump_server(c, d.h2d, false);
+          pump_server(c, d.d2h, false);
+        }
+      }
+      for (auto &d : c->dev) {
+        backlog |= !d.copy.sched.empty() || !d.h2d.sched.empty() || !d.d2h.sched.empty();
+        busy |= !d.copy.inflight.empty() || !d.h2d.inflight.empty() || !d.d2h.inflight.empty();
+        if (!c->replay) {
+          retire(d.copy);
+          retire(d.h2d);
+          retire(d.d2h);
+        }
+      }
+      auto now = std::chrono::steady_clock::now();
+      if (now - last_trim > std::chrono::milliseconds(50)) {  // I/O thread: reclaim (L269)
+        last_trim = now;
+        for (auto &d : c->dev) {
+          DeviceGuard g(d.phys);
+          d.pool.heap.reclaim();
+          uint64_t floor_ = std::min<uint64_t>(c->cfg.pool_floor_bytes, d.cap);
+          d.pool.trim(std::max<uint64_t>(d.used, floor_) + (64ull << 20));
+        }
+        c->host.heap.reclaim();
+      }
+    } catch (const Error &e) {
+      set_error(e.what());
+      c->sticky_error = true;
+    }
+    if (backlog && !c->replay) {
+      lk.unlock();
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+      lk.lock();
+    } else {
+      c->cv.wait_for(lk, busy ? std::chrono::milliseconds(1) : std::chrono::milliseconds(20));
+    }
+  }
+}
+
+void engine_init(grouter_ctx *c) {
+  const int n = (int)c->cfg.n_gpus;
+  int ndev = 0;
+  GR_CUDA(cudaGetDeviceCount(&ndev));
+  for (int i = 0; i < n; ++i) {
+    int p = c->cfg.device_map[i];
+    if (p < 0 || p >= ndev) throw Error(GROUTER_EINVAL, "device_map entry out of range");
+    if (!c->phys.count(p)) {
+      auto pd = std::make_unique<PhysDev>();
+      pd->ordinal = p;
+      pd->events.phys = p;
+      GR_CUDA(cudaDeviceGetAttribute(&pd->sm_count, cudaDevAttrMultiProcessorCount, p));
+      c->phys[p] = std::move(pd);
+    }
+  }
+  // peer access between every pair of physical GPUs that supports it
+  std::vector<int> phys_list;
+  for (auto &kv : c->phys) phys_list.push_back(kv.first);
+  for (int a : phys_list)
+    for (int b : phys_list) {
+      if (a == b) continue;
+      int ok = 0;
+      cudaDeviceCanAccessPeer(&ok, a, b);
+      if (ok) {
+        DeviceGuard g(a);
+        cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+          throw Error(GROUTER_ECUDA, "cudaDeviceEnablePeerAccess failed");
+        cudaGetLastError();
+      }
+    }
+  // completion words (pinned, mapped; written by kernels and copy engines)
+  c->n_slots = kSlots;
+  GR_CUDA(cudaHostAlloc((void **)&c->words, (size_t)kSlots * GROUTER_MAX_PATHS * 4,
+                        cudaHostAllocMapped | cudaHostAllocPortable));
+  std::memset(c->words, 0, (size_t)kSlots * GROUTER_MAX_PATHS * 4);
+  c->slot_final.assign(kSlots, {});
+  // circular pinned bounce ring for pageable host sources (L229)
+  c->bounce_slots = kBounceSlots;
+  GR_CUDA(cudaHostAlloc((void **)&c->bounce, (size_t)kBounceSlots * c->cfg.chunk_bytes,
+                        cudaHostAllocPortable));
+  c->bounce_ev.assign(kBounceSlots, nullptr);
+  // pinned host store (+ headroom so page fragmentation never decides a
+  // placement that the capacity accounting admitted)
+  c->host_cap = c->cfg.host_store_bytes / kPage * kPage;
+  c->host.size = c->host_cap * 2 + (64ull << 20);
+  GR_CUDA(cudaHostAlloc((void **)&c->host.base, c->host.size,
+                        cudaHostAllocMapped | cudaHostAllocPortable));
+  c->host.heap.give(0, c->host.size / kPage * kPage);
+  // per logical GPU: pool, servers
+  const bool multi = n > 1 && !(c->cfg.flags & GROUTER_NO_MULTIPATH);
+  for (int i = 0; i < n; ++i) {
+    gr::LogicalDev &d = c->dev[i];
+    d.phys = c->cfg.device_map[i];
+    DeviceGuard g(d.phys);
+    size_t fr = 0, tot = 0;
+    GR_CUDA(cudaMemGetInfo(&fr, &tot));
+    if (c->cfg.pool_cap_bytes[i]) d.cap = c->cfg.pool_cap_bytes[i];
+    else d.cap = (uint64_t)((unsigned __int128)fr * c->cfg.pool_cap_permille / 1000) / kPage * kPage;
+    uint64_t prewarm = std::min<uint64_t>(c->cfg.pool_floor_bytes, d.cap == GROUTER_UNLIMITED ? c->cfg.pool_floor_bytes : d.cap);
+    d.pool.init(i, d.phys, (uint64_t)tot * 2 / kPage * kPage, phys_list, prewarm / kPage * kPage);
+    Server *ss[3] = {&d.copy, &d.h2d, &d.d2h};
+    for (int k = 0; k < 3; ++k) {
+      Server &s = *ss[k];
+      s.kind = k;
+      s.logical = i;
+      s.phys = d.phys;
+      s.sched.batch = c->cfg.batch_chunks;
+      int lo = 0, hi = 0;
+      cudaDeviceGetStreamPriorityRange(&lo, &hi);
+      GR_CUDA(cudaStreamCreateWithPriority(&s.stream, cudaStreamNonBlocking, hi));
+    }
+    GR_CUDA(cudaMalloc(&d.copy.scratch, 64));
+    GR_CUDA(cudaMemset(d.copy.scratch, 0, 64));
+    if (multi) {
+      int lo = 0, hi = 0;
+      cudaDeviceGetStreamPriorityRange(&lo, &hi);
+      GR_CUDA(cudaStreamCreateWithPriority(&d.h2d.fwd_stream, cudaStreamNonBlocking, hi));
+      GR_CUDA(cudaMalloc(&d.h2d.fwd_scratch, 64));
+      GR_CUDA(cudaMemset(d.h2d.fwd_scratch, 0, 64));
+      d.h2d.n_slots = 4 * c->cfg.batch_chunks;  // two rounds of two batches in flight
+      d.h2d.slot_bytes = c->cfg.chunk_bytes;
+      GR_CUDA(cudaMalloc(&d.h2d.staging, (size_t)d.h2d.n_slots * d.h2d.slot_bytes));
+      d.h2d.slot_free.assign(d.h2d.n_slots, nullptr);
+    }
+    GR_CUDA(cudaDeviceSynchronize());
+  }
+  c->daemon = std::thread(daemon_main, c);
+}
+
+void engine_shutdown(grouter_ctx *c) {
+  {
+    std::lock_guard<std::mutex> lk(c->mu);
+    c->stop = true;
+  }
+  c->cv.notify_all();
+  if (c->daemon.joinable()) c->daemon.join();
+  for (auto &d : c->dev) {
+    DeviceGuard g(d.phys);
+    cudaDeviceSynchronize();
+    Server *ss[3] = {&d.copy, &d.h2d, &d.d2h};
+    for (Server *s : ss) {
+      s->inflight.clear();
+      s->slot_free.clear();
+      if (s->stream) cudaStreamDestroy(s->stream);
+      if (s->fwd_stream) cudaStreamDestroy(s->fwd_stream);
+      if (s->scratch) cudaFree(s->scratch);
+      if (s->fwd_scratch) cudaFree(s->fwd_scratch);
+      if (s->staging) cudaFree(s->staging);
+    }
+    d.pool.heap.quarantine.clear();
+    d.pool.destroy();
+  }
+  c->bounce_ev.clear();
+  c->host.heap.quarantine.clear();
+  if (c->host.base) cudaFreeHost(c->host.base);
+  if (c->bounce) cudaFreeHost(c->bounce);
+  if (c->words) cudaFreeHost(c->words);
+  c->phys.clear();
+}
+
+}  // namespace gr

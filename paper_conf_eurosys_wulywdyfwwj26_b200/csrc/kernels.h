@@ -1,0 +1,46 @@
+// kernels.h -- host-side launch interface of the sm_100a data-movement kernels.
+//
+// gr_copy (SURVEY K2'/K4'): one launch moves a whole dispatch ROUND -- a list
+// of chunks in stride order (L229) -- with a persistent grid whose CTAs claim
+// 64 KiB tiles from a ticket in device scratch, in round order.  The same
+// kernel is the NVLink D2D push (dst = peer VA), the same-GPU HBM copy, and
+// the relay forward hop of striped host->GPU transfers (src = staging slot
+// on the route GPU, dst = lease on the destination).  When the last CTA
+// finishes it publishes per-(transfer, path) completion values with
+// system-scope release stores (L182 "synchronization primitives ensuring
+// in-order delivery": consumers see nothing until the whole payload landed).
+#pragma once
+
+#include <cstdint>
+
+namespace gr {
+
+constexpr int kMaxRoundChunks = 128;
+constexpr int kMaxPublish = 64;
+
+struct KChunk {
+  uint64_t src, dst, bytes;
+};
+struct KPublish {
+  uint64_t word;   // address of a u32 completion word (host-mapped or device)
+  uint32_t value;
+  uint32_t pad;
+};
+
+struct CopyParams {
+  uint32_t n_chunks = 0, n_pub = 0;
+  uint32_t tile_log2 = 16;
+  uint32_t _pad = 0;
+  uint32_t *scratch = nullptr;   // [0] tile ticket, [1] finished CTAs; zero between launches
+  uint32_t *counts = nullptr;    // test only: bytes written per 16 B granule
+  uint64_t count_base = 0;
+  uint64_t tile_prefix[kMaxRoundChunks + 1] = {};
+  KChunk chunk[kMaxRoundChunks];
+  KPublish pub[kMaxPublish];
+};
+
+// Launch gr_copy on `stream` (current device must own the stream).  grid =
+// min(tiles, sm_count * ctas_per_sm).  Returns cudaError_t as int.
+int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream);
+
+}  // namespace gr

@@ -1,0 +1,39 @@
+// plan.h -- route sets and the chunk splitter (host side, integer only).
+//
+// PAPER.md L178 (stage host data over route GPUs' PCIe links, exclude GPUs
+// behind the same PCIe switch), L131 (shared switches contend), L182 (2 MB
+// chunks, precomputed plan), L242 (chunk size proportional to path
+// capacity), L271 (routes pre-generated at init).  The split objective (exact
+// minimum makespan, canonical fill in route order, interleaved layout) is
+// the reading R3/R4 in DESIGN.md.  All arithmetic is integer (R30).
+#pragma once
+
+#include <cstdint>
+#include <vector>
+
+#include "../../include/grouter.h"
+
+namespace gr {
+
+struct PathModel {
+  int route_gpu;
+  uint64_t alpha_ps;  // per-chunk overhead
+  uint64_t beta_Bps;  // bandwidth
+  uint64_t phi_ps;    // fill latency
+  uint64_t chunk;     // C_p
+};
+
+struct Planner {
+  grouter_config cfg;
+  std::vector<std::vector<int>> groups;          // uplink groups, each sorted
+  std::vector<std::vector<int>> routes;          // R(d) per destination
+  std::vector<std::vector<PathModel>> paths;     // per destination, in route order
+
+  void build(const grouter_config &c);
+  // host -> d striped plan (O6); D2D/same-GPU/D2H single-path plan.
+  void plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const;
+  void plan_single(uint64_t n, int route_gpu, std::vector<grouter_chunk> &out) const;
+  void plan(int src_loc, int dst_loc, uint64_t n, std::vector<grouter_chunk> &out) const;
+};
+
+}  // namespace gr

@@ -1,0 +1,284 @@
+// pool.cpp -- elastic GPU object pool, pinned host store, error/driver plumbing.
+//
+// PAPER.md L248 (cudaMalloc/cudaFree are millisecond-level -> pool), L256
+// (minimum warm pool "e.g., 300 MB", scale with demand), L262 (storage kept
+// under 50% of free memory), L269 (per-GPU elastic pool; an I/O thread
+// reclaims unused memory), L394 ("enforced alignment" of mapped storage).
+//
+// Device pool = one CUDA VMM virtual range per logical GPU, backed by
+// physical segments mapped contiguously from its base; objects and leases
+// are page-aligned runs (2 MiB, R14) of that range.  Freed runs go to a
+// quarantine until every GPU operation that may still touch them has
+// completed (stream-ordered reuse without host synchronisation on the hot
+// path); the pool grows by mapping more segments at its end and trims
+// trailing free segments back toward the warm floor.
+#include <chrono>
+#include <cstdio>
+#include <thread>
+
+#include "ctx.h"
+
+namespace gr {
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string tl_error;
+void set_error(const std::string &msg) { tl_error = msg; }
+const char *last_error() { return tl_error.c_str(); }
+
+// ------------------------------------------------------------------ driver
+template <class F>
+static void resolve(const char *name, F &fn) {
+  void *p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || !p)
+    throw Error(GROUTER_ECUDA, std::string("driver entry point missing: ") + name);
+  fn = reinterpret_cast<F>(p);
+}
+
+const Driver &drv() {
+  static Driver d;
+  static std::once_flag once;
+  static std::string err;
+  std::call_once(once, [] {
+    try {
+      resolve("cuMemCreate", d.memCreate);
+      resolve("cuMemRelease", d.memRelease);
+      resolve("cuMemAddressReserve", d.memAddressReserve);
+      resolve("cuMemAddressFree", d.memAddressFree);
+      resolve("cuMemMap", d.memMap);
+      resolve("cuMemUnmap", d.memUnmap);
+      resolve("cuMemSetAccess", d.memSetAccess);
+      resolve("cuMemGetAllocationGranularity", d.memGetAllocationGranularity);
+      resolve("cuStreamWaitValue32", d.streamWaitValue32);
+      resolve("cuStreamWriteValue32", d.streamWriteValue32);
+    } catch (const Error &e) {
+      err = e.what();
+    }
+  });
+  if (!err.empty()) throw Error(GROUTER_ECUDA, err);
+  return d;
+}
+
+// ------------------------------------------------------------------ events
+EventRef EventPool::get() {
+  Event *e = nullptr;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    if (!free_list.empty()) {
+      e = free_list.back();
+      free_list.pop_back();
+    }
+  }
+  if (!e) {
+    e = new Event();
+    e->phys = phys;
+    e->pool = this;
+    GR_CUDA(cudaEventCreateWithFlags(&e->ev, cudaEventDisableTiming));
+  }
+  return EventRef(e, [](Event *ev) {
+    std::lock_guard<std::mutex> g(ev->pool->mu);
+    ev->pool->free_list.push_back(ev);
+  });
+}
+
+EventPool::~EventPool() {
+  for (Event *e : free_list) {
+    cudaEventDestroy(e->ev);
+    delete e;
+  }
+}
+
+// ------------------------------------------------------------------ page heap
+bool PageHeap::take(uint64_t len, uint64_t *off) {
+  for (auto it = free_runs.begin(); it != free_runs.end(); ++it) {
+    if (it->second >= len) {
+      *off = it->first;
+      uint64_t rest = it->second - len, o = it->first;
+      free_runs.erase(it);
+      if (rest) free_runs[o + len] = rest;
+      return true;
+    }
+  }
+  return false;
+}
+
+void PageHeap::give(uint64_t off, uint64_t len) {
+  if (!len) return;
+  auto nx = free_runs.lower_bound(off);
+  if (nx != free_runs.end() && off + len == nx->first) {
+    len += nx->second;
+    nx = free_runs.erase(nx);
+  }
+  if (nx != free_runs.begin()) {
+    auto pv = std::prev(nx);
+    if (pv->first + pv->second == off) {
+      pv->second += len;
+      return;
+    }
+  }
+  free_runs[off] = len;
+}
+
+void PageHeap::reclaim() {
+  size_t w = 0;
+  for (size_t i = 0; i < quarantine.size(); ++i) {
+    bool done = true;
+    for (auto &f : quarantine[i].fences)
+      if (!f.done()) {
+        done = false;
+        break;
+      }
+    if (done) give(quarantine[i].off, quarantine[i].len);
+    else quarantine[w++] = std::move(quarantine[i]);
+  }
+  quarantine.resize(w);
+}
+
+uint64_t PageHeap::free_bytes() const {
+  uint64_t s = 0;
+  for (auto &kv : free_runs) s += kv.second;
+  return s;
+}
+
+uint64_t PageHeap::tail_free(uint64_t end) const {
+  if (free_runs.empty()) return 0;
+  auto it = std::prev(free_runs.end());
+  return it->first + it->second == end ? it->second : 0;
+}
+
+// ------------------------------------------------------------------ device pool
+void DevicePool::init(int lg, int ph, uint64_t va, const std::vector<int> &acc, uint64_t prewarm) {
+  logical = lg;
+  phys = ph;
+  access = acc;
+  va_size = va;
+  GR_CU(drv().memAddressReserve(&base, va_size, kPage, 0, 0));
+  if (prewarm) grow(prewarm);
+}
+
+void DevicePool::grow(uint64_t need) {
+  need = charge(need);
+  uint64_t seg = std::max<uint64_t>(need, 64ull << 20);
+  if (mapped + seg > va_size) seg = need;
+  if (mapped + seg > va_size) throw Error(GROUTER_ENOMEM, "pool VA range exhausted");
+  CUmemAllocationProp prop = {};
+  prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  prop.location.id = phys;
+  prop.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;  // IPC-exportable (L167)
+  CUmemGenericAllocationHandle h;
+  CUresult r = drv().memCreate(&h, seg, &prop, 0);
+  if (r != CUDA_SUCCESS && seg > need) {
+    seg = need;
+    r = drv().memCreate(&h, seg, &prop, 0);
+  }
+  if (r != CUDA_SUCCESS) throw Error(GROUTER_ENOMEM, "cuMemCreate failed (HBM exhausted)");
+  GR_CU(drv().memMap(base + mapped, seg, 0, h, 0));
+  std::vector<CUmemAccessDesc> ad;
+  for (int p : access) {
+    CUmemAccessDesc a = {};
+    a.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    a.location.id = p;
+    a.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+    ad.push_back(a);
+  }
+  GR_CU(drv().memSetAccess(base + mapped, seg, ad.data(), ad.size()));
+  segs.push_back({mapped, seg, h});
+  heap.give(mapped, seg);
+  mapped += seg;
+}
+
+// Unmaps trailing segments that are entirely free while the mapping stays >= keep.
+void DevicePool::trim(uint64_t keep) {
+  heap.reclaim();
+  while (!segs.empty()) {
+    Seg s = segs.back();
+    if (mapped - s.size < keep) break;
+    if (heap.tail_free(mapped) < s.size) break;
+    uint64_t off = 0;
+    // carve the segment out of the trailing free run
+    auto it = std::prev(heap.free_runs.end());
+    uint64_t run_off = it->first;
+    heap.free_runs.erase(it);
+    if (s.off > run_off) heap.free_runs[run_off] = s.off - run_off;
+    (void)off;
+    drv().memUnmap(base + s.off, s.size);
+    drv().memRelease(s.h);
+    mapped -= s.size;
+    segs.pop_back();
+  }
+}
+
+void DevicePool::destroy() {
+  for (auto &s : segs) {
+    drv().memUnmap(base + s.off, s.size);
+    drv().memRelease(s.h);
+  }
+  segs.clear();
+  if (base) drv().memAddressFree(base, va_size);
+  base = 0;
+  mapped = 0;
+}
+
+static bool all_grounded(const grouter_ctx *c, const Quarantined &q) {
+  return grounded(c, q.fences);
+}
+
+// Physical pages for `len` bytes (a multiple of 2 MiB) on a logical GPU.
+// Order: free runs; reclaimed quarantine; wait for grounded quarantine (after
+// draining queued work so no wait depends on the caller); grow the mapping.
+uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
+  DevicePool &P = c->dev[logical].pool;
+  uint64_t off;
+  P.heap.reclaim();
+  if (P.heap.take(len, &off)) return (uint8_t *)(P.base + off);
+  bool any = false;
+  for (auto &q : P.heap.quarantine) any |= all_grounded(c, q);
+  if (any) {
+    if (!c->replay) pump(c, true);
+    for (auto &q : P.heap.quarantine)
+      if (all_grounded(c, q)) host_wait(q.fences);
+    P.heap.reclaim();
+    if (P.heap.take(len, &off)) return (uint8_t *)(P.base + off);
+  }
+  P.grow(len - std::min(len, P.heap.tail_free(P.mapped)));
+  if (!P.heap.take(len, &off)) throw Error(GROUTER_ENOMEM, "pool fragmentation");
+  return (uint8_t *)(P.base + off);
+}
+
+void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f) {
+  if (!len) return;
+  DevicePool &P = c->dev[logical].pool;
+  uint64_t off = (uint64_t)p - P.base;
+  bool done = true;
+  for (auto &w : f) done &= w.done();
+  if (done) P.heap.give(off, len);
+  else P.heap.quarantine.push_back({off, len, std::move(f)});
+}
+
+uint8_t *host_alloc(grouter_ctx *c, uint64_t len) {
+  uint64_t off;
+  c->host.heap.reclaim();
+  if (c->host.heap.take(len, &off)) return c->host.base + off;
+  bool any = false;
+  for (auto &q : c->host.heap.quarantine) any |= all_grounded(c, q);
+  if (any) {
+    if (!c->replay) pump(c, true);
+    for (auto &q : c->host.heap.quarantine)
+      if (all_grounded(c, q)) host_wait(q.fences);
+    c->host.heap.reclaim();
+    if (c->host.heap.take(len, &off)) return c->host.base + off;
+  }
+  throw Error(GROUTER_ENOMEM, "host store arena fragmented or busy");
+}
+
+void host_free(grouter_ctx *c, uint8_t *p, uint64_t len, Fences &&f) {
+  if (!len) return;
+  uint64_t off = (uint64_t)(p - c->host.base);
+  bool done = true;
+  for (auto &w : f) done &= w.done();
+  if (done) c->host.heap.give(off, len);
+  else c->host.heap.quarantine.push_back({off, len, std::move(f)});
+}
+
+}  // namespace gr

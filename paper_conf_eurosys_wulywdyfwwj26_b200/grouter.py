@@ -1,0 +1,367 @@
+"""Thin ctypes binding of include/grouter.h and include/grouter_testing.h.
+
+Argument marshalling only: every step of the data path (placement, planning,
+scheduling, eviction, copies, completion) runs inside libgrouter.so and its
+sm_100a kernels.  There is no Python or CPU fallback: if the library is not
+built, importing this module raises.
+
+Names follow the C ABI (``grouter_put`` ...).  ``Ctx`` is a small
+convenience wrapper returning ``(status, outputs...)`` tuples; PyTorch
+tensors/streams can be passed as raw integers (``t.data_ptr()``,
+``torch.cuda.current_stream().cuda_stream``).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libgrouter.so")
+
+MAX_GPUS = 16
+MAX_PATHS = 8
+HOST = -1
+NOHINT = -2
+UNLIMITED = (1 << 64) - 1
+
+REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA = 0x1, 0x2, 0x4, 0x8, 0x10
+
+OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
+STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]
+
+
+class grouter_fn(C.Structure):
+    _fields_ = [("workflow_id", C.c_uint32), ("function_id", C.c_uint32), ("device", C.c_int32)]
+
+
+class grouter_chunk(C.Structure):
+    _fields_ = [("offset", C.c_uint64), ("bytes", C.c_uint64), ("path", C.c_int32),
+                ("route_gpu", C.c_int32)]
+
+
+class grouter_config(C.Structure):
+    _fields_ = [
+        ("n_gpus", C.c_uint32),
+        ("device_map", C.c_int32 * MAX_GPUS),
+        ("nvl_Bps", C.c_uint64),
+        ("h2d_Bps", C.c_uint64 * MAX_GPUS),
+        ("h2d_alpha_ps", C.c_uint64 * MAX_GPUS),
+        ("h2d_phi_ps", C.c_uint64 * MAX_GPUS),
+        ("relay_phi_ps", C.c_uint64),
+        ("h2d_pair_Bps", (C.c_uint64 * MAX_GPUS) * MAX_GPUS),
+        ("uplink_group", C.c_int32 * MAX_GPUS),
+        ("p2p", (C.c_uint8 * MAX_GPUS) * MAX_GPUS),
+        ("chunk_bytes", C.c_uint64),
+        ("batch_chunks", C.c_uint32),
+        ("granule", C.c_uint64),
+        ("pool_floor_bytes", C.c_uint64),
+        ("pool_cap_permille", C.c_uint32),
+        ("pool_cap_bytes", C.c_uint64 * MAX_GPUS),
+        ("host_store_bytes", C.c_uint64),
+        ("round_bytes", C.c_uint64),
+        ("copy_ctas_per_sm", C.c_uint32),
+        ("flags", C.c_uint32),
+    ]
+
+
+class grouter_stats_t(C.Structure):
+    _fields_ = [
+        ("used", C.c_uint64 * MAX_GPUS), ("cap", C.c_uint64 * MAX_GPUS),
+        ("mapped", C.c_uint64 * MAX_GPUS), ("host_used", C.c_uint64), ("host_cap", C.c_uint64),
+        ("spill_count", C.c_uint64), ("spill_bytes", C.c_uint64), ("xfer_count", C.c_uint64),
+        ("link_bytes", (C.c_uint64 * MAX_GPUS) * 3), ("kernel_launches", C.c_uint64),
+        ("rounds", C.c_uint64),
+    ]
+
+
+class grouter_dispatch(C.Structure):
+    _fields_ = [("server_kind", C.c_int32), ("server_dev", C.c_int32), ("tenant", C.c_uint32),
+                ("n_chunks", C.c_uint32), ("chunk_ids", C.c_uint64 * 8), ("bytes", C.c_uint64)]
+
+
+_P = C.c_void_p
+_U64, _U32, _I32 = C.c_uint64, C.c_uint32, C.c_int32
+_ST = C.c_int
+_CTX = C.c_void_p
+
+# name -> (restype, argtypes); every symbol declared in include/*.h
+SIGNATURES = {
+    "grouter_config_default": (None, [C.POINTER(grouter_config)]),
+    "grouter_init": (_ST, [C.POINTER(grouter_config), C.POINTER(_CTX)]),
+    "grouter_finalize": (_ST, [_CTX]),
+    "grouter_put": (_ST, [_CTX, C.POINTER(grouter_fn), _P, _U64, _I32, _U32, _P, C.POINTER(_U64)]),
+    "grouter_alloc": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _I32, _U32, C.POINTER(_P),
+                            C.POINTER(_U64)]),
+    "grouter_seal": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P]),
+    "grouter_get": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, C.POINTER(_P), C.POINTER(_U64)]),
+    "grouter_get_into": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, _U64, _P, C.POINTER(_U64)]),
+    "grouter_release": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, _P]),
+    "grouter_free": (_ST, [_CTX, C.POINTER(grouter_fn), _U64]),
+    "grouter_set_tenant_weight": (_ST, [_CTX, _U32, _U32]),
+    "grouter_set_next_use": (_ST, [_CTX, _U64, _U64]),
+    "grouter_set_pool_limit": (_ST, [_CTX, _I32, _U64]),
+    "grouter_flush": (_ST, [_CTX]),
+    "grouter_sync": (_ST, [_CTX]),
+    "grouter_plan": (_ST, [_CTX, _I32, _I32, _U64, C.POINTER(grouter_chunk), _U64, C.POINTER(_U64)]),
+    "grouter_route_set": (_ST, [_CTX, _I32, C.POINTER(_I32), _U32, C.POINTER(_U32)]),
+    "grouter_where": (_ST, [_CTX, _U64, C.POINTER(_I32)]),
+    "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
+    "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
+    "grouter_dispatch_log": (_ST, [_CTX, C.POINTER(grouter_dispatch), _U64, C.POINTER(_U64)]),
+    "grouter_sched_new": (_ST, [_U32, C.POINTER(_P)]),
+    "grouter_sched_set_weight": (_ST, [_P, _U32, _U32]),
+    "grouter_sched_enqueue": (_ST, [_P, _U32, _U64, _U64]),
+    "grouter_sched_dispatch": (_ST, [_P, C.POINTER(_U32), C.POINTER(_U64), C.POINTER(_U32),
+                                     C.POINTER(_U64), C.POINTER(_U64)]),
+    "grouter_sched_free": (None, [_P]),
+    "grouter_strerror": (C.c_char_p, [_ST]),
+    "grouter_last_error": (C.c_char_p, []),
+    "grouter_test_fill": (_ST, [_P, _U64, _U64, _U64, _P]),
+    "grouter_test_verify": (_ST, [_P, _U64, _U64, _U64, _P, C.POINTER(_U64), C.POINTER(_U64)]),
+    "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
+}
+
+_lib = None
+
+
+def load(build_if_missing: bool = False):
+    """Loads libgrouter.so (built in-tree).  Raises if missing: no fallback."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        if not build_if_missing:
+            raise ImportError(f"{LIB_PATH} not built; run __graft_entry__.build()")
+        from . import _build
+        _build.build()
+    lib = C.CDLL(LIB_PATH)
+    for name, (res, args) in SIGNATURES.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = lib
+    return lib
+
+
+def last_error() -> str:
+    s = load().grouter_last_error()
+    return s.decode() if s else ""
+
+
+class GrouterError(RuntimeError):
+    def __init__(self, st, what=""):
+        super().__init__(f"{STATUS[st] if 0 <= st < 8 else st}: {what} ({last_error()})")
+        self.status = st
+
+
+def check(st, what=""):
+    if st != OK:
+        raise GrouterError(st, what)
+    return st
+
+
+# ------------------------------------------------------------------ config
+def config_from_calib(calib: dict | None = None, **kw) -> grouter_config:
+    """grouter_config from a calibration dict (synth/calib.py format) plus
+    overrides (chunk_bytes, host_store_bytes, pool_cap=[...], flags, ...)."""
+    lib = load()
+    cfg = grouter_config()
+    lib.grouter_config_default(C.byref(cfg))
+    if calib is not None:
+        n = calib["n_gpus"]
+        cfg.n_gpus = n
+        dm = calib.get("device_map", list(range(n)))
+        for i in range(n):
+            cfg.device_map[i] = dm[i]
+            cfg.h2d_Bps[i] = calib["h2d_Bps"][i]
+            cfg.h2d_alpha_ps[i] = calib["h2d_alpha_ps"][i]
+            cfg.h2d_phi_ps[i] = calib["h2d_phi_ps"][i]
+            for j in range(n):
+                cfg.p2p[i][j] = calib["p2p"][i][j]
+        cfg.nvl_Bps = calib["nvl_Bps"]
+        cfg.relay_phi_ps = calib["relay_phi_ps"]
+        if "uplink_groups" in calib:
+            for gi, g in enumerate(calib["uplink_groups"]):
+                for x in g:
+                    cfg.uplink_group[x] = gi
+        else:
+            for i in range(MAX_GPUS):
+                cfg.uplink_group[i] = -1
+            for i in range(n):
+                for j in range(n):
+                    cfg.h2d_pair_Bps[i][j] = calib["h2d_pair_Bps"][i][j]
+    caps = kw.pop("pool_cap", None)
+    if caps is not None:
+        for i, v in enumerate(caps):
+            cfg.pool_cap_bytes[i] = v
+    for k, v in kw.items():
+        setattr(cfg, k, v)
+    return cfg
+
+
+def fn(wf: int, fid: int, dev: int) -> grouter_fn:
+    return grouter_fn(wf, fid, dev)
+
+
+class Ctx:
+    """Owns a grouter_ctx; methods mirror the C calls and return statuses."""
+
+    def __init__(self, cfg: grouter_config):
+        self.lib = load()
+        h = C.c_void_p()
+        check(self.lib.grouter_init(C.byref(cfg), C.byref(h)), "grouter_init")
+        self.h = h
+
+    def close(self):
+        if self.h:
+            self.lib.grouter_finalize(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # data path
+    def put(self, f, src: int, n: int, hint=NOHINT, consumers=0, stream=0):
+        oid = C.c_uint64(0)
+        st = self.lib.grouter_put(self.h, C.byref(f), src or None, n, hint, consumers, stream or None,
+                                  C.byref(oid))
+        return st, oid.value
+
+    def alloc(self, f, n: int, hint=NOHINT, consumers=0):
+        buf, oid = C.c_void_p(), C.c_uint64(0)
+        st = self.lib.grouter_alloc(self.h, C.byref(f), n, hint, consumers, C.byref(buf), C.byref(oid))
+        return st, (buf.value or 0), oid.value
+
+    def seal(self, f, oid: int, stream=0):
+        return self.lib.grouter_seal(self.h, C.byref(f), oid, stream or None)
+
+    def get(self, f, oid: int, stream=0):
+        p, n = C.c_void_p(), C.c_uint64(0)
+        st = self.lib.grouter_get(self.h, C.byref(f), oid, stream or None, C.byref(p), C.byref(n))
+        return st, (p.value or 0), n.value
+
+    def get_into(self, f, oid: int, dst: int, cap: int, stream=0):
+        n = C.c_uint64(0)
+        st = self.lib.grouter_get_into(self.h, C.byref(f), oid, dst or None, cap, stream or None,
+                                       C.byref(n))
+        return st, n.value
+
+    def release(self, f, oid: int, ptr: int, stream=0):
+        return self.lib.grouter_release(self.h, C.byref(f), oid, ptr or None, stream or None)
+
+    def free(self, f, oid: int):
+        return self.lib.grouter_free(self.h, C.byref(f), oid)
+
+    # control
+    def set_tenant_weight(self, wf, w):
+        return self.lib.grouter_set_tenant_weight(self.h, wf, w)
+
+    def set_next_use(self, oid, pos):
+        return self.lib.grouter_set_next_use(self.h, oid, pos)
+
+    def set_pool_limit(self, dev, nbytes):
+        return self.lib.grouter_set_pool_limit(self.h, dev, nbytes)
+
+    def flush(self):
+        return self.lib.grouter_flush(self.h)
+
+    def sync(self):
+        return self.lib.grouter_sync(self.h)
+
+    # introspection
+    def plan(self, src, dst, n):
+        cnt = C.c_uint64(0)
+        st = self.lib.grouter_plan(self.h, src, dst, n, None, 0, C.byref(cnt))
+        if st not in (OK, EINVAL) or (st == EINVAL and cnt.value == 0):
+            return st, []
+        arr = (grouter_chunk * max(cnt.value, 1))()
+        st = self.lib.grouter_plan(self.h, src, dst, n, arr, cnt.value, C.byref(cnt))
+        return st, [(c.offset, c.bytes, c.path, c.route_gpu) for c in arr[:cnt.value]]
+
+    def route_set(self, d):
+        arr, cnt = (C.c_int32 * MAX_GPUS)(), C.c_uint32(0)
+        st = self.lib.grouter_route_set(self.h, d, arr, MAX_GPUS, C.byref(cnt))
+        return st, list(arr[:cnt.value])
+
+    def where(self, oid):
+        loc = C.c_int32(0)
+        st = self.lib.grouter_where(self.h, oid, C.byref(loc))
+        return st, loc.value
+
+    def stats(self) -> grouter_stats_t:
+        s = grouter_stats_t()
+        check(self.lib.grouter_stats(self.h, C.byref(s)), "stats")
+        return s
+
+    def victims(self):
+        arr, cnt = (C.c_uint64 * 4096)(), C.c_uint64(0)
+        check(self.lib.grouter_victims(self.h, arr, 4096, C.byref(cnt)), "victims")
+        return list(arr[:cnt.value])
+
+    def dispatch_log(self):
+        out = []
+        arr, cnt = (grouter_dispatch * 4096)(), C.c_uint64(0)
+        while True:
+            check(self.lib.grouter_dispatch_log(self.h, arr, 4096, C.byref(cnt)), "dispatch_log")
+            for d in arr[:cnt.value]:
+                out.append({"kind": d.server_kind, "dev": d.server_dev, "tenant": d.tenant,
+                            "chunks": [(x >> 32, x & 0xFFFFFFFF) for x in d.chunk_ids[:d.n_chunks]],
+                            "bytes": d.bytes})
+            if cnt.value < 4096:
+                return out
+
+
+# ------------------------------------------------------------------ test kernels (K9)
+def test_fill(ptr: int, n: int, seed: int, offset: int = 0, stream: int = 0):
+    return load().grouter_test_fill(ptr or None, n, seed, offset, stream or None)
+
+
+def test_verify(ptr: int, n: int, seed: int, offset: int = 0, stream: int = 0):
+    mism, first = C.c_uint64(0), C.c_uint64(0)
+    st = load().grouter_test_verify(ptr or None, n, seed, offset, stream or None, C.byref(mism),
+                                    C.byref(first))
+    return st, mism.value, first.value
+
+
+def test_copy(dst: int, src: int, chunks, counts: int = 0, tma: bool = False, stream: int = 0):
+    arr = (grouter_chunk * max(len(chunks), 1))(*[grouter_chunk(o, b, p, r) for o, b, p, r in chunks])
+    return load().grouter_test_copy(dst or None, src or None, arr, len(chunks), counts or None,
+                                    int(tma), stream or None)
+
+
+class Sched:
+    """The library's stride scheduler (standalone; no GPU needed)."""
+
+    def __init__(self, batch=5):
+        self.lib = load()
+        self.h = C.c_void_p()
+        check(self.lib.grouter_sched_new(batch, C.byref(self.h)), "sched_new")
+
+    def set_weight(self, t, w):
+        return self.lib.grouter_sched_set_weight(self.h, t, w)
+
+    def enqueue(self, t, cid, nbytes):
+        return self.lib.grouter_sched_enqueue(self.h, t, cid, nbytes)
+
+    def dispatch(self):
+        t, n, b, p = C.c_uint32(0), C.c_uint32(0), C.c_uint64(0), C.c_uint64(0)
+        ids = (C.c_uint64 * 8)()
+        st = self.lib.grouter_sched_dispatch(self.h, C.byref(t), ids, C.byref(n), C.byref(b), C.byref(p))
+        if st != OK:
+            return None
+        return t.value, list(ids[:n.value]), b.value, p.value
+
+    def __del__(self):
+        try:
+            self.lib.grouter_sched_free(self.h)
+        except Exception:
+            pass

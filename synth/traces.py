@@ -274,6 +274,7 @@ def random_trace(rng: random.Random, n_gpus: int, n_ops: int = 200, max_n: int =
             b.get_into(f, i, dst_align=rng.choice([0, 0, 1, 5, 16]))
         elif r < 0.80 and gets:
             g, f = gets.pop(rng.randrange(len(gets)))
+            b.flush()            # the consumer has read its lease before releasing it
             b.release(f, g)
         elif r < 0.86 and live:
             i, _ = live.pop(rng.randrange(len(live)))

@@ -1,0 +1,144 @@
+"""Host-side (no GPU) tests of libgrouter.so: exported ABI, and parity of the
+C++ planner and stride scheduler against the oracle (SURVEY §7 step 1:
+replay-mode parity on synthetic calibrations for 1/2/4/8 GPUs).
+
+These call only GPU-free entry points (GROUTER_PLAN_ONLY contexts and the
+standalone scheduler)."""
+import os
+import random
+import re
+
+import pytest
+
+from oracle import routes as oroutes
+from oracle import splitter as osplit
+from oracle import stride as ostride
+from paper_conf_eurosys_wulywdyfwwj26_b200 import _build
+from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G
+from synth import calib as C
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    _build.build()
+    G.load()
+
+
+def _declared():
+    names = set()
+    for h in ("grouter.h", "grouter_testing.h"):
+        txt = open(os.path.join(ROOT, "include", h)).read()
+        txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+        names |= set(re.findall(r"\b(grouter_[a-z0-9_]+)\s*\(", txt))
+    return names
+
+
+def test_every_declared_symbol_is_exported():
+    lib = G.load()
+    declared = _declared()
+    assert len(declared) >= 30
+    for name in declared:
+        assert hasattr(lib, name), name
+        assert name in G.SIGNATURES, f"binding lacks {name}"
+    # nothing but the ABI leaks out of the library (static cudart is hidden)
+    out = os.popen(f"nm -D --defined-only {G.LIB_PATH}").read().split()
+    exported = {w for w in out if w.startswith("grouter_") or w.startswith("cuda")}
+    assert exported == declared
+
+
+def _plan_ctx(calib, **kw):
+    return G.Ctx(G.config_from_calib(calib, flags=G.PLAN_ONLY | kw.pop("flags", 0), **kw))
+
+
+def _oracle_plan(calib, src, dst, n, multipath=True):
+    if n == 0 or (src == -1 and dst == -1):
+        return []
+    if src == -1:
+        p = osplit.plan_h2d(calib, dst, n, multipath)
+    else:
+        p = osplit.plan_single(n, src)
+    return [(c["offset"], c["bytes"], c["path"], c["route_gpu"]) for c in p]
+
+
+SIZES = [0, 1, 15, 16, 17, 4095, 4096, 4097, 2**21 - 1, 2**21, 2**21 + 1, 38_535_168,
+         39_321_600, 602_112, 33_554_432, 67_108_864, 1 << 30]
+
+
+@pytest.mark.parametrize("topo", ["pairs8", "solo8", "solo4", "solo2", "one", "fig5a"])
+def test_plan_parity_config_topologies(topo):
+    calib = {"pairs8": C.b200_hgx(8), "solo8": C.b200_hgx(8, shared_pairs=False),
+             "solo4": C.b200_hgx(4, shared_pairs=False), "solo2": C.b200_hgx(2, shared_pairs=False),
+             "one": C.b200_hgx(1), "fig5a": C.fig5a()}[topo]
+    with _plan_ctx(calib) as ctx:
+        n = calib["n_gpus"]
+        for d in range(n):
+            assert ctx.route_set(d)[1] == oroutes.route_set(calib, d)
+        for src in [-1] + list(range(n)):
+            for dst in [-1] + list(range(n)):
+                for size in SIZES:
+                    st, got = ctx.plan(src, dst, size)
+                    assert st == G.OK
+                    assert got == _oracle_plan(calib, src, dst, size), (src, dst, size)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_plan_parity_random_calibrations(seed):
+    rng = random.Random(seed)
+    n = rng.choice([1, 2, 3, 4, 5, 8])
+    calib = C.random_calib(rng, n)
+    chunk = rng.choice([1 << 20, 2 << 20, 4 << 20])
+    with _plan_ctx(calib, chunk_bytes=chunk) as ctx:
+        for d in range(n):
+            assert ctx.route_set(d)[1] == oroutes.route_set(calib, d)
+            for _ in range(6):
+                size = rng.choice([rng.randint(0, 1 << 22), rng.randint(0, 1 << 31), rng.choice(SIZES)])
+                st, got = ctx.plan(-1, d, size)
+                exp = osplit.plan_h2d(calib, d, size, C=chunk)
+                assert got == [(c["offset"], c["bytes"], c["path"], c["route_gpu"]) for c in exp]
+
+
+def test_no_multipath_flag():
+    calib = C.b200_hgx(8, shared_pairs=False)
+    with _plan_ctx(calib, flags=G.NO_MULTIPATH) as ctx:
+        assert ctx.route_set(3)[1] == [3]
+        st, got = ctx.plan(-1, 3, 1 << 30)
+        assert got == _oracle_plan(calib, -1, 3, 1 << 30, multipath=False)
+
+
+def test_plan_bad_arguments():
+    with _plan_ctx(C.b200_hgx(2)) as ctx:
+        assert ctx.plan(-1, 2, 10)[0] == G.EINVAL
+        assert ctx.plan(-3, 0, 10)[0] == G.EINVAL
+        assert ctx.route_set(5)[0] == G.EINVAL
+        # data-path calls are refused by a planner-only context (no CPU fallback)
+        st, _ = ctx.put(G.fn(1, 1, -1), 0, 0)
+        assert st == G.EINVAL
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_sched_parity_with_oracle(seed):
+    rng = random.Random(seed)
+    w = {t: rng.choice([1, 2, 3, 4, 8]) for t in range(1, rng.randint(2, 7))}
+    lib, orc = G.Sched(5), ostride.StrideServer()
+    for t, x in w.items():
+        lib.set_weight(t, x)
+    cid = 0
+    for step in range(300):
+        if rng.random() < 0.55:
+            for _ in range(rng.randint(1, 8)):
+                t = rng.choice(list(w))
+                nb = rng.randint(1, 4 << 20)
+                lib.enqueue(t, cid, nb)
+                orc.enqueue(t, cid, nb)
+                cid += 1
+        else:
+            a = lib.dispatch()
+            b = orc.dispatch(w.get)
+            if b is None:
+                assert a is None
+            else:
+                assert a is not None
+                assert (a[0], a[1], a[2]) == (b[0], b[1], b[2])
+                assert a[3] == orc.pass_[b[0]]

@@ -62,8 +62,8 @@ def test_golden_small_trace():
         assert r["victims"] == e["victims"], r["i"]
         if "plan" in e:
             assert _plan_tuples(r["plan"]) == e["plan"], r["i"]
-    disp = [{"server": d["server"], "tenant": d["tenant"], "chunks": d["chunks"]}
-            for d in recs[-1]["dispatched"]]
+    disp = [{"server": d["server"], "tenant": d["tenant"], "chunks": d["chunks"], "at_op": r["i"]}
+            for r in recs for d in r.get("dispatched", [])]
     assert disp == g["dispatch"]
     orc = out["oracle"]
     assert orc.used == g["final"]["used"] and orc.host_used == g["final"]["host_used"]
