@@ -37,6 +37,11 @@ grouter_status grouter_test_verify(const void *src, uint64_t n, uint64_t seed, u
 grouter_status grouter_test_copy(void *dst_base, const void *src_base, const grouter_chunk *chunks,
                                  uint32_t n_chunks, uint32_t *counts, int tma, void *stream);
 
+/* Text dump of the context's internal state (servers, objects, leases,
+ * pending completion words) for debugging; truncated to cap bytes.  Returns
+ * the full length needed in *len (may be NULL). */
+grouter_status grouter_test_dump(grouter_ctx *ctx, char *buf, uint64_t cap, uint64_t *len);
+
 #ifdef __cplusplus
 }
 #endif

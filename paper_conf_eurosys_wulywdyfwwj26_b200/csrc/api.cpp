@@ -11,6 +11,9 @@
 #include <cstring>
 
 #include "../../include/grouter.h"
+#include "../../include/grouter_testing.h"
+
+#include <sstream>
 #include "ctx.h"
 
 using namespace gr;
@@ -168,6 +171,21 @@ void block_on(grouter_ctx *c, const Fences &f) {
   host_wait(f);
 }
 
+// Stream-ordered completion for device callers: work enqueued on `s` after
+// the call sees the bytes.  In real-time mode everything the fences depend
+// on is submitted first, so the caller's wait is enqueued now; in replay
+// mode waits on unsubmitted transfers are attached to them and enqueued at
+// grouter_flush() (R31).
+void order_after(grouter_ctx *c, cudaStream_t s, const Fences &f) {
+  if (!c->replay)
+    for (auto &w : f)
+      if (!is_submitted(w)) {
+        pump(c, true);
+        break;
+      }
+  caller_wait(c, s, f);
+}
+
 int server_kind_for(int src, int dst) {
   if (src == GROUTER_HOST) return SK_H2D;
   if (dst == GROUTER_HOST) return SK_D2H;
@@ -321,13 +339,13 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
       std::memcpy(ptr, src, n);  // cFn -> host store: plain memcpy
     } else {
       Fences deps;
-      if (!blocking) deps.push_back({record(c, (cudaStream_t)stream, phys_of(c, from)), nullptr, 0, c->epoch});
+      if (!blocking) deps.push_back(signal(c, (cudaStream_t)stream, phys_of(c, from)));
       bool pageable = from == GROUTER_HOST && is_pageable(src);
       XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr,
                                  std::move(deps), pageable);
-      x->add_done_fences(done);
+      done_fences(x, done);
       o.ready = done;
-      if (!blocking) stream_wait(c, (cudaStream_t)stream, phys_of(c, from), done);
+      if (!blocking) order_after(c, (cudaStream_t)stream, done);
     }
   }
   *out = o.oid;
@@ -385,7 +403,7 @@ grouter_status grouter_seal(grouter_ctx *c, const grouter_fn *fn, grouter_oid oi
   o.state = OBJ_SEALED;
   o.last_access = c->seq;
   if (stream && o.loc != GROUTER_HOST)
-    o.ready.push_back({record(c, (cudaStream_t)stream, phys_of(c, o.loc)), nullptr, 0, c->epoch});
+    o.ready.push_back(signal(c, (cudaStream_t)stream, phys_of(c, o.loc)));
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -432,7 +450,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
     uint8_t *lease = storage(c, d, ch);
     XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false);
     Fences done;
-    x->add_done_fences(done);
+    done_fences(x, done);
     for (auto &w : done) o.readers.push_back(w);
     Lease L{oid, o.wf, d, lease, n, done};
     c->leases[(uintptr_t)lease] = std::move(L);
@@ -444,7 +462,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
   *n_out = n;
   consume(c, o);  // may release the object's storage (quarantined behind `wait`)
   if (blocking) block_on(c, wait);
-  else stream_wait(c, (cudaStream_t)stream, phys_of(c, d), wait);
+  else order_after(c, (cudaStream_t)stream, wait);
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -475,10 +493,10 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
     } else {
       Fences deps = o.ready;
       if (!blocking)  // the copy must not overwrite dst before prior work on the stream
-        deps.push_back({record(c, (cudaStream_t)stream, phys_of(c, d)), nullptr, 0, c->epoch});
+        deps.push_back(signal(c, (cudaStream_t)stream, phys_of(c, d)));
       XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, (uint8_t *)dst,
                                  std::move(deps), false);
-      x->add_done_fences(wait);
+      done_fences(x, wait);
       for (auto &w : wait) o.readers.push_back(w);
     }
   }
@@ -486,7 +504,7 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
   if (n_out) *n_out = n;
   consume(c, o);
   if (blocking) block_on(c, wait);
-  else stream_wait(c, (cudaStream_t)stream, phys_of(c, d), wait);
+  else order_after(c, (cudaStream_t)stream, wait);
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -506,7 +524,7 @@ grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid
     if (o.wf != fn->workflow_id) return fail(GROUTER_EPERM, "release: workflow mismatch");
     o.pins--;
     if (dev_stream)
-      o.readers.push_back({record(c, (cudaStream_t)stream, phys_of(c, fn->device)), nullptr, 0, c->epoch});
+      o.readers.push_back(signal(c, (cudaStream_t)stream, phys_of(c, fn->device)));
     release_storage_if_dead(c, o);
     return GROUTER_OK;
   }
@@ -515,7 +533,7 @@ grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid
   Lease &L = lt->second;
   if (L.wf != fn->workflow_id) return fail(GROUTER_EPERM, "release: workflow mismatch");
   Fences f = std::move(L.fill);
-  if (dev_stream) f.push_back({record(c, (cudaStream_t)stream, phys_of(c, fn->device)), nullptr, 0, c->epoch});
+  if (dev_stream) f.push_back(signal(c, (cudaStream_t)stream, phys_of(c, fn->device)));
   const uint64_t ch = charge(L.n);
   if (L.dev == GROUTER_HOST) {
     c->host_used -= ch;
@@ -727,5 +745,64 @@ grouter_status grouter_sched_dispatch(grouter_sched *s, uint32_t *tenant, uint64
 }
 
 void grouter_sched_free(grouter_sched *s) { delete s; }
+
+static void dump_fences(std::ostringstream &o, grouter_ctx *c, const Fences &f) {
+  o << "[";
+  for (auto &w : f) {
+    if (w.word)
+      o << " w" << (w.word - c->words) << "=" << *w.word << "/" << w.target << (w.done() ? "ok" : "WAIT");
+    else if (w.ev)
+      o << " ev" << (w.done() ? "ok" : "WAIT");
+    o << "@" << w.epoch;
+  }
+  o << " ]";
+}
+
+grouter_status grouter_test_dump(grouter_ctx *c, char *buf, uint64_t cap, uint64_t *len) {
+  if (!c) return GROUTER_EINVAL;
+  Guard g(c);
+  std::ostringstream o;
+  o << "epoch " << c->epoch << " replay " << c->replay << " sticky " << c->sticky_error << "\n";
+  for (size_t i = 0; i < c->dev.size(); ++i) {
+    auto &d = c->dev[i];
+    o << "dev " << i << " phys " << d.phys << " used " << d.used << " cap " << d.cap << " mapped "
+      << d.pool.mapped << " quarantine " << d.pool.heap.quarantine.size() << "\n";
+    for (Server *s : {&d.copy, &d.h2d, &d.d2h}) {
+      o << "  server " << s->kind << " backlog " << s->sched.backlog_items << " inflight";
+      for (auto &e : s->inflight) o << (cudaEventQuery(e->ev) == cudaSuccess ? " done" : " busy");
+      if (s->stream) o << " stream " << (cudaStreamQuery(s->stream) == cudaSuccess ? "idle" : "busy");
+      if (s->fwd_stream) o << " fwd " << (cudaStreamQuery(s->fwd_stream) == cudaSuccess ? "idle" : "busy");
+      o << "\n";
+    }
+  }
+  for (auto &kv : c->objects) {
+    const Obj &ob = kv.second;
+    o << "obj " << ob.oid << " loc " << ob.loc << " n " << ob.n << " state " << ob.state << " pins "
+      << ob.pins << " ready";
+    dump_fences(o, c, ob.ready);
+    o << " readers";
+    dump_fences(o, c, ob.readers);
+    o << "\n";
+  }
+  for (auto &kv : c->leases) {
+    o << "lease " << kv.first << " oid " << kv.second.oid << " dev " << kv.second.dev << " fill";
+    dump_fences(o, c, kv.second.fill);
+    o << "\n";
+  }
+  for (uint32_t sl = 0; sl < c->n_slots; ++sl)
+    for (int p = 0; p < GROUTER_MAX_PATHS; ++p) {
+      uint32_t w = c->words[sl * GROUTER_MAX_PATHS + p];
+      if ((int32_t)(w - c->slot_final[sl][p]) < 0)
+        o << "pending slot " << sl << " path " << p << " word " << w << " final " << c->slot_final[sl][p] << "\n";
+    }
+  std::string str = o.str();
+  if (len) *len = str.size();
+  if (buf && cap) {
+    uint64_t k = std::min<uint64_t>(cap - 1, str.size());
+    std::memcpy(buf, str.data(), k);
+    buf[k] = 0;
+  }
+  return GROUTER_OK;
+}
 
 }  // extern "C"

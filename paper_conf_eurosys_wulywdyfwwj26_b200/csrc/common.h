@@ -103,6 +103,8 @@ struct EventPool {
   ~EventPool();
 };
 
+struct Xfer;  // ctx.h
+
 // Something the library can wait for: a CUDA event, or a completion word
 // (host-mapped u32) reaching a target value (wrap-safe compare, the same
 // rule as CU_STREAM_WAIT_VALUE_GEQ).  `epoch` = replay epoch of creation.
@@ -111,6 +113,10 @@ struct Waitable {
   volatile uint32_t *word = nullptr;
   uint32_t target = 0;
   uint64_t epoch = 0;
+  // transfer whose chunks publish `word`; null when the producing GPU work is
+  // already submitted (events, caller-stream signals).  A wait is never
+  // enqueued before its producer is submitted (see engine.cpp).
+  std::shared_ptr<Xfer> producer;
   bool done() const {
     if (word) return (int32_t)(*word - target) >= 0;
     if (ev) return cudaEventQuery(ev->ev) == cudaSuccess;

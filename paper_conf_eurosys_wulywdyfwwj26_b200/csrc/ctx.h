@@ -84,7 +84,13 @@ struct Xfer {
   uint64_t deps_waited = 0;                 // bitmask of servers that already waited
   uint64_t epoch = 0;
   bool pageable_src = false;
-  void add_done_fences(Fences &f) const;    // "all chunks complete"
+  uint32_t nchunks = 0, submitted_chunks = 0;
+  bool submitted() const { return submitted_chunks == nchunks; }
+  struct Waiter {
+    cudaStream_t stream;
+    Waitable w;
+  };
+  std::vector<Waiter> waiters;              // caller-stream waits deferred until submission
   bool done() const;
 };
 using XferRef = std::shared_ptr<Xfer>;
@@ -106,6 +112,8 @@ struct Server {
   uint32_t *scratch = nullptr;        // device scratch of the copy kernel on `stream`
   uint32_t *fwd_scratch = nullptr;    // ... on `fwd_stream`
   std::deque<EventRef> inflight;
+  std::deque<ChunkItem> carry;        // scheduled (stride order) but not yet submitted
+  std::deque<ChunkItem> urgent;       // unscheduled work (spills), FIFO
   // H2D relay staging ring on this GPU (device memory)
   uint8_t *staging = nullptr;
   uint32_t n_slots = 0, next_slot = 0;
@@ -202,8 +210,14 @@ void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_ch
                   int kind, uint64_t src_base, uint64_t dst_base, int dst_logical);
 void pump(grouter_ctx *c, bool force_all);            // dispatch rounds (caller holds mu)
 void flush_all(grouter_ctx *c);                        // replay flush
-void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);
-EventRef record(grouter_ctx *c, cudaStream_t s, int phys);
+void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);  // submitted fences only
+// Waits on a CALLER stream: submitted fences now, the others as soon as their
+// producer transfer is submitted.
+void caller_wait(grouter_ctx *c, cudaStream_t s, const Fences &f);
+void done_fences(const XferRef &x, Fences &f);
+bool is_submitted(const Waitable &w);
+EventRef record(grouter_ctx *c, cudaStream_t s, int phys);       // library streams only
+Waitable signal(grouter_ctx *c, cudaStream_t s, int phys);       // caller streams
 void host_wait(const Fences &f, double timeout_s = 120.0);
 bool grounded(const grouter_ctx *c, const Fences &f);
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst);  // D2H of a victim (unscheduled)

@@ -36,9 +36,16 @@
 namespace gr {
 
 static const uint32_t kSlots = 4096;
+XferRef new_xfer_slot(grouter_ctx *c, const std::vector<grouter_chunk> &plan);
 static const uint32_t kBounceSlots = 16;
 
 // ------------------------------------------------------------------ waits
+// Deadlock rule: a stream wait (cuStreamWaitValue32 / cudaStreamWaitEvent) is
+// only ever enqueued once the GPU work that satisfies it has been SUBMITTED.
+// Streams share hardware channels, so a wait enqueued ahead of its producer
+// can park the very channel the producer would run on.
+bool is_submitted(const Waitable &w) { return !w.producer || w.producer->submitted(); }
+
 bool grounded(const grouter_ctx *c, const Fences &f) {
   if (!c->replay) return true;
   for (auto &w : f)
@@ -51,6 +58,7 @@ void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f) {
   (void)phys;
   for (auto &w : f) {
     if (w.done()) continue;  // fast path: already satisfied, no GPU wait
+    if (!is_submitted(w)) throw Error(GROUTER_ECUDA, "internal: wait before submission");
     if (w.word) {
       GR_CU(drv().streamWaitValue32((CUstream)s, (CUdeviceptr)(uintptr_t)w.word, w.target,
                                     CU_STREAM_WAIT_VALUE_GEQ));
@@ -58,6 +66,30 @@ void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f) {
       GR_CUDA(cudaStreamWaitEvent(s, w.ev->ev, 0));
     }
   }
+}
+
+void caller_wait(grouter_ctx *c, cudaStream_t s, const Fences &f) {
+  for (auto &w : f) {
+    if (w.done()) continue;
+    if (is_submitted(w)) stream_wait(c, s, -1, Fences{w});
+    else w.producer->waiters.push_back({s, w});
+  }
+}
+
+// A point on a CALLER's stream: the library writes a fresh completion word
+// from that stream (cuStreamWriteValue32) and waits for / polls the word.
+// Caller streams may come from another runtime instance (PyTorch's), so no
+// event handle crosses that boundary.
+Waitable signal(grouter_ctx *c, cudaStream_t s, int phys) {
+  (void)phys;
+  std::vector<grouter_chunk> one(1, grouter_chunk{0, 0, 0, 0});
+  XferRef x = new_xfer_slot(c, one);
+  GR_CU(drv().streamWriteValue32((CUstream)s, (CUdeviceptr)(uintptr_t)&x->words[0], x->target[0], 0));
+  Waitable w;
+  w.word = &x->words[0];
+  w.target = x->target[0];
+  w.epoch = c->epoch;
+  return w;
 }
 
 EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
@@ -85,13 +117,14 @@ void host_wait(const Fences &f, double timeout_s) {
 }
 
 // ------------------------------------------------------------------ transfers
-void Xfer::add_done_fences(Fences &f) const {
-  for (uint32_t p = 0; p < npath; ++p) {
-    if (!total[p]) continue;
+void done_fences(const XferRef &x, Fences &f) {
+  for (uint32_t p = 0; p < x->npath; ++p) {
+    if (!x->total[p]) continue;
     Waitable w;
-    w.word = &words[p];
-    w.target = target[p];
-    w.epoch = epoch;
+    w.word = &x->words[p];
+    w.target = x->target[p];
+    w.epoch = x->epoch;
+    w.producer = x;
     f.push_back(w);
   }
 }
@@ -103,9 +136,16 @@ bool Xfer::done() const {
 }
 
 XferRef new_xfer(grouter_ctx *c, uint32_t tenant, const std::vector<grouter_chunk> &plan) {
-  auto x = std::make_shared<Xfer>();
+  XferRef x = new_xfer_slot(c, plan);
   x->id = ++c->xfer_seq;
   x->tenant = tenant;
+  c->stats.xfer_count++;
+  return x;
+}
+
+// Completion slot for `plan` (one word per path) without a transfer id.
+XferRef new_xfer_slot(grouter_ctx *c, const std::vector<grouter_chunk> &plan) {
+  auto x = std::make_shared<Xfer>();
   x->epoch = c->epoch;
   uint32_t np = 1;
   for (auto &ch : plan) {
@@ -113,7 +153,8 @@ XferRef new_xfer(grouter_ctx *c, uint32_t tenant, const std::vector<grouter_chun
     np = std::max<uint32_t>(np, (uint32_t)ch.path + 1);
   }
   x->npath = np;
-  // a slot is reusable once its previous transfer has completed
+  x->nchunks = (uint32_t)plan.size();
+  // a slot is reusable once its previous user has completed
   for (uint32_t tries = 0; tries < c->n_slots; ++tries) {
     uint32_t s = c->next_slot;
     c->next_slot = (c->next_slot + 1) % c->n_slots;
@@ -128,7 +169,6 @@ XferRef new_xfer(grouter_ctx *c, uint32_t tenant, const std::vector<grouter_chun
       x->target[p] = c->slot_final[s][p] + x->total[p];
       c->slot_final[s][p] = x->target[p];
     }
-    c->stats.xfer_count++;
     return x;
   }
   throw Error(GROUTER_EBUSY, "no free completion slot (too many transfers in flight)");
@@ -139,20 +179,24 @@ static Server &server_of(grouter_ctx *c, int kind, int logical) {
   return kind == SK_COPY ? d.copy : kind == SK_H2D ? d.h2d : d.d2h;
 }
 
+static ChunkItem make_item(const XferRef &x, uint32_t i, const grouter_chunk &ch, uint64_t src_base,
+                           uint64_t dst_base, int dst_logical) {
+  ChunkItem it;
+  it.x = x;
+  it.idx = i;
+  it.path = (uint32_t)ch.path;
+  it.src = src_base + ch.offset;
+  it.dst = dst_base + ch.offset;
+  it.bytes = ch.bytes;
+  it.dst_logical = dst_logical;
+  return it;
+}
+
 void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_chunk> &plan, int kind,
                   uint64_t src_base, uint64_t dst_base, int dst_logical) {
-  for (uint32_t i = 0; i < plan.size(); ++i) {
-    const grouter_chunk &ch = plan[i];
-    ChunkItem it;
-    it.x = x;
-    it.idx = i;
-    it.path = (uint32_t)ch.path;
-    it.src = src_base + ch.offset;
-    it.dst = dst_base + ch.offset;
-    it.bytes = ch.bytes;
-    it.dst_logical = dst_logical;
-    server_of(c, kind, ch.route_gpu).sched.enqueue(x->tenant, it);
-  }
+  for (uint32_t i = 0; i < plan.size(); ++i)
+    server_of(c, kind, plan[i].route_gpu)
+        .sched.enqueue(x->tenant, make_item(x, i, plan[i], src_base, dst_base, dst_logical));
 }
 
 // ------------------------------------------------------------------ rounds
@@ -175,39 +219,61 @@ static void log_batch(grouter_ctx *c, const Server &s, uint32_t tenant,
   if (c->dlog.size() > (1u << 20)) c->dlog.pop_front();
 }
 
-// Pops whole batches (stride order) for one round.
-static void take_round(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes,
-                       uint32_t max_chunks, std::vector<ChunkItem> &round) {
-  round.clear();
-  std::vector<ChunkItem> b;
+// Moves whole batches (stride order, logged) from the scheduler into the
+// carry queue until the round budget is covered.
+static void refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes) {
   uint64_t bytes = 0;
-  uint32_t nb = 0, npub = 0;
+  for (auto &it : s.carry) bytes += it.bytes;
+  uint32_t nb = 0;
+  std::vector<ChunkItem> b;
   const uint32_t batch = s.sched.batch;
   while (!s.sched.empty() && nb < max_batches && bytes < max_bytes &&
-         round.size() + batch <= max_chunks && npub + batch <= (uint32_t)kMaxPublish) {
+         s.carry.size() + batch <= (size_t)kMaxRoundChunks) {
     uint64_t bb = 0;
     uint32_t t = s.sched.dispatch([&](uint32_t tn) { return weight_of(c, tn); }, b, &bb);
     if (t == UINT32_MAX) break;
     log_batch(c, s, t, b, bb);
-    round.insert(round.end(), b.begin(), b.end());
+    for (auto &it : b) s.carry.push_back(it);
     bytes += bb;
-    npub += (uint32_t)b.size();
     ++nb;
   }
-  c->stats.rounds++;
 }
 
-static void wait_deps(grouter_ctx *c, Server &s, cudaStream_t st, const std::vector<ChunkItem> &items) {
-  for (auto &it : items) {
-    Xfer &x = *it.x;
-    if (x.deps_waited & s.id_bit()) continue;
-    x.deps_waited |= s.id_bit();
-    stream_wait(c, st, s.phys, x.deps);
+// Takes the longest submittable prefix of urgent + carry (bounded by the
+// round limits).  An item is submittable unless it is the first item of a
+// transfer on this server whose dependencies are not all submitted; cut[i]
+// says a stream wait for the transfer's dependencies must precede item i.
+static void take(Server &s, uint64_t max_bytes, std::vector<ChunkItem> &items, std::vector<char> &cut) {
+  items.clear();
+  cut.clear();
+  uint64_t bytes = 0;
+  uint32_t npub = 0;
+  for (int q = 0; q < 2; ++q) {
+    std::deque<ChunkItem> &dq = q == 0 ? s.urgent : s.carry;
+    while (!dq.empty() && items.size() < (size_t)kMaxRoundChunks && bytes < max_bytes &&
+           npub < (uint32_t)kMaxPublish) {
+      const ChunkItem &it = dq.front();
+      Xfer &x = *it.x;
+      bool first = !(x.deps_waited & s.id_bit());
+      bool need_wait = false;
+      if (first) {
+        for (auto &w : x.deps) {
+          if (!is_submitted(w)) return;  // producer not submitted yet: stop here
+          need_wait |= !w.done();
+        }
+        x.deps_waited |= s.id_bit();
+      }
+      items.push_back(it);
+      cut.push_back(need_wait);
+      bytes += it.bytes;
+      ++npub;
+      dq.pop_front();
+    }
+    if (items.size() >= (size_t)kMaxRoundChunks || bytes >= max_bytes) return;
   }
 }
 
-// Marks the items as issued and returns the distinct (xfer, path) pairs with
-// their absolute word values after these items complete.
+// Marks the items as issued and returns the distinct (xfer, path) pairs.
 struct Pub {
   Xfer *x;
   uint32_t path;
@@ -222,6 +288,19 @@ static std::vector<Pub> issue(const std::vector<ChunkItem> &items) {
     if (!found) pubs.push_back({x, it.path});
   }
   return pubs;
+}
+
+// After a round is submitted: count chunks, release caller-stream waits of
+// transfers that are now fully submitted.
+static void after_submit(grouter_ctx *c, const std::vector<ChunkItem> &items) {
+  for (auto &it : items) it.x->submitted_chunks++;
+  for (auto &it : items) {
+    Xfer &x = *it.x;
+    if (!x.submitted() || x.waiters.empty()) continue;
+    auto ws = std::move(x.waiters);
+    x.waiters.clear();
+    for (auto &wt : ws) stream_wait(c, wt.stream, -1, Fences{wt.w});
+  }
 }
 
 static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *scratch,
@@ -251,49 +330,87 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
   c->stats.kernel_launches++;
 }
 
-// SM-copy server: one kernel launch per round (D2D push over NVLink, or a
-// same-GPU HBM copy).
-static void round_copy(grouter_ctx *c, Server &s) {
-  std::vector<ChunkItem> items;
-  take_round(c, s, UINT32_MAX, c->cfg.round_bytes, (uint32_t)kMaxRoundChunks, items);
-  if (items.empty()) return;
+// SM-copy server: one kernel launch per round segment (D2D push over
+// NVLink, or a same-GPU HBM copy).
+static size_t round_copy(grouter_ctx *c, Server &s) {
+  refill(c, s, UINT32_MAX, c->cfg.round_bytes);
+  std::vector<ChunkItem> items, seg;
+  std::vector<char> cut;
+  take(s, c->cfg.round_bytes, items, cut);
+  if (items.empty()) return 0;
   DeviceGuard g(s.phys);
-  wait_deps(c, s, s.stream, items);
-  launch_round(c, s, s.stream, s.scratch, items, nullptr);
-  for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
+  for (size_t i = 0; i < items.size(); ++i) {
+    if (cut[i]) {
+      if (!seg.empty()) launch_round(c, s, s.stream, s.scratch, seg, nullptr);
+      seg.clear();
+      stream_wait(c, s.stream, s.phys, items[i].x->deps);
+    }
+    seg.push_back(items[i]);
+    c->stats.link_bytes[0][s.logical] += items[i].bytes;
+  }
+  launch_round(c, s, s.stream, s.scratch, seg, nullptr);
   s.inflight.push_back(record(c, s.stream, s.phys));
+  c->stats.rounds++;
+  after_submit(c, items);
+  return items.size();
 }
 
 // Copies a pageable host chunk into the circular pinned buffer (L229) and
-// returns the pinned address to DMA from.
-static uint64_t bounce(grouter_ctx *c, cudaStream_t st, int phys, uint64_t src, uint64_t bytes) {
+// returns the pinned address to DMA from; the slot is reused once the DMA
+// that last read it has completed.
+static uint64_t bounce(grouter_ctx *c, uint64_t src, uint64_t bytes, uint32_t *slot_out) {
   uint32_t k = c->bounce_next;
   c->bounce_next = (k + 1) % c->bounce_slots;
   if (c->bounce_ev[k]) GR_CUDA(cudaEventSynchronize(c->bounce_ev[k]->ev));
   uint8_t *slot = c->bounce + (uint64_t)k * c->cfg.chunk_bytes;
   std::memcpy(slot, (const void *)src, bytes);
-  (void)st;
-  (void)phys;
+  *slot_out = k;
   return (uint64_t)slot;
 }
 
-// H2D server of route GPU r: CE copies of up to two batches (L229); chunks
-// for r itself land in the lease, relayed chunks go through r's staging
-// ring and one forward round kernel on r pushes them to their destination.
-static void round_h2d(grouter_ctx *c, Server &s) {
-  std::vector<ChunkItem> items;
-  take_round(c, s, 2, UINT64_MAX, (uint32_t)kMaxRoundChunks, items);
-  if (items.empty()) return;
+static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg) {
+  for (auto &p : issue(seg))
+    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
+                                   p.x->value_after(p.path), 0));
+  seg.clear();
+}
+
+// H2D server of route GPU r: CE copies of up to two batches (L229).  Chunks
+// for r itself land in the lease; relayed chunks go through r's staging ring
+// and a forward round kernel on r pushes them to their destination.
+static size_t round_h2d(grouter_ctx *c, Server &s) {
+  const uint64_t budget = 2ull * s.sched.batch * c->cfg.chunk_bytes;
+  refill(c, s, 2, budget);
+  std::vector<ChunkItem> items, direct, relay;
+  std::vector<char> cut;
+  take(s, budget, items, cut);
+  if (items.empty()) return 0;
   DeviceGuard g(s.phys);
-  wait_deps(c, s, s.stream, items);
-  std::vector<ChunkItem> direct, relay;
   std::vector<uint64_t> slot_src;
   std::vector<uint32_t> slots_used;
-  for (auto &it : items) {
-    uint64_t src = it.src;
-    if (it.x->pageable_src) {
-      src = bounce(c, s.stream, s.phys, it.src, it.bytes);
+  EventRef last_fwd;
+  auto end_segment = [&]() {
+    publish_ce(c, s, direct);
+    if (!relay.empty()) {
+      EventRef ce = record(c, s.stream, s.phys);
+      GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
+      launch_round(c, s, s.fwd_stream, s.fwd_scratch, relay, slot_src.data());
+      last_fwd = record(c, s.fwd_stream, s.phys);
+      for (uint32_t k : slots_used) s.slot_free[k] = last_fwd;
+      relay.clear();
+      slot_src.clear();
+      slots_used.clear();
     }
+  };
+  for (size_t i = 0; i < items.size(); ++i) {
+    const ChunkItem &it = items[i];
+    if (cut[i]) {
+      end_segment();
+      stream_wait(c, s.stream, s.phys, it.x->deps);
+    }
+    uint64_t src = it.src;
+    uint32_t bslot = 0;
+    if (it.x->pageable_src) src = bounce(c, it.src, it.bytes, &bslot);
     if (it.dst_logical == s.logical) {
       GR_CUDA(cudaMemcpyAsync((void *)it.dst, (const void *)src, it.bytes, cudaMemcpyHostToDevice,
                               s.stream));
@@ -308,42 +425,48 @@ static void round_h2d(grouter_ctx *c, Server &s) {
       slot_src.push_back((uint64_t)slot);
       slots_used.push_back(k);
     }
-    if (it.x->pageable_src) c->bounce_ev[(c->bounce_next + c->bounce_slots - 1) % c->bounce_slots] =
-        record(c, s.stream, s.phys);
+    if (it.x->pageable_src) c->bounce_ev[bslot] = record(c, s.stream, s.phys);
     c->stats.link_bytes[1][s.logical] += it.bytes;
   }
-  for (auto &p : issue(direct))
-    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
-                                   p.x->value_after(p.path), 0));
-  if (!relay.empty()) {
-    EventRef ce = record(c, s.stream, s.phys);
-    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
-    launch_round(c, s, s.fwd_stream, s.fwd_scratch, relay, slot_src.data());
-    EventRef fwd = record(c, s.fwd_stream, s.phys);
-    for (uint32_t k : slots_used) s.slot_free[k] = fwd;
-    s.inflight.push_back(fwd);
+  end_segment();
+  EventRef ce_end = record(c, s.stream, s.phys);
+  if (last_fwd) {  // one in-flight marker covering both the CE and the forward stream
+    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce_end->ev, 0));
+    s.inflight.push_back(record(c, s.fwd_stream, s.phys));
   } else {
-    s.inflight.push_back(record(c, s.stream, s.phys));
+    s.inflight.push_back(ce_end);
   }
+  c->stats.rounds++;
+  after_submit(c, items);
+  return items.size();
 }
 
 // D2H server: CE copies device -> host (host store, host leases, caller
-// host buffers).
-static void round_d2h(grouter_ctx *c, Server &s) {
-  std::vector<ChunkItem> items;
-  take_round(c, s, 2, UINT64_MAX, (uint32_t)kMaxRoundChunks, items);
-  if (items.empty()) return;
+// host buffers, and urgent spills).
+static size_t round_d2h(grouter_ctx *c, Server &s) {
+  const uint64_t budget = 2ull * s.sched.batch * c->cfg.chunk_bytes;
+  refill(c, s, 2, budget);
+  std::vector<ChunkItem> items, seg;
+  std::vector<char> cut;
+  take(s, UINT64_MAX, items, cut);
+  if (items.empty()) return 0;
   DeviceGuard g(s.phys);
-  wait_deps(c, s, s.stream, items);
-  for (auto &it : items) {
+  for (size_t i = 0; i < items.size(); ++i) {
+    const ChunkItem &it = items[i];
+    if (cut[i]) {
+      publish_ce(c, s, seg);
+      stream_wait(c, s.stream, s.phys, it.x->deps);
+    }
     GR_CUDA(cudaMemcpyAsync((void *)it.dst, (const void *)it.src, it.bytes, cudaMemcpyDeviceToHost,
                             s.stream));
+    seg.push_back(it);
     c->stats.link_bytes[2][s.logical] += it.bytes;
   }
-  for (auto &p : issue(items))
-    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
-                                   p.x->value_after(p.path), 0));
+  publish_ce(c, s, seg);
   s.inflight.push_back(record(c, s.stream, s.phys));
+  c->stats.rounds++;
+  after_submit(c, items);
+  return items.size();
 }
 
 static void retire(Server &s) {
@@ -351,53 +474,68 @@ static void retire(Server &s) {
     s.inflight.pop_front();
 }
 
-static void pump_server(grouter_ctx *c, Server &s, bool force) {
-  if (!s.stream) return;
-  retire(s);
-  while (!s.sched.empty() && (force || s.inflight.size() < 2)) {
-    if (s.kind == SK_COPY) round_copy(c, s);
-    else if (s.kind == SK_H2D) round_h2d(c, s);
-    else round_d2h(c, s);
-  }
+static bool has_work(const Server &s) {
+  return !s.sched.empty() || !s.carry.empty() || !s.urgent.empty();
 }
 
+static size_t pump_server(grouter_ctx *c, Server &s, bool force) {
+  if (!s.stream) return 0;
+  retire(s);
+  size_t total = 0;
+  while (has_work(s) && (force || s.inflight.size() < 2)) {
+    size_t n = s.kind == SK_COPY ? round_copy(c, s) : s.kind == SK_H2D ? round_h2d(c, s) : round_d2h(c, s);
+    if (!n) break;  // blocked on another server's submission
+    total += n;
+  }
+  return total;
+}
+
+// Dispatches rounds.  force: ignore the in-flight limit and iterate over the
+// servers until every queued chunk is submitted (a server blocked on another
+// server's submission is retried after that one progressed).
 void pump(grouter_ctx *c, bool force_all) {
   if (c->replay && !force_all) return;
-  for (auto &d : c->dev) {
-    pump_server(c, d.copy, force_all);
-    pump_server(c, d.h2d, force_all);
-    pump_server(c, d.d2h, force_all);
+  for (;;) {
+    size_t progress = 0;
+    for (auto &d : c->dev) {
+      progress += pump_server(c, d.copy, force_all);
+      progress += pump_server(c, d.h2d, force_all);
+      progress += pump_server(c, d.d2h, force_all);
+    }
+    if (!force_all || !progress) break;
   }
   bool backlog = false;
-  for (auto &d : c->dev) backlog |= !d.copy.sched.empty() || !d.h2d.sched.empty() || !d.d2h.sched.empty();
+  for (auto &d : c->dev) backlog |= has_work(d.copy) || has_work(d.h2d) || has_work(d.d2h);
   if (backlog) c->cv.notify_one();
 }
 
 void flush_all(grouter_ctx *c) {
   pump(c, true);
-  c->epoch++;   // everything created before is now dispatched (grounded)
+  c->epoch++;  // everything created before is now submitted (grounded)
 }
 
-// Unscheduled D2H of an eviction victim (L258-L262; the per-GPU I/O path of L269).
+// D2H of an eviction victim (L258-L262; the per-GPU I/O path of L269): an
+// urgent, unscheduled transfer on the victim GPU's D2H engine.
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
+  std::vector<grouter_chunk> plan;
+  c->planner.plan_single(o.n, o.loc, plan);
+  XferRef x = new_xfer_slot(c, plan);
+  x->deps = o.ready;
   Server &s = c->dev[o.loc].d2h;
-  DeviceGuard g(s.phys);
-  stream_wait(c, s.stream, s.phys, o.ready);
-  if (o.n)
-    GR_CUDA(cudaMemcpyAsync(host_dst, o.ptr, o.n, cudaMemcpyDeviceToHost, s.stream));
-  Waitable w;
-  w.ev = record(c, s.stream, s.phys);
-  w.epoch = c->epoch;
+  for (uint32_t i = 0; i < plan.size(); ++i)
+    s.urgent.push_back(make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)host_dst,
+                                 GROUTER_HOST));
+  Fences done;
+  done_fences(x, done);
   Fences old = std::move(o.readers);
   for (auto &f : o.ready) old.push_back(f);
-  old.push_back(w);
+  for (auto &f : done) old.push_back(f);
   dev_free(c, o.loc, o.ptr, charge(o.n), std::move(old));
-  o.ready.clear();
-  o.ready.push_back(w);
+  o.ready = done;
   o.readers.clear();
   c->stats.spill_count++;
   c->stats.spill_bytes += o.n;
-  c->stats.link_bytes[2][o.loc] += o.n;
+  pump(c, false);
 }
 
 // ------------------------------------------------------------------ lifecycle
@@ -407,15 +545,9 @@ static void daemon_main(grouter_ctx *c) {
   while (!c->stop) {
     bool backlog = false, busy = false;
     try {
-      if (!c->replay) {
-        for (auto &d : c->dev) {
-          pump_server(c, d.copy, false);
-          pump_server(c, d.h2d, false);
-          pump_server(c, d.d2h, false);
-        }
-      }
+      if (!c->replay) pump(c, false);
       for (auto &d : c->dev) {
-        backlog |= !d.copy.sched.empty() || !d.h2d.sched.empty() || !d.d2h.sched.empty();
+        backlog |= has_work(d.copy) || has_work(d.h2d) || has_work(d.d2h);
         busy |= !d.copy.inflight.empty() || !d.h2d.inflight.empty() || !d.d2h.inflight.empty();
         if (!c->replay) {
           retire(d.copy);
@@ -545,9 +677,19 @@ void engine_shutdown(grouter_ctx *c) {
   }
   c->cv.notify_all();
   if (c->daemon.joinable()) c->daemon.join();
+  // drain the library's own streams (never the device: a caller stream may be
+  // parked on a completion word that will not arrive after an error)
+  auto t0 = std::chrono::steady_clock::now();
   for (auto &d : c->dev) {
     DeviceGuard g(d.phys);
-    cudaDeviceSynchronize();
+    for (Server *s : {&d.copy, &d.h2d, &d.d2h})
+      for (cudaStream_t st : {s->stream, s->fwd_stream})
+        while (st && cudaStreamQuery(st) == cudaErrorNotReady &&
+               std::chrono::steady_clock::now() - t0 < std::chrono::seconds(10))
+          std::this_thread::sleep_for(std::chrono::microseconds(100));
+  }
+  for (auto &d : c->dev) {
+    DeviceGuard g(d.phys);
     Server *ss[3] = {&d.copy, &d.h2d, &d.d2h};
     for (Server *s : ss) {
       s->inflight.clear();

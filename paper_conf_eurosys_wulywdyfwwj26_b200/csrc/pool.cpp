@@ -128,8 +128,12 @@ void PageHeap::reclaim() {
         done = false;
         break;
       }
-    if (done) give(quarantine[i].off, quarantine[i].len);
-    else quarantine[w++] = std::move(quarantine[i]);
+    if (done) {
+      give(quarantine[i].off, quarantine[i].len);
+    } else {
+      if (w != i) quarantine[w] = std::move(quarantine[i]);  // never self-move: it empties the fences
+      ++w;
+    }
   }
   quarantine.resize(w);
 }
@@ -195,13 +199,11 @@ void DevicePool::trim(uint64_t keep) {
     Seg s = segs.back();
     if (mapped - s.size < keep) break;
     if (heap.tail_free(mapped) < s.size) break;
-    uint64_t off = 0;
     // carve the segment out of the trailing free run
     auto it = std::prev(heap.free_runs.end());
     uint64_t run_off = it->first;
     heap.free_runs.erase(it);
     if (s.off > run_off) heap.free_runs[run_off] = s.off - run_off;
-    (void)off;
     drv().memUnmap(base + s.off, s.size);
     drv().memRelease(s.h);
     mapped -= s.size;

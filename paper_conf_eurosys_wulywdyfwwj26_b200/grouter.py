@@ -118,6 +118,7 @@ SIGNATURES = {
     "grouter_last_error": (C.c_char_p, []),
     "grouter_test_fill": (_ST, [_P, _U64, _U64, _U64, _P]),
     "grouter_test_verify": (_ST, [_P, _U64, _U64, _U64, _P, C.POINTER(_U64), C.POINTER(_U64)]),
+    "grouter_test_dump": (_ST, [_CTX, C.c_char_p, _U64, C.POINTER(_U64)]),
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
 }
 
@@ -301,6 +302,13 @@ class Ctx:
         s = grouter_stats_t()
         check(self.lib.grouter_stats(self.h, C.byref(s)), "stats")
         return s
+
+    def dump(self) -> str:
+        n = C.c_uint64(0)
+        self.lib.grouter_test_dump(self.h, None, 0, C.byref(n))
+        buf = C.create_string_buffer(n.value + 1)
+        self.lib.grouter_test_dump(self.h, buf, n.value + 1, C.byref(n))
+        return buf.value.decode()
 
     def victims(self):
         arr, cnt = (C.c_uint64 * 4096)(), C.c_uint64(0)

@@ -10,6 +10,7 @@ kernel (test infrastructure) or copied from the host generator.
 from __future__ import annotations
 
 import ctypes
+import os
 import time
 
 import numpy as np
@@ -67,6 +68,7 @@ class LibRunner:
         self.ctx = G.Ctx(G.config_from_calib(calib, **kw))
         self.replay = replay
         self.streams = [torch.cuda.Stream(device=p) for p in self.phys]
+        self.upload = [torch.cuda.Stream(device=p) for p in self.phys]
         self.keep_bytes = keep_bytes
         self.keep = []          # buffers that must outlive their use
         self.pending = []       # (rec, verifier) to check after the next flush
@@ -86,7 +88,11 @@ class LibRunner:
             rec["bytes"] = got
 
     def _flush_and_verify(self):
-        wait_streams(self.streams)
+        try:
+            wait_streams(self.streams)
+        except TimeoutError:
+            print(self.ctx.dump(), flush=True)
+            raise
         for rec, fnv in self.pending:
             self._verify(rec, fnv())
         self.pending = []
@@ -94,9 +100,12 @@ class LibRunner:
     def run(self, ops):
         recs = []
         ctx = self.ctx
+        trace = bool(os.environ.get("GR_TRACE"))
         for i, op in enumerate(ops):
             k = op["op"]
             rec = {"i": i, "op": k}
+            if trace:
+                print("op", i, {a: b for a, b in op.items() if a != "seed"}, flush=True)
             oid = 0
             if "ref" in op and op["ref"] < len(recs):
                 oid = recs[op["ref"]].get("oid", 0)
@@ -116,9 +125,13 @@ class LibRunner:
                 else:
                     dev = self.phys[f["dev"]]
                     buf = torch.empty(n + align + 1, dtype=torch.uint8, device=f"cuda:{dev}")
-                    with torch.cuda.stream(self.streams[f["dev"]]):
+                    # upload on a side stream: in replay mode the caller stream may be
+                    # parked on a completion word until the next flush
+                    up = self.upload[f["dev"]]
+                    with torch.cuda.stream(up):
                         buf[align:align + n].copy_(torch.from_numpy(data).to(f"cuda:{dev}",
                                                                              non_blocking=False))
+                    self.streams[f["dev"]].wait_stream(up)
                     ptr = buf.data_ptr() + align
                 self.keep.append(buf)
                 st, o = ctx.put(self._fnc(f), ptr, n, op["hint"], op["consumers"],
@@ -130,9 +143,11 @@ class LibRunner:
                 st, buf, o = ctx.alloc(self._fnc(f), n, op["hint"], op["consumers"])
                 if st == G.OK:
                     rec["oid"] = oid = o
+                    rec["buf"] = buf
                     if n:
                         if f["dev"] == HOST:
-                            ctypes.memmove(buf, payload(op["seed"], n).ctypes.data, n)
+                            data = payload(op["seed"], n)   # keep alive across memmove
+                            ctypes.memmove(buf, data.ctypes.data, n)
                         else:
                             with torch.cuda.device(self.phys[f["dev"]]):
                                 G.check(G.test_fill(buf, n, op["seed"], 0, self._stream(f["dev"])))
@@ -210,6 +225,8 @@ class LibRunner:
             if st == G.OK and k in ("put", "alloc"):
                 self._size_of[rec["oid"]] = op["n"]
             rec["status"] = G.STATUS[st]
+            if trace:
+                print("   ->", G.STATUS[st], G.last_error() if st else "", flush=True)
             rec["victims"] = ctx.victims()
             s = ctx.stats()
             rec["used"] = [s.used[d] for d in range(self.n)]
@@ -247,7 +264,11 @@ def compare(orc_out, lib_out, check_dispatch=True):
         if o["status"] == "OK" and o["op"] in ("get", "get_into"):
             assert l["n"] == o["n"], ctx
             if "bytes" in o and "bytes" in l:
-                assert np.array_equal(l["bytes"], o["bytes"]), ctx
+                if not np.array_equal(l["bytes"], o["bytes"]):
+                    bad = np.nonzero(l["bytes"] != o["bytes"])[0]
+                    raise AssertionError(f"{ctx}: {bad.size} of {o['n']} bytes differ, first at "
+                                         f"{bad[0]}, last at {bad[-1]}; lib[:8]={l['bytes'][bad[0]:bad[0]+8]} "
+                                         f"orc[:8]={o['bytes'][bad[0]:bad[0]+8]}")
             assert l["digest"] == o["digest"], ctx
             compared += 1
     if check_dispatch:
