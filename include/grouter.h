@@ -57,6 +57,7 @@ extern "C" {
 #define GROUTER_PLAN_ONLY     0x4u /* no CUDA at all: planner/introspection only            */
 #define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
 #define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
+#define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;
@@ -127,6 +128,11 @@ typedef struct {
   uint64_t link_bytes[3][GROUTER_MAX_GPUS]; /* [0]=SM copy egress, [1]=H2D, [2]=D2H */
   uint64_t kernel_launches;              /* copy/forward kernels launched       */
   uint64_t rounds;                       /* dispatch rounds                     */
+  /* GROUTER_PROFILE: completed, timed copy-kernel launches (CUDA events
+   * recorded on the launching stream around each launch) */
+  uint64_t timed_launches;
+  uint64_t timed_ns;                     /* sum of their durations              */
+  uint64_t timed_bytes;                  /* sum of the bytes they moved         */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE

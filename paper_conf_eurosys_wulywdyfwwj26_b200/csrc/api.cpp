@@ -192,16 +192,30 @@ int server_kind_for(int src, int dst) {
   return SK_COPY;
 }
 
-// Plans, enqueues and starts one transfer; returns it.
+// Plans, enqueues and starts one transfer; returns it.  `caller` (a device
+// caller's stream, else null): a same-GPU SM copy may run directly on it
+// (*direct = true: stream order alone sequences it, no signal or wait
+// needed); otherwise `caller_dep` adds a point on the caller's stream to the
+// transfer's dependencies (the copy reads src / overwrites dst only after
+// prior work on that stream).
 XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc, uint64_t n,
-                       const uint8_t *src, uint8_t *dst, Fences deps, bool pageable_src) {
+                       const uint8_t *src, uint8_t *dst, Fences deps, bool pageable_src,
+                       cudaStream_t caller = nullptr, int caller_logical = -1, bool caller_dep = false,
+                       bool *direct = nullptr) {
   std::vector<grouter_chunk> plan;
   c->planner.plan(src_loc, dst_loc, n, plan);
   XferRef x = new_xfer(c, tenant, plan);
   x->deps = std::move(deps);
   x->pageable_src = pageable_src;
-  enqueue_plan(c, x, plan, server_kind_for(src_loc, dst_loc), (uint64_t)(uintptr_t)src,
-               (uint64_t)(uintptr_t)dst, dst_loc);
+  const int kind = server_kind_for(src_loc, dst_loc);
+  enqueue_plan(c, x, plan, kind, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, dst_loc);
+  if (direct) *direct = false;
+  if (caller && kind == SK_COPY && direct &&
+      try_direct(c, x, src_loc, caller, c->dev[caller_logical].phys)) {
+    *direct = true;
+    return x;
+  }
+  if (caller && caller_dep) x->deps.push_back(signal(c, caller, c->dev[caller_logical].phys));
   pump(c, false);  // inline dispatch when the server has room (no-op in replay mode)
   return x;
 }
@@ -338,14 +352,14 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
     if (from == GROUTER_HOST && home == GROUTER_HOST) {
       std::memcpy(ptr, src, n);  // cFn -> host store: plain memcpy
     } else {
-      Fences deps;
-      if (!blocking) deps.push_back(signal(c, (cudaStream_t)stream, phys_of(c, from)));
       bool pageable = from == GROUTER_HOST && is_pageable(src);
-      XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr,
-                                 std::move(deps), pageable);
+      bool direct = false;
+      XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr, Fences{},
+                                 pageable, blocking ? nullptr : (cudaStream_t)stream, from, true,
+                                 &direct);
       done_fences(x, done);
       o.ready = done;
-      if (!blocking) order_after(c, (cudaStream_t)stream, done);
+      if (!blocking && !direct) order_after(c, (cudaStream_t)stream, done);
     }
   }
   *out = o.oid;
@@ -448,14 +462,16 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
     if (d == GROUTER_HOST ? !host_reserve(c, ch) : !reserve(c, d, ch))
       return fail(GROUTER_ENOMEM, "get: lease does not fit after eviction");
     uint8_t *lease = storage(c, d, ch);
-    XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false);
+    bool direct = false;
+    XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false,
+                               blocking ? nullptr : (cudaStream_t)stream, d, false, &direct);
     Fences done;
     done_fences(x, done);
     for (auto &w : done) o.readers.push_back(w);
     Lease L{oid, o.wf, d, lease, n, done};
     c->leases[(uintptr_t)lease] = std::move(L);
     result = lease;
-    wait = done;
+    if (!direct) wait = done;
   }
   o.last_access = c->seq;
   *ptr = result;
@@ -491,13 +507,15 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
       host_wait(o.ready);
       std::memcpy(dst, o.ptr, n);
     } else {
-      Fences deps = o.ready;
-      if (!blocking)  // the copy must not overwrite dst before prior work on the stream
-        deps.push_back(signal(c, (cudaStream_t)stream, phys_of(c, d)));
-      XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, (uint8_t *)dst,
-                                 std::move(deps), false);
-      done_fences(x, wait);
-      for (auto &w : wait) o.readers.push_back(w);
+      // the copy must not overwrite dst before prior work on the stream:
+      // a direct launch on that stream, or a signal from it as a dependency
+      bool direct = false;
+      XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, (uint8_t *)dst, o.ready,
+                                 false, blocking ? nullptr : (cudaStream_t)stream, d, true, &direct);
+      Fences done;
+      done_fences(x, done);
+      for (auto &w : done) o.readers.push_back(w);
+      if (!direct) wait = done;
     }
   }
   o.last_access = c->seq;
@@ -665,6 +683,11 @@ grouter_status grouter_where(grouter_ctx *c, grouter_oid oid, int32_t *loc) {
 grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
   if (!c || !out) return fail(GROUTER_EINVAL, "null argument");
   Guard g(c);
+  if (!c->plan_only) {
+    API_TRY
+    harvest_profile(c, false);
+    API_CATCH(c)
+  }
   *out = c->stats;
   for (size_t i = 0; i < c->dev.size(); ++i) {
     out->used[i] = c->dev[i].used;
@@ -769,7 +792,7 @@ grouter_status grouter_test_dump(grouter_ctx *c, char *buf, uint64_t cap, uint64
       << d.pool.mapped << " quarantine " << d.pool.heap.quarantine.size() << "\n";
     for (Server *s : {&d.copy, &d.h2d, &d.d2h}) {
       o << "  server " << s->kind << " backlog " << s->sched.backlog_items << " inflight";
-      for (auto &e : s->inflight) o << (cudaEventQuery(e->ev) == cudaSuccess ? " done" : " busy");
+      for (auto &e : s->inflight) o << (e.w.done() ? " done" : " busy") << (e.direct ? "(direct)" : "");
       if (s->stream) o << " stream " << (cudaStreamQuery(s->stream) == cudaSuccess ? "idle" : "busy");
       if (s->fwd_stream) o << " fwd " << (cudaStreamQuery(s->fwd_stream) == cudaSuccess ? "idle" : "busy");
       o << "\n";

@@ -111,7 +111,11 @@ struct Server {
   cudaStream_t fwd_stream = nullptr;  // H2D: relay forward kernel stream
   uint32_t *scratch = nullptr;        // device scratch of the copy kernel on `stream`
   uint32_t *fwd_scratch = nullptr;    // ... on `fwd_stream`
-  std::deque<EventRef> inflight;
+  struct Inflight {
+    Waitable w;                  // completion of a dispatched round
+    cudaStream_t direct;         // caller stream of a direct launch, null for the server stream
+  };
+  std::deque<Inflight> inflight;
   std::deque<ChunkItem> carry;        // scheduled (stride order) but not yet submitted
   std::deque<ChunkItem> urgent;       // unscheduled work (spills), FIFO
   // H2D relay staging ring on this GPU (device memory)
@@ -161,6 +165,18 @@ struct PhysDev {
   int ordinal = -1;
   int sm_count = 148;
   EventPool events;
+  // copy-kernel scratch pairs for direct launches on caller streams; a pair
+  // is reusable once the launch that used it has completed
+  uint32_t *scratch = nullptr;
+  uint32_t n_scratch = 0, next_scratch = 0;
+  std::vector<Fences> scratch_busy;
+  std::vector<cudaEvent_t> timing_free;  // timing-enabled events (GROUTER_PROFILE)
+};
+
+struct ProfRec {
+  int phys;
+  cudaEvent_t start, stop;
+  uint64_t bytes;
 };
 
 }  // namespace gr
@@ -189,6 +205,7 @@ struct grouter_ctx {
   uint64_t seq = 0, next_oid = 1, xfer_seq = 0;
   uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
   std::vector<grouter_oid> victims;
+  std::deque<gr::ProfRec> prof;                        // GROUTER_PROFILE launches not yet harvested
   std::deque<grouter_dispatch> dlog;
   grouter_stats_t stats{};
   // background I/O + dispatch thread (L269, L271)
@@ -210,6 +227,11 @@ void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_ch
                   int kind, uint64_t src_base, uint64_t dst_base, int dst_logical);
 void pump(grouter_ctx *c, bool force_all);            // dispatch rounds (caller holds mu)
 void flush_all(grouter_ctx *c);                        // replay flush
+void harvest_profile(grouter_ctx *c, bool wait);       // completed timed launches -> stats
+// Same-GPU SM copy run directly on the caller's stream when its copy server
+// is idle (or only busy with direct launches on that same stream).  Returns
+// false (nothing done) when the server path must be used.
+bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys);
 void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);  // submitted fences only
 // Waits on a CALLER stream: submitted fences now, the others as soon as their
 // producer transfer is submitted.

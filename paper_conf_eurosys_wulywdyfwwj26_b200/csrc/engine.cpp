@@ -92,6 +92,13 @@ Waitable signal(grouter_ctx *c, cudaStream_t s, int phys) {
   return w;
 }
 
+static Waitable ev_wait(grouter_ctx *c, EventRef e) {
+  Waitable w;
+  w.ev = std::move(e);
+  w.epoch = c->epoch;
+  return w;
+}
+
 EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
   EventRef e = c->phys.at(phys)->events.get();
   GR_CUDA(cudaEventRecord(e->ev, s));
@@ -323,11 +330,46 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
     p->pub[i].value = pubs[i].x->value_after(pubs[i].path);
   }
   PhysDev &pd = *c->phys.at(s.phys);
+  const bool prof = (c->cfg.flags & GROUTER_PROFILE) != 0;
+  ProfRec pr{s.phys, nullptr, nullptr, 0};
+  if (prof) {
+    for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
+      if (!pd.timing_free.empty()) {
+        *e = pd.timing_free.back();
+        pd.timing_free.pop_back();
+      } else {
+        GR_CUDA(cudaEventCreate(e));
+      }
+    }
+    for (auto &it : items) pr.bytes += it.bytes;
+    GR_CUDA(cudaEventRecord(pr.start, st));
+  }
   int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm,
                       (c->cfg.flags & GROUTER_COPY_TMA) != 0, st);
   if (e != 0)
     throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
+  if (prof) {
+    GR_CUDA(cudaEventRecord(pr.stop, st));
+    c->prof.push_back(pr);
+  }
   c->stats.kernel_launches++;
+}
+
+void harvest_profile(grouter_ctx *c, bool wait) {
+  while (!c->prof.empty()) {
+    ProfRec &r = c->prof.front();
+    if (wait) GR_CUDA(cudaEventSynchronize(r.stop));
+    else if (cudaEventQuery(r.stop) != cudaSuccess) break;
+    float ms = 0.f;
+    GR_CUDA(cudaEventElapsedTime(&ms, r.start, r.stop));
+    c->stats.timed_launches++;
+    c->stats.timed_ns += (uint64_t)((double)ms * 1e6);
+    c->stats.timed_bytes += r.bytes;
+    auto &fl = c->phys.at(r.phys)->timing_free;
+    fl.push_back(r.start);
+    fl.push_back(r.stop);
+    c->prof.pop_front();
+  }
 }
 
 // SM-copy server: one kernel launch per round segment (D2D push over
@@ -349,7 +391,7 @@ static size_t round_copy(grouter_ctx *c, Server &s) {
     c->stats.link_bytes[0][s.logical] += items[i].bytes;
   }
   launch_round(c, s, s.stream, s.scratch, seg, nullptr);
-  s.inflight.push_back(record(c, s.stream, s.phys));
+  s.inflight.push_back({ev_wait(c, record(c, s.stream, s.phys)), nullptr});
   c->stats.rounds++;
   after_submit(c, items);
   return items.size();
@@ -432,9 +474,9 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   EventRef ce_end = record(c, s.stream, s.phys);
   if (last_fwd) {  // one in-flight marker covering both the CE and the forward stream
     GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce_end->ev, 0));
-    s.inflight.push_back(record(c, s.fwd_stream, s.phys));
+    s.inflight.push_back({ev_wait(c, record(c, s.fwd_stream, s.phys)), nullptr});
   } else {
-    s.inflight.push_back(ce_end);
+    s.inflight.push_back({ev_wait(c, ce_end), nullptr});
   }
   c->stats.rounds++;
   after_submit(c, items);
@@ -463,15 +505,14 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
     c->stats.link_bytes[2][s.logical] += it.bytes;
   }
   publish_ce(c, s, seg);
-  s.inflight.push_back(record(c, s.stream, s.phys));
+  s.inflight.push_back({ev_wait(c, record(c, s.stream, s.phys)), nullptr});
   c->stats.rounds++;
   after_submit(c, items);
   return items.size();
 }
 
 static void retire(Server &s) {
-  while (!s.inflight.empty() && cudaEventQuery(s.inflight.front()->ev) == cudaSuccess)
-    s.inflight.pop_front();
+  while (!s.inflight.empty() && s.inflight.front().w.done()) s.inflight.pop_front();
 }
 
 static bool has_work(const Server &s) {
@@ -512,6 +553,42 @@ void pump(grouter_ctx *c, bool force_all) {
 void flush_all(grouter_ctx *c) {
   pump(c, true);
   c->epoch++;  // everything created before is now submitted (grounded)
+}
+
+bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys) {
+  if (c->replay || !caller) return false;
+  Server &s = c->dev[server_logical].copy;
+  if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty()) return false;
+  if (s.sched.backlog_items != x->nchunks) return false;  // only this transfer is queued
+  retire(s);
+  for (auto &f : s.inflight)
+    if (f.direct != caller) return false;  // server-stream work in flight: keep order there
+  for (auto &w : x->deps)
+    if (!is_submitted(w)) return false;
+  PhysDev &pd = *c->phys.at(s.phys);
+  DeviceGuard g(s.phys);
+  std::vector<ChunkItem> items;
+  std::vector<char> cut;
+  while (has_work(s)) {
+    refill(c, s, UINT32_MAX, c->cfg.round_bytes);
+    take(s, c->cfg.round_bytes, items, cut);
+    if (items.empty()) throw Error(GROUTER_ECUDA, "internal: direct launch made no progress");
+    if (cut[0]) stream_wait(c, caller, s.phys, x->deps);
+    // scratch pair for this launch (the server's own pair belongs to its stream)
+    uint32_t k = pd.next_scratch;
+    pd.next_scratch = (k + 1) % pd.n_scratch;
+    for (auto &w : pd.scratch_busy[k])
+      if (!w.done()) host_wait(Fences{w});
+    launch_round(c, s, caller, pd.scratch + 2 * k, items, nullptr);
+    for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
+    c->stats.rounds++;
+    after_submit(c, items);
+    Fences done;
+    done_fences(x, done);
+    pd.scratch_busy[k] = done;
+    s.inflight.push_back({done.empty() ? Waitable{} : done.front(), caller});
+  }
+  return true;
 }
 
 // D2H of an eviction victim (L258-L262; the per-GPU I/O path of L269): an
@@ -592,6 +669,13 @@ void engine_init(grouter_ctx *c) {
       pd->ordinal = p;
       pd->events.phys = p;
       GR_CUDA(cudaDeviceGetAttribute(&pd->sm_count, cudaDevAttrMultiProcessorCount, p));
+      {
+        DeviceGuard g(p);
+        pd->n_scratch = 256;
+        GR_CUDA(cudaMalloc(&pd->scratch, (size_t)pd->n_scratch * 2 * sizeof(uint32_t)));
+        GR_CUDA(cudaMemset(pd->scratch, 0, (size_t)pd->n_scratch * 2 * sizeof(uint32_t)));
+        pd->scratch_busy.assign(pd->n_scratch, {});
+      }
       c->phys[p] = std::move(pd);
     }
   }
@@ -703,6 +787,13 @@ void engine_shutdown(grouter_ctx *c) {
     d.pool.heap.quarantine.clear();
     d.pool.destroy();
   }
+  for (auto &kv : c->phys) {
+    DeviceGuard g(kv.first);
+    if (kv.second->scratch) cudaFree(kv.second->scratch);
+    for (cudaEvent_t e : kv.second->timing_free) cudaEventDestroy(e);
+    kv.second->scratch_busy.clear();
+  }
+  c->prof.clear();
   c->bounce_ev.clear();
   c->host.heap.quarantine.clear();
   if (c->host.base) cudaFreeHost(c->host.base);

@@ -13,6 +13,8 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
+#include <string>
 
 #include "../../include/grouter.h"
 #include "../../include/grouter_testing.h"
@@ -43,14 +45,14 @@ __device__ __forceinline__ void st_release_sys(uint64_t addr, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(addr), "r"(v) : "memory");
 }
 
-template <bool COUNT>
-__device__ __forceinline__ void count_bytes(const CopyParams &p, uint64_t dst_addr, uint32_t nbytes) {
+template <bool COUNT, class KP>
+__device__ __forceinline__ void count_bytes(const KP &p, uint64_t dst_addr, uint32_t nbytes) {
   if (COUNT) atomicAdd(&p.counts[(dst_addr - p.count_base) >> 4], nbytes);
 }
 
 // dst[0,len) <- src[0,len), all threads of the CTA; any alignment.
-template <bool COUNT>
-__device__ void tile_ldst(const CopyParams &p, uint8_t *dst, const uint8_t *src, uint64_t len) {
+template <bool COUNT, int U, class KP>
+__device__ void tile_ldst(const KP &p, uint8_t *dst, const uint8_t *src, uint64_t len) {
   const uint32_t tid = threadIdx.x;
   uintptr_t d = (uintptr_t)dst, s = (uintptr_t)src;
   // head: bytes until dst is 16-aligned
@@ -68,8 +70,9 @@ __device__ void tile_ldst(const CopyParams &p, uint8_t *dst, const uint8_t *src,
   const uint64_t nvec = len >> 4;
   int4 *vd = reinterpret_cast<int4 *>(dst);
   if ((s & 15) == 0) {
+    // 8 x 16 B in flight per thread before the first store (32 KiB per
+    // CTA pass); tiles are 8-64 KiB, chosen per launch to balance waves
     const int4 *vs = reinterpret_cast<const int4 *>(src);
-    constexpr int U = 4;
     uint64_t i = tid;
     for (; i + (U - 1) * kThreads < nvec; i += U * kThreads) {
       int4 v[U];
@@ -163,42 +166,9 @@ __device__ __forceinline__ void bulk_wait_read() {
 }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
-struct TmaState {
-  uint32_t phase_bits;  // one parity bit per stage
-};
-
-// One elected thread moves [src, src+len) -> [dst, ...) in kTmaStage pieces.
-// Requires 16 B alignment of src, dst and len.  Stage s is refilled with
-// piece k+S only after the store of piece k has finished READING shared
-// memory (wait_group.read 1 while the newest store may still be reading).
-__device__ void tile_tma(uint8_t *dst, const uint8_t *src, uint64_t len, uint8_t *smem,
-                         uint64_t *bars, TmaState &st) {
-  const uint32_t pieces = (uint32_t)((len + kTmaStage - 1) / kTmaStage);
-  auto piece_bytes = [&](uint32_t k) {
-    return (uint32_t)umin64(kTmaStage, len - (uint64_t)k * kTmaStage);
-  };
-  auto load = [&](uint32_t k) {
-    const uint32_t s = k % kTmaStages;
-    mbar_expect_tx(&bars[s], piece_bytes(k));
-    bulk_g2s(smem + s * kTmaStage, src + (uint64_t)k * kTmaStage, piece_bytes(k), &bars[s]);
-  };
-  for (uint32_t k = 0; k < pieces && k < (uint32_t)kTmaStages; ++k) load(k);
-  for (uint32_t k = 0; k < pieces; ++k) {
-    const uint32_t s = k % kTmaStages;
-    mbar_wait(&bars[s], (st.phase_bits >> s) & 1u);
-    st.phase_bits ^= (1u << s);
-    bulk_s2g(dst + (uint64_t)k * kTmaStage, smem + s * kTmaStage, piece_bytes(k));
-    bulk_commit();
-    if (k >= 1 && k - 1 + kTmaStages < pieces) {
-      bulk_wait_read<1>();
-      load(k - 1 + kTmaStages);
-    }
-  }
-  bulk_wait_read<0>();  // stages free for the next tile
-}
-
-// ------------------------------------------------------------------ round kernel
-__device__ __forceinline__ int find_chunk(const CopyParams &p, uint32_t t) {
+// ------------------------------------------------------------------ round kernels
+template <class KP>
+__device__ __forceinline__ int find_chunk(const KP &p, uint32_t t) {
   int lo = 0, hi = (int)p.n_chunks - 1;
   while (lo < hi) {
     int mid = (lo + hi + 1) >> 1;
@@ -208,10 +178,15 @@ __device__ __forceinline__ int find_chunk(const CopyParams &p, uint32_t t) {
   return lo;
 }
 
-__device__ __forceinline__ void finish_round(const CopyParams &p) {
-  __threadfence_system();
+// Round completion: the CTA barrier orders every thread's stores before
+// thread 0's system-scope fence (fences are cumulative), so ONE fence per
+// CTA suffices; the last CTA to finish publishes the completion words with
+// release stores (no partial visibility).
+template <class KP>
+__device__ __forceinline__ void finish_round(const KP &p) {
   __syncthreads();
   if (threadIdx.x == 0) {
+    __threadfence_system();
     unsigned prev = atomicAdd(&p.scratch[1], 1u);
     if (prev == gridDim.x - 1) {
       __threadfence_system();
@@ -224,8 +199,8 @@ __device__ __forceinline__ void finish_round(const CopyParams &p) {
   }
 }
 
-template <bool COUNT>
-__global__ void __launch_bounds__(kThreads) gr_copy_ldst(const __grid_constant__ CopyParams p) {
+template <bool COUNT, int U, int MINB, class KP>
+__global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_constant__ KP p) {
   __shared__ uint32_t s_tile;
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   for (;;) {
@@ -238,45 +213,86 @@ __global__ void __launch_bounds__(kThreads) gr_copy_ldst(const __grid_constant__
     const KChunk &ch = p.chunk[c];
     const uint64_t off = (uint64_t)(t - (uint32_t)p.tile_prefix[c]) << p.tile_log2;
     const uint64_t len = umin64(ch.bytes - off, 1ull << p.tile_log2);
-    tile_ldst<COUNT>(p, reinterpret_cast<uint8_t *>(ch.dst + off),
+    tile_ldst<COUNT, U>(p, reinterpret_cast<uint8_t *>(ch.dst + off),
                      reinterpret_cast<const uint8_t *>(ch.src + off), len);
   }
   finish_round(p);
 }
 
-__global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant__ CopyParams p) {
+// Continuous TMA stream: ONE elected thread per CTA claims tiles and keeps a
+// STAGES-deep ring of kTmaStage-byte pieces in flight across tile
+// boundaries -- bulk loads (global -> shared, mbarrier complete_tx) and bulk
+// stores (shared -> global, bulk groups); piece k+STAGES-1 is loaded into the
+// stage of piece k-1 once that piece's store has finished reading shared
+// memory.  Requires 16 B aligned chunks (checked by the launcher).
+template <int STAGES, class KP>
+__global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant__ KP p) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ __align__(8) uint64_t bars[kTmaStages];
-  __shared__ uint32_t s_tile;
+  __shared__ __align__(8) uint64_t bars[STAGES];
   if (threadIdx.x == 0) {
-    for (int i = 0; i < kTmaStages; ++i) mbar_init(&bars[i], 1);
+    for (int i = 0; i < STAGES; ++i) mbar_init(&bars[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  TmaState st{0};
-  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
-  for (;;) {
-    if (threadIdx.x == 0) s_tile = atomicAdd(&p.scratch[0], 1u);
-    __syncwarp();
-    __syncthreads();
-    const uint32_t t = s_tile;
-    __syncthreads();
-    if (t >= total) break;
-    const int c = find_chunk(p, t);
-    const KChunk &ch = p.chunk[c];
-    const uint64_t off = (uint64_t)(t - (uint32_t)p.tile_prefix[c]) << p.tile_log2;
-    const uint64_t len = umin64(ch.bytes - off, 1ull << p.tile_log2);
-    uint8_t *dst = reinterpret_cast<uint8_t *>(ch.dst + off);
-    const uint8_t *src = reinterpret_cast<const uint8_t *>(ch.src + off);
-    if ((((uintptr_t)dst | (uintptr_t)src | len) & 15) == 0) {
-      if (threadIdx.x == 0) tile_tma(dst, src, len, smem, bars, st);
-      __syncwarp();
-    } else {
-      // rare misaligned tile: plain byte copy by the warp
-      for (uint64_t i = threadIdx.x; i < len; i += kTmaThreads) dst[i] = src[i];
+    const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
+    // piece generator over claimed tiles
+    uint64_t cur_src = 0, cur_dst = 0, cur_left = 0;
+    auto next_piece = [&](uint64_t &ps, uint64_t &pd, uint32_t &pb) -> bool {
+      if (cur_left == 0) {
+        const uint32_t t = atomicAdd(&p.scratch[0], 1u);
+        if (t >= total) return false;
+        const int c = find_chunk(p, t);
+        const KChunk &ch = p.chunk[c];
+        const uint64_t off = (uint64_t)(t - (uint32_t)p.tile_prefix[c]) << p.tile_log2;
+        cur_src = ch.src + off;
+        cur_dst = ch.dst + off;
+        cur_left = umin64(ch.bytes - off, 1ull << p.tile_log2);
+      }
+      pb = (uint32_t)umin64(cur_left, kTmaStage);
+      ps = cur_src;
+      pd = cur_dst;
+      cur_src += pb;
+      cur_dst += pb;
+      cur_left -= pb;
+      return true;
+    };
+    uint64_t dst_of[STAGES];
+    uint32_t bytes_of[STAGES];
+    uint32_t phase = 0;
+    auto load = [&](uint32_t k, uint64_t ps, uint64_t pd, uint32_t pb) {
+      const uint32_t s = k % STAGES;
+      dst_of[s] = pd;
+      bytes_of[s] = pb;
+      mbar_expect_tx(&bars[s], pb);
+      bulk_g2s(smem + s * kTmaStage, reinterpret_cast<const void *>(ps), pb, &bars[s]);
+    };
+    uint32_t loaded = 0;
+    bool more = true;
+    for (; loaded < (uint32_t)STAGES; ++loaded) {
+      uint64_t ps, pd;
+      uint32_t pb;
+      if (!next_piece(ps, pd, pb)) {
+        more = false;
+        break;
+      }
+      load(loaded, ps, pd, pb);
     }
-  }
-  if (threadIdx.x == 0) {
+    for (uint32_t k = 0; k < loaded; ++k) {
+      const uint32_t s = k % STAGES;
+      mbar_wait(&bars[s], (phase >> s) & 1u);
+      phase ^= (1u << s);
+      bulk_s2g(reinterpret_cast<void *>(dst_of[s]), smem + s * kTmaStage, bytes_of[s]);
+      bulk_commit();
+      if (more && k >= 1) {
+        uint64_t ps, pd;
+        uint32_t pb;
+        if (next_piece(ps, pd, pb)) {
+          bulk_wait_read<1>();  // the store of piece k-1 has left its stage
+          load(loaded, ps, pd, pb);
+          ++loaded;
+        } else {
+          more = false;
+        }
+      }
+    }
     bulk_wait_all();
     asm volatile("fence.proxy.async.global;" ::: "memory");
   }
@@ -284,25 +300,223 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
   finish_round(p);
 }
 
-int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream) {
-  const uint64_t tiles = p.tile_prefix[p.n_chunks];
-  if (tiles == 0) return (int)cudaSuccess;
-  cudaStream_t s = (cudaStream_t)stream;
-  if (tma) {
-    static bool attr_set = false;
-    const int smem = kTmaStages * kTmaStage;
-    if (!attr_set) {
-      cudaFuncSetAttribute(gr_copy_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-      attr_set = true;
+// Warp-strided streaming copy: the round is cut into 4 KiB units; warp w of
+// W takes units w, w+W, w+2W ... and keeps U units (U x 8 x 16 B per lane)
+// in flight before storing.  No tile claims, no CTA barriers on the hot
+// loop; consecutive warps touch consecutive 4 KiB units (DRAM/L2-slice
+// friendly).  Partial or misaligned units fall back to the CTA-less warp
+// byte path.
+template <bool COUNT, int U, class KP>
+__global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ KP p) {
+  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t W = gridDim.x * (kThreads / 32);
+  const uint32_t w0 = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+  for (uint32_t base = w0; base < total; base += W * U) {
+    int4 v[U][8];
+    uint64_t dsts[U];
+    uint32_t lens[U];
+    uint64_t srcs[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t id = base + u * W;
+      lens[u] = 0;
+      if (id < total) {
+        const int c = find_chunk(p, id);
+        const KChunk &ch = p.chunk[c];
+        const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << 12;
+        srcs[u] = ch.src + off;
+        dsts[u] = ch.dst + off;
+        lens[u] = (uint32_t)umin64(ch.bytes - off, 4096);
+        if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
+          const int4 *sv = reinterpret_cast<const int4 *>(srcs[u]);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[u][j] = ld_stream(sv + j * 32 + lane);
+        }
+      }
     }
-    uint64_t grid = (uint64_t)sm_count * 3;
-    if (grid > tiles) grid = tiles;
-    gr_copy_tma<<<(unsigned)grid, kTmaThreads, smem, s>>>(p);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (!lens[u]) continue;
+      uint8_t *d = reinterpret_cast<uint8_t *>(dsts[u]);
+      const uint8_t *sp = reinterpret_cast<const uint8_t *>(srcs[u]);
+      if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
+        int4 *dv = reinterpret_cast<int4 *>(d);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          st_stream(dv + j * 32 + lane, v[u][j]);
+          count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
+        }
+      } else {
+        for (uint32_t i = lane; i < lens[u]; i += 32) {
+          d[i] = sp[i];
+          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
+        }
+      }
+    }
+  }
+  finish_round(p);
+}
+
+// Tile size per launch.  Tiles are claimed dynamically, so the makespan is
+// ~ceil(tiles / grid) tiles: take the LARGEST tile (fewest claims, longest
+// streams per claim) whose wave quantisation costs <= 5% over a perfect
+// split of the round's bytes; min_lg keeps a tile at least one full pass of
+// the engine (LD/ST: U x 256 x 16 B; TMA: 4 pieces).
+template <class KP>
+static void choose_tiles(KP &p, uint64_t grid_cap, uint32_t min_lg, uint32_t max_lg) {
+  uint64_t total = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
+  uint32_t best = min_lg;
+  double best_q = 1e30;
+  for (uint32_t lg = max_lg; lg >= min_lg; --lg) {
+    uint64_t tiles = 0;
+    for (uint32_t i = 0; i < p.n_chunks; ++i) tiles += (p.chunk[i].bytes + (1ull << lg) - 1) >> lg;
+    // makespan in bytes per CTA slot vs a perfect split over ALL slots
+    const double q = (double)(((tiles + grid_cap - 1) / grid_cap) << lg) * (double)grid_cap / (double)total;
+    if (q <= 1.05) {
+      best = lg;
+      break;
+    }
+    if (q < best_q) {
+      best_q = q;
+      best = lg;
+    }
+  }
+  p.tile_log2 = best;
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += (p.chunk[i].bytes + (1ull << best) - 1) >> best;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+}
+
+// Kernel variant: GR_COPY env (tuning) = ldst8 | ldst16 | tma4 | tma8 | tma12 |
+// ws1 | ws2 | ws4; default ws1, or tma8 for 16-B aligned rounds when `tma`.
+static int variant_from_env() {
+  static int v = -2;
+  if (v == -2) {
+    const char *e = getenv("GR_COPY");
+    v = -1;
+    if (e) {
+      std::string s(e);
+      v = s == "ldst8" ? 0 : s == "ldst16" ? 1 : s == "tma4" ? 2 : s == "tma8" ? 3 : s == "tma12" ? 4
+        : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : -1;
+    }
+  }
+  return v;
+}
+
+template <int STAGES, class KP>
+static void launch_tma(KP &p, int sm_count, cudaStream_t s) {
+  static bool attr_set = false;
+  const int smem = STAGES * kTmaStage;
+  if (!attr_set) {
+    cudaFuncSetAttribute(gr_copy_tma<STAGES, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr_set = true;
+  }
+  const int per_sm = STAGES <= 4 ? 3 : STAGES <= 8 ? 1 : 1;
+  const uint64_t cap = (uint64_t)sm_count * per_sm;
+  choose_tiles(p, cap, 16, 20);
+  uint64_t tiles = p.tile_prefix[p.n_chunks];
+  uint64_t grid = cap > tiles ? tiles : cap;
+  gr_copy_tma<STAGES, KP><<<(unsigned)grid, kTmaThreads, smem, s>>>(p);
+}
+
+template <int U, int MINB, class KP>
+static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  static int occ = 0;
+  if (!occ) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ldst<false, U, MINB, KP>, kThreads, 0);
+    if (occ <= 0) occ = 1;
+  }
+  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
+  const uint64_t cap = (uint64_t)sm_count * (uint64_t)per_sm;
+  choose_tiles(p, cap, U == 16 ? 16 : 15, 18);
+  uint64_t tiles = p.tile_prefix[p.n_chunks];
+  uint64_t grid = cap > tiles ? tiles : cap;
+  if (p.counts) gr_copy_ldst<true, U, MINB, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+  else gr_copy_ldst<false, U, MINB, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+}
+
+template <int U, class KP>
+static void launch_ws(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  static int occ = 0;
+  if (!occ) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ws<false, U, KP>, kThreads, 0);
+    if (occ <= 0) occ = 1;
+  }
+  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
+  p.tile_log2 = 12;
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += (p.chunk[i].bytes + 4095) >> 12;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+  // enough warps that every warp has U units in flight at least once
+  uint64_t warps = (t + U - 1) / U;
+  uint64_t grid = (warps + (kThreads / 32) - 1) / (kThreads / 32);
+  const uint64_t cap = (uint64_t)sm_count * per_sm;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  if (p.counts) gr_copy_ws<true, U, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+  else gr_copy_ws<false, U, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+}
+
+template <class KP>
+static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  switch (v) {
+    case 5: launch_ws<1>(p, sm_count, ctas_per_sm, s); break;
+    case 6: launch_ws<2>(p, sm_count, ctas_per_sm, s); break;
+    case 7: launch_ws<4>(p, sm_count, ctas_per_sm, s); break;
+    case 1: launch_ldst<16, 4>(p, sm_count, ctas_per_sm, s); break;
+    case 2: launch_tma<4>(p, sm_count, s); break;
+    case 3: launch_tma<8>(p, sm_count, s); break;
+    case 4: launch_tma<12>(p, sm_count, s); break;
+    default: launch_ldst<8, 1>(p, sm_count, ctas_per_sm, s); break;
+  }
+}
+
+int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream) {
+  if (p.n_chunks == 0) return (int)cudaSuccess;
+  static int ctas_env = -1;
+  if (ctas_env < 0) {
+    const char *e = getenv("GR_CTAS");
+    ctas_env = e ? atoi(e) : 0;
+  }
+  if (ctas_env > 0) ctas_per_sm = ctas_env;
+  cudaStream_t s = (cudaStream_t)stream;
+  // coalesce chunks that are contiguous in both source and destination (the
+  // plan's 2 MiB chunks of one transfer are): fewer, longer runs per launch
+  uint32_t w = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    if (w && p.chunk[w - 1].src + p.chunk[w - 1].bytes == p.chunk[i].src &&
+        p.chunk[w - 1].dst + p.chunk[w - 1].bytes == p.chunk[i].dst)
+      p.chunk[w - 1].bytes += p.chunk[i].bytes;
+    else
+      p.chunk[w++] = p.chunk[i];
+  }
+  p.n_chunks = w;
+  bool aligned = true;
+  for (uint32_t i = 0; i < p.n_chunks; ++i)
+    aligned &= ((p.chunk[i].src | p.chunk[i].dst | p.chunk[i].bytes) & 15) == 0;
+  int v = variant_from_env();
+  if (v < 0) v = tma ? 3 : 5;  // default: warp-strided LD/ST; GROUTER_COPY_TMA: 8-stage bulk ring
+  if (v >= 2 && v <= 4 && (!aligned || p.counts)) v = 0;  // TMA needs 16 B alignment; counting is LD/ST
+  if (p.n_chunks <= (uint32_t)SmallParams::kChunks && p.n_pub <= (uint32_t)SmallParams::kPubs) {
+    SmallParams q;
+    q.n_chunks = p.n_chunks;
+    q.n_pub = p.n_pub;
+    q.scratch = p.scratch;
+    q.counts = p.counts;
+    q.count_base = p.count_base;
+    for (uint32_t i = 0; i < p.n_chunks; ++i) q.chunk[i] = p.chunk[i];
+    for (uint32_t i = 0; i < p.n_pub; ++i) q.pub[i] = p.pub[i];
+    launch_variant(q, v, sm_count, ctas_per_sm, s);
   } else {
-    uint64_t grid = (uint64_t)sm_count * (uint64_t)ctas_per_sm;
-    if (grid > tiles) grid = tiles;
-    if (p.counts) gr_copy_ldst<true><<<(unsigned)grid, kThreads, 0, s>>>(p);
-    else gr_copy_ldst<false><<<(unsigned)grid, kThreads, 0, s>>>(p);
+    launch_variant(p, v, sm_count, ctas_per_sm, s);
   }
   return (int)cudaGetLastError();
 }

@@ -27,17 +27,25 @@ struct KPublish {
   uint32_t pad;
 };
 
-struct CopyParams {
+// Kernel parameters (passed by value, __grid_constant__).  Two capacities:
+// the large one for rounds with many distinct chunks, a small one (a few
+// hundred bytes -- cheaper to launch) for the common round whose chunks
+// coalesce into a handful of contiguous runs.
+template <int C, int P>
+struct KParams {
+  static constexpr int kChunks = C, kPubs = P;
   uint32_t n_chunks = 0, n_pub = 0;
   uint32_t tile_log2 = 16;
   uint32_t _pad = 0;
   uint32_t *scratch = nullptr;   // [0] tile ticket, [1] finished CTAs; zero between launches
   uint32_t *counts = nullptr;    // test only: bytes written per 16 B granule
   uint64_t count_base = 0;
-  uint64_t tile_prefix[kMaxRoundChunks + 1] = {};
-  KChunk chunk[kMaxRoundChunks];
-  KPublish pub[kMaxPublish];
+  uint64_t tile_prefix[C + 1] = {};
+  KChunk chunk[C];
+  KPublish pub[P];
 };
+using CopyParams = KParams<kMaxRoundChunks, kMaxPublish>;   // host-side builder
+using SmallParams = KParams<8, 8>;
 
 // Launch gr_copy on `stream` (current device must own the stream).  grid =
 // min(tiles, sm_count * ctas_per_sm).  Returns cudaError_t as int.

@@ -24,7 +24,7 @@ HOST = -1
 NOHINT = -2
 UNLIMITED = (1 << 64) - 1
 
-REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA = 0x1, 0x2, 0x4, 0x8, 0x10
+REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]
@@ -70,7 +70,8 @@ class grouter_stats_t(C.Structure):
         ("mapped", C.c_uint64 * MAX_GPUS), ("host_used", C.c_uint64), ("host_cap", C.c_uint64),
         ("spill_count", C.c_uint64), ("spill_bytes", C.c_uint64), ("xfer_count", C.c_uint64),
         ("link_bytes", (C.c_uint64 * MAX_GPUS) * 3), ("kernel_launches", C.c_uint64),
-        ("rounds", C.c_uint64),
+        ("rounds", C.c_uint64), ("timed_launches", C.c_uint64), ("timed_ns", C.c_uint64),
+        ("timed_bytes", C.c_uint64),
     ]
 
 

@@ -65,6 +65,27 @@ def test_verify_kernel_detects_corruption():
 @pytest.mark.parametrize("tma", [False, True])
 @pytest.mark.parametrize("src_off,dst_off", [(0, 0), (16, 32), (3, 3), (1, 0), (0, 5), (7, 13), (15, 1)])
 def test_copy_kernel_exactly_once(tma, src_off, dst_off):
+    _copy_exactly_once(tma, src_off, dst_off)
+
+
+VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4"]
+
+
+@pytest.mark.parametrize("variant", VARIANTS)
+def test_copy_kernel_variants(variant):
+    """Every engine variant (GR_COPY) in a subprocess: byte-exact over aligned
+    and misaligned chunk lists, exactly-once counts where it can count."""
+    import os
+    import subprocess
+    import sys
+    code = ("import sys; sys.path.insert(0, '.'); from tests.test_gpu_parity import _copy_exactly_once as f; "
+            "[f(t, a, b) for t in (False, True) for a, b in ((0, 0), (3, 3), (1, 0), (7, 13))]")
+    r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, GR_COPY=variant),
+                       capture_output=True, text=True, timeout=240)
+    assert r.returncode == 0, r.stderr[-2000:]
+
+
+def _copy_exactly_once(tma, src_off, dst_off):
     """Invariant I1 on the production kernel: every destination byte of a
     chunk list tiling [0, n) is written exactly once; bytes are identical;
     guard bands stay untouched."""
