@@ -328,7 +328,7 @@ def run_gpu(args, rank, world, local_rank):
             "config": {"workload": WORKLOAD, "requests_per_step": R, "bytes": N_BYTES,
                        "parallelism": f"replicas x{world}",
                        "l2": "inputs larger than L2: 20 resident 38.5 MB objects, 8 rotating bindings",
-                       "copy_kernel": "tma" if args.tma else f"ldst {args.ctas} CTA/SM"},
+                       "copy_kernel": os.environ.get("GR_COPY", "tma8" if args.tma else "ws1") + f", {args.ctas} CTA/SM cap"},
             "gbps": value * N_BYTES / 1e9,
             "host_us_per_request": host_us,
             "latency_us": {"p50": pct(lat, 50), "p99": pct(lat, 99), "samples": len(lat),
