@@ -213,10 +213,12 @@ def run_gpu(args, rank, world, local_rank):
         G.check(st, "put")
         resident.append(oid)
 
+    bptr = [bindings[i % B].data_ptr() for i in range(R)]
+    work = list(zip(resident, bptr))
+
     def value_step():
-        for i, oid in enumerate(resident):
-            b = bindings[i % B]
-            st, _ = ctx.get_into(gfn, oid, b.data_ptr(), n, s)
+        for oid, dst in work:
+            st, _ = ctx.get_into(gfn, oid, dst, n, s)
             if st:
                 G.check(st, "get_into")
 

@@ -96,7 +96,7 @@ struct Xfer {
 using XferRef = std::shared_ptr<Xfer>;
 
 struct ChunkItem {
-  XferRef x;
+  Xfer *x;            // kept alive by grouter_ctx::live until fully submitted
   uint32_t idx;       // chunk index in the plan
   uint32_t path;
   uint64_t src, dst;  // absolute addresses (device VA or host)
@@ -161,6 +161,8 @@ struct LogicalDev {
   Server copy, h2d, d2h;
 };
 
+struct CopyParamsHost;  // kernels.h CopyParams, boxed (keeps kernels.h out of this header)
+
 struct PhysDev {
   int ordinal = -1;
   int sm_count = 148;
@@ -206,6 +208,8 @@ struct grouter_ctx {
   uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
   std::vector<grouter_oid> victims;
   std::deque<gr::ProfRec> prof;                        // GROUTER_PROFILE launches not yet harvested
+  std::unordered_map<gr::Xfer *, gr::XferRef> live;    // transfers with chunks not yet submitted
+  gr::CopyParamsHost *params = nullptr;                // reused kernel-parameter builder (engine.cpp)
   std::deque<grouter_dispatch> dlog;
   grouter_stats_t stats{};
   // background I/O + dispatch thread (L269, L271)
@@ -216,6 +220,7 @@ struct grouter_ctx {
 };
 
 namespace gr {
+struct CopyParamsHost;
 // engine.cpp
 void engine_init(grouter_ctx *c);
 void engine_shutdown(grouter_ctx *c);

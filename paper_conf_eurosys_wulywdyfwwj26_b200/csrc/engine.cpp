@@ -35,6 +35,10 @@
 
 namespace gr {
 
+struct CopyParamsHost {
+  CopyParams p;
+};
+
 static const uint32_t kSlots = 4096;
 XferRef new_xfer_slot(grouter_ctx *c, const std::vector<grouter_chunk> &plan);
 static const uint32_t kBounceSlots = 16;
@@ -189,7 +193,7 @@ static Server &server_of(grouter_ctx *c, int kind, int logical) {
 static ChunkItem make_item(const XferRef &x, uint32_t i, const grouter_chunk &ch, uint64_t src_base,
                            uint64_t dst_base, int dst_logical) {
   ChunkItem it;
-  it.x = x;
+  it.x = x.get();
   it.idx = i;
   it.path = (uint32_t)ch.path;
   it.src = src_base + ch.offset;
@@ -201,6 +205,7 @@ static ChunkItem make_item(const XferRef &x, uint32_t i, const grouter_chunk &ch
 
 void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_chunk> &plan, int kind,
                   uint64_t src_base, uint64_t dst_base, int dst_logical) {
+  if (!plan.empty()) c->live.emplace(x.get(), x);
   for (uint32_t i = 0; i < plan.size(); ++i)
     server_of(c, kind, plan[i].route_gpu)
         .sched.enqueue(x->tenant, make_item(x, i, plan[i], src_base, dst_base, dst_logical));
@@ -288,7 +293,7 @@ struct Pub {
 static std::vector<Pub> issue(const std::vector<ChunkItem> &items) {
   std::vector<Pub> pubs;
   for (auto &it : items) {
-    Xfer *x = it.x.get();
+    Xfer *x = it.x;
     x->issued[it.path]++;
     bool found = false;
     for (auto &p : pubs) found |= (p.x == x && p.path == it.path);
@@ -301,19 +306,32 @@ static std::vector<Pub> issue(const std::vector<ChunkItem> &items) {
 // transfers that are now fully submitted.
 static void after_submit(grouter_ctx *c, const std::vector<ChunkItem> &items) {
   for (auto &it : items) it.x->submitted_chunks++;
+  Xfer *last = nullptr;
   for (auto &it : items) {
-    Xfer &x = *it.x;
-    if (!x.submitted() || x.waiters.empty()) continue;
-    auto ws = std::move(x.waiters);
-    x.waiters.clear();
-    for (auto &wt : ws) stream_wait(c, wt.stream, -1, Fences{wt.w});
+    Xfer *x = it.x;
+    if (x == last || !x->submitted()) continue;
+    last = x;
+    if (!x->waiters.empty()) {
+      auto ws = std::move(x->waiters);
+      x->waiters.clear();
+      for (auto &wt : ws) stream_wait(c, wt.stream, -1, Fences{wt.w});
+    }
   }
+  // release ownership of fully submitted transfers (collect first: erasing
+  // may destroy the transfer, and a round may hold several of its chunks)
+  std::vector<Xfer *> fin;
+  for (auto &it : items)
+    if (it.x->submitted() && std::find(fin.begin(), fin.end(), it.x) == fin.end()) fin.push_back(it.x);
+  for (Xfer *x : fin) c->live.erase(x);
 }
 
 static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *scratch,
                          const std::vector<ChunkItem> &items, const uint64_t *src_override) {
-  auto p = std::make_unique<CopyParams>();
+  if (!c->params) c->params = new CopyParamsHost();
+  CopyParams *p = &c->params->p;
   p->n_chunks = (uint32_t)items.size();
+  p->counts = nullptr;
+  p->count_base = 0;
   p->scratch = scratch;
   p->tile_log2 = 16;
   uint64_t t = 0;
@@ -794,6 +812,9 @@ void engine_shutdown(grouter_ctx *c) {
     kv.second->scratch_busy.clear();
   }
   c->prof.clear();
+  c->live.clear();
+  delete c->params;
+  c->params = nullptr;
   c->bounce_ev.clear();
   c->host.heap.quarantine.clear();
   if (c->host.base) cudaFreeHost(c->host.base);

@@ -41,6 +41,13 @@ __device__ __forceinline__ void st_stream(int4 *p, const int4 &v) {
                "r"(v.w)
                : "memory");
 }
+// Programmatic dependent launch (sm_90+): a copy kernel is launched while
+// its predecessor on the stream drains; it waits here (before touching any
+// memory or its scratch) until the predecessor completed and flushed, and
+// lets its own successor launch once its main loop is done.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ void st_release_sys(uint64_t addr, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(addr), "r"(v) : "memory");
 }
@@ -201,6 +208,7 @@ __device__ __forceinline__ void finish_round(const KP &p) {
 
 template <bool COUNT, int U, int MINB, class KP>
 __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_constant__ KP p) {
+  pdl_wait();
   __shared__ uint32_t s_tile;
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   for (;;) {
@@ -216,6 +224,7 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
     tile_ldst<COUNT, U>(p, reinterpret_cast<uint8_t *>(ch.dst + off),
                      reinterpret_cast<const uint8_t *>(ch.src + off), len);
   }
+  pdl_trigger();
   finish_round(p);
 }
 
@@ -227,6 +236,7 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
 // memory.  Requires 16 B aligned chunks (checked by the launcher).
 template <int STAGES, class KP>
 __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant__ KP p) {
+  pdl_wait();
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
   if (threadIdx.x == 0) {
@@ -297,6 +307,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
     asm volatile("fence.proxy.async.global;" ::: "memory");
   }
   __syncthreads();
+  pdl_trigger();
   finish_round(p);
 }
 
@@ -308,6 +319,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
 // byte path.
 template <bool COUNT, int U, class KP>
 __global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ KP p) {
+  pdl_wait();
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t W = gridDim.x * (kThreads / 32);
@@ -355,7 +367,141 @@ __global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ K
       }
     }
   }
+  pdl_trigger();
   finish_round(p);
+}
+
+// Warp-dynamic streaming copy: like ws, but each warp CLAIMS U consecutive
+// 4 KiB units from the round's ticket (lane 0, atomicAdd), and claims the
+// next batch while this batch's loads are in flight, so faster SMs take
+// more units (the per-SM latency spread no longer sets the launch length).
+template <bool COUNT, int U, class KP>
+__global__ void __launch_bounds__(kThreads) gr_copy_wd(const __grid_constant__ KP p) {
+  pdl_wait();
+  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
+  const uint32_t lane = threadIdx.x & 31;
+  uint32_t next = 0;
+  if (lane == 0) next = atomicAdd(&p.scratch[0], (uint32_t)U);
+  next = __shfl_sync(0xffffffffu, next, 0);
+  while (next < total) {
+    const uint32_t base = next;
+    int4 v[U][8];
+    uint64_t dsts[U], srcs[U];
+    uint32_t lens[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint32_t id = base + u;
+      lens[u] = 0;
+      if (id < total) {
+        const int c = find_chunk(p, id);
+        const KChunk &ch = p.chunk[c];
+        const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << 12;
+        srcs[u] = ch.src + off;
+        dsts[u] = ch.dst + off;
+        lens[u] = (uint32_t)umin64(ch.bytes - off, 4096);
+        if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
+          const int4 *sv = reinterpret_cast<const int4 *>(srcs[u]);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[u][j] = ld_stream(sv + j * 32 + lane);
+        }
+      }
+    }
+    if (lane == 0) next = atomicAdd(&p.scratch[0], (uint32_t)U);  // overlaps the loads
+    next = __shfl_sync(0xffffffffu, next, 0);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (!lens[u]) continue;
+      uint8_t *d = reinterpret_cast<uint8_t *>(dsts[u]);
+      const uint8_t *sp = reinterpret_cast<const uint8_t *>(srcs[u]);
+      if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
+        int4 *dv = reinterpret_cast<int4 *>(d);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          st_stream(dv + j * 32 + lane, v[u][j]);
+          count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
+        }
+      } else {
+        for (uint32_t i = lane; i < lens[u]; i += 32) {
+          d[i] = sp[i];
+          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
+        }
+      }
+    }
+  }
+  pdl_trigger();
+  finish_round(p);
+}
+
+// Grid-stride streaming copy over the round's 16 B vectors: thread t moves
+// vectors t, t+S, t+2S, ... (S = grid threads), U loads in flight spread a
+// whole grid-width apart -- every DRAM channel/L2 slice is busy at once and
+// no two warps contend for the same lines.  Requires 16 B aligned chunks
+// (launcher checks); the flattened vector space maps to chunks through a
+// prefix (in vectors) -- a single coalesced chunk skips the search.
+template <int U, class KP>
+__global__ void __launch_bounds__(kThreads) gr_copy_gs(const __grid_constant__ KP p) {
+  pdl_wait();
+  const uint64_t total = p.tile_prefix[p.n_chunks];           // vectors
+  const uint64_t S = (uint64_t)gridDim.x * kThreads;
+  const bool one = p.n_chunks == 1;
+  const int4 *s0 = reinterpret_cast<const int4 *>(p.chunk[0].src);
+  int4 *d0 = reinterpret_cast<int4 *>(p.chunk[0].dst);
+  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < total; i += S * U) {
+    int4 v[U];
+    int4 *dp[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t j = i + (uint64_t)u * S;
+      dp[u] = nullptr;
+      if (j < total) {
+        const int4 *sp;
+        if (one) {
+          sp = s0 + j;
+          dp[u] = d0 + j;
+        } else {
+          int lo = 0, hi = (int)p.n_chunks - 1;
+          while (lo < hi) {
+            int mid = (lo + hi + 1) >> 1;
+            if (p.tile_prefix[mid] <= j) lo = mid;
+            else hi = mid - 1;
+          }
+          const uint64_t o = j - p.tile_prefix[lo];
+          sp = reinterpret_cast<const int4 *>(p.chunk[lo].src) + o;
+          dp[u] = reinterpret_cast<int4 *>(p.chunk[lo].dst) + o;
+        }
+        v[u] = ld_stream(sp);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (dp[u]) st_stream(dp[u], v[u]);
+  }
+  pdl_trigger();
+  finish_round(p);
+}
+
+// Launch with programmatic stream serialization (PDL) when GR_PDL=1 (hides
+// the inter-kernel gap, ~0.8 us/launch, but the Ex launch path costs host
+// time and the data path is near host-bound; measured both ways).
+template <class KP>
+static void launch_pdl(void (*kern)(KP), uint64_t grid, int block, int smem, cudaStream_t s, const KP &p) {
+  static int pdl = -1;
+  if (pdl < 0) {
+    const char *e = getenv("GR_PDL");
+    pdl = (e && e[0] == '1') ? 1 : 0;  // opt-in: cudaLaunchKernelEx costs host time
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  if (pdl) cudaLaunchKernelEx(&cfg, kern, p);
+  else kern<<<cfg.gridDim, cfg.blockDim, cfg.dynamicSmemBytes, s>>>(p);
 }
 
 // Tile size per launch.  Tiles are claimed dynamically, so the makespan is
@@ -402,7 +548,8 @@ static int variant_from_env() {
     if (e) {
       std::string s(e);
       v = s == "ldst8" ? 0 : s == "ldst16" ? 1 : s == "tma4" ? 2 : s == "tma8" ? 3 : s == "tma12" ? 4
-        : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : -1;
+        : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : s == "wd1" ? 8 : s == "wd2" ? 9
+        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : -1;
     }
   }
   return v;
@@ -421,7 +568,7 @@ static void launch_tma(KP &p, int sm_count, cudaStream_t s) {
   choose_tiles(p, cap, 16, 20);
   uint64_t tiles = p.tile_prefix[p.n_chunks];
   uint64_t grid = cap > tiles ? tiles : cap;
-  gr_copy_tma<STAGES, KP><<<(unsigned)grid, kTmaThreads, smem, s>>>(p);
+  launch_pdl(gr_copy_tma<STAGES, KP>, grid, kTmaThreads, smem, s, p);
 }
 
 template <int U, int MINB, class KP>
@@ -436,8 +583,8 @@ static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   choose_tiles(p, cap, U == 16 ? 16 : 15, 18);
   uint64_t tiles = p.tile_prefix[p.n_chunks];
   uint64_t grid = cap > tiles ? tiles : cap;
-  if (p.counts) gr_copy_ldst<true, U, MINB, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
-  else gr_copy_ldst<false, U, MINB, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+  if (p.counts) launch_pdl(gr_copy_ldst<true, U, MINB, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_ldst<false, U, MINB, KP>, grid, kThreads, 0, s, p);
 }
 
 template <int U, class KP>
@@ -461,13 +608,59 @@ static void launch_ws(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   const uint64_t cap = (uint64_t)sm_count * per_sm;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
-  if (p.counts) gr_copy_ws<true, U, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
-  else gr_copy_ws<false, U, KP><<<(unsigned)grid, kThreads, 0, s>>>(p);
+  if (p.counts) launch_pdl(gr_copy_ws<true, U, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_ws<false, U, KP>, grid, kThreads, 0, s, p);
+}
+
+template <int U, class KP>
+static void launch_wd(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  static int occ = 0;
+  if (!occ) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wd<false, U, KP>, kThreads, 0);
+    if (occ <= 0) occ = 1;
+  }
+  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
+  p.tile_log2 = 12;
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += (p.chunk[i].bytes + 4095) >> 12;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+  uint64_t warps = (t + U - 1) / U;
+  uint64_t grid = (warps + (kThreads / 32) - 1) / (kThreads / 32);
+  const uint64_t cap = (uint64_t)sm_count * per_sm;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  if (p.counts) launch_pdl(gr_copy_wd<true, U, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_wd<false, U, KP>, grid, kThreads, 0, s, p);
+}
+
+template <int U, class KP>
+static void launch_gs(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += p.chunk[i].bytes >> 4;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+  p.tile_log2 = 4;
+  // enough threads for U vectors each, capped at ctas_per_sm CTAs per SM
+  uint64_t grid = (t + (uint64_t)kThreads * U - 1) / ((uint64_t)kThreads * U);
+  const uint64_t cap = (uint64_t)sm_count * (uint64_t)ctas_per_sm;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  launch_pdl(gr_copy_gs<U, KP>, grid, kThreads, 0, s, p);
 }
 
 template <class KP>
 static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
   switch (v) {
+    case 10: launch_gs<8>(p, sm_count, ctas_per_sm, s); break;
+    case 11: launch_gs<4>(p, sm_count, ctas_per_sm, s); break;
+    case 12: launch_gs<16>(p, sm_count, ctas_per_sm, s); break;
+    case 8: launch_wd<1>(p, sm_count, ctas_per_sm, s); break;
+    case 9: launch_wd<2>(p, sm_count, ctas_per_sm, s); break;
     case 5: launch_ws<1>(p, sm_count, ctas_per_sm, s); break;
     case 6: launch_ws<2>(p, sm_count, ctas_per_sm, s); break;
     case 7: launch_ws<4>(p, sm_count, ctas_per_sm, s); break;
@@ -504,7 +697,7 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
     aligned &= ((p.chunk[i].src | p.chunk[i].dst | p.chunk[i].bytes) & 15) == 0;
   int v = variant_from_env();
   if (v < 0) v = tma ? 3 : 5;  // default: warp-strided LD/ST; GROUTER_COPY_TMA: 8-stage bulk ring
-  if (v >= 2 && v <= 4 && (!aligned || p.counts)) v = 0;  // TMA needs 16 B alignment; counting is LD/ST
+  if (((v >= 2 && v <= 4) || v >= 10) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
   if (p.n_chunks <= (uint32_t)SmallParams::kChunks && p.n_pub <= (uint32_t)SmallParams::kPubs) {
     SmallParams q;
     q.n_chunks = p.n_chunks;

@@ -68,7 +68,7 @@ def test_copy_kernel_exactly_once(tma, src_off, dst_off):
     _copy_exactly_once(tma, src_off, dst_off)
 
 
-VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4"]
+VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4", "wd1", "wd2", "gs4", "gs8", "gs16"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
