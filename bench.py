@@ -41,6 +41,11 @@ WORKLOAD = ("cfg1 2-function workflow, 38,535,168 B tensor; value: gFn get_into 
             "from pinned host + get_into + 8 B D2H")
 
 
+WORKLOAD_N = ("cfg1 2-function workflow at N GPUs, 38,535,168 B tensor; value: gFn on GPU r get_into "
+              "of objects resident on GPU r+1 (exported/imported via CUDA VMM IPC, SM pull copy over "
+              "NVLink), e2e: cFn put(hint=own GPU) from pinned host + local get_into + 8 B D2H")
+
+
 def _peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -90,6 +95,37 @@ class ClockSampler:
                     reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
                 "samples": len(sm), "reasons": sorted(reasons)}
+
+
+# ------------------------------------------------------------------ multi-rank plumbing (gloo-tested)
+def peer_of(rank: int, world: int) -> int:
+    """cfg1 at N GPUs: the object produced on GPU r+1 is consumed on GPU r
+    (a ring of disjoint producer->consumer pairs: every GPU's NVLink egress
+    and ingress carry one stream, no link is shared)."""
+    return (rank + 1) % world
+
+
+def exchange(obj, world: int, group=None):
+    """all_gather of a picklable object (export descriptors) over the
+    process group; world == 1 returns [obj]."""
+    if world == 1:
+        return [obj]
+    import torch.distributed as dist
+    out = [None] * world
+    dist.all_gather_object(out, obj, group=group)
+    return out
+
+
+def max_over_ranks(x: float, world: int, device=None) -> float:
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    if dist.get_backend() != "nccl":
+        device = None
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
 
 
 # ------------------------------------------------------------------ reference / oracle arm
@@ -216,6 +252,23 @@ def run_gpu(args, rank, world, local_rank):
     bptr = [bindings[i % B].data_ptr() for i in range(R)]
     work = list(zip(resident, bptr))
 
+    remote = world > 1
+    exports = []
+    if remote:
+        # export every resident object, import the peer's (CUDA VMM IPC, L167/L269)
+        for oid in resident:
+            st, desc = ctx.export_ipc(gfn, oid)
+            G.check(st, "export_ipc")
+            exports.append((oid, desc))
+        all_descs = exchange([d for _, d in exports], world)
+        peer = peer_of(rank, world)
+        imported = []
+        for desc in all_descs[peer]:
+            st, roid = ctx.import_ipc(gfn, desc)
+            G.check(st, "import_ipc")
+            imported.append(roid)
+        work = list(zip(imported, bptr))
+
     def value_step():
         for oid, dst in work:
             st, _ = ctx.get_into(gfn, oid, dst, n, s)
@@ -249,10 +302,7 @@ def run_gpu(args, rank, world, local_rank):
     ms = e0.elapsed_time(e1)
     G.check(ctx.sync(), "sync")
     st1 = ctx.stats()
-    t = torch.tensor([ms], device=f"cuda:{dev}", dtype=torch.float64)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
+    ms_max = max_over_ranks(ms, world, f"cuda:{dev}")
     total_req = R * args.steps * world
     value = total_req / (ms_max / 1e3)
     launches = st1.kernel_launches - st0.kernel_launches
@@ -261,10 +311,15 @@ def run_gpu(args, rank, world, local_rank):
     # launches, GPU-bound: host submission < GPU time), so the event-timed
     # region on that stream / launches = average launch duration (incl. the
     # inter-launch gap, i.e. conservative).
-    alg_bytes_per_launch = 2 * moved / max(launches, 1)      # read + write (same-GPU HBM copy)
     avg_ns = ms * 1e6 / max(launches, 1)
+    if remote:   # pull over NVLink: n bytes cross the link per request
+        alg_bytes_per_launch = moved / max(launches, 1)
+        bound, peak, peak_src = "nvlink", 770.0, "B200_PROFILING.md measured peer copy 770 GB/s/direction"
+    else:        # same-GPU HBM copy: read + write
+        alg_bytes_per_launch = 2 * moved / max(launches, 1)
+        bound = "hbm"
+        peak, peak_src = _peaks()
     achieved = alg_bytes_per_launch / avg_ns if launches else None  # bytes/ns == GB/s
-    peak, peak_src = _peaks()
 
     # per-request latency (separate, untimed pass): device events around one get_into
     lat = []
@@ -302,10 +357,15 @@ def run_gpu(args, rank, world, local_rank):
         e2e_step()
     barrier()
     e2e_s = time.perf_counter() - h0
-    t = torch.tensor([e2e_s], device=f"cuda:{dev}", dtype=torch.float64)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    e2e_val = R * e2e_steps * world / float(t.item())
+    e2e_val = R * e2e_steps * world / max_over_ranks(e2e_s, world, f"cuda:{dev}")
+
+    if remote:   # drop imports and our export pins once every rank is done reading
+        barrier()
+        for roid in imported:
+            ctx.free(gfn, roid)
+        barrier()
+        for oid, desc in exports:
+            ctx.release(gfn, oid, G.Ctx.desc_exporter_ptr(desc), 0)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -327,15 +387,17 @@ def run_gpu(args, rank, world, local_rank):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (SplitMix64 payload, verified on device before timing)",
-            "config": {"workload": WORKLOAD, "requests_per_step": R, "bytes": N_BYTES,
-                       "parallelism": f"replicas x{world}",
+            "config": {"workload": WORKLOAD if not remote else WORKLOAD_N, "requests_per_step": R,
+                       "bytes": N_BYTES,
+                       "parallelism": f"replicas x{world}" if not remote else
+                       f"{world} GPUs, GPU r pulls from GPU r+1 over NVLink (IPC-mapped pool pages)",
                        "l2": "inputs larger than L2: 20 resident 38.5 MB objects, 8 rotating bindings",
                        "copy_kernel": os.environ.get("GR_COPY", "tma8" if args.tma else "ws1") + f", {args.ctas} CTA/SM cap"},
             "gbps": value * N_BYTES / 1e9,
             "host_us_per_request": host_us,
             "latency_us": {"p50": pct(lat, 50), "p99": pct(lat, 99), "samples": len(lat),
                            "what": "one get_into of 38,535,168 B, CUDA events on the consumer stream"},
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": (achieved / peak) if achieved else None, "traffic": traffic,
                          "kernel": "gr_copy (K2')", "peak_source": peak_src,
                          "launches": launches, "avg_launch_us": avg_ns / 1e3,
@@ -374,11 +436,19 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank)
         return
+    # GR_BENCH_SAME_GPU=1 + GR_BENCH_BACKEND=gloo: every rank on GPU 0 (exercises the
+    # N>1 IPC pull path on a 1-GPU box; NCCL refuses two ranks on one GPU)
+    if os.environ.get("GR_BENCH_SAME_GPU") == "1":
+        local_rank = 0
     if world > 1:
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
+        backend = os.environ.get("GR_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
+        else:
+            dist.init_process_group(backend)
     run_gpu(args, rank, world, local_rank)
     if world > 1:
         import torch.distributed as dist

@@ -49,6 +49,7 @@ extern "C" {
 #define GROUTER_MAX_PATHS 8
 #define GROUTER_HOST (-1)          /* location / device of a CPU function  */
 #define GROUTER_NOHINT (-2)        /* put: no placement hint               */
+#define GROUTER_REMOTE (-3)        /* location of an object imported from another process */
 #define GROUTER_UNLIMITED UINT64_MAX
 
 /* flags for grouter_config.flags */
@@ -187,6 +188,44 @@ grouter_status grouter_release(grouter_ctx *ctx, const grouter_fn *fn, grouter_o
 /* Frees an object (L260); later gets fail with ENOENT.  Pages are reclaimed
  * once zero-copy pins drain.  EBUSY if unsealed. */
 grouter_status grouter_free(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid);
+
+/* ------------------------------------------------------------ cross-process handoff
+ * L167 (1) / L269: GROUTER maps stored data into the address space of the
+ * consuming function through CUDA IPC.  Pool pages are CUDA VMM allocations
+ * exported as POSIX file descriptors; the descriptor below is plain bytes
+ * that any channel can carry; the file descriptors themselves travel over
+ * an abstract Unix socket served by the exporting context. */
+#define GROUTER_IPC_MAX_SEGS 8
+typedef struct {
+  uint32_t magic, version;
+  int32_t pid;                    /* exporting process                          */
+  uint32_t ctx_id;                /* exporting context (socket name)            */
+  uint8_t gpu_uuid[16];           /* GPU holding the bytes                      */
+  uint32_t workflow_id;           /* owner workflow: importer must match (L394) */
+  int32_t logical;                /* exporter's logical GPU                     */
+  grouter_oid oid;                /* exporter-side object id                    */
+  uint64_t n;                     /* bytes                                      */
+  uint64_t exporter_ptr;          /* object address in the exporter (release)   */
+  uint64_t first_offset;          /* object start within the first segment      */
+  uint32_t n_segs, pad;
+  uint64_t seg_off[GROUTER_IPC_MAX_SEGS];   /* segment offsets in the exporter's pool */
+  uint64_t seg_size[GROUTER_IPC_MAX_SEGS];
+} grouter_ipc_desc;
+
+/* Exports a sealed object resident on a GPU for use by another process.
+ * Blocks until the object's bytes are in place, pins the object like a
+ * zero-copy lease and consumes one consumer; the exporter drops the pin
+ * with grouter_release(fn, oid, (void*)desc.exporter_ptr, stream). */
+grouter_status grouter_export_ipc(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid,
+                                  grouter_ipc_desc *desc);
+/* Imports an exported object as a local, sealed, read-only object owned by
+ * fn's workflow (EPERM if desc's workflow differs).  No bytes move: gets on
+ * the GPU that holds the bytes alias them (zero copy); gets on another GPU
+ * copy them with the SM copy kernel on the consumer GPU reading over
+ * NVLink.  Its location is GROUTER_REMOTE; grouter_free (or `consumers`)
+ * unmaps it.  consumers as in grouter_put. */
+grouter_status grouter_import_ipc(grouter_ctx *ctx, const grouter_fn *fn, const grouter_ipc_desc *desc,
+                                  uint32_t consumers, grouter_oid *out);
 
 /* ------------------------------------------------------------ control */
 /* Tenant (workflow) bandwidth weight, >= 1 (north star; L193-L197). */

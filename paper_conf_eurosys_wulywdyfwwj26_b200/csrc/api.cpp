@@ -7,6 +7,8 @@
 // L248-L262 (elastic pool, 50% cap, queue-aware migration, prompt removal),
 // L394 (authentication by function id + workflow id).  Readings R14-R24 in
 // DESIGN.md.  Byte movement is delegated to engine.cpp.
+#include <unistd.h>
+
 #include <algorithm>
 #include <cstring>
 
@@ -64,6 +66,13 @@ void release_storage_if_dead(grouter_ctx *c, Obj &o) {
   const uint64_t ch = charge(o.n);
   Fences f = std::move(o.readers);
   for (auto &w : o.ready) f.push_back(w);
+  if (o.loc == GROUTER_REMOTE) {  // imported mapping: unmap once local reads are done
+    if (!c->replay) pump(c, true);
+    host_wait(f);
+    if (o.remote) ipc_unmap(*o.remote);
+    c->objects.erase(o.oid);
+    return;
+  }
   if (o.loc == GROUTER_HOST) {
     c->host_used -= ch;
     host_free(c, o.ptr, ch, std::move(f));
@@ -187,6 +196,7 @@ void order_after(grouter_ctx *c, cudaStream_t s, const Fences &f) {
 }
 
 int server_kind_for(int src, int dst) {
+  if (src == GROUTER_REMOTE) return SK_COPY;
   if (src == GROUTER_HOST) return SK_H2D;
   if (dst == GROUTER_HOST) return SK_D2H;
   return SK_COPY;
@@ -203,7 +213,8 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
                        cudaStream_t caller = nullptr, int caller_logical = -1, bool caller_dep = false,
                        bool *direct = nullptr) {
   std::vector<grouter_chunk> plan;
-  c->planner.plan(src_loc, dst_loc, n, plan);
+  if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
+  else c->planner.plan(src_loc, dst_loc, n, plan);
   XferRef x = new_xfer(c, tenant, plan);
   x->deps = std::move(deps);
   x->pageable_src = pageable_src;
@@ -211,7 +222,7 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   enqueue_plan(c, x, plan, kind, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, dst_loc);
   if (direct) *direct = false;
   if (caller && kind == SK_COPY && direct &&
-      try_direct(c, x, src_loc, caller, c->dev[caller_logical].phys)) {
+      try_direct(c, x, src_loc == GROUTER_REMOTE ? dst_loc : src_loc, caller, c->dev[caller_logical].phys)) {
     *direct = true;
     return x;
   }
@@ -311,7 +322,10 @@ grouter_status grouter_finalize(grouter_ctx *c) {
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
   if (!c->plan_only) {
     API_TRY
+    ipc_shutdown(c);
     engine_shutdown(c);
+    for (auto &kv : c->objects)
+      if (kv.second.remote) ipc_unmap(*kv.second.remote);
     API_CATCH(c)
   }
   delete c;
@@ -451,9 +465,11 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
   const uint64_t n = o.n;
   Fences wait;
   const void *result = nullptr;
+  const bool remote = o.loc == GROUTER_REMOTE;
+  if (remote && d == GROUTER_HOST) return fail(GROUTER_EINVAL, "get: CPU get of an imported object");
   if (n == 0) {
     result = nullptr;
-  } else if (o.loc == d) {  // zero copy: share the address (L167 (1))
+  } else if (o.loc == d || (remote && o.remote->phys == c->dev[d].phys)) {  // zero copy (L167 (1))
     o.pins++;
     result = o.ptr;
     wait = o.ready;
@@ -498,6 +514,8 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
   const uint64_t n = o.n;
   if (dst_cap < n || (!dst && n)) return fail(GROUTER_EINVAL, "get_into: dst too small");
   const int d = fn->device;
+  if (o.loc == GROUTER_REMOTE && d == GROUTER_HOST)
+    return fail(GROUTER_EINVAL, "get_into: CPU get of an imported object");
   const bool blocking = !stream || d == GROUTER_HOST;
   Fences wait;
   if (n) {
@@ -577,6 +595,91 @@ grouter_status grouter_free(grouter_ctx *c, const grouter_fn *fn, grouter_oid oi
   if (o->state == OBJ_OPEN) return fail(GROUTER_EBUSY, "free: object not sealed");
   o->state = OBJ_FREED;
   release_storage_if_dead(c, *o);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+// ------------------------------------------------------------------ cross-process handoff
+grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid,
+                                  grouter_ipc_desc *desc) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (!desc) return fail(GROUTER_EINVAL, "export_ipc: null desc");
+  Obj *op = nullptr;
+  grouter_status st = get_common(c, fn, oid, &op);
+  if (st) return st;
+  Obj &o = *op;
+  if (o.loc < 0) return fail(GROUTER_EINVAL, "export_ipc: object is not in a GPU pool");
+  if (c->replay) flush_all(c);
+  else pump(c, true);
+  host_wait(o.ready);  // the importer sees finished bytes
+  ipc_serve_start(c);
+  grouter_ipc_desc d{};
+  d.magic = 0x47524f55u;
+  d.version = 1;
+  d.pid = (int32_t)getpid();
+  d.ctx_id = c->ctx_id;
+  cudaDeviceProp prop;
+  GR_CUDA(cudaGetDeviceProperties(&prop, c->dev[o.loc].phys));
+  std::memcpy(d.gpu_uuid, &prop.uuid, 16);
+  d.workflow_id = o.wf;
+  d.logical = o.loc;
+  d.oid = oid;
+  d.n = o.n;
+  d.exporter_ptr = (uint64_t)(uintptr_t)o.ptr;
+  const DevicePool &P = c->dev[o.loc].pool;
+  const uint64_t lo = (uint64_t)(o.ptr - (uint8_t *)P.base), hi = lo + std::max<uint64_t>(o.n, 1);
+  for (auto &sg : P.segs) {
+    if (sg.off + sg.size <= lo || sg.off >= hi) continue;
+    if (d.n_segs == GROUTER_IPC_MAX_SEGS) return fail(GROUTER_EINVAL, "export_ipc: object spans too many segments");
+    if (d.n_segs == 0) d.first_offset = lo - sg.off;
+    d.seg_off[d.n_segs] = sg.off;
+    d.seg_size[d.n_segs] = sg.size;
+    d.n_segs++;
+  }
+  o.pins++;  // like a zero-copy lease: released with grouter_release(ptr = exporter_ptr)
+  o.last_access = c->seq;
+  *desc = d;
+  consume(c, o);
+  return GROUTER_OK;
+  API_CATCH(c)
+}
+
+grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const grouter_ipc_desc *d,
+                                  uint32_t consumers, grouter_oid *out) {
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  API_TRY
+  if (!fn || !d || !out || d->magic != 0x47524f55u || d->version != 1 || d->n_segs > GROUTER_IPC_MAX_SEGS)
+    return fail(GROUTER_EINVAL, "import_ipc: bad descriptor");
+  if (!valid_loc(c, fn->device)) return fail(GROUTER_EINVAL, "import_ipc: bad function");
+  if (d->workflow_id != fn->workflow_id) return fail(GROUTER_EPERM, "import_ipc: workflow mismatch (L394)");
+  // which local GPU (if any) holds the bytes
+  int local_phys = -1;
+  for (auto &kv : c->phys) {
+    cudaDeviceProp prop;
+    GR_CUDA(cudaGetDeviceProperties(&prop, kv.first));
+    if (std::memcmp(&prop.uuid, d->gpu_uuid, 16) == 0) local_phys = kv.first;
+  }
+  std::shared_ptr<RemoteMap> map;
+  if (d->n) map = ipc_map(c, *d, local_phys);
+  else map = std::make_shared<RemoteMap>();
+  Obj o;
+  o.oid = c->next_oid++;
+  o.wf = fn->workflow_id;
+  o.fid = fn->function_id;
+  o.n = d->n;
+  o.loc = GROUTER_REMOTE;
+  o.ptr = d->n ? (uint8_t *)(uintptr_t)(map->va + d->first_offset) : nullptr;
+  o.state = OBJ_SEALED;
+  o.consumers_left = consumers;
+  o.last_access = c->seq;
+  o.remote = map;
+  *out = o.oid;
+  c->objects.emplace(o.oid, std::move(o));
   return GROUTER_OK;
   API_CATCH(c)
 }

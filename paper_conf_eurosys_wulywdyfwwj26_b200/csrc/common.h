@@ -62,6 +62,9 @@ struct Driver {
   CUresult (*memSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc *, size_t);
   CUresult (*memGetAllocationGranularity)(size_t *, const CUmemAllocationProp *,
                                           CUmemAllocationGranularity_flags);
+  CUresult (*memExportToShareableHandle)(void *, CUmemGenericAllocationHandle, CUmemAllocationHandleType,
+                                         unsigned long long);
+  CUresult (*memImportFromShareableHandle)(CUmemGenericAllocationHandle *, void *, CUmemAllocationHandleType);
   CUresult (*streamWaitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
   CUresult (*streamWriteValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 };

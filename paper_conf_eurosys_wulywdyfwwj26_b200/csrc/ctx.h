@@ -127,6 +127,16 @@ struct Server {
 };
 
 // ------------------------------------------------------------------ objects
+// An object imported from another process (grouter_import_ipc): its bytes
+// live in the exporter's pool; this process maps the exporter's segments.
+struct RemoteMap {
+  CUdeviceptr va = 0;
+  uint64_t size = 0;
+  std::vector<CUmemGenericAllocationHandle> handles;
+  std::vector<uint64_t> sizes;
+  int phys = -1;   // local CUDA ordinal holding the bytes, -1 if not visible
+};
+
 enum ObjState { OBJ_OPEN, OBJ_SEALED, OBJ_CONSUMED, OBJ_FREED };
 
 struct Obj {
@@ -143,6 +153,7 @@ struct Obj {
   uint64_t next_use = 0;
   Fences ready;                    // the bytes are in place once these complete
   Fences readers;                  // in-flight library reads of the bytes
+  std::shared_ptr<RemoteMap> remote;  // loc == GROUTER_REMOTE
 };
 
 struct Lease {
@@ -217,6 +228,11 @@ struct grouter_ctx {
   std::condition_variable cv;
   bool stop = false;
   std::atomic<bool> sticky_error{false};
+  // cross-process export (ipc.cpp)
+  uint32_t ctx_id = 0;
+  int ipc_listen = -1;
+  std::thread ipc_thread;
+  std::map<std::pair<int, uint64_t>, int> exported_fds;  // (logical, seg offset) -> fd
 };
 
 namespace gr {
@@ -248,6 +264,11 @@ Waitable signal(grouter_ctx *c, cudaStream_t s, int phys);       // caller strea
 void host_wait(const Fences &f, double timeout_s = 120.0);
 bool grounded(const grouter_ctx *c, const Fences &f);
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst);  // D2H of a victim (unscheduled)
+// ipc.cpp
+void ipc_serve_start(grouter_ctx *c);
+void ipc_shutdown(grouter_ctx *c);
+std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, int local_phys);
+void ipc_unmap(RemoteMap &m);
 // pool.cpp
 uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len);   // may grow the pool
 void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f);

@@ -49,6 +49,8 @@ const Driver &drv() {
       resolve("cuMemUnmap", d.memUnmap);
       resolve("cuMemSetAccess", d.memSetAccess);
       resolve("cuMemGetAllocationGranularity", d.memGetAllocationGranularity);
+      resolve("cuMemExportToShareableHandle", d.memExportToShareableHandle);
+      resolve("cuMemImportFromShareableHandle", d.memImportFromShareableHandle);
       resolve("cuStreamWaitValue32", d.streamWaitValue32);
       resolve("cuStreamWriteValue32", d.streamWriteValue32);
     } catch (const Error &e) {

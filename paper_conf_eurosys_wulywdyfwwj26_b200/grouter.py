@@ -22,6 +22,7 @@ MAX_GPUS = 16
 MAX_PATHS = 8
 HOST = -1
 NOHINT = -2
+REMOTE = -3
 UNLIMITED = (1 << 64) - 1
 
 REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20
@@ -75,6 +76,18 @@ class grouter_stats_t(C.Structure):
     ]
 
 
+IPC_MAX_SEGS = 8
+
+
+class grouter_ipc_desc(C.Structure):
+    _fields_ = [("magic", C.c_uint32), ("version", C.c_uint32), ("pid", C.c_int32),
+                ("ctx_id", C.c_uint32), ("gpu_uuid", C.c_uint8 * 16), ("workflow_id", C.c_uint32),
+                ("logical", C.c_int32), ("oid", C.c_uint64), ("n", C.c_uint64),
+                ("exporter_ptr", C.c_uint64), ("first_offset", C.c_uint64), ("n_segs", C.c_uint32),
+                ("pad", C.c_uint32), ("seg_off", C.c_uint64 * IPC_MAX_SEGS),
+                ("seg_size", C.c_uint64 * IPC_MAX_SEGS)]
+
+
 class grouter_dispatch(C.Structure):
     _fields_ = [("server_kind", C.c_int32), ("server_dev", C.c_int32), ("tenant", C.c_uint32),
                 ("n_chunks", C.c_uint32), ("chunk_ids", C.c_uint64 * 8), ("bytes", C.c_uint64)]
@@ -109,6 +122,9 @@ SIGNATURES = {
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_dispatch_log": (_ST, [_CTX, C.POINTER(grouter_dispatch), _U64, C.POINTER(_U64)]),
+    "grouter_export_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, C.POINTER(grouter_ipc_desc)]),
+    "grouter_import_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), C.POINTER(grouter_ipc_desc), _U32,
+                                 C.POINTER(_U64)]),
     "grouter_sched_new": (_ST, [_U32, C.POINTER(_P)]),
     "grouter_sched_set_weight": (_ST, [_P, _U32, _U32]),
     "grouter_sched_enqueue": (_ST, [_P, _U32, _U64, _U64]),
@@ -263,6 +279,22 @@ class Ctx:
 
     def free(self, f, oid: int):
         return self.lib.grouter_free(self.h, C.byref(f), oid)
+
+    # cross-process handoff
+    def export_ipc(self, f, oid):
+        d = grouter_ipc_desc()
+        st = self.lib.grouter_export_ipc(self.h, C.byref(f), oid, C.byref(d))
+        return st, bytes(d)
+
+    def import_ipc(self, f, desc: bytes, consumers=0):
+        d = grouter_ipc_desc.from_buffer_copy(desc)
+        oid = C.c_uint64(0)
+        st = self.lib.grouter_import_ipc(self.h, C.byref(f), C.byref(d), consumers, C.byref(oid))
+        return st, oid.value
+
+    @staticmethod
+    def desc_exporter_ptr(desc: bytes) -> int:
+        return grouter_ipc_desc.from_buffer_copy(desc).exporter_ptr
 
     # control
     def set_tenant_weight(self, wf, w):
