@@ -665,8 +665,21 @@ grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const gr
     if (std::memcmp(&prop.uuid, d->gpu_uuid, 16) == 0) local_phys = kv.first;
   }
   std::shared_ptr<RemoteMap> map;
-  if (d->n) map = ipc_map(c, *d, local_phys);
-  else map = std::make_shared<RemoteMap>();
+  if (d->n) {
+    // the round trip to the exporter runs WITHOUT our lock: two contexts may
+    // import from each other at once, and each server thread needs its
+    // context's lock to look its segments up
+    g.lk.unlock();
+    try {
+      map = ipc_map(c, *d, local_phys);
+    } catch (...) {
+      g.lk.lock();
+      throw;
+    }
+    g.lk.lock();
+  } else {
+    map = std::make_shared<RemoteMap>();
+  }
   Obj o;
   o.oid = c->next_oid++;
   o.wf = fn->workflow_id;
