@@ -151,6 +151,17 @@ typedef struct {
 
 /* ------------------------------------------------------------ lifecycle */
 void grouter_config_default(grouter_config *cfg);
+/* Calibration probe (the topology matrix of Alg. 1,
+ * and the PCIe-switch sharing of L131/L178, measured on this box): for the
+ * n_gpus CUDA ordinals in cfg->device_map, measures solo pinned H2D
+ * bandwidth (h2d_Bps, from `probe_bytes` copies), per-chunk copy-engine cost
+ * (h2d_alpha_ps, from back-to-back 4 KiB copies), first-chunk latency
+ * (h2d_phi_ps), concurrent H2D sums for every pair (h2d_pair_Bps; uplink
+ * groups are then derived by grouter_init), peer access (p2p) and a D2D
+ * peer copy (nvl_Bps, if any pair has P2P).  Writes into *cfg (sets
+ * uplink_group to -1 so groups come from the pair matrix).  Blocking; uses
+ * the GPUs exclusively for a few seconds. */
+grouter_status grouter_probe(grouter_config *cfg, uint64_t probe_bytes);
 /* Creates the context: per-GPU pools (VMM reservations), host store, streams,
  * route sets R(d) (precomputed, L271).  cfg is copied. */
 grouter_status grouter_init(const grouter_config *cfg, grouter_ctx **out);

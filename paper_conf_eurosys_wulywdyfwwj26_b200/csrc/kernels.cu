@@ -359,6 +359,18 @@ __global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ K
           st_stream(dv + j * 32 + lane, v[u][j]);
           count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
         }
+      } else if (((srcs[u] | dsts[u]) & 15) == 0) {  // aligned partial unit: vectors + byte tail
+        const uint32_t nv = lens[u] >> 4;
+        const int4 *sv = reinterpret_cast<const int4 *>(sp);
+        int4 *dv = reinterpret_cast<int4 *>(d);
+        for (uint32_t i = lane; i < nv; i += 32) {
+          st_stream(dv + i, ld_stream(sv + i));
+          count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
+        }
+        for (uint32_t i = (nv << 4) + lane; i < lens[u]; i += 32) {
+          d[i] = sp[i];
+          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
+        }
       } else {
         for (uint32_t i = lane; i < lens[u]; i += 32) {
           d[i] = sp[i];
@@ -419,6 +431,18 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wd(const __grid_constant__ K
         for (int j = 0; j < 8; ++j) {
           st_stream(dv + j * 32 + lane, v[u][j]);
           count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
+        }
+      } else if (((srcs[u] | dsts[u]) & 15) == 0) {  // aligned partial unit: vectors + byte tail
+        const uint32_t nv = lens[u] >> 4;
+        const int4 *sv = reinterpret_cast<const int4 *>(sp);
+        int4 *dv = reinterpret_cast<int4 *>(d);
+        for (uint32_t i = lane; i < nv; i += 32) {
+          st_stream(dv + i, ld_stream(sv + i));
+          count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
+        }
+        for (uint32_t i = (nv << 4) + lane; i < lens[u]; i += 32) {
+          d[i] = sp[i];
+          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
         }
       } else {
         for (uint32_t i = lane; i < lens[u]; i += 32) {
@@ -695,8 +719,13 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   bool aligned = true;
   for (uint32_t i = 0; i < p.n_chunks; ++i)
     aligned &= ((p.chunk[i].src | p.chunk[i].dst | p.chunk[i].bytes) & 15) == 0;
+  uint64_t total = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
   int v = variant_from_env();
-  if (v < 0) v = tma ? 3 : 5;  // default: warp-strided LD/ST; GROUTER_COPY_TMA: 8-stage bulk ring
+  // default: the 8-stage TMA bulk ring for large aligned rounds (best at
+  // >= 64 MiB), the warp-strided LD/ST engine otherwise; GROUTER_COPY_TMA
+  // forces the bulk ring for every aligned round
+  if (v < 0) v = (tma || (aligned && total >= (64ull << 20))) ? 3 : 5;
   if (((v >= 2 && v <= 4) || v >= 10) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
   if (p.n_chunks <= (uint32_t)SmallParams::kChunks && p.n_pub <= (uint32_t)SmallParams::kPubs) {
     SmallParams q;

@@ -101,6 +101,7 @@ _CTX = C.c_void_p
 # name -> (restype, argtypes); every symbol declared in include/*.h
 SIGNATURES = {
     "grouter_config_default": (None, [C.POINTER(grouter_config)]),
+    "grouter_probe": (_ST, [C.POINTER(grouter_config), _U64]),
     "grouter_init": (_ST, [C.POINTER(grouter_config), C.POINTER(_CTX)]),
     "grouter_finalize": (_ST, [_CTX]),
     "grouter_put": (_ST, [_CTX, C.POINTER(grouter_fn), _P, _U64, _I32, _U32, _P, C.POINTER(_U64)]),
@@ -215,6 +216,26 @@ def config_from_calib(calib: dict | None = None, **kw) -> grouter_config:
     for k, v in kw.items():
         setattr(cfg, k, v)
     return cfg
+
+
+def probe(devices, probe_bytes: int = 256 << 20) -> dict:
+    """Runs grouter_probe on CUDA ordinals `devices`; returns a calibration
+    dict in synth/calib.py format (device_map = devices)."""
+    lib = load()
+    cfg = grouter_config()
+    lib.grouter_config_default(C.byref(cfg))
+    cfg.n_gpus = len(devices)
+    for i, d in enumerate(devices):
+        cfg.device_map[i] = d
+    check(lib.grouter_probe(C.byref(cfg), probe_bytes), "grouter_probe")
+    n = len(devices)
+    return {"name": "probed", "n_gpus": n, "device_map": list(devices), "nvl_Bps": cfg.nvl_Bps,
+            "h2d_Bps": [cfg.h2d_Bps[i] for i in range(n)],
+            "h2d_alpha_ps": [cfg.h2d_alpha_ps[i] for i in range(n)],
+            "h2d_phi_ps": [cfg.h2d_phi_ps[i] for i in range(n)],
+            "relay_phi_ps": cfg.relay_phi_ps,
+            "h2d_pair_Bps": [[cfg.h2d_pair_Bps[i][j] for j in range(n)] for i in range(n)],
+            "p2p": [[cfg.p2p[i][j] for j in range(n)] for i in range(n)]}
 
 
 def fn(wf: int, fid: int, dev: int) -> grouter_fn:
