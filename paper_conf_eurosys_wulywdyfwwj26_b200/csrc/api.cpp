@@ -171,27 +171,43 @@ bool is_pageable(const void *p) {
   return a.type == cudaMemoryTypeUnregistered;
 }
 
-// Blocking completion for host callers: in replay mode the call flushes
-// (R31), otherwise everything queued is dispatched so the wait
-// cannot depend on the daemon (we hold the lock).
-void block_on(grouter_ctx *c, const Fences &f) {
-  if (c->replay) flush_all(c);
-  else pump(c, true);
+// Blocking completion for host callers.  Replay mode: the call flushes
+// (R31).  Real-time: the transfer competes in the servers'
+// schedulers like any other (no forced dispatch); the context lock is
+// dropped while the caller polls its completion words, so the daemon and
+// other callers keep running.  Nothing touches context state afterwards.
+void block_on(grouter_ctx *c, Guard &g, const Fences &f) {
+  if (c->replay) {
+    flush_all(c);
+    host_wait(f);
+    return;
+  }
+  pump(c, false);
+  c->cv.notify_one();
+  g.lk.unlock();
   host_wait(f);
 }
 
 // Stream-ordered completion for device callers: work enqueued on `s` after
-// the call sees the bytes.  In real-time mode everything the fences depend
-// on is submitted first, so the caller's wait is enqueued now; in replay
-// mode waits on unsubmitted transfers are attached to them and enqueued at
-// grouter_flush() (R31).
-void order_after(grouter_ctx *c, cudaStream_t s, const Fences &f) {
-  if (!c->replay)
-    for (auto &w : f)
-      if (!is_submitted(w)) {
-        pump(c, true);
-        break;
-      }
+// the call sees the bytes.  A wait may only be enqueued once its producer
+// is submitted, so in real-time mode the caller blocks (lock released,
+// condition variable) until the servers have submitted the transfer --
+// backpressure, not a forced dispatch that would bypass the tenant
+// scheduler.  Replay mode: waits on unsubmitted transfers are attached to
+// them and enqueued at grouter_flush() (R31).
+void order_after(grouter_ctx *c, Guard &g, cudaStream_t s, const Fences &f) {
+  if (!c->replay) {
+    auto all_submitted = [&] {
+      for (auto &w : f)
+        if (!is_submitted(w)) return false;
+      return true;
+    };
+    if (!all_submitted()) {
+      pump(c, false);
+      c->cv.notify_one();
+      c->submit_cv.wait(g.lk, all_submitted);
+    }
+  }
   caller_wait(c, s, f);
 }
 
@@ -373,12 +389,12 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
                                  &direct);
       done_fences(x, done);
       o.ready = done;
-      if (!blocking && !direct) order_after(c, (cudaStream_t)stream, done);
+      if (!blocking && !direct) order_after(c, g, (cudaStream_t)stream, done);
     }
   }
   *out = o.oid;
   c->objects.emplace(o.oid, std::move(o));
-  if (blocking && (c->replay || !done.empty())) block_on(c, done);
+  if (blocking && (c->replay || !done.empty())) block_on(c, g, done);
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -493,8 +509,8 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
   *ptr = result;
   *n_out = n;
   consume(c, o);  // may release the object's storage (quarantined behind `wait`)
-  if (blocking) block_on(c, wait);
-  else order_after(c, (cudaStream_t)stream, wait);
+  if (blocking) block_on(c, g, wait);
+  else order_after(c, g, (cudaStream_t)stream, wait);
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -539,8 +555,8 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
   o.last_access = c->seq;
   if (n_out) *n_out = n;
   consume(c, o);
-  if (blocking) block_on(c, wait);
-  else order_after(c, (cudaStream_t)stream, wait);
+  if (blocking) block_on(c, g, wait);
+  else order_after(c, g, (cudaStream_t)stream, wait);
   return GROUTER_OK;
   API_CATCH(c)
 }

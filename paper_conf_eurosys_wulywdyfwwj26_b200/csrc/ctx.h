@@ -226,6 +226,7 @@ struct grouter_ctx {
   // background I/O + dispatch thread (L269, L271)
   std::thread daemon;
   std::condition_variable cv;
+  std::condition_variable submit_cv;                   // a transfer became fully submitted
   bool stop = false;
   std::atomic<bool> sticky_error{false};
   // cross-process export (ipc.cpp)

@@ -329,6 +329,7 @@ static void after_submit(grouter_ctx *c, const std::vector<ChunkItem> &items) {
   for (auto &it : items)
     if (it.x->submitted() && std::find(fin.begin(), fin.end(), it.x) == fin.end()) fin.push_back(it.x);
   for (Xfer *x : fin) c->live.erase(x);
+  if (!fin.empty()) c->submit_cv.notify_all();
 }
 
 // One or more kernel launches for `items` (in order): contiguous chunks are
@@ -780,10 +781,10 @@ void engine_init(grouter_ctx *c) {
   GR_CUDA(cudaHostAlloc((void **)&c->bounce, (size_t)kBounceSlots * c->cfg.chunk_bytes,
                         cudaHostAllocPortable));
   c->bounce_ev.assign(kBounceSlots, nullptr);
-  // pinned host store (+ headroom so page fragmentation never decides a
+  // pinned host store (+ headroom so page fragmentation does not decide a
   // placement that the capacity accounting admitted)
   c->host_cap = c->cfg.host_store_bytes / kPage * kPage;
-  c->host.size = c->host_cap * 2 + (64ull << 20);
+  c->host.size = (c->host_cap + c->host_cap / 4 + (64ull << 20)) / kPage * kPage;
   GR_CUDA(cudaHostAlloc((void **)&c->host.base, c->host.size,
                         cudaHostAllocMapped | cudaHostAllocPortable));
   c->host.heap.give(0, c->host.size / kPage * kPage);

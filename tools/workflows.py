@@ -1,0 +1,175 @@
+"""Workflow-level measurements on one B200.
+
+cfg4  8 tenants (workflows) with weights 1,1,2,2,4,4,8,8 share GPU0's
+      host->GPU engine: each tenant's CPU function loops blocking puts of a
+      38,535,168 B tensor (hint GPU0) for T seconds; per-tenant GB/s and the
+      share error |x_t/sum x - w_t/sum w| / (w_t/sum w) (pass <= 10%), plus a
+      run with all weights 1 (no partitioning) for the Fig. 17 analog: the
+      w=8 tenant's put latency alone vs with the others.
+cfg5  LLM pipeline (Llama-3-8B public shapes): per request stage A allocs 32
+      KV objects of 33,554,432 B + 67,108,864 B hidden states on GPU0, stage
+      B (same GPU) gets them into its own buffers in queue order; pool limit
+      = 10% / 1% of the working set; queue-aware (next_use = queue position)
+      vs LRU (no hints).  Per-request latency p50/p99, spilled bytes, req/s.
+"""
+import json
+import sys
+import threading
+import time
+
+sys.path.insert(0, ".")
+
+import torch  # noqa: E402
+
+from paper_conf_eurosys_wulywdyfwwj26_b200 import _build  # noqa: E402
+from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G  # noqa: E402
+from synth.calib import b200_hgx  # noqa: E402
+
+MiB = 1 << 20
+N1 = 38_535_168
+
+
+def pct(xs, q):
+    xs = sorted(xs)
+    return xs[max(0, min(len(xs) - 1, -(-len(xs) * q // 100) - 1))] if xs else None
+
+
+def mkctx(**kw):
+    c = b200_hgx(1)
+    c["device_map"] = [0]
+    return G.Ctx(G.config_from_calib(c, **kw))
+
+
+def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8)):
+    ctx = mkctx(host_store_bytes=256 * MiB, pool_cap=[G.UNLIMITED])
+    T = len(weights)
+    for t, w in enumerate(weights):
+        ctx.set_tenant_weight(100 + t, w)
+    srcs = [torch.empty(N1, dtype=torch.uint8, pin_memory=True) for _ in range(T)]
+    done = [0] * T
+    lat = [[] for _ in range(T)]
+    stop = [False]
+    start = threading.Barrier(T + 1)
+
+    def worker(t):
+        f = G.fn(100 + t, 1, G.HOST)
+        start.wait()
+        while not stop[0]:
+            t0 = time.perf_counter()
+            st, oid = ctx.put(f, srcs[t].data_ptr(), N1, 0, 0)
+            lat[t].append(time.perf_counter() - t0)
+            if st == G.OK:
+                ctx.free(f, oid)
+                done[t] += 1
+
+    ths = [threading.Thread(target=worker, args=(t,)) for t in range(T)]
+    for th in ths:
+        th.start()
+    start.wait()
+    t0 = time.perf_counter()
+    time.sleep(seconds)
+    stop[0] = True
+    for th in ths:
+        th.join()
+    dt = time.perf_counter() - t0
+    gbps = [d * N1 / dt / 1e9 for d in done]
+    tot, wsum = sum(gbps), sum(weights)
+    err = [abs(g / tot - w / wsum) / (w / wsum) for g, w in zip(gbps, weights)] if tot else []
+    ctx.close()
+    return {"weights": list(weights), "seconds": dt, "puts": done, "GBps": [round(g, 2) for g in gbps],
+            "aggregate_GBps": round(tot, 2), "share_error": [round(e, 3) for e in err],
+            "max_share_error": round(max(err), 3) if err else None,
+            "p50_ms": [round(pct(l, 50) * 1e3, 2) if l else None for l in lat],
+            "p99_ms": [round(pct(l, 99) * 1e3, 2) if l else None for l in lat]}
+
+
+def cfg4_isolation(seconds=2.0):
+    """Fig. 17 analog: latency of a w=8 tenant alone, then next to 7 others
+    with weights (partitioned) and with all weights 1 (unpartitioned)."""
+    alone = cfg4(seconds, weights=(8,))
+    part = cfg4(seconds, weights=(8, 1, 1, 1, 1, 1, 1, 1))
+    flat = cfg4(seconds, weights=(1, 1, 1, 1, 1, 1, 1, 1))
+    return {"alone_p50_ms": alone["p50_ms"][0], "weighted_p50_ms": part["p50_ms"][0],
+            "unweighted_p50_ms": flat["p50_ms"][0], "alone_GBps": alone["GBps"][0],
+            "weighted_GBps": part["GBps"][0], "unweighted_GBps": flat["GBps"][0]}
+
+
+def cfg5(requests=4, limit_frac=0.1, hints=True, layers=32):
+    KV, HID = 33_554_432, 67_108_864
+    page = 2 * MiB
+    charge = lambda x: -(-x // page) * page
+    ws = requests * (layers * charge(KV) + charge(HID))
+    limit = int(ws * limit_frac) // page * page if limit_frac else G.UNLIMITED
+    ctx = mkctx(host_store_bytes=ws + 512 * MiB, pool_cap=[G.UNLIMITED], pool_floor_bytes=64 * MiB)
+    if limit_frac:
+        G.check(ctx.set_pool_limit(0, limit), "limit")
+    s = torch.cuda.Stream()
+    scratch = torch.empty(HID, dtype=torch.uint8, device="cuda")
+    objs = []
+    t_start = time.perf_counter()
+    for r in range(requests):
+        A = G.fn(500 + r, 1, 0)
+        mine = []
+        for nb in [KV] * layers + [HID]:
+            st, buf, oid = ctx.alloc(A, nb, G.NOHINT, 1)
+            if st == G.ENOMEM:
+                # larger than the pool limit: the producer keeps its own output
+                # buffer and puts it by copy -> stored in host memory (R16)
+                G.check(G.test_fill(scratch.data_ptr(), nb, r * 1000 + len(mine), 0, s.cuda_stream))
+                st, oid = ctx.put(A, scratch.data_ptr(), nb, G.NOHINT, 1, s.cuda_stream)
+                G.check(st, "put")
+            else:
+                G.check(st, "alloc")
+                G.check(G.test_fill(buf, nb, oid, 0, s.cuda_stream))
+                G.check(ctx.seal(A, oid, s.cuda_stream))
+            if hints:
+                ctx.set_next_use(oid, r)
+            mine.append((oid, nb))
+        objs.append(mine)
+    dst = torch.empty(HID, dtype=torch.uint8, device="cuda")
+    lat = []
+    for r in range(requests):
+        B = G.fn(500 + r, 2, 0)
+        t0 = time.perf_counter()
+        for oid, nb in objs[r]:
+            st, n = ctx.get_into(B, oid, dst.data_ptr(), nb, s.cuda_stream)
+            G.check(st, "get_into")
+        s.synchronize()
+        lat.append(time.perf_counter() - t0)
+    total = time.perf_counter() - t_start
+    stt = ctx.stats()
+    out = {"requests": requests, "limit_frac": limit_frac, "queue_aware": hints,
+           "working_set_GB": round(ws / 1e9, 3), "pool_limit_GB": round(limit / 1e9, 3) if limit_frac else None,
+           "stageB_p50_ms": round(pct(lat, 50) * 1e3, 2), "stageB_p99_ms": round(pct(lat, 99) * 1e3, 2),
+           "stageB_ms": [round(x * 1e3, 2) for x in lat],
+           "spill_count": stt.spill_count, "spill_GB": round(stt.spill_bytes / 1e9, 3),
+           "req_per_s": round(requests / total, 2)}
+    ctx.close()
+    return out
+
+
+def main():
+    _build.build()
+    G.load()
+    res = {"gpu": torch.cuda.get_device_name(0)}
+    out = sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/workflows.json"
+
+    def save():
+        json.dump(res, open(out, "w"), indent=1)
+    res["cfg4"] = cfg4(3.0)
+    print("cfg4", json.dumps(res["cfg4"]), flush=True)
+    save()
+    res["cfg4_isolation"] = cfg4_isolation(2.0)
+    print("cfg4_isolation", json.dumps(res["cfg4_isolation"]), flush=True)
+    save()
+    res["cfg5"] = []
+    for frac in (None, 0.1, 0.01):
+        for hints in ((True, False) if frac else (True,)):
+            r = cfg5(4, frac, hints)
+            res["cfg5"].append(r)
+            print("cfg5", json.dumps(r), flush=True)
+            save()
+
+
+if __name__ == "__main__":
+    main()
