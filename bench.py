@@ -199,6 +199,36 @@ def run_reference(args, rank):
     print(json.dumps(line), flush=True)
 
 
+def measure_multipath(world, G, nbytes=1 << 30, reps=3):
+    """Probe every GPU (solo/pairwise H2D -> uplink groups, P2P, NVLink), then
+    time a blocking cFn put of `nbytes` from pinned host into GPU0 striped over
+    R(0) vs the direct link only (GROUTER_NO_MULTIPATH)."""
+    import torch
+    devs = [0] * world if os.environ.get("GR_BENCH_SAME_GPU") == "1" else list(range(world))
+    calib = G.probe(devs, 256 << 20)
+    host = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    out = {"probe_h2d_GBps": [round(b / 1e9, 2) for b in calib["h2d_Bps"]],
+           "probe_nvl_GBps": round(calib["nvl_Bps"] / 1e9, 1)}
+    for name, flags in (("direct", G.NO_MULTIPATH), ("striped", 0)):
+        ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, flags=flags,
+                                        pool_cap=[G.UNLIMITED] * world, pool_floor_bytes=64 << 20))
+        st, routes = ctx.route_set(0)
+        f = G.fn(9, 1, G.HOST)
+        ts = []
+        for r in range(reps + 1):
+            t0 = time.perf_counter()
+            st, oid = ctx.put(f, host.data_ptr(), nbytes, 0, 0)
+            G.check(st, "put")
+            dt = time.perf_counter() - t0
+            ctx.free(f, oid)
+            if r:
+                ts.append(dt)
+        out[name] = {"routes": routes, "GBps": round(nbytes / min(ts) / 1e9, 2)}
+        ctx.close()
+    out["speedup"] = round(out["striped"]["GBps"] / out["direct"]["GBps"], 2)
+    return out
+
+
 # ------------------------------------------------------------------ GPU arm
 def run_gpu(args, rank, world, local_rank):
     import torch
@@ -367,6 +397,15 @@ def run_gpu(args, rank, world, local_rank):
         for oid, desc in exports:
             ctx.release(gfn, oid, G.Ctx.desc_exporter_ptr(desc), 0)
 
+    # N > 1: host->GPU striping over the other GPUs' PCIe links (L120, L178), measured by
+    # rank 0 alone on a context spanning every GPU of the node while the others wait
+    multipath = None
+    if world > 1 and not args.no_multipath_probe:
+        barrier()
+        if rank == 0:
+            multipath = measure_multipath(world, G)
+        barrier()
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, done, dt = oracle_rate(4, args.cpu_seconds)
@@ -410,6 +449,8 @@ def run_gpu(args, rank, world, local_rank):
             "gpu_launches": launches,
             "clocks": clocks,
         }
+        if multipath is not None:
+            line["h2d_multipath"] = multipath
         print(json.dumps(line), flush=True)
     ctx.close()
 
@@ -427,6 +468,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--tma", action="store_true")
     ap.add_argument("--ctas", type=int, default=4)
+    ap.add_argument("--no-multipath-probe", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
