@@ -283,7 +283,7 @@ def run_gpu(args, rank, world, local_rank):
     work = list(zip(resident, bptr))
 
     remote = world > 1
-    exports = []
+    exports, imported, ipc_error = [], [], None
     if remote:
         # export every resident object, import the peer's (CUDA VMM IPC, L167/L269)
         for oid in resident:
@@ -292,12 +292,23 @@ def run_gpu(args, rank, world, local_rank):
             exports.append((oid, desc))
         all_descs = exchange([d for _, d in exports], world)
         peer = peer_of(rank, world)
-        imported = []
         for desc in all_descs[peer]:
             st, roid = ctx.import_ipc(gfn, desc)
-            G.check(st, "import_ipc")
+            if st != G.OK:
+                ipc_error = f"import_ipc from rank {peer}: {G.STATUS[st]} ({G.last_error()})"
+                break
             imported.append(roid)
-        work = list(zip(imported, bptr))
+        # every rank must take the same branch: agree on success
+        ok = max_over_ranks(1.0 if ipc_error else 0.0, world, f"cuda:{dev}") == 0.0
+        if ok:
+            work = list(zip(imported, bptr))
+        else:  # measured honestly as local replicas, error reported in the line
+            print(f"[bench] rank {rank}: IPC pull unavailable ({ipc_error}); local replicas",
+                  file=sys.stderr, flush=True)
+            for roid in imported:
+                ctx.free(gfn, roid)
+            imported = []
+            remote = False
 
     def value_step():
         for oid, dst in work:
@@ -389,7 +400,7 @@ def run_gpu(args, rank, world, local_rank):
     e2e_s = time.perf_counter() - h0
     e2e_val = R * e2e_steps * world / max_over_ranks(e2e_s, world, f"cuda:{dev}")
 
-    if remote:   # drop imports and our export pins once every rank is done reading
+    if world > 1:   # drop imports and our export pins once every rank is done reading
         barrier()
         for roid in imported:
             ctx.free(gfn, roid)
@@ -403,7 +414,10 @@ def run_gpu(args, rank, world, local_rank):
     if world > 1 and not args.no_multipath_probe:
         barrier()
         if rank == 0:
-            multipath = measure_multipath(world, G)
+            try:
+                multipath = measure_multipath(world, G)
+            except Exception as e:  # report, never abort the scaling line
+                multipath = {"error": f"{type(e).__name__}: {e}"[:300]}
         barrier()
 
     cpu = None
@@ -451,6 +465,11 @@ def run_gpu(args, rank, world, local_rank):
         }
         if multipath is not None:
             line["h2d_multipath"] = multipath
+        if world > 1 and not remote:
+            line["ipc_pull_error"] = ipc_error or "another rank failed to import"
+            line["config"]["workload"] = WORKLOAD
+            line["config"]["parallelism"] = f"replicas x{world}"
+
         print(json.dumps(line), flush=True)
     ctx.close()
 

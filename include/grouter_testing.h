@@ -37,6 +37,12 @@ grouter_status grouter_test_verify(const void *src, uint64_t n, uint64_t seed, u
 grouter_status grouter_test_copy(void *dst_base, const void *src_base, const grouter_chunk *chunks,
                                  uint32_t n_chunks, uint32_t *counts, int tma, void *stream);
 
+/* Host cost of kernel launches from this library (tuning probe): kind 0 =
+ * empty kernel with an int parameter, 1 = small copy-parameter block, 2 =
+ * large copy-parameter block; n launches of `blocks` x 256 on `stream`;
+ * *us_per_launch = host time per launch call. */
+grouter_status grouter_test_launch_cost(int kind, int n, int blocks, void *stream, double *us_per_launch);
+
 /* Text dump of the context's internal state (servers, objects, leases,
  * pending completion words) for debugging; truncated to cap bytes.  Returns
  * the full length needed in *len (may be NULL). */

@@ -15,6 +15,7 @@
 #include "../../include/grouter.h"
 #include "../../include/grouter_testing.h"
 
+#include <cstdio>
 #include <sstream>
 #include "ctx.h"
 
@@ -228,6 +229,7 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
                        const uint8_t *src, uint8_t *dst, Fences deps, bool pageable_src,
                        cudaStream_t caller = nullptr, int caller_logical = -1, bool caller_dep = false,
                        bool *direct = nullptr) {
+  const uint64_t tst = hprof().on ? now_ns() : 0;
   std::vector<grouter_chunk> plan;
   if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
   else c->planner.plan(src_loc, dst_loc, n, plan);
@@ -236,6 +238,7 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   x->pageable_src = pageable_src;
   const int kind = server_kind_for(src_loc, dst_loc);
   enqueue_plan(c, x, plan, kind, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, dst_loc);
+  if (hprof().on) hprof().t[4] += now_ns() - tst;
   if (direct) *direct = false;
   if (caller && kind == SK_COPY && direct &&
       try_direct(c, x, src_loc == GROUTER_REMOTE ? dst_loc : src_loc, caller, c->dev[caller_logical].phys)) {
@@ -336,6 +339,17 @@ grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
 
 grouter_status grouter_finalize(grouter_ctx *c) {
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  if (hprof().on && hprof().calls) {
+    HostProf &h = hprof();
+    fprintf(stderr, "[grouter host profile] get_into calls %llu: lock+lookup %.2f us, transfer+launch %.2f us, "
+                    "fences+consume %.2f us, ordering %.2f us\n",
+            (unsigned long long)h.calls, h.t[0] / h.calls / 1e3, h.t[1] / h.calls / 1e3,
+            h.t[2] / h.calls / 1e3, h.t[3] / h.calls / 1e3);
+    if (h.t[4] > 0)
+      fprintf(stderr, "[grouter host profile] inside transfer: plan+xfer+enqueue %.2f us, take %.2f us, "
+                      "params %.2f us, launch %.2f us\n",
+              h.t[4] / h.calls / 1e3, h.t[5] / h.calls / 1e3, h.t[6] / h.calls / 1e3, h.t[7] / h.calls / 1e3);
+  }
   if (!c->plan_only) {
     API_TRY
     ipc_shutdown(c);
@@ -499,6 +513,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
                                blocking ? nullptr : (cudaStream_t)stream, d, false, &direct);
     Fences done;
     done_fences(x, done);
+    if (o.readers.size() > 8) prune(o.readers);
     for (auto &w : done) o.readers.push_back(w);
     Lease L{oid, o.wf, d, lease, n, done};
     c->leases[(uintptr_t)lease] = std::move(L);
@@ -518,6 +533,8 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
 grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *dst,
                                 uint64_t dst_cap, void *stream, uint64_t *n_out) {
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  HostProf &hp = hprof();
+  uint64_t t0 = hp.on ? now_ns() : 0, t1 = 0, t2 = 0, t3 = 0;
   Guard g(c);
   c->seq++;
   c->victims.clear();
@@ -534,6 +551,7 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
     return fail(GROUTER_EINVAL, "get_into: CPU get of an imported object");
   const bool blocking = !stream || d == GROUTER_HOST;
   Fences wait;
+  if (hp.on) t1 = t2 = now_ns();
   if (n) {
     if (o.loc == GROUTER_HOST && d == GROUTER_HOST) {
       if (c->replay) flush_all(c);
@@ -546,8 +564,10 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
       bool direct = false;
       XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, (uint8_t *)dst, o.ready,
                                  false, blocking ? nullptr : (cudaStream_t)stream, d, true, &direct);
+      if (hp.on) t2 = now_ns();
       Fences done;
       done_fences(x, done);
+      if (o.readers.size() > 8) prune(o.readers);
       for (auto &w : done) o.readers.push_back(w);
       if (!direct) wait = done;
     }
@@ -555,8 +575,17 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
   o.last_access = c->seq;
   if (n_out) *n_out = n;
   consume(c, o);
+  if (hp.on) t3 = now_ns();
   if (blocking) block_on(c, g, wait);
   else order_after(c, g, (cudaStream_t)stream, wait);
+  if (hp.on) {
+    const uint64_t t4 = now_ns();
+    hp.calls++;
+    hp.t[0] += t1 - t0;  // lock + lookup + checks
+    hp.t[1] += t2 - t1;  // plan + transfer + enqueue + dispatch/launch
+    hp.t[2] += t3 - t2;  // fences + consume
+    hp.t[3] += t4 - t3;  // ordering
+  }
   return GROUTER_OK;
   API_CATCH(c)
 }

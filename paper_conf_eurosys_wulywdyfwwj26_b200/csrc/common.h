@@ -128,4 +128,25 @@ struct Waitable {
 };
 using Fences = std::vector<Waitable>;
 
+// Drops completed fences (keeps long-lived objects' reader lists short).
+inline void prune(Fences &f) {
+  size_t w = 0;
+  for (size_t i = 0; i < f.size(); ++i)
+    if (!f[i].done()) {
+      if (w != i) f[w] = std::move(f[i]);
+      ++w;
+    }
+  f.resize(w);
+}
+
+// GROUTER_HOST_PROFILE=1: per-stage host time of the data-path calls,
+// printed to stderr at grouter_finalize (tuning aid).
+struct HostProf {
+  bool on = false;
+  uint64_t calls = 0;
+  double t[8] = {};
+};
+HostProf &hprof();
+uint64_t now_ns();
+
 }  // namespace gr

@@ -344,6 +344,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
   size_t i = 0;
   std::vector<ChunkItem> part;
   while (i < items.size()) {
+    const uint64_t tparams = hprof().on ? now_ns() : 0;
     p->n_chunks = 0;
     p->n_pub = 0;
     p->scratch = scratch;
@@ -385,8 +386,12 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       }
       GR_CUDA(cudaEventRecord(pr.start, st));
     }
+    HostProf &hp = hprof();
+    uint64_t tl = hp.on ? now_ns() : 0;
+    if (hp.on) hp.t[6] += tl - tparams;
     int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm,
                         (c->cfg.flags & GROUTER_COPY_TMA) != 0, st);
+    if (hp.on) hp.t[7] += now_ns() - tl;
     if (e != 0)
       throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
     if (prof) {
@@ -644,9 +649,12 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
   DeviceGuard g(s.phys);
   std::vector<ChunkItem> items;
   std::vector<char> cut;
+  HostProf &hp = hprof();
   while (has_work(s)) {
+    uint64_t ta = hp.on ? now_ns() : 0;
     refill(c, s, UINT32_MAX, kDirectBytes, kDirectItems);
     take(s, kDirectBytes, items, cut, kDirectItems);
+    if (hp.on) hp.t[5] += now_ns() - ta;
     if (items.empty()) throw Error(GROUTER_ECUDA, "internal: direct launch made no progress");
     if (cut[0]) stream_wait(c, caller, s.phys, x->deps);
     // scratch pair for this launch (the server's own pair belongs to its stream)

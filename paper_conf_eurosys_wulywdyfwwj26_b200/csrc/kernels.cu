@@ -13,6 +13,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <chrono>
 #include <cstdlib>
 #include <string>
 
@@ -801,6 +802,27 @@ static unsigned fill_grid(uint64_t words) {
   uint64_t g = (words + 255) / 256;
   if (g > 148 * 16) g = 148 * 16;
   return (unsigned)(g ? g : 1);
+}
+
+__global__ void gr_empty_kernel(const __grid_constant__ SmallParams p) { (void)p; }
+__global__ void gr_empty_kernel_big(const __grid_constant__ CopyParams p) { (void)p; }
+__global__ void gr_empty_kernel_tiny(int x) { (void)x; }
+
+extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, void *stream, double *us_per_launch) {
+  if (!us_per_launch || n <= 0) return GROUTER_EINVAL;
+  cudaStream_t s = (cudaStream_t)stream;
+  static SmallParams sp;
+  static CopyParams bp;
+  auto t0 = std::chrono::steady_clock::now();
+  for (int i = 0; i < n; ++i) {
+    if (kind == 0) gr_empty_kernel_tiny<<<blocks, 256, 0, s>>>(i);
+    else if (kind == 1) gr_empty_kernel<<<blocks, 256, 0, s>>>(sp);
+    else gr_empty_kernel_big<<<blocks, 256, 0, s>>>(bp);
+  }
+  auto t1 = std::chrono::steady_clock::now();
+  cudaStreamSynchronize(s);
+  *us_per_launch = std::chrono::duration<double, std::micro>(t1 - t0).count() / n;
+  return cudaGetLastError() == cudaSuccess ? GROUTER_OK : GROUTER_ECUDA;
 }
 
 extern "C" grouter_status grouter_test_fill(void *dst, uint64_t n, uint64_t seed, uint64_t offset,

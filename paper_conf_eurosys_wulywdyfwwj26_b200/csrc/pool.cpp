@@ -20,6 +20,22 @@
 
 namespace gr {
 
+// ------------------------------------------------------------------ host profile
+HostProf &hprof() {
+  static HostProf h = [] {
+    HostProf x;
+    const char *e = getenv("GROUTER_HOST_PROFILE");
+    x.on = e && e[0] == '1';
+    return x;
+  }();
+  return h;
+}
+uint64_t now_ns() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
 // ------------------------------------------------------------------ errors
 static thread_local std::string tl_error;
 void set_error(const std::string &msg) { tl_error = msg; }

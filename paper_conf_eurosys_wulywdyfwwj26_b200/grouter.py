@@ -136,6 +136,7 @@ SIGNATURES = {
     "grouter_last_error": (C.c_char_p, []),
     "grouter_test_fill": (_ST, [_P, _U64, _U64, _U64, _P]),
     "grouter_test_verify": (_ST, [_P, _U64, _U64, _U64, _P, C.POINTER(_U64), C.POINTER(_U64)]),
+    "grouter_test_launch_cost": (_ST, [C.c_int, C.c_int, C.c_int, _P, C.POINTER(C.c_double)]),
     "grouter_test_dump": (_ST, [_CTX, C.c_char_p, _U64, C.POINTER(_U64)]),
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
 }
