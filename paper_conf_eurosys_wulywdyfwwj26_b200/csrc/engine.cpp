@@ -343,8 +343,12 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
   const bool prof = (c->cfg.flags & GROUTER_PROFILE) != 0;
   size_t i = 0;
   std::vector<ChunkItem> part;
+  bool local = true;  // every destination in the launching GPU's memory -> GPU-scope fences
+  for (auto &it : items)
+    local &= it.dst_logical >= 0 && c->dev[it.dst_logical].phys == s.phys;
   while (i < items.size()) {
     const uint64_t tparams = hprof().on ? now_ns() : 0;
+    p->flags = local ? kFlagLocalDst : 0;
     p->n_chunks = 0;
     p->n_pub = 0;
     p->scratch = scratch;
@@ -389,11 +393,15 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
     HostProf &hp = hprof();
     uint64_t tl = hp.on ? now_ns() : 0;
     if (hp.on) hp.t[6] += tl - tparams;
+    bool host_pub = false;
     int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm,
-                        (c->cfg.flags & GROUTER_COPY_TMA) != 0, st);
+                        (c->cfg.flags & GROUTER_COPY_TMA) != 0, st, &host_pub);
     if (hp.on) hp.t[7] += now_ns() - tl;
     if (e != 0)
       throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
+    if (host_pub)  // stream order: the writes land after every byte of the launch
+      for (uint32_t k = 0; k < p->n_pub; ++k)
+        GR_CU(drv().streamWriteValue32((CUstream)st, (CUdeviceptr)p->pub[k].word, p->pub[k].value, 0));
     if (prof) {
       GR_CUDA(cudaEventRecord(pr.stop, st));
       c->prof.push_back(pr);

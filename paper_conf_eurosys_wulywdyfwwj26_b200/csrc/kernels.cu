@@ -46,7 +46,11 @@ __device__ __forceinline__ void st_stream(int4 *p, const int4 &v) {
 // its predecessor on the stream drains; it waits here (before touching any
 // memory or its scratch) until the predecessor completed and flushed, and
 // lets its own successor launch once its main loop is done.
-__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait_raw() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+#define pdl_wait() \
+  do {                                   \
+    if (p.flags & kFlagPdl) pdl_wait_raw(); \
+  } while (0)
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 __device__ __forceinline__ void st_release_sys(uint64_t addr, uint32_t v) {
@@ -192,9 +196,13 @@ __device__ __forceinline__ int find_chunk(const KP &p, uint32_t t) {
 // release stores (no partial visibility).
 template <class KP>
 __device__ __forceinline__ void finish_round(const KP &p) {
+  if (p.flags & kFlagNoPublish) return;  // a stream write after the launch publishes
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence_system();
+    // local destinations only need GPU-scope ordering before the counter;
+    // peer (NVLink) destinations need the system-scope fence
+    if (p.flags & kFlagLocalDst) __threadfence();
+    else __threadfence_system();
     unsigned prev = atomicAdd(&p.scratch[1], 1u);
     if (prev == gridDim.x - 1) {
       __threadfence_system();
@@ -525,6 +533,7 @@ static void launch_pdl(void (*kern)(KP), uint64_t grid, int block, int smem, cud
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl ? 1 : 0;
+  if (pdl) const_cast<KP &>(p).flags |= kFlagPdl;
   if (pdl) cudaLaunchKernelEx(&cfg, kern, p);
   else kern<<<cfg.gridDim, cfg.blockDim, cfg.dynamicSmemBytes, s>>>(p);
 }
@@ -697,7 +706,8 @@ static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStre
   }
 }
 
-int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream) {
+int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream, bool *host_publish) {
+  if (host_publish) *host_publish = false;
   if (p.n_chunks == 0) return (int)cudaSuccess;
   static int ctas_env = -1;
   if (ctas_env < 0) {
@@ -728,8 +738,18 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   // forces the bulk ring for every aligned round
   if (v < 0) v = (tma || (aligned && total >= (64ull << 20))) ? 3 : 5;
   if (((v >= 2 && v <= 4) || v >= 10) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
+  // static-assignment engines (ws, gs) need no scratch: their completion can
+  // be published by a stream write after the launch, which costs the GPU
+  // ~2 us less than the in-kernel fence + counter + last-CTA protocol
+  const bool is_static = (v >= 5 && v <= 7) || v >= 10;
+  p.flags &= ~kFlagNoPublish;
+  if (host_publish && is_static && !p.counts) {
+    p.flags |= kFlagNoPublish;
+    *host_publish = true;
+  }
   if (p.n_chunks <= (uint32_t)SmallParams::kChunks && p.n_pub <= (uint32_t)SmallParams::kPubs) {
     SmallParams q;
+    q.flags = p.flags;
     q.n_chunks = p.n_chunks;
     q.n_pub = p.n_pub;
     q.scratch = p.scratch;
@@ -870,6 +890,7 @@ extern "C" grouter_status grouter_test_copy(void *dst_base, const void *src_base
     cudaMemset(scratch[dev], 0, 2 * sizeof(uint32_t));
   }
   CopyParams *p = new CopyParams();
+  p->flags = kFlagLocalDst;  // test copies stay on the current device
   p->n_chunks = n_chunks;
   p->scratch = scratch[dev];
   p->counts = counts;

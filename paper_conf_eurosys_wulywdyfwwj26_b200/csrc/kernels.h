@@ -27,6 +27,10 @@ struct KPublish {
   uint32_t pad;
 };
 
+constexpr uint32_t kFlagPdl = 1;        // launched with programmatic stream serialization
+constexpr uint32_t kFlagLocalDst = 2;   // every destination is in this GPU's memory
+constexpr uint32_t kFlagNoPublish = 4;  // completion written by the host after the launch
+
 // Kernel parameters (passed by value, __grid_constant__).  Two capacities:
 // the large one for rounds with many distinct chunks, a small one (a few
 // hundred bytes -- cheaper to launch) for the common round whose chunks
@@ -36,7 +40,7 @@ struct KParams {
   static constexpr int kChunks = C, kPubs = P;
   uint32_t n_chunks = 0, n_pub = 0;
   uint32_t tile_log2 = 16;
-  uint32_t _pad = 0;
+  uint32_t flags = 0;            // kFlag* below
   uint32_t *scratch = nullptr;   // [0] tile ticket, [1] finished CTAs; zero between launches
   uint32_t *counts = nullptr;    // test only: bytes written per 16 B granule
   uint64_t count_base = 0;
@@ -48,7 +52,12 @@ using CopyParams = KParams<kMaxRoundChunks, kMaxPublish>;   // host-side builder
 using SmallParams = KParams<8, 8>;
 
 // Launch gr_copy on `stream` (current device must own the stream).  grid =
-// min(tiles, sm_count * ctas_per_sm).  Returns cudaError_t as int.
-int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream);
+// min(tiles, sm_count * ctas_per_sm).  Returns cudaError_t as int.  When
+// `host_publish` is non-null and the engine chosen has static work
+// assignment (no ticket scratch to reset), the kernel skips its completion
+// protocol and *host_publish = true: the CALLER must publish p.pub with
+// stream writes right after the launch on the same stream.
+int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream,
+                bool *host_publish = nullptr);
 
 }  // namespace gr
