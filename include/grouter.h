@@ -59,6 +59,9 @@ extern "C" {
 #define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
 #define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
 #define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream */
+#define GROUTER_RESTORE       0x40u/* proactive restore (L260-L262): when pool storage is released
+                                      or a cap is raised, objects migrated away from that GPU come
+                                      back while they fit (R42)                      */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;
@@ -134,6 +137,7 @@ typedef struct {
   uint64_t timed_launches;
   uint64_t timed_ns;                     /* sum of their durations              */
   uint64_t timed_bytes;                  /* sum of the bytes they moved         */
+  uint64_t restore_count, restore_bytes; /* host -> home GPU restores (L260)    */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
@@ -265,6 +269,11 @@ grouter_status grouter_where(grouter_ctx *ctx, grouter_oid oid, int32_t *loc);
 grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
 /* Takes (and clears) the objects spilled since the last call, in order. */
 grouter_status grouter_victims(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
+/* Takes (and clears) the objects proactively restored to a GPU pool since the
+ * last call, in order (GROUTER_RESTORE, R42).
+ * Like grouter_victims the list is also reset at the start of every data-path
+ * call, so it reports the restores of the latest call. */
+grouter_status grouter_restored(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
 /* Takes (and clears) up to cap dispatch records, oldest first. */
 grouter_status grouter_dispatch_log(grouter_ctx *ctx, grouter_dispatch *out, uint64_t cap,
                                     uint64_t *n_out);

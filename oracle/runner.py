@@ -27,9 +27,9 @@ def digest(b: np.ndarray) -> str:
 
 
 def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
-        multipath: bool = True, keep_bytes: bool = False) -> dict:
+        multipath: bool = True, keep_bytes: bool = False, restore: bool = False) -> dict:
     orc = Oracle(calib, host_store_bytes=host_store_bytes, pool_cap=pool_cap,
-                 multipath=multipath)
+                 multipath=multipath, restore=restore)
     recs = []
     seed_of = {}          # oid -> payload seed
     for i, op in enumerate(ops):
@@ -106,12 +106,13 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
         if st == 0 and k in ("put", "get", "get_into") and op["fn"]["dev"] == HOST:
             # a CPU caller blocks until its bytes are in place; in replay mode
             # that dispatches everything queued (R31)
-            victims = list(orc.victims)
+            victims, restored = list(orc.victims), list(orc.restored)
             _, fl = orc.flush()
-            orc.victims = victims
+            orc.victims, orc.restored = victims, restored
             rec["dispatched"] = fl["dispatched"]
         rec["status"] = STATUS[st]
         rec["victims"] = list(orc.victims)
+        rec["restored"] = list(orc.restored)
         rec["used"] = list(orc.used)
         rec["host_used"] = orc.host_used
         if oid:

@@ -60,6 +60,39 @@ Obj *lookup_live(grouter_ctx *c, grouter_oid oid) {
   return &it->second;
 }
 
+// Proactive restore (L260-L262, R42): once storage on GPU d is
+// released (or its cap raised), objects migrated away from d come back while
+// they fit under the cap -- objects with a next-use hint first, queue head
+// first; then most recently used; then lower oid.  Stops at the first misfit.
+void restore(grouter_ctx *c, int d) {
+  if (!c->restore_on || d < 0) return;
+  std::vector<Obj *> v;
+  for (auto &kv : c->objects) {
+    Obj &o = kv.second;
+    if (o.loc == GROUTER_HOST && o.home == d && o.state == OBJ_SEALED && o.pins == 0 && o.n > 0)
+      v.push_back(&o);
+  }
+  std::sort(v.begin(), v.end(), [](const Obj *a, const Obj *b) {
+    if (a->has_next_use != b->has_next_use) return a->has_next_use;
+    if (a->has_next_use && a->next_use != b->next_use) return a->next_use < b->next_use;
+    if (a->last_access != b->last_access) return a->last_access > b->last_access;
+    return a->oid < b->oid;
+  });
+  LogicalDev &D = c->dev[d];
+  for (Obj *o : v) {
+    const uint64_t ch = charge(o->n);
+    if (D.cap != GROUTER_UNLIMITED && D.used + ch > D.cap) break;
+    uint8_t *p = dev_alloc(c, d, ch);
+    restore_copy(c, *o, d, p);   // frees the host pages behind the copy
+    D.used += ch;
+    c->host_used -= ch;
+    o->loc = d;
+    o->ptr = p;
+    o->home = -1;
+    c->restored.push_back(o->oid);
+  }
+}
+
 // Storage of a consumed/freed object goes back to its pool once no zero-copy
 // lease pins it ("promptly removes intermediate data", L260).
 void release_storage_if_dead(grouter_ctx *c, Obj &o) {
@@ -78,8 +111,12 @@ void release_storage_if_dead(grouter_ctx *c, Obj &o) {
     c->host_used -= ch;
     host_free(c, o.ptr, ch, std::move(f));
   } else {
-    c->dev[o.loc].used -= ch;
-    dev_free(c, o.loc, o.ptr, ch, std::move(f));
+    const int d = o.loc;
+    c->dev[d].used -= ch;
+    dev_free(c, d, o.ptr, ch, std::move(f));
+    c->objects.erase(o.oid);
+    restore(c, d);
+    return;
   }
   c->objects.erase(o.oid);
 }
@@ -115,6 +152,7 @@ void spill(grouter_ctx *c, Obj &o) {
   uint8_t *h = host_alloc(c, ch);
   const int d = o.loc;
   spill_copy(c, o, h);            // D2H + device pages to quarantine
+  o.home = d;
   o.loc = GROUTER_HOST;
   o.ptr = h;
   c->dev[d].used -= ch;
@@ -311,6 +349,7 @@ grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
   auto *c = new grouter_ctx();
   c->cfg = cfg;
   c->replay = (cfg.flags & GROUTER_REPLAY) != 0;
+  c->restore_on = (cfg.flags & GROUTER_RESTORE) != 0;
   c->plan_only = (cfg.flags & GROUTER_PLAN_ONLY) != 0;
   c->planner.build(cfg);
   c->dev.resize(cfg.n_gpus);
@@ -369,6 +408,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
   Guard g(c);
   c->seq++;
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!check_ready(c)) return GROUTER_ECUDA;
   if (!fn || !out || !valid_loc(c, fn->device) ||
@@ -419,6 +459,7 @@ grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, i
   Guard g(c);
   c->seq++;
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!check_ready(c)) return GROUTER_ECUDA;
   if (!fn || !buf || !out || !valid_loc(c, fn->device) ||
@@ -451,6 +492,7 @@ grouter_status grouter_seal(grouter_ctx *c, const grouter_fn *fn, grouter_oid oi
   Guard g(c);
   c->seq++;
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!fn) return fail(GROUTER_EINVAL, "seal: null fn");
   auto it = c->objects.find(oid);
@@ -483,6 +525,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
   Guard g(c);
   c->seq++;
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!check_ready(c)) return GROUTER_ECUDA;
   if (!ptr || !n_out) return fail(GROUTER_EINVAL, "get: null output");
@@ -538,6 +581,7 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
   Guard g(c);
   c->seq++;
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!check_ready(c)) return GROUTER_ECUDA;
   Obj *op = nullptr;
@@ -596,6 +640,7 @@ grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!fn || !ptr) return fail(GROUTER_EINVAL, "release: bad argument");
   const bool dev_stream = stream && fn->device != GROUTER_HOST && valid_gpu(c, fn->device);
@@ -619,11 +664,14 @@ grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid
   if (L.dev == GROUTER_HOST) {
     c->host_used -= ch;
     host_free(c, L.ptr, ch, std::move(f));
+    c->leases.erase(lt);
   } else {
-    c->dev[L.dev].used -= ch;
-    dev_free(c, L.dev, L.ptr, ch, std::move(f));
+    const int d = L.dev;
+    c->dev[d].used -= ch;
+    dev_free(c, d, L.ptr, ch, std::move(f));
+    c->leases.erase(lt);
+    restore(c, d);
   }
-  c->leases.erase(lt);
   return GROUTER_OK;
   API_CATCH(c)
 }
@@ -632,6 +680,7 @@ grouter_status grouter_free(grouter_ctx *c, const grouter_fn *fn, grouter_oid oi
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!fn) return fail(GROUTER_EINVAL, "free: null fn");
   Obj *o = lookup_live(c, oid);
@@ -650,6 +699,7 @@ grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!desc) return fail(GROUTER_EINVAL, "export_ipc: null desc");
   Obj *op = nullptr;
@@ -697,6 +747,7 @@ grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const gr
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!fn || !d || !out || d->magic != 0x47524f55u || d->version != 1 || d->n_segs > GROUTER_IPC_MAX_SEGS)
     return fail(GROUTER_EINVAL, "import_ipc: bad descriptor");
@@ -747,6 +798,7 @@ grouter_status grouter_set_tenant_weight(grouter_ctx *c, uint32_t wf, uint32_t w
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   if (w < 1) return fail(GROUTER_EINVAL, "weight must be >= 1");
   c->weights[wf] = w;
   return GROUTER_OK;
@@ -756,6 +808,7 @@ grouter_status grouter_set_next_use(grouter_ctx *c, grouter_oid oid, uint64_t po
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   Obj *o = lookup_live(c, oid);
   if (!o) return fail(GROUTER_ENOENT, "set_next_use: unknown oid");
   o->has_next_use = true;
@@ -767,6 +820,7 @@ grouter_status grouter_set_pool_limit(grouter_ctx *c, int32_t d, uint64_t bytes)
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (!valid_gpu(c, d)) return fail(GROUTER_EINVAL, "set_pool_limit: bad device");
   LogicalDev &D = c->dev[d];
@@ -777,6 +831,7 @@ grouter_status grouter_set_pool_limit(grouter_ctx *c, int32_t d, uint64_t bytes)
       if (c->host_used + charge(o->n) > c->host_cap) break;
       spill(c, *o);
     }
+  if (bytes == GROUTER_UNLIMITED || D.used <= D.cap) restore(c, d);
   return (bytes == GROUTER_UNLIMITED || D.used <= D.cap) ? GROUTER_OK
                                                          : fail(GROUTER_ENOMEM, "pool above cap");
   API_CATCH(c)
@@ -786,6 +841,7 @@ grouter_status grouter_flush(grouter_ctx *c) {
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
+  c->restored.clear();
   API_TRY
   if (c->replay) flush_all(c);
   else pump(c, true);
@@ -857,6 +913,17 @@ grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
   }
   out->host_used = c->host_used;
   out->host_cap = c->host_cap;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_restored(grouter_ctx *c, grouter_oid *out, uint64_t cap, uint64_t *n_out) {
+  if (!c || !n_out) return fail(GROUTER_EINVAL, "restored: bad argument");
+  Guard g(c);
+  *n_out = c->restored.size();
+  if (c->restored.size() > cap || (!out && !c->restored.empty()))
+    return fail(GROUTER_EINVAL, "restored: cap too small");
+  for (size_t i = 0; i < c->restored.size(); ++i) out[i] = c->restored[i];
+  c->restored.clear();
   return GROUTER_OK;
 }
 

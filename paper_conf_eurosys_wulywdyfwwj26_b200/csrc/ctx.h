@@ -151,6 +151,7 @@ struct Obj {
   uint64_t last_access = 0;
   bool has_next_use = false;
   uint64_t next_use = 0;
+  int home = -1;                   // GPU it was migrated away from (proactive restore)
   Fences ready;                    // the bytes are in place once these complete
   Fences readers;                  // in-flight library reads of the bytes
   std::shared_ptr<RemoteMap> remote;  // loc == GROUTER_REMOTE
@@ -218,6 +219,8 @@ struct grouter_ctx {
   uint64_t seq = 0, next_oid = 1, xfer_seq = 0;
   uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
   std::vector<grouter_oid> victims;
+  std::vector<grouter_oid> restored;                   // GROUTER_RESTORE (L260)
+  bool restore_on = false;
   std::deque<gr::ProfRec> prof;                        // GROUTER_PROFILE launches not yet harvested
   std::unordered_map<gr::Xfer *, gr::XferRef> live;    // transfers with chunks not yet submitted
   gr::CopyParamsHost *params = nullptr;                // reused kernel-parameter builder (engine.cpp)
@@ -265,6 +268,7 @@ Waitable signal(grouter_ctx *c, cudaStream_t s, int phys);       // caller strea
 void host_wait(const Fences &f, double timeout_s = 120.0);
 bool grounded(const grouter_ctx *c, const Fences &f);
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst);  // D2H of a victim (unscheduled)
+void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst);  // H2D back home (unscheduled)
 // ipc.cpp
 void ipc_serve_start(grouter_ctx *c);
 void ipc_shutdown(grouter_ctx *c);

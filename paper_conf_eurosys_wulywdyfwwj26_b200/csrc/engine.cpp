@@ -706,6 +706,30 @@ void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
   pump(c, false);
 }
 
+// H2D of a proactively restored object (L260-L262) back to its home GPU d: an
+// urgent, unscheduled single-path transfer on d's own H2D engine (no relay:
+// restores are background work, they should not load other GPUs' links).
+void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst) {
+  std::vector<grouter_chunk> plan;
+  c->planner.plan_single(o.n, d, plan);
+  XferRef x = new_xfer_slot(c, plan);
+  x->deps = o.ready;
+  Server &s = c->dev[d].h2d;
+  for (uint32_t i = 0; i < plan.size(); ++i)
+    s.urgent.push_back(make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)dev_dst, d));
+  Fences done;
+  done_fences(x, done);
+  Fences old = std::move(o.readers);
+  for (auto &f : o.ready) old.push_back(f);
+  for (auto &f : done) old.push_back(f);
+  host_free(c, o.ptr, charge(o.n), std::move(old));
+  o.ready = done;
+  o.readers.clear();
+  c->stats.restore_count++;
+  c->stats.restore_bytes += o.n;
+  pump(c, false);
+}
+
 // ------------------------------------------------------------------ lifecycle
 static void daemon_main(grouter_ctx *c) {
   std::unique_lock<std::mutex> lk(c->mu);

@@ -25,7 +25,7 @@ NOHINT = -2
 REMOTE = -3
 UNLIMITED = (1 << 64) - 1
 
-REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20
+REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE, RESTORE = 0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]
@@ -72,7 +72,7 @@ class grouter_stats_t(C.Structure):
         ("spill_count", C.c_uint64), ("spill_bytes", C.c_uint64), ("xfer_count", C.c_uint64),
         ("link_bytes", (C.c_uint64 * MAX_GPUS) * 3), ("kernel_launches", C.c_uint64),
         ("rounds", C.c_uint64), ("timed_launches", C.c_uint64), ("timed_ns", C.c_uint64),
-        ("timed_bytes", C.c_uint64),
+        ("timed_bytes", C.c_uint64), ("restore_count", C.c_uint64), ("restore_bytes", C.c_uint64),
     ]
 
 
@@ -122,6 +122,7 @@ SIGNATURES = {
     "grouter_where": (_ST, [_CTX, _U64, C.POINTER(_I32)]),
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
+    "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_dispatch_log": (_ST, [_CTX, C.POINTER(grouter_dispatch), _U64, C.POINTER(_U64)]),
     "grouter_export_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, C.POINTER(grouter_ipc_desc)]),
     "grouter_import_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), C.POINTER(grouter_ipc_desc), _U32,
@@ -369,6 +370,11 @@ class Ctx:
     def victims(self):
         arr, cnt = (C.c_uint64 * 4096)(), C.c_uint64(0)
         check(self.lib.grouter_victims(self.h, arr, 4096, C.byref(cnt)), "victims")
+        return list(arr[:cnt.value])
+
+    def restored(self):
+        arr, cnt = (C.c_uint64 * 4096)(), C.c_uint64(0)
+        check(self.lib.grouter_restored(self.h, arr, 4096, C.byref(cnt)), "restored")
         return list(arr[:cnt.value])
 
     def dispatch_log(self):

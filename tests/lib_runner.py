@@ -228,6 +228,7 @@ class LibRunner:
             if trace:
                 print("   ->", G.STATUS[st], G.last_error() if st else "", flush=True)
             rec["victims"] = ctx.victims()
+            rec["restored"] = ctx.restored()
             s = ctx.stats()
             rec["used"] = [s.used[d] for d in range(self.n)]
             rec["host_used"] = s.host_used
@@ -259,6 +260,7 @@ def compare(orc_out, lib_out, check_dispatch=True):
         assert l.get("oid") == o.get("oid"), ctx
         assert l.get("where") == o.get("where"), (ctx, o.get("where"), l.get("where"))
         assert l["victims"] == o["victims"], (ctx, o["victims"], l["victims"])
+        assert l.get("restored", []) == o.get("restored", []), (ctx, o.get("restored"), l.get("restored"))
         assert l["used"] == o["used"], (ctx, o["used"], l["used"])
         assert l["host_used"] == o["host_used"], ctx
         if o["status"] == "OK" and o["op"] in ("get", "get_into"):

@@ -116,9 +116,11 @@ def _copy_exactly_once(tma, src_off, dst_off):
 
 
 # ------------------------------------------------------------------ trace parity
-def _both(ops, calib, replay=True, keep=True, **kw):
+def _both(ops, calib, replay=True, keep=True, restore=False, **kw):
     orc = orun.run(ops, calib, host_store_bytes=kw.get("host_store_bytes", 1 << 30),
-                   pool_cap=kw.get("pool_cap"), keep_bytes=keep)
+                   pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore)
+    if restore:
+        kw["flags"] = kw.get("flags", 0) | G.RESTORE
     r = LibRunner(calib, replay=replay, keep_bytes=keep, **kw)
     try:
         lib_out = r(ops)
@@ -180,6 +182,33 @@ def test_random_traces_realtime(seed):
     caps = [rng.choice([8, 16, 64]) * MiB for _ in range(k)]
     orc, lib_out = _both(ops, calib, replay=False, host_store_bytes=48 * MiB, pool_cap=caps)
     compare(orc, lib_out, check_dispatch=False)
+
+
+def test_fig11b_restore():
+    """PAPER.md L260-L262 worked example on the device: a2's output is
+    migrated, then reloaded once a1's output has been processed."""
+    from tests.test_oracle_model import _fig11b_restore_ops
+    calib = dict(C.b200_hgx(1), device_map=[0])
+    orc, lib_out = _both(_fig11b_restore_ops(), calib, restore=True, pool_cap=[4 * MiB])
+    compare(orc, lib_out)
+    assert lib_out["records"][-1]["restored"] == [2]
+    assert lib_out["stats"].restore_count == 1
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_restore(seed, replay):
+    """Random traces with proactive restore on: statuses, placements, victims,
+    restores, pool usage and bytes equal the oracle's (restore=True)."""
+    rng = random.Random(3000 + seed)
+    k = rng.choice([1, 2, 3]) if replay else rng.choice([2, 3])
+    calib = C.virtual(k) if k > 1 else dict(C.b200_hgx(1), device_map=[0])
+    ops = T.random_trace(rng, k, n_ops=120, max_n=5 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, restore=True, host_store_bytes=64 * MiB,
+                         pool_cap=caps)
+    compare(orc, lib_out, check_dispatch=replay)
+    assert sum(len(r["restored"]) for r in lib_out["records"]) == lib_out["stats"].restore_count
 
 
 def test_full_size_cfg1_sampled():

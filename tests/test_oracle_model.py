@@ -160,3 +160,119 @@ def test_capacity_never_exceeded_by_reserve():
         for r in res["records"]:
             assert all(u <= c for u, c in zip(r["used"], caps)), r
         assert any(r["victims"] for r in res["records"]) or True
+
+
+# ---------------------------------------------------------------- proactive restore
+def _fig11b_restore(restore):
+    """Fig. 11(b) continued: "after the output of a1 is
+    processed, the output of a2 is reloaded into GPU memory"."""
+    return runner.run(_fig11b_restore_ops(), C.b200_hgx(1), pool_cap=[4 * MiB], restore=restore)
+
+
+def _fig11b_restore_ops():
+    b = T.Builder(3)
+    a1, a2, a3, b1 = T.fn(1, 1, 0), T.fn(1, 2, 0), T.fn(1, 3, 0), T.fn(1, 4, 0)
+    o1 = b.alloc(a1, MiB, consumers=1)
+    b.seal(a1, o1)
+    o2 = b.alloc(a2, MiB, consumers=1)
+    b.seal(a2, o2)
+    b.next_use(o1, 0)
+    b.next_use(o2, 1)
+    b.put(a3, MiB)                      # evicts O2 (queue-aware)
+    g = b.get(b1, o1)                   # b1 processes a1's output (zero copy)
+    b.release(b1, g)                    # ... and is done with it
+    return b.ops
+
+
+def test_fig11b_restore_after_a1_output_processed():
+    out = _fig11b_restore(True)
+    recs = out["records"]
+    assert recs[6]["victims"] == [2]
+    assert recs[-1]["restored"] == [2]             # a2's output reloaded
+    orc = out["oracle"]
+    assert orc.where(2) == 0 and orc.host_used == 0 and orc.used == [4 * MiB]
+    # without restore the object stays on the host; restore moves, never changes, bytes
+    out2 = _fig11b_restore(False)
+    assert out2["records"][-1]["restored"] == [] and out2["oracle"].where(2) == model.HOST
+    assert bytes(orc.objects[2].buf) == bytes(out2["oracle"].objects[2].buf)
+
+
+def _restore_setup(hints, cap_after):
+    """Four spilled 1-page objects (oids 1-4), then the limit is raised."""
+    b = T.Builder(5)
+    f = T.fn(1, 1, 0)
+    refs = [b.put(f, MiB) for _ in range(4)]
+    for r, h in zip(refs, hints):
+        if h is not None:
+            b.next_use(r, h)
+    b.pool_limit(0, 0)                  # spill everything
+    b.pool_limit(0, cap_after)
+    out = runner.run(b.ops, C.b200_hgx(1), restore=True)
+    return out["records"]
+
+
+def test_restore_order_hinted_first_then_mru():
+    # hints: oid1 -> 5, oid2 none, oid3 -> 2, oid4 none
+    recs = _restore_setup([5, None, 2, None], 8 * MiB)
+    assert sorted(recs[-2]["victims"]) == [1, 2, 3, 4]
+    # queue head first among hinted (3 then 1), then most recently used (4, 2)
+    assert recs[-1]["restored"] == [3, 1, 4, 2]
+
+
+def test_restore_stops_at_cap():
+    recs = _restore_setup([5, None, 2, None], 5 * MiB)    # room for 2 pages
+    assert recs[-1]["restored"] == [3, 1]
+    assert recs[-1]["used"] == [4 * MiB]
+
+
+def test_restore_stops_at_first_misfit():
+    """Strict priority: a small later object is not restored past a large
+    earlier one that does not fit (R42)."""
+    b = T.Builder(5)
+    f = T.fn(1, 1, 0)
+    big, small = b.put(f, 3 * MiB), b.put(f, MiB)
+    b.next_use(big, 0)
+    b.next_use(small, 1)
+    b.pool_limit(0, 0)
+    b.pool_limit(0, 2 * MiB)            # small fits, big (4 MiB) does not
+    recs = runner.run(b.ops, C.b200_hgx(1), restore=True)["records"]
+    assert recs[-1]["restored"] == [] and recs[-1]["used"] == [0]
+
+
+def test_restore_respects_home_gpu():
+    """Only objects migrated away from the GPU that gained room come back."""
+    b = T.Builder(6)
+    f0, f1 = T.fn(1, 1, 0), T.fn(1, 2, 1)
+    b.put(f0, MiB)
+    o2 = b.put(f1, MiB)
+    b.pool_limit(0, 0)
+    b.pool_limit(1, 0)
+    b.pool_limit(0, 8 * MiB)
+    recs = runner.run(b.ops, C.b200_hgx(2), restore=True)["records"]
+    assert recs[-1]["restored"] == [1]
+    del o2
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_restore_preserves_bytes_and_caps(seed):
+    """Restore moves data, never changes it: every get/get_into that succeeds
+    both with and without restore reads identical bytes; and restore never
+    takes a pool above its cap (I4 holds after restore-only ops)."""
+    rng = random.Random(100 + seed)
+    n = rng.choice([1, 2, 4])
+    c = C.b200_hgx(n)
+    ops = T.random_trace(rng, n, n_ops=150, max_n=5 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16]) * MiB for _ in range(n)]
+    a = runner.run(ops, c, host_store_bytes=1 << 30, pool_cap=caps, restore=False)["records"]
+    r = runner.run(ops, c, host_store_bytes=1 << 30, pool_cap=caps, restore=True)
+    moved = 0
+    caps = list(caps)
+    for op, x, y in zip(ops, a, r["records"]):
+        if op["op"] == "pool_limit":
+            caps[op["dev"]] = op["bytes"]
+        moved += len(y["restored"])
+        if x["op"] in ("get", "get_into") and x["status"] == y["status"] == "OK":
+            assert x.get("digest") == y.get("digest"), x["i"]
+        if y["restored"] and y["op"] in ("release", "free", "get", "get_into"):
+            assert all(u <= cp for u, cp in zip(y["used"], caps))
+    assert moved > 0 or seed % 3 == 0     # most traces exercise restore
