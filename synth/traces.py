@@ -222,6 +222,46 @@ def cfg5(n_gpus: int, requests: int = 8, limit_frac=None, run_seed: int = 5000,
     return b.ops
 
 
+def cfg5_interleaved(n_gpus: int, requests: int = 8, window: int = 3, limit_frac=0.3,
+                     run_seed: int = 5500, scale: int = 1, layers: int = CFG5_LAYERS,
+                     hints: bool = True) -> list:
+    """Config 5 with interleaved arrivals (Fig. 18 setting):
+    ``window`` requests are in flight; stage B of request r consumes (get_into)
+    its objects, then stage A of request r + window produces.  The pool limit
+    is ``limit_frac`` of the in-flight working set, so consumption releases
+    storage that proactive restore (L260) can refill with the queue head."""
+    b = Builder(run_seed)
+    kv, hid = CFG5_KV // scale, CFG5_HIDDEN // scale
+    a_dev, b_dev = 0, (1 if n_gpus > 1 else 0)
+    pages = lambda x: -(-x // (2 * MiB)) * (2 * MiB)
+    ws = window * (layers * pages(kv) + pages(hid))
+    if limit_frac is not None:
+        b.pool_limit(a_dev, max(2 * MiB, int(ws * limit_frac) // (2 * MiB) * (2 * MiB)))
+    objs = {}
+
+    def produce(r):
+        A = fn(500 + r, 1, a_dev)
+        mine = []
+        for nb in [kv] * layers + [hid]:
+            o = b.alloc(A, nb, consumers=1)
+            b.seal(A, o)
+            if hints:
+                b.next_use(o, r)
+            mine.append(o)
+        objs[r] = mine
+
+    for r in range(min(window, requests)):
+        produce(r)
+    for r in range(requests):
+        B = fn(500 + r, 2, b_dev)
+        for o in objs.pop(r):
+            b.get_into(B, o)
+        b.flush()
+        if r + window < requests:
+            produce(r + window)
+    return b.ops
+
+
 def random_trace(rng: random.Random, n_gpus: int, n_ops: int = 200, max_n: int = 9 * MiB,
                  n_wf: int = 3, host_ok: bool = True, run_seed: int = 7, flush_every: int = 4,
                  limits: bool = True, small_sizes: bool = True) -> list:

@@ -211,6 +211,18 @@ def test_random_traces_restore(seed, replay):
     assert sum(len(r["restored"]) for r in lib_out["records"]) == lib_out["stats"].restore_count
 
 
+@pytest.mark.parametrize("k", [1, 2])
+@pytest.mark.parametrize("replay", [True, False])
+def test_cfg5_interleaved_restore(k, replay):
+    """Interleaved cfg5 with queue hints and proactive restore (Fig. 18
+    setting): library == oracle op by op, bytes included."""
+    calib = C.virtual(k) if k > 1 else dict(C.b200_hgx(1), device_map=[0])
+    ops = T.cfg5_interleaved(k, requests=6, window=3, limit_frac=0.3, scale=64, layers=8)
+    orc, lib_out = _both(ops, calib, replay=replay, restore=True)
+    assert compare(orc, lib_out, check_dispatch=replay) > 0
+    assert lib_out["stats"].restore_count > 0
+
+
 def test_full_size_cfg1_sampled():
     """cfg1 at its real size (38,535,168 B): striped put into GPU0 then get on
     logical GPU1 (virtual), verified in full on the device against the

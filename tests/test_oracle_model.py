@@ -276,3 +276,24 @@ def test_restore_preserves_bytes_and_caps(seed):
         if y["restored"] and y["op"] in ("release", "free", "get", "get_into"):
             assert all(u <= cp for u, cp in zip(y["used"], caps))
     assert moved > 0 or seed % 3 == 0     # most traces exercise restore
+
+
+@pytest.mark.parametrize("restore", [False, True])
+@pytest.mark.parametrize("hints", [False, True])
+def test_cfg5_interleaved_drains(restore, hints):
+    """Interleaved cfg5 (Fig. 18 setting): every op succeeds, the pools drain,
+    and with queue hints + restore the head of the queue is reloaded."""
+    ops = T.cfg5_interleaved(2, requests=6, window=3, limit_frac=0.3, scale=64, layers=8, hints=hints)
+    out = runner.run(ops, C.b200_hgx(2), restore=restore)
+    assert all(r["status"] == "OK" for r in out["records"])
+    orc = out["oracle"]
+    assert orc.used == [0, 0] and orc.host_used == 0 and not orc.objects
+    restored = [o for r in out["records"] for o in r["restored"]]
+    assert bool(restored) == (restore and hints)
+    if restored:
+        # restores follow consumption: each restored object belongs to a
+        # request later than the one whose get_into released the room
+        by_oid = {r["oid"]: ops[r["i"]]["fn"]["wf"] for r in out["records"] if r["op"] == "alloc"}
+        for r in out["records"]:
+            if r["op"] == "get_into" and r["restored"]:
+                assert all(by_oid[o] > ops[r["i"]]["fn"]["wf"] for o in r["restored"])

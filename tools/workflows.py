@@ -148,6 +148,69 @@ def cfg5(requests=4, limit_frac=0.1, hints=True, layers=32):
     return out
 
 
+def cfg5_interleaved(requests=12, window=3, limit_frac=0.3, hints=True, restore=True,
+                     layers=32, compute_ms=30.0):
+    """Fig. 18 analog: `window` requests in flight; stage B of
+    request r reads its 33 objects (get_into), "computes" for compute_ms
+    (host sleep: the model's inference time, during which the background
+    restores run), then stage A of request r + window produces.  The pool
+    limit is limit_frac of the in-flight working set."""
+    KV, HID = 33_554_432, 67_108_864
+    page = 2 * MiB
+    charge = lambda x: -(-x // page) * page
+    ws = window * (layers * charge(KV) + charge(HID))
+    limit = int(ws * limit_frac) // page * page
+    flags = G.RESTORE if restore else 0
+    ctx = mkctx(host_store_bytes=ws + 512 * MiB, pool_cap=[G.UNLIMITED], pool_floor_bytes=64 * MiB,
+                flags=flags)
+    G.check(ctx.set_pool_limit(0, limit), "limit")
+    s = torch.cuda.Stream()
+    dst = torch.empty(HID, dtype=torch.uint8, device="cuda")
+    objs = {}
+
+    def produce(r):
+        A = G.fn(500 + r, 1, 0)
+        mine = []
+        for nb in [KV] * layers + [HID]:
+            st, buf, oid = ctx.alloc(A, nb, G.NOHINT, 1)
+            G.check(st, "alloc")
+            G.check(G.test_fill(buf, nb, oid, 0, s.cuda_stream))
+            G.check(ctx.seal(A, oid, s.cuda_stream))
+            if hints:
+                ctx.set_next_use(oid, r)
+            mine.append((oid, nb))
+        objs[r] = mine
+
+    t_start = time.perf_counter()
+    for r in range(window):
+        produce(r)
+    s.synchronize()
+    lat, from_host = [], []
+    for r in range(requests):
+        B = G.fn(500 + r, 2, 0)
+        where = [ctx.where(oid)[1] for oid, _ in objs[r]]
+        from_host.append(sum(1 for w in where if w == G.HOST))
+        t0 = time.perf_counter()
+        for oid, nb in objs.pop(r):
+            G.check(ctx.get_into(B, oid, dst.data_ptr(), nb, s.cuda_stream)[0], "get_into")
+        s.synchronize()
+        lat.append(time.perf_counter() - t0)
+        time.sleep(compute_ms / 1e3)          # stage-B inference
+        if r + window < requests:
+            produce(r + window)
+    total = time.perf_counter() - t_start
+    stt = ctx.stats()
+    out = {"requests": requests, "window": window, "limit_frac": limit_frac, "queue_aware": hints,
+           "restore": restore, "compute_ms": compute_ms, "pool_limit_GB": round(limit / 1e9, 3),
+           "stageB_p50_ms": round(pct(lat, 50) * 1e3, 2), "stageB_p99_ms": round(pct(lat, 99) * 1e3, 2),
+           "stageB_mean_ms": round(sum(lat) / len(lat) * 1e3, 2),
+           "objects_read_from_host": sum(from_host),
+           "spill_GB": round(stt.spill_bytes / 1e9, 3), "restore_GB": round(stt.restore_bytes / 1e9, 3),
+           "req_per_s": round(requests / total, 2)}
+    ctx.close()
+    return out
+
+
 def main():
     _build.build()
     G.load()
@@ -156,6 +219,15 @@ def main():
 
     def save():
         json.dump(res, open(out, "w"), indent=1)
+    if len(sys.argv) > 2 and sys.argv[2] == "cfg5i":
+        res["cfg5_interleaved"] = []
+        for frac in (0.3, 0.1):
+            for hints, restore in ((True, True), (True, False), (False, False), (False, True)):
+                r = cfg5_interleaved(12, 3, frac, hints, restore)
+                res["cfg5_interleaved"].append(r)
+                print("cfg5i", json.dumps(r), flush=True)
+                save()
+        return
     res["cfg4"] = cfg4(3.0)
     print("cfg4", json.dumps(res["cfg4"]), flush=True)
     save()
