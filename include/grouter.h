@@ -245,6 +245,25 @@ grouter_status grouter_import_ipc(grouter_ctx *ctx, const grouter_fn *fn, const 
 /* ------------------------------------------------------------ control */
 /* Tenant (workflow) bandwidth weight, >= 1 (north star; L193-L197). */
 grouter_status grouter_set_tenant_weight(grouter_ctx *ctx, uint32_t workflow_id, uint32_t weight);
+/* Transfer rate control (§4.3.2; R43):
+ * declares workflow wf's SLO -- it must move data_bytes within
+ * slo_ns - infer_ns.  Rate_least = ceil(data_bytes * 1e9 / (slo_ns - infer_ns))
+ * B/s; Rate_idle = max(0, BW_all - sum Rate_least) with BW_all = sum of the
+ * calibrated h2d_Bps; the tightest SLO (min slo_ns, ties -> lower id) also
+ * gets Rate_idle; every SLO workflow's stride weight becomes its rate in
+ * MiB/s, rounded up (>= 1).  Workflows without an SLO keep their weight.
+ * data_bytes == 0 removes wf's SLO (weight back to 1); a later
+ * grouter_set_tenant_weight(wf) also removes it; both re-weight the other SLO
+ * workflows.  EINVAL if slo_ns <= infer_ns. */
+grouter_status grouter_set_tenant_slo(grouter_ctx *ctx, uint32_t workflow_id, uint64_t data_bytes,
+                                      uint64_t slo_ns, uint64_t infer_ns);
+/* The same allocation as a pure function (no context, no GPU): n workflows
+ * with ids[i] and SLO triples; writes weights_out[i].  EINVAL on a null
+ * pointer with n > 0 or slo_ns[i] <= infer_ns[i]. */
+grouter_status grouter_slo_weights(uint32_t n, const uint32_t *ids, const uint64_t *data_bytes,
+                                   const uint64_t *slo_ns, const uint64_t *infer_ns, uint64_t bw_all_Bps,
+                                   uint32_t *weights_out);
+
 /* Queue position of the object's next consumer (D8; L258 queue-aware eviction). */
 grouter_status grouter_set_next_use(grouter_ctx *ctx, grouter_oid oid, uint64_t queue_pos);
 /* Pool cap of a GPU (GROUTER_UNLIMITED = no cap); evicts at once until used <= cap

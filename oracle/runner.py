@@ -94,6 +94,8 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
             st, out = orc.free(op["fn"], oid)
         elif k == "weight":
             st, out = orc.set_weight(op["wf"], op["w"])
+        elif k == "slo":
+            st, out = orc.set_slo(op["wf"], op["data"], op["slo_ns"], op["infer_ns"])
         elif k == "next_use":
             st, out = orc.set_next_use(oid, op["pos"])
         elif k == "pool_limit":

@@ -794,6 +794,8 @@ grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const gr
 }
 
 // ------------------------------------------------------------------ control
+static grouter_status reweight_slos(grouter_ctx *c);
+
 grouter_status grouter_set_tenant_weight(grouter_ctx *c, uint32_t wf, uint32_t w) {
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
   Guard g(c);
@@ -801,6 +803,68 @@ grouter_status grouter_set_tenant_weight(grouter_ctx *c, uint32_t wf, uint32_t w
   c->restored.clear();
   if (w < 1) return fail(GROUTER_EINVAL, "weight must be >= 1");
   c->weights[wf] = w;
+  if (c->slos.erase(wf)) return reweight_slos(c);  // an explicit weight replaces an SLO (R43)
+  return GROUTER_OK;
+}
+
+// Rate_least (L195) = ceil(data * 1e9 / (slo - infer)) B/s; Rate_idle (L197)
+// to the tightest SLO (L227); weight = rate in MiB/s rounded up (R43).
+grouter_status grouter_slo_weights(uint32_t n, const uint32_t *ids, const uint64_t *data,
+                                   const uint64_t *slo, const uint64_t *infer, uint64_t bw_all,
+                                   uint32_t *out) {
+  if (n && (!ids || !data || !slo || !infer || !out)) return fail(GROUTER_EINVAL, "slo_weights: null");
+  std::vector<unsigned __int128> least(n);
+  unsigned __int128 sum = 0;
+  uint32_t tight = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (slo[i] <= infer[i]) return fail(GROUTER_EINVAL, "slo_weights: slo_ns <= infer_ns");
+    const unsigned __int128 num = (unsigned __int128)data[i] * 1000000000u, den = slo[i] - infer[i];
+    least[i] = (num + den - 1) / den;
+    sum += least[i];
+    if (slo[i] < slo[tight] || (slo[i] == slo[tight] && ids[i] < ids[tight])) tight = i;
+  }
+  const unsigned __int128 idle = sum < bw_all ? bw_all - sum : 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    const unsigned __int128 rate = least[i] + (i == tight ? idle : 0);
+    unsigned __int128 w = (rate + (1u << 20) - 1) >> 20;
+    if (w < 1) w = 1;
+    if (w > 0xFFFFFFFFu) w = 0xFFFFFFFFu;
+    out[i] = (uint32_t)w;
+  }
+  return GROUTER_OK;
+}
+
+grouter_status grouter_set_tenant_slo(grouter_ctx *c, uint32_t wf, uint64_t data, uint64_t slo_ns,
+                                      uint64_t infer_ns) {
+  if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  Guard g(c);
+  c->victims.clear();
+  c->restored.clear();
+  if (data == 0) {
+    c->slos.erase(wf);
+    c->weights.erase(wf);
+  } else {
+    if (slo_ns <= infer_ns) return fail(GROUTER_EINVAL, "set_tenant_slo: slo_ns <= infer_ns");
+    c->slos[wf] = {data, slo_ns, infer_ns};
+  }
+  return reweight_slos(c);
+}
+
+static grouter_status reweight_slos(grouter_ctx *c) {
+  const uint32_t n = (uint32_t)c->slos.size();
+  std::vector<uint32_t> ids, w(n);
+  std::vector<uint64_t> d, s, inf;
+  for (auto &kv : c->slos) {
+    ids.push_back(kv.first);
+    d.push_back(kv.second[0]);
+    s.push_back(kv.second[1]);
+    inf.push_back(kv.second[2]);
+  }
+  uint64_t bw_all = 0;
+  for (uint32_t i = 0; i < c->cfg.n_gpus; ++i) bw_all += c->cfg.h2d_Bps[i];
+  grouter_status st = grouter_slo_weights(n, ids.data(), d.data(), s.data(), inf.data(), bw_all, w.data());
+  if (st) return st;
+  for (uint32_t i = 0; i < n; ++i) c->weights[ids[i]] = w[i];
   return GROUTER_OK;
 }
 

@@ -216,6 +216,7 @@ struct grouter_ctx {
   std::unordered_map<grouter_oid, gr::Obj> objects;
   std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
   std::unordered_map<uint32_t, uint32_t> weights;
+  std::map<uint32_t, std::array<uint64_t, 3>> slos;    // wf -> (data, slo_ns, infer_ns), R43
   uint64_t seq = 0, next_oid = 1, xfer_seq = 0;
   uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
   std::vector<grouter_oid> victims;

@@ -123,6 +123,9 @@ SIGNATURES = {
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
+    "grouter_set_tenant_slo": (_ST, [_CTX, C.c_uint32, _U64, _U64, _U64]),
+    "grouter_slo_weights": (_ST, [C.c_uint32, C.POINTER(C.c_uint32), C.POINTER(_U64), C.POINTER(_U64),
+                                  C.POINTER(_U64), _U64, C.POINTER(C.c_uint32)]),
     "grouter_dispatch_log": (_ST, [_CTX, C.POINTER(grouter_dispatch), _U64, C.POINTER(_U64)]),
     "grouter_export_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, C.POINTER(grouter_ipc_desc)]),
     "grouter_import_ipc": (_ST, [_CTX, C.POINTER(grouter_fn), C.POINTER(grouter_ipc_desc), _U32,
@@ -323,6 +326,9 @@ class Ctx:
     def set_tenant_weight(self, wf, w):
         return self.lib.grouter_set_tenant_weight(self.h, wf, w)
 
+    def set_tenant_slo(self, wf, data_bytes, slo_ns, infer_ns):
+        return self.lib.grouter_set_tenant_slo(self.h, wf, data_bytes, slo_ns, infer_ns)
+
     def set_next_use(self, oid, pos):
         return self.lib.grouter_set_next_use(self.h, oid, pos)
 
@@ -391,6 +397,19 @@ class Ctx:
 
 
 # ------------------------------------------------------------------ test kernels (K9)
+def slo_weights(slos: dict, bw_all: int) -> dict:
+    """grouter_slo_weights: {wf: (data_bytes, slo_ns, infer_ns)} -> {wf: weight}."""
+    lib = load()
+    n = len(slos)
+    ids = (C.c_uint32 * max(n, 1))(*slos.keys())
+    d = (C.c_uint64 * max(n, 1))(*[v[0] for v in slos.values()])
+    s = (C.c_uint64 * max(n, 1))(*[v[1] for v in slos.values()])
+    i = (C.c_uint64 * max(n, 1))(*[v[2] for v in slos.values()])
+    out = (C.c_uint32 * max(n, 1))()
+    check(lib.grouter_slo_weights(n, ids, d, s, i, bw_all, out), "slo_weights")
+    return dict(zip(slos.keys(), out[:n]))
+
+
 def test_fill(ptr: int, n: int, seed: int, offset: int = 0, stream: int = 0):
     return load().grouter_test_fill(ptr or None, n, seed, offset, stream or None)
 

@@ -85,6 +85,9 @@ class Builder:
     def weight(self, wf, w):
         return self._add({"op": "weight", "wf": wf, "w": w})
 
+    def slo(self, wf, data, slo_ns, infer_ns):
+        return self._add({"op": "slo", "wf": wf, "data": data, "slo_ns": slo_ns, "infer_ns": infer_ns})
+
     def next_use(self, ref, pos):
         return self._add({"op": "next_use", "ref": ref, "pos": pos})
 
@@ -155,17 +158,24 @@ def cfg2(n_gpus: int, requests: int = 8, run_seed: int = 2000, scale: int = 1) -
 
 
 def cfg4(n_gpus: int, rounds: int = 4, run_seed: int = 4000, scale: int = 1,
-         weights=(1, 1, 2, 2, 4, 4, 8, 8)) -> list:
+         weights=(1, 1, 2, 2, 4, 4, 8, 8), slos=None) -> list:
     """Config 4: 8 workflows with weights; each round every tenant puts a
     tensor from host, gets it on GPU t%N, allocs an output and the next GPU
     gets it.  The gets of one round are flushed together (replay-mode
     dispatch log is the compared artefact)."""
     b = Builder(run_seed)
     n = CFG1_BYTES // scale
-    T = len(weights)
-    for t, w in enumerate(weights):
-        b.weight(100 + t, w)
-    for _ in range(rounds):
+    T = len(weights) if slos is None else len(slos)
+    if slos is None:
+        for t, w in enumerate(weights):
+            b.weight(100 + t, w)
+    else:
+        for t, (data, slo_ns, infer_ns) in enumerate(slos):
+            b.slo(100 + t, data, slo_ns, infer_ns)
+    for r in range(rounds):
+        if slos is not None and r == 1:
+            b.slo(100, 0, 0, 0)          # tenant 100 drops its SLO: everyone re-weighted
+            b.weight(101, 3)             # an explicit weight replaces 101's SLO
         puts = []
         for t in range(T):
             puts.append(b.put(fn(100 + t, 1, HOST), n, hint=NOHINT, consumers=1))
@@ -188,6 +198,13 @@ def cfg4(n_gpus: int, rounds: int = 4, run_seed: int = 4000, scale: int = 1,
             b.release(fn(100 + t, 2, t % n_gpus), gets[t])
             b.release(fn(100 + t, 3, (t + 1) % n_gpus), gets2[t])
     return b.ops
+
+
+# SLO variant of cfg4 (L193-L197): (data_bytes, slo_ns, infer_ns) per tenant;
+# data = the cfg1 tensor, SLOs 1.5-2x inference time as in L193.
+CFG4_SLOS = [(CFG1_BYTES, 60_000_000, 40_000_000), (CFG1_BYTES, 80_000_000, 40_000_000),
+             (CFG1_BYTES, 30_000_000, 20_000_000), (2 * CFG1_BYTES, 100_000_000, 50_000_000),
+             (CFG1_BYTES, 45_000_000, 30_000_000), (4 * CFG1_BYTES, 200_000_000, 100_000_000)]
 
 
 def cfg5(n_gpus: int, requests: int = 8, limit_frac=None, run_seed: int = 5000,

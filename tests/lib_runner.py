@@ -213,6 +213,8 @@ class LibRunner:
                 st = ctx.free(self._fnc(op["fn"]), oid)
             elif k == "weight":
                 st = ctx.set_tenant_weight(op["wf"], op["w"])
+            elif k == "slo":
+                st = ctx.set_tenant_slo(op["wf"], op["data"], op["slo_ns"], op["infer_ns"])
             elif k == "next_use":
                 st = ctx.set_next_use(oid, op["pos"])
             elif k == "pool_limit":

@@ -223,6 +223,16 @@ def test_cfg5_interleaved_restore(k, replay):
     assert lib_out["stats"].restore_count > 0
 
 
+@pytest.mark.parametrize("k", [1, 2, 4])
+def test_cfg4_slo_dispatch_parity(k):
+    """SLO-derived shares (L193-L197, R43): with replay dispatch the library's
+    per-server batch order equals the oracle's -- so its weights do."""
+    calib = C.virtual(k) if k > 1 else dict(C.b200_hgx(1), device_map=[0])
+    ops = T.cfg4(k, rounds=2, scale=64, slos=T.CFG4_SLOS)
+    orc, lib_out = _both(ops, calib)
+    assert compare(orc, lib_out) > 0
+
+
 def test_full_size_cfg1_sampled():
     """cfg1 at its real size (38,535,168 B): striped put into GPU0 then get on
     logical GPU1 (virtual), verified in full on the device against the

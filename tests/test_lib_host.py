@@ -142,3 +142,26 @@ def test_sched_parity_with_oracle(seed):
                 assert a is not None
                 assert (a[0], a[1], a[2]) == (b[0], b[1], b[2])
                 assert a[3] == orc.pass_[b[0]]
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_slo_weights_parity_with_oracle(seed):
+    """grouter_slo_weights (C) == oracle/slo.weights on random SLO sets,
+    including oversubscribed ones and 64-bit-overflowing data sizes."""
+    import random
+    from oracle import slo as oslo
+    rng = random.Random(seed)
+    s = {}
+    for _ in range(rng.randint(1, 8)):
+        wf = rng.randint(1, 50)
+        slo_ns = rng.choice([1, 7, 10 ** 6, 5 * 10 ** 7, 10 ** 9, 3 * 10 ** 10])
+        infer = rng.randint(0, slo_ns - 1)
+        data = rng.choice([1, 4096, 38_535_168, rng.randint(1, 1 << 40), (1 << 63) + rng.randint(0, 1 << 20)])
+        s[wf] = (data, slo_ns, infer)
+    bw = rng.choice([0, 55 * 10 ** 9, 8 * 55 * 10 ** 9, 1 << 62])
+    assert G.slo_weights(s, bw) == oslo.weights(s, bw)
+
+
+def test_slo_weights_rejects_infeasible():
+    with pytest.raises(RuntimeError):
+        G.slo_weights({1: (10, 5, 5)}, 10 ** 9)

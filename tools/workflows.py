@@ -34,17 +34,22 @@ def pct(xs, q):
     return xs[max(0, min(len(xs) - 1, -(-len(xs) * q // 100) - 1))] if xs else None
 
 
-def mkctx(**kw):
+def mkctx(h2d_Bps=None, **kw):
     c = b200_hgx(1)
     c["device_map"] = [0]
+    if h2d_Bps:
+        c["h2d_Bps"] = [h2d_Bps]
     return G.Ctx(G.config_from_calib(c, **kw))
 
 
-def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8)):
-    ctx = mkctx(host_store_bytes=256 * MiB, pool_cap=[G.UNLIMITED])
+def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8), slos=None, h2d_Bps=None):
+    ctx = mkctx(h2d_Bps=h2d_Bps, host_store_bytes=256 * MiB, pool_cap=[G.UNLIMITED])
     T = len(weights)
     for t, w in enumerate(weights):
-        ctx.set_tenant_weight(100 + t, w)
+        if slos:
+            G.check(ctx.set_tenant_slo(100 + t, *slos[t]), "slo")
+        else:
+            ctx.set_tenant_weight(100 + t, w)
     srcs = [torch.empty(N1, dtype=torch.uint8, pin_memory=True) for _ in range(T)]
     done = [0] * T
     lat = [[] for _ in range(T)]
@@ -81,6 +86,22 @@ def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8)):
             "max_share_error": round(max(err), 3) if err else None,
             "p50_ms": [round(pct(l, 50) * 1e3, 2) if l else None for l in lat],
             "p99_ms": [round(pct(l, 99) * 1e3, 2) if l else None for l in lat]}
+
+
+def cfg4_slo(seconds=3.0, bw=53e9):
+    """Transfer rate control (L193-L197, L227): 8 CPU tenants loop blocking
+    puts of 38,535,168 B; tenant t must finish each put within budget_t
+    (SLO = 2x inference time, L193, so budget = slo - infer = infer).  With
+    SLO-derived weights vs all weights 1: per-tenant p99 put latency vs budget."""
+    budgets_ms = [3, 4, 6, 8, 12, 16, 24, 32]
+    slos = [(N1, int(2 * b * 1e6), int(b * 1e6)) for b in budgets_ms]
+    res = {"budgets_ms": budgets_ms, "bw_all_GBps": bw / 1e9,
+           "rate_least_GBps": [round(N1 / (b / 1e3) / 1e9, 2) for b in budgets_ms]}
+    for name, kw in (("slo", dict(slos=slos, h2d_Bps=int(bw))), ("equal", {})):
+        r = cfg4(seconds, weights=(1,) * 8, **kw)
+        r["met"] = [p <= b for p, b in zip(r["p99_ms"], budgets_ms)]
+        res[name] = r
+    return res
 
 
 def cfg4_isolation(seconds=2.0):
@@ -219,6 +240,11 @@ def main():
 
     def save():
         json.dump(res, open(out, "w"), indent=1)
+    if len(sys.argv) > 2 and sys.argv[2] == "slo":
+        res["cfg4_slo"] = cfg4_slo(3.0)
+        print("cfg4_slo", json.dumps(res["cfg4_slo"]), flush=True)
+        save()
+        return
     if len(sys.argv) > 2 and sys.argv[2] == "cfg5i":
         res["cfg5_interleaved"] = []
         for frac in (0.3, 0.1):
