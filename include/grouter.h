@@ -138,6 +138,7 @@ typedef struct {
   uint64_t timed_ns;                     /* sum of their durations              */
   uint64_t timed_bytes;                  /* sum of the bytes they moved         */
   uint64_t restore_count, restore_bytes; /* host -> home GPU restores (L260)    */
+  uint64_t pool_target[GROUTER_MAX_GPUS]; /* histogram-driven pool size (R44)    */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
@@ -283,6 +284,16 @@ grouter_status grouter_plan(grouter_ctx *ctx, int32_t src_loc, int32_t dst_dev, 
 /* Route set R(dst) (L178, precomputed at init, L271). */
 grouter_status grouter_route_set(grouter_ctx *ctx, int32_t dst_dev, int32_t *out, uint32_t cap,
                                  uint32_t *n_out);
+/* Histogram-driven pool size of GPU dev at the current clock (PAPER.md
+ * §4.4.1, Fig. 11a; R44): per function (workflow,
+ * function id, GPU) the library samples, at every put/alloc placed in that
+ * GPU's pool, the arrival time, the page charge and the function's resident
+ * object count; R_window/R_size/R_con are nearest-rank p99s over the last
+ * 1024 samples; target = min(cap, max(pool_floor_bytes, sum of
+ * R_size * R_con over functions with now <= last arrival + R_window)).
+ * The background thread pre-maps the pool up to the target (pre-warming)
+ * and trims it down to max(used, target) + one 64 MiB segment. */
+grouter_status grouter_pool_target(grouter_ctx *ctx, int32_t dev, uint64_t *target);
 /* Current location of an object: GPU index or GROUTER_HOST. */
 grouter_status grouter_where(grouter_ctx *ctx, grouter_oid oid, int32_t *loc);
 grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);

@@ -48,6 +48,11 @@ grouter_status grouter_test_launch_cost(int kind, int n, int blocks, void *strea
  * the full length needed in *len (may be NULL). */
 grouter_status grouter_test_dump(grouter_ctx *ctx, char *buf, uint64_t cap, uint64_t *len);
 
+/* Fixes the clock the pool-sizing samples and targets use (fixed != 0) to
+ * t_ns, or returns to the monotonic clock (fixed == 0).  For deterministic
+ * parity traces (R44). */
+grouter_status grouter_test_set_clock(grouter_ctx *ctx, int32_t fixed, uint64_t t_ns);
+
 #ifdef __cplusplus
 }
 #endif

@@ -27,9 +27,11 @@ def digest(b: np.ndarray) -> str:
 
 
 def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
-        multipath: bool = True, keep_bytes: bool = False, restore: bool = False) -> dict:
+        multipath: bool = True, keep_bytes: bool = False, restore: bool = False,
+        pool_floor: int | None = None, targets: bool = False) -> dict:
+    kw = {} if pool_floor is None else {"pool_floor": pool_floor}
     orc = Oracle(calib, host_store_bytes=host_store_bytes, pool_cap=pool_cap,
-                 multipath=multipath, restore=restore)
+                 multipath=multipath, restore=restore, **kw)
     recs = []
     seed_of = {}          # oid -> payload seed
     for i, op in enumerate(ops):
@@ -94,6 +96,8 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
             st, out = orc.free(op["fn"], oid)
         elif k == "weight":
             st, out = orc.set_weight(op["wf"], op["w"])
+        elif k == "tick":
+            st, out = orc.tick(op["t_ns"])
         elif k == "slo":
             st, out = orc.set_slo(op["wf"], op["data"], op["slo_ns"], op["infer_ns"])
         elif k == "next_use":
@@ -115,6 +119,8 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
         rec["status"] = STATUS[st]
         rec["victims"] = list(orc.victims)
         rec["restored"] = list(orc.restored)
+        if targets:
+            rec["pool_target"] = [orc.pool_target(d) for d in range(orc.ngpu)]
         rec["used"] = list(orc.used)
         rec["host_used"] = orc.host_used
         if oid:

@@ -60,6 +60,21 @@ Obj *lookup_live(grouter_ctx *c, grouter_oid oid) {
   return &it->second;
 }
 
+// Resident-object counts per (wf, fid, gpu) and the pool-sizing sample of a
+// placement (L250-L256, R44).
+static void resident_add(grouter_ctx *c, const Obj &o, int64_t delta) {
+  if (o.loc < 0) return;
+  uint64_t &r = c->resident[std::make_tuple(o.wf, o.fid, o.loc)];
+  r += delta;
+}
+
+static void observe(grouter_ctx *c, const Obj &o) {
+  if (o.loc < 0) return;
+  resident_add(c, o, 1);
+  const auto key = std::make_tuple(o.wf, o.fid, o.loc);
+  c->hists[key].observe(c->clock_fixed ? c->clock_ns : now_ns(), charge(o.n), c->resident[key]);
+}
+
 // Proactive restore (L260-L262, R42): once storage on GPU d is
 // released (or its cap raised), objects migrated away from d come back while
 // they fit under the cap -- objects with a next-use hint first, queue head
@@ -87,6 +102,7 @@ void restore(grouter_ctx *c, int d) {
     D.used += ch;
     c->host_used -= ch;
     o->loc = d;
+    resident_add(c, *o, 1);
     o->ptr = p;
     o->home = -1;
     c->restored.push_back(o->oid);
@@ -112,6 +128,7 @@ void release_storage_if_dead(grouter_ctx *c, Obj &o) {
     host_free(c, o.ptr, ch, std::move(f));
   } else {
     const int d = o.loc;
+    resident_add(c, o, -1);
     c->dev[d].used -= ch;
     dev_free(c, d, o.ptr, ch, std::move(f));
     c->objects.erase(o.oid);
@@ -152,6 +169,7 @@ void spill(grouter_ctx *c, Obj &o) {
   uint8_t *h = host_alloc(c, ch);
   const int d = o.loc;
   spill_copy(c, o, h);            // D2H + device pages to quarantine
+  resident_add(c, o, -1);
   o.home = d;
   o.loc = GROUTER_HOST;
   o.ptr = h;
@@ -447,6 +465,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
     }
   }
   *out = o.oid;
+  observe(c, o);
   c->objects.emplace(o.oid, std::move(o));
   if (blocking && (c->replay || !done.empty())) block_on(c, g, done);
   return GROUTER_OK;
@@ -482,6 +501,7 @@ grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, i
   o.last_access = c->seq;
   *buf = ptr;
   *out = o.oid;
+  observe(c, o);
   c->objects.emplace(o.oid, std::move(o));
   return GROUTER_OK;
   API_CATCH(c)
@@ -974,9 +994,26 @@ grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
     out->used[i] = c->dev[i].used;
     out->cap[i] = c->dev[i].cap;
     out->mapped[i] = c->dev[i].pool.mapped;
+    out->pool_target[i] = pool_target(c, (int)i);
   }
   out->host_used = c->host_used;
   out->host_cap = c->host_cap;
+  return GROUTER_OK;
+}
+
+grouter_status grouter_pool_target(grouter_ctx *c, int32_t d, uint64_t *target) {
+  if (!c || !target) return fail(GROUTER_EINVAL, "pool_target: null argument");
+  Guard g(c);
+  if (d < 0 || d >= (int)c->dev.size()) return fail(GROUTER_EINVAL, "pool_target: bad device");
+  *target = pool_target(c, d);
+  return GROUTER_OK;
+}
+
+grouter_status grouter_test_set_clock(grouter_ctx *c, int32_t fixed, uint64_t t_ns) {
+  if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  Guard g(c);
+  c->clock_fixed = fixed != 0;
+  c->clock_ns = t_ns;
   return GROUTER_OK;
 }
 

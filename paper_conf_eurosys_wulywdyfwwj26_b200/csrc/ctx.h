@@ -60,6 +60,17 @@ struct DevicePool {
   void destroy();
 };
 
+// Pool-sizing samples of one function on one GPU (L250-L256, Fig. 11a; R44):
+// arrival times, page charges and resident-object counts, last kHist each.
+struct FuncHist {
+  static constexpr size_t kHist = 1024;
+  std::deque<uint64_t> arrivals, sizes, cons;
+  void observe(uint64_t t, uint64_t size, uint64_t con);
+  uint64_t r_window() const;   // p99 inter-arrival interval, 0 with < 2 arrivals
+  uint64_t data_size() const;  // Data_size = R_size * R_con (saturating)
+  bool active(uint64_t t) const { return !arrivals.empty() && t <= arrivals.back() + r_window(); }
+};
+
 struct HostStore {
   uint8_t *base = nullptr;
   uint64_t size = 0;
@@ -217,6 +228,11 @@ struct grouter_ctx {
   std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
   std::unordered_map<uint32_t, uint32_t> weights;
   std::map<uint32_t, std::array<uint64_t, 3>> slos;    // wf -> (data, slo_ns, infer_ns), R43
+  // pool sizing (R44): per (wf, fid, gpu) histograms and resident counts
+  std::map<std::tuple<uint32_t, uint32_t, int>, gr::FuncHist> hists;
+  std::map<std::tuple<uint32_t, uint32_t, int>, uint64_t> resident;
+  bool clock_fixed = false;                            // grouter_test_set_clock
+  uint64_t clock_ns = 0;
   uint64_t seq = 0, next_oid = 1, xfer_seq = 0;
   uint64_t epoch = 1, flushed_epoch = 0;               // replay grounding
   std::vector<grouter_oid> victims;
@@ -276,6 +292,7 @@ void ipc_shutdown(grouter_ctx *c);
 std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, int local_phys);
 void ipc_unmap(RemoteMap &m);
 // pool.cpp
+uint64_t pool_target(grouter_ctx *c, int logical);   // R44 target at the current clock
 uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len);   // may grow the pool
 void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f);
 uint8_t *host_alloc(grouter_ctx *c, uint64_t len);

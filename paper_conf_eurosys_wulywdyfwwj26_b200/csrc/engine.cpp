@@ -750,11 +750,21 @@ static void daemon_main(grouter_ctx *c) {
       auto now = std::chrono::steady_clock::now();
       if (now - last_trim > std::chrono::milliseconds(50)) {  // I/O thread: reclaim (L269)
         last_trim = now;
-        for (auto &d : c->dev) {
+        for (size_t i = 0; i < c->dev.size(); ++i) {
+          LogicalDev &d = c->dev[i];
           DeviceGuard g(d.phys);
           d.pool.heap.reclaim();
-          uint64_t floor_ = std::min<uint64_t>(c->cfg.pool_floor_bytes, d.cap);
-          d.pool.trim(std::max<uint64_t>(d.used, floor_) + (64ull << 20));
+          // histogram-driven size (L250-L256, R44): pre-warm one segment per
+          // tick toward the target, trim back to max(used, target)
+          const uint64_t tgt = pool_target(c, (int)i);
+          if (d.pool.mapped < tgt) {
+            try {
+              d.pool.grow(std::min<uint64_t>(tgt - d.pool.mapped, 64ull << 20));
+            } catch (const Error &) {
+              // HBM short: pre-warming is best effort
+            }
+          }
+          d.pool.trim(std::max<uint64_t>(d.used, tgt) + (64ull << 20));
         }
         c->host.heap.reclaim();
       }

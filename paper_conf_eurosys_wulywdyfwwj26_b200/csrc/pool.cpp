@@ -12,6 +12,7 @@
 // completed (stream-ordered reuse without host synchronisation on the hot
 // path); the pool grows by mapping more segments at its end and trims
 // trailing free segments back toward the warm floor.
+#include <algorithm>
 #include <chrono>
 #include <cstdio>
 #include <thread>
@@ -166,6 +167,50 @@ uint64_t PageHeap::tail_free(uint64_t end) const {
   if (free_runs.empty()) return 0;
   auto it = std::prev(free_runs.end());
   return it->first + it->second == end ? it->second : 0;
+}
+
+// ------------------------------------------------------------------ pool sizing (R44)
+// Nearest-rank p99: the ceil(0.99 m)-th smallest sample.
+static uint64_t p99(const std::deque<uint64_t> &xs) {
+  if (xs.empty()) return 0;
+  std::vector<uint64_t> v(xs.begin(), xs.end());
+  const size_t k = (99 * v.size() + 99) / 100;
+  std::nth_element(v.begin(), v.begin() + (k - 1), v.end());
+  return v[k - 1];
+}
+
+void FuncHist::observe(uint64_t t, uint64_t size, uint64_t con) {
+  arrivals.push_back(t);
+  sizes.push_back(size);
+  cons.push_back(con);
+  if (arrivals.size() > kHist + 1) arrivals.pop_front();
+  if (sizes.size() > kHist) sizes.pop_front();
+  if (cons.size() > kHist) cons.pop_front();
+}
+
+uint64_t FuncHist::r_window() const {
+  std::deque<uint64_t> iv;
+  for (size_t i = 1; i < arrivals.size(); ++i) iv.push_back(arrivals[i] - arrivals[i - 1]);
+  return p99(iv);
+}
+
+uint64_t FuncHist::data_size() const {
+  const unsigned __int128 d = (unsigned __int128)p99(sizes) * p99(cons);
+  return d > UINT64_MAX ? UINT64_MAX : (uint64_t)d;
+}
+
+static uint64_t clock_now(const grouter_ctx *c) { return c->clock_fixed ? c->clock_ns : now_ns(); }
+
+// target(d, now) = min(cap, max(floor, MemPool_size)), MemPool_size = sum of
+// Data_size over the functions whose reservation window is open (L254-L256).
+uint64_t pool_target(grouter_ctx *c, int d) {
+  const uint64_t t = clock_now(c);
+  unsigned __int128 sum = 0;
+  for (auto &kv : c->hists)
+    if (std::get<2>(kv.first) == d && kv.second.active(t)) sum += kv.second.data_size();
+  uint64_t m = sum > UINT64_MAX ? UINT64_MAX : (uint64_t)sum;
+  m = std::max<uint64_t>(m, c->cfg.pool_floor_bytes);
+  return std::min<uint64_t>(m, c->dev[d].cap);
 }
 
 // ------------------------------------------------------------------ device pool

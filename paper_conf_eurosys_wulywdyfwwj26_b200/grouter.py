@@ -73,6 +73,7 @@ class grouter_stats_t(C.Structure):
         ("link_bytes", (C.c_uint64 * MAX_GPUS) * 3), ("kernel_launches", C.c_uint64),
         ("rounds", C.c_uint64), ("timed_launches", C.c_uint64), ("timed_ns", C.c_uint64),
         ("timed_bytes", C.c_uint64), ("restore_count", C.c_uint64), ("restore_bytes", C.c_uint64),
+        ("pool_target", C.c_uint64 * MAX_GPUS),
     ]
 
 
@@ -123,6 +124,8 @@ SIGNATURES = {
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
+    "grouter_pool_target": (_ST, [_CTX, C.c_int32, C.POINTER(_U64)]),
+    "grouter_test_set_clock": (_ST, [_CTX, C.c_int32, _U64]),
     "grouter_set_tenant_slo": (_ST, [_CTX, C.c_uint32, _U64, _U64, _U64]),
     "grouter_slo_weights": (_ST, [C.c_uint32, C.POINTER(C.c_uint32), C.POINTER(_U64), C.POINTER(_U64),
                                   C.POINTER(_U64), _U64, C.POINTER(C.c_uint32)]),
@@ -325,6 +328,15 @@ class Ctx:
     # control
     def set_tenant_weight(self, wf, w):
         return self.lib.grouter_set_tenant_weight(self.h, wf, w)
+
+    def pool_target(self, dev):
+        v = C.c_uint64(0)
+        check(self.lib.grouter_pool_target(self.h, dev, C.byref(v)), "pool_target")
+        return v.value
+
+    def set_clock(self, t_ns=None):
+        """Fix the pool-sizing clock to t_ns (None: back to the monotonic clock)."""
+        return self.lib.grouter_test_set_clock(self.h, 0 if t_ns is None else 1, t_ns or 0)
 
     def set_tenant_slo(self, wf, data_bytes, slo_ns, infer_ns):
         return self.lib.grouter_set_tenant_slo(self.h, wf, data_bytes, slo_ns, infer_ns)

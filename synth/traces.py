@@ -85,6 +85,9 @@ class Builder:
     def weight(self, wf, w):
         return self._add({"op": "weight", "wf": wf, "w": w})
 
+    def tick(self, t_ns):
+        return self._add({"op": "tick", "t_ns": t_ns})
+
     def slo(self, wf, data, slo_ns, infer_ns):
         return self._add({"op": "slo", "wf": wf, "data": data, "slo_ns": slo_ns, "infer_ns": infer_ns})
 
@@ -353,4 +356,37 @@ def random_trace(rng: random.Random, n_gpus: int, n_ops: int = 200, max_n: int =
     for g, f in gets:
         b.release(f, g)
     b.flush()
+    return b.ops
+
+
+def sizing_trace(rng: random.Random, n_gpus: int, n_ops: int = 150, run_seed: int = 77) -> list:
+    """Pool-sizing trace (L250-L256, R44): a clock that advances by bursty
+    intervals (tick ops), functions on several GPUs that put/alloc outputs of
+    varying size, consumers that drain some of them, and idle gaps long
+    enough for reservation windows to lapse."""
+    b = Builder(run_seed)
+    t = 0
+    live = []
+    fns = [fn(rng.randint(1, 3), rng.randint(1, 3), rng.randrange(n_gpus)) for _ in range(5)]
+    for _ in range(n_ops):
+        r = rng.random()
+        if r < 0.25:
+            t += rng.choice([1, 10, 100, 1000]) * 10 ** 3 * rng.randint(1, 5)
+            if rng.random() < 0.1:
+                t += 10 ** 9                       # idle gap: windows lapse
+            b.tick(t)
+        elif r < 0.6:
+            f = rng.choice(fns)
+            n = rng.choice([0, 1, 4096, 2 * MiB, 3 * MiB + 5, rng.randint(1, 9 * MiB)])
+            if rng.random() < 0.5:
+                live.append((f, b.put(f, n, consumers=1)))
+            else:
+                o = b.alloc(f, n, consumers=1)
+                b.seal(f, o)
+                live.append((f, o))
+        elif live:
+            f, o = live.pop(rng.randrange(len(live)))
+            c = fn(f["wf"], 9, rng.randrange(n_gpus))
+            b.get_into(c, o)
+    b.flush()                                      # replay mode dispatches on flush (R31)
     return b.ops

@@ -55,7 +55,7 @@ def wait_streams(streams, timeout=60.0):
 
 class LibRunner:
     def __init__(self, calib, host_store_bytes=1 << 30, pool_cap=None, replay=True, flags=0,
-                 keep_bytes=False, pool_floor=64 << 20, chunk_bytes=None):
+                 keep_bytes=False, pool_floor=64 << 20, chunk_bytes=None, targets=False):
         self.calib = calib
         n = calib["n_gpus"]
         self.n = n
@@ -67,6 +67,9 @@ class LibRunner:
             kw["chunk_bytes"] = chunk_bytes
         self.ctx = G.Ctx(G.config_from_calib(calib, **kw))
         self.replay = replay
+        self.targets = targets
+        if targets:
+            self.ctx.set_clock(0)        # the oracle's clock starts at 0 (R44)
         self.streams = [torch.cuda.Stream(device=p) for p in self.phys]
         self.upload = [torch.cuda.Stream(device=p) for p in self.phys]
         self.keep_bytes = keep_bytes
@@ -213,6 +216,8 @@ class LibRunner:
                 st = ctx.free(self._fnc(op["fn"]), oid)
             elif k == "weight":
                 st = ctx.set_tenant_weight(op["wf"], op["w"])
+            elif k == "tick":
+                st = ctx.set_clock(op["t_ns"])
             elif k == "slo":
                 st = ctx.set_tenant_slo(op["wf"], op["data"], op["slo_ns"], op["infer_ns"])
             elif k == "next_use":
@@ -231,6 +236,8 @@ class LibRunner:
                 print("   ->", G.STATUS[st], G.last_error() if st else "", flush=True)
             rec["victims"] = ctx.victims()
             rec["restored"] = ctx.restored()
+            if self.targets:
+                rec["pool_target"] = [ctx.pool_target(d) for d in range(self.n)]
             s = ctx.stats()
             rec["used"] = [s.used[d] for d in range(self.n)]
             rec["host_used"] = s.host_used
@@ -263,6 +270,8 @@ def compare(orc_out, lib_out, check_dispatch=True):
         assert l.get("where") == o.get("where"), (ctx, o.get("where"), l.get("where"))
         assert l["victims"] == o["victims"], (ctx, o["victims"], l["victims"])
         assert l.get("restored", []) == o.get("restored", []), (ctx, o.get("restored"), l.get("restored"))
+        if "pool_target" in o and "pool_target" in l:
+            assert l["pool_target"] == o["pool_target"], (ctx, o["pool_target"], l["pool_target"])
         assert l["used"] == o["used"], (ctx, o["used"], l["used"])
         assert l["host_used"] == o["host_used"], ctx
         if o["status"] == "OK" and o["op"] in ("get", "get_into"):

@@ -118,7 +118,8 @@ def _copy_exactly_once(tma, src_off, dst_off):
 # ------------------------------------------------------------------ trace parity
 def _both(ops, calib, replay=True, keep=True, restore=False, **kw):
     orc = orun.run(ops, calib, host_store_bytes=kw.get("host_store_bytes", 1 << 30),
-                   pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore)
+                   pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore,
+                   pool_floor=kw.get("pool_floor", 64 << 20), targets=kw.get("targets", False))
     if restore:
         kw["flags"] = kw.get("flags", 0) | G.RESTORE
     r = LibRunner(calib, replay=replay, keep_bytes=keep, **kw)
@@ -231,6 +232,56 @@ def test_cfg4_slo_dispatch_parity(k):
     ops = T.cfg4(k, rounds=2, scale=64, slos=T.CFG4_SLOS)
     orc, lib_out = _both(ops, calib)
     assert compare(orc, lib_out) > 0
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_pool_sizing_targets(seed):
+    """Histogram-driven pool size (L250-L256, R44): with a fixed clock the
+    library's per-GPU target equals the oracle's after every op."""
+    rng = random.Random(4000 + seed)
+    k = rng.choice([1, 2, 3])
+    calib = C.virtual(k) if k > 1 else dict(C.b200_hgx(1), device_map=[0])
+    ops = T.sizing_trace(rng, k)
+    caps = [rng.choice([16, 64, 1024]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, pool_cap=caps, pool_floor=8 * MiB, targets=True,
+                         host_store_bytes=256 * MiB)
+    compare(orc, lib_out)
+    assert any(t > 8 * MiB for r in lib_out["records"] for t in r["pool_target"])
+
+
+def test_pool_prewarm_and_trim():
+    """The background thread maps the pool up to the target and trims it
+    back once the reservation windows lapse (real clock)."""
+    import time as _t
+    calib = dict(C.b200_hgx(1), device_map=[0])
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED],
+                                    pool_floor_bytes=64 * MiB))
+    try:
+        f = G.fn(1, 1, 0)
+        src = torch.empty(9 * MiB, dtype=torch.uint8, device="cuda")
+        ctx.set_clock(0)
+        oids = []
+        for i in range(40):                     # 40 live 10 MiB outputs, 1 ms apart
+            ctx.set_clock(i * 10 ** 6)
+            st, oid = ctx.put(f, src.data_ptr(), 9 * MiB, G.NOHINT, 0, 0)
+            assert st == G.OK
+            oids.append(oid)
+        for oid in oids:
+            assert ctx.free(f, oid) == G.OK
+        tgt = ctx.pool_target(0)
+        assert tgt == 40 * 10 * MiB                 # R_size 10 MiB x R_con 40
+        t0 = _t.time()
+        while ctx.stats().mapped[0] < tgt and _t.time() - t0 < 5:
+            _t.sleep(0.05)
+        assert ctx.stats().mapped[0] >= tgt         # pre-warmed (already grown by the puts)
+        ctx.set_clock(10 ** 12)                     # long idle: window lapsed
+        assert ctx.pool_target(0) == 64 * MiB
+        t0 = _t.time()
+        while ctx.stats().mapped[0] > 64 * MiB + 64 * MiB and _t.time() - t0 < 5:
+            _t.sleep(0.05)
+        assert ctx.stats().mapped[0] <= 128 * MiB   # trimmed to floor + one segment
+    finally:
+        ctx.close()
 
 
 def test_full_size_cfg1_sampled():
