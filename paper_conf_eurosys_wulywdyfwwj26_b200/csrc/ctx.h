@@ -102,6 +102,10 @@ struct Xfer {
     Waitable w;
   };
   std::vector<Waiter> waiters;              // caller-stream waits deferred until submission
+  // completion evidence when no word is published: an event recorded on the
+  // caller stream after a direct launch that moved the whole transfer (its
+  // completion slot is handed back at once)
+  EventRef done_ev;
   bool done() const;
 };
 using XferRef = std::shared_ptr<Xfer>;

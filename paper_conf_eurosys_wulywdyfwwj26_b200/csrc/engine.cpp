@@ -132,6 +132,13 @@ void host_wait(const Fences &f, double timeout_s) {
 
 // ------------------------------------------------------------------ transfers
 void done_fences(const XferRef &x, Fences &f) {
+  if (x->done_ev) {
+    Waitable w;
+    w.ev = x->done_ev;
+    w.epoch = x->epoch;
+    f.push_back(w);
+    return;
+  }
   for (uint32_t p = 0; p < x->npath; ++p) {
     if (!x->total[p]) continue;
     Waitable w;
@@ -144,6 +151,7 @@ void done_fences(const XferRef &x, Fences &f) {
 }
 
 bool Xfer::done() const {
+  if (done_ev) return cudaEventQuery(done_ev->ev) == cudaSuccess;
   for (uint32_t p = 0; p < npath; ++p)
     if (total[p] && (int32_t)(words[p] - target[p]) < 0) return false;
   return true;
@@ -335,14 +343,21 @@ static void after_submit(grouter_ctx *c, const std::vector<ChunkItem> &items) {
 // One or more kernel launches for `items` (in order): contiguous chunks are
 // coalesced into one run while the parameter block is built; a launch ends
 // when its block is full (kMaxRoundChunks runs or kMaxPublish publishes).
+// deferred_pub (direct launches of one whole transfer): when the engine needs
+// a host-side publish, skip the stream writes and report it -- the caller
+// records an event instead (a stream write after a kernel costs ~3.5 us of
+// GPU time per launch and breaks programmatic dependent launch; an event
+// record costs neither).
 static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *scratch,
-                         const std::vector<ChunkItem> &items, const uint64_t *src_override) {
+                         const std::vector<ChunkItem> &items, const uint64_t *src_override,
+                         bool *deferred_pub = nullptr) {
   if (!c->params) c->params = new CopyParamsHost();
   CopyParams *p = &c->params->p;
   PhysDev &pd = *c->phys.at(s.phys);
   const bool prof = (c->cfg.flags & GROUTER_PROFILE) != 0;
   size_t i = 0;
   std::vector<ChunkItem> part;
+  bool first = true;
   bool local = true;  // every destination in the launching GPU's memory -> GPU-scope fences
   for (auto &it : items)
     local &= it.dst_logical >= 0 && c->dev[it.dst_logical].phys == s.phys;
@@ -393,15 +408,19 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
     HostProf &hp = hprof();
     uint64_t tl = hp.on ? now_ns() : 0;
     if (hp.on) hp.t[6] += tl - tparams;
+    // host-side completion only where an event can stand in for the words
+    // (a whole direct transfer); elsewhere the kernel publishes in-kernel,
+    // which costs less GPU time than a stream write after the launch
     bool host_pub = false;
+    const bool only = first && i == items.size();  // one launch moves every item
+    first = false;
     int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm,
-                        (c->cfg.flags & GROUTER_COPY_TMA) != 0, st, &host_pub);
+                        (c->cfg.flags & GROUTER_COPY_TMA) != 0, st,
+                        deferred_pub && only ? &host_pub : nullptr);
     if (hp.on) hp.t[7] += now_ns() - tl;
     if (e != 0)
       throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
-    if (host_pub)  // stream order: the writes land after every byte of the launch
-      for (uint32_t k = 0; k < p->n_pub; ++k)
-        GR_CU(drv().streamWriteValue32((CUstream)st, (CUdeviceptr)p->pub[k].word, p->pub[k].value, 0));
+    if (host_pub) *deferred_pub = true;
     if (prof) {
       GR_CUDA(cudaEventRecord(pr.stop, st));
       c->prof.push_back(pr);
@@ -670,7 +689,15 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     pd.next_scratch = (k + 1) % pd.n_scratch;
     for (auto &w : pd.scratch_busy[k])
       if (!w.done()) host_wait(Fences{w});
-    launch_round(c, s, caller, pd.scratch + 2 * k, items, nullptr);
+    // one launch moves the whole transfer: complete it by an event, not words
+    static const bool ev_done = !getenv("GR_NO_EVDONE");
+    const bool whole = ev_done && x->submitted_chunks == 0 && items.size() == x->nchunks && x->waiters.empty();
+    bool deferred = false;
+    launch_round(c, s, caller, pd.scratch + 2 * k, items, nullptr, whole ? &deferred : nullptr);
+    if (deferred) {
+      x->done_ev = record(c, caller, s.phys);
+      for (uint32_t p = 0; p < x->npath; ++p) c->slot_final[x->slot][p] -= x->total[p];  // slot back
+    }
     for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
     c->stats.rounds++;
     after_submit(c, items);
@@ -927,6 +954,12 @@ void engine_shutdown(grouter_ctx *c) {
   if (c->host.base) cudaFreeHost(c->host.base);
   if (c->bounce) cudaFreeHost(c->bounce);
   if (c->words) cudaFreeHost(c->words);
+  // fences may hold pooled events: drop them while the pools are alive
+  for (auto &kv : c->objects) {
+    kv.second.ready.clear();
+    kv.second.readers.clear();
+  }
+  for (auto &kv : c->leases) kv.second.fill.clear();
   c->phys.clear();
 }
 

@@ -21,6 +21,8 @@
 #include "../../include/grouter_testing.h"
 #include "kernels.h"
 
+typedef int CUresult_t;
+
 namespace gr {
 
 constexpr int kThreads = 256;
@@ -513,15 +515,19 @@ __global__ void __launch_bounds__(kThreads) gr_copy_gs(const __grid_constant__ K
   finish_round(p);
 }
 
-// Launch with programmatic stream serialization (PDL) when GR_PDL=1 (hides
-// the inter-kernel gap, ~0.8 us/launch, but the Ex launch path costs host
-// time and the data path is near host-bound; measured both ways).
+// Launch with programmatic stream serialization (PDL; GR_PDL=0 disables):
+// the next copy's CTAs are scheduled while this one drains and block in
+// griddepcontrol.wait before touching memory, which hides the inter-kernel
+// gap (~1.2-2.2 us per 38.5 MB launch measured, tools/pubbench.sh).  It pays
+// only when nothing but kernels/events sit between launches: a stream write
+// (cuStreamWriteValue32) after a kernel breaks the overlap, which is why
+// direct launches complete by an event (engine.cpp try_direct).
 template <class KP>
 static void launch_pdl(void (*kern)(KP), uint64_t grid, int block, int smem, cudaStream_t s, const KP &p) {
   static int pdl = -1;
   if (pdl < 0) {
     const char *e = getenv("GR_PDL");
-    pdl = (e && e[0] == '1') ? 1 : 0;  // opt-in: cudaLaunchKernelEx costs host time
+    pdl = (e && e[0] == '0') ? 0 : 1;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
@@ -905,7 +911,29 @@ extern "C" grouter_status grouter_test_copy(void *dst_base, const void *src_base
   p->tile_prefix[n_chunks] = t;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  int e = launch_copy(*p, sms, 2, tma && !counts, stream);
+  // diagnostic knob GR_TEST_PUB: 0 = in-kernel completion (default), 1 = no
+  // completion, 2 = host-published (stream write after the launch), 3 =
+  // event record after the launch
+  static int pub = getenv("GR_TEST_PUB") ? atoi(getenv("GR_TEST_PUB")) : 0;
+  static uint32_t *word = nullptr;
+  static cudaEvent_t ev = nullptr;
+  typedef CUresult_t (*WriteFn)(cudaStream_t, unsigned long long, unsigned, unsigned);
+  static WriteFn wv = nullptr;
+  if (pub >= 2 && !word) {
+    cudaHostAlloc(&word, 64, cudaHostAllocMapped);
+    cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+    cudaDriverEntryPointQueryResult q;
+    cudaGetDriverEntryPoint("cuStreamWriteValue32", (void **)&wv, cudaEnableDefault, &q);
+  }
+  bool host_pub = false;
+  int e = launch_copy(*p, sms, 2, tma && !counts, stream, pub >= 1 ? &host_pub : nullptr);
+  if (pub == 2 && wv) {
+    void *dptr = nullptr;
+    cudaHostGetDevicePointer(&dptr, word, 0);
+    wv((cudaStream_t)stream, (unsigned long long)dptr, 1, 0);
+  } else if (pub == 3) {
+    cudaEventRecord(ev, (cudaStream_t)stream);
+  }
   delete p;
   return e == 0 ? GROUTER_OK : GROUTER_ECUDA;
 }

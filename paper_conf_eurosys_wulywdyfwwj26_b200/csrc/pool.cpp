@@ -13,6 +13,10 @@
 // path); the pool grows by mapping more segments at its end and trims
 // trailing free segments back toward the warm floor.
 #include <algorithm>
+#include <csignal>
+#include <cstdio>
+#include <dlfcn.h>
+#include <execinfo.h>
 #include <chrono>
 #include <cstdio>
 #include <thread>
@@ -22,6 +26,28 @@
 namespace gr {
 
 // ------------------------------------------------------------------ host profile
+// GROUTER_BT=1: print a raw backtrace on SIGABRT/SIGSEGV (debug aid; map
+// the offsets with addr2line -e libgrouter.so).
+static void bt_handler(int sig) {
+  void *fr[64];
+  int n = backtrace(fr, 64);
+  Dl_info di;
+  for (int i = 0; i < n; ++i) {
+    if (dladdr(fr[i], &di) && di.dli_fname)
+      fprintf(stderr, "  #%d %s +0x%lx\n", i, di.dli_fname, (unsigned long)((char *)fr[i] - (char *)di.dli_fbase));
+  }
+  ::signal(sig, SIG_DFL);
+  ::raise(sig);
+}
+static int bt_init = [] {
+  const char *e = getenv("GROUTER_BT");
+  if (e && e[0] == '1') {
+    ::signal(SIGABRT, bt_handler);
+    ::signal(SIGSEGV, bt_handler);
+  }
+  return 0;
+}();
+
 HostProf &hprof() {
   static HostProf h = [] {
     HostProf x;
