@@ -226,6 +226,28 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
         out[name] = {"routes": routes, "GBps": round(nbytes / min(ts) / 1e9, 2)}
         ctx.close()
     out["speedup"] = round(out["striped"]["GBps"] / out["direct"]["GBps"], 2)
+    # gFn-host (L178, Fig. 5a): a GPU0 object read into host memory by a cFn,
+    # direct D2H vs striped over R(0) (GROUTER_D2H_MULTIPATH)
+    src = torch.empty(nbytes, dtype=torch.uint8, device="cuda:0")
+    for name, flags in (("d2h_direct", 0), ("d2h_striped", G.D2H_MULTIPATH)):
+        ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, flags=flags,
+                                        pool_cap=[G.UNLIMITED] * world, pool_floor_bytes=64 << 20))
+        g0, c0 = G.fn(9, 1, 0), G.fn(9, 2, G.HOST)
+        st, oid = ctx.put(g0, src.data_ptr(), nbytes, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        ctx.sync()
+        ts = []
+        for r in range(reps + 1):
+            t0 = time.perf_counter()
+            st, nn = ctx.get_into(c0, oid, host.data_ptr(), nbytes, 0)
+            G.check(st, "get_into")
+            dt = time.perf_counter() - t0
+            if r:
+                ts.append(dt)
+        out[name] = {"GBps": round(nbytes / min(ts) / 1e9, 2)}
+        ctx.free(g0, oid)
+        ctx.close()
+    out["d2h_speedup"] = round(out["d2h_striped"]["GBps"] / out["d2h_direct"]["GBps"], 2)
     return out
 
 

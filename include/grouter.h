@@ -59,6 +59,9 @@ extern "C" {
 #define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
 #define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
 #define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream */
+#define GROUTER_D2H_MULTIPATH 0x80u/* gFn-host striping (L178, Fig. 5a; R45): a GPU
+                                      object read into host memory is split over R(src) like a
+                                      host->GPU plan; route r's copy engine moves its share      */
 #define GROUTER_RESTORE       0x40u/* proactive restore (L260-L262): when pool storage is released
                                       or a cap is raised, objects migrated away from that GPU come
                                       back while they fit (R42)                      */
@@ -276,8 +279,9 @@ grouter_status grouter_flush(grouter_ctx *ctx);
 grouter_status grouter_sync(grouter_ctx *ctx);
 
 /* ------------------------------------------------------------ introspection */
-/* Transfer plan (L182) for n bytes from src_loc (GPU or GROUTER_HOST) to
- * dst_dev (GPU or GROUTER_HOST).  *n_out = chunk count even if cap is short
+/* Transfer plan (L182) for n bytes of pool data from src_loc (GPU or
+ * GROUTER_HOST) to dst_dev (GPU or GROUTER_HOST); GPU -> host plans are
+ * striped when GROUTER_D2H_MULTIPATH is set.  *n_out = chunk count even if cap is short
  * (then EINVAL and nothing written). */
 grouter_status grouter_plan(grouter_ctx *ctx, int32_t src_loc, int32_t dst_dev, uint64_t n,
                             grouter_chunk *out, uint64_t cap, uint64_t *n_out);

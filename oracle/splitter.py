@@ -110,6 +110,18 @@ def plan_h2d(calib: dict, d: int, n: int, multipath: bool = True,
     return layout(n, shares, Cps, routes, g)
 
 
+def plan_d2h(calib: dict, s: int, n: int, multipath: bool = True,
+             C: int = CHUNK, g: int = GRANULE) -> list:
+    """gFn-host plan (L178, Fig. 5a: "data from GPU1 is first routed via NVLink
+    to peer GPUs ..., which concurrently stage it to host memory through their
+    PCIe links"): GPU s -> r in R(s) -> host.  The calibration measures PCIe in
+    the host->GPU direction and the reading takes it as symmetric (R45), so a
+    path s -> r -> host has the parameters of host -> r -> s and the split is
+    the O6 split of plan_h2d(s, n); route_gpu = the GPU whose copy engine
+    moves the chunk to host memory."""
+    return plan_h2d(calib, s, n, multipath, C, g)
+
+
 def plan_single(n: int, route_gpu: int, C: int = CHUNK) -> list:
     """k = 1 plan (D2D, same-GPU copy, D2H): consecutive chunks of C bytes,
     the last one clipped (L182 chunking on a single direct path)."""

@@ -284,11 +284,11 @@ int server_kind_for(int src, int dst) {
 XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc, uint64_t n,
                        const uint8_t *src, uint8_t *dst, Fences deps, bool pageable_src,
                        cudaStream_t caller = nullptr, int caller_logical = -1, bool caller_dep = false,
-                       bool *direct = nullptr) {
+                       bool *direct = nullptr, bool pool_src = true) {
   const uint64_t tst = hprof().on ? now_ns() : 0;
   std::vector<grouter_chunk> plan;
   if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
-  else c->planner.plan(src_loc, dst_loc, n, plan);
+  else c->planner.plan(src_loc, dst_loc, n, plan, pool_src);
   XferRef x = new_xfer(c, tenant, plan);
   x->deps = std::move(deps);
   x->pageable_src = pageable_src;
@@ -458,7 +458,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
       bool direct = false;
       XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr, Fences{},
                                  pageable, blocking ? nullptr : (cudaStream_t)stream, from, true,
-                                 &direct);
+                                 &direct, /*pool_src=*/false);  // the caller's buffer
       done_fences(x, done);
       o.ready = done;
       if (!blocking && !direct) order_after(c, g, (cudaStream_t)stream, done);

@@ -159,10 +159,14 @@ void Planner::plan_single(uint64_t n, int route_gpu, std::vector<grouter_chunk> 
     out.push_back({o, std::min<uint64_t>(cfg.chunk_bytes, n - o), 0, route_gpu});
 }
 
-void Planner::plan(int src, int dst, uint64_t n, std::vector<grouter_chunk> &out) const {
+void Planner::plan(int src, int dst, uint64_t n, std::vector<grouter_chunk> &out, bool pool_src) const {
   out.clear();
   if (n == 0 || (src == GROUTER_HOST && dst == GROUTER_HOST)) return;
   if (src == GROUTER_HOST) plan_h2d(dst, n, out);
+  // gFn-host (L178, Fig. 5a): GPU src -> route GPUs -> host.  PCIe is
+  // calibrated in the host->GPU direction and taken as symmetric, so the
+  // split over R(src) is the host->GPU plan of src (R45)
+  else if (dst == GROUTER_HOST && pool_src && (cfg.flags & GROUTER_D2H_MULTIPATH)) plan_h2d(src, n, out);
   else plan_single(n, src, out);  // D2D / same-GPU copy / D2H: source GPU's engine
 }
 

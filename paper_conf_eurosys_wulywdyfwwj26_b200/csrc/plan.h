@@ -33,7 +33,9 @@ struct Planner {
   // host -> d striped plan (O6); D2D/same-GPU/D2H single-path plan.
   void plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const;
   void plan_single(uint64_t n, int route_gpu, std::vector<grouter_chunk> &out) const;
-  void plan(int src_loc, int dst_loc, uint64_t n, std::vector<grouter_chunk> &out) const;
+  // pool_src: the source is library pool memory (readable by every route
+  // GPU), so a GPU -> host plan may be striped (GROUTER_D2H_MULTIPATH, R45)
+  void plan(int src_loc, int dst_loc, uint64_t n, std::vector<grouter_chunk> &out, bool pool_src = true) const;
 };
 
 }  // namespace gr

@@ -116,12 +116,15 @@ def _copy_exactly_once(tma, src_off, dst_off):
 
 
 # ------------------------------------------------------------------ trace parity
-def _both(ops, calib, replay=True, keep=True, restore=False, **kw):
+def _both(ops, calib, replay=True, keep=True, restore=False, d2h=False, **kw):
     orc = orun.run(ops, calib, host_store_bytes=kw.get("host_store_bytes", 1 << 30),
                    pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore,
-                   pool_floor=kw.get("pool_floor", 64 << 20), targets=kw.get("targets", False))
+                   pool_floor=kw.get("pool_floor", 64 << 20), targets=kw.get("targets", False),
+                   d2h_multipath=d2h)
     if restore:
         kw["flags"] = kw.get("flags", 0) | G.RESTORE
+    if d2h:
+        kw["flags"] = kw.get("flags", 0) | G.D2H_MULTIPATH
     r = LibRunner(calib, replay=replay, keep_bytes=keep, **kw)
     try:
         lib_out = r(ops)
@@ -282,6 +285,25 @@ def test_pool_prewarm_and_trim():
         assert ctx.stats().mapped[0] <= 128 * MiB   # trimmed to floor + one segment
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_d2h_striped(seed, replay):
+    """gFn-host striping (L178, R45) on virtual topologies: every GPU object
+    read into host memory is split over R(src); statuses, bytes, placements
+    and (replay) the per-server dispatch logs equal the oracle's."""
+    rng = random.Random(5000 + seed)
+    k = rng.choice([2, 3, 4])
+    calib = C.virtual(k)
+    ops = T.random_trace(rng, k, n_ops=120, max_n=9 * MiB, run_seed=seed)
+    caps = [rng.choice([16, 64]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, d2h=True, host_store_bytes=64 * MiB, pool_cap=caps)
+    compare(orc, lib_out, check_dispatch=replay)
+    striped = [r for r in orc["records"] if r["op"] in ("get", "get_into") and r["status"] == "OK"
+               and len({c["route_gpu"] for c in r.get("plan", [])}) > 1
+               and all(c.get("path", 0) >= 0 for c in r["plan"])]
+    assert striped or seed % 2, "trace should read some GPU object into host memory"
 
 
 def test_full_size_cfg1_sampled():

@@ -165,3 +165,29 @@ def test_slo_weights_parity_with_oracle(seed):
 def test_slo_weights_rejects_infeasible():
     with pytest.raises(RuntimeError):
         G.slo_weights({1: (10, 5, 5)}, 10 ** 9)
+
+
+@pytest.mark.parametrize("topo", ["pairs8", "solo4", "fig5a", "one"])
+@pytest.mark.parametrize("multipath", [True, False])
+def test_d2h_striped_plan_parity(topo, multipath):
+    """GROUTER_D2H_MULTIPATH (L178 gFn-host, R45): GPU -> host plans equal
+    oracle.splitter.plan_d2h; other directions are unchanged."""
+    calib = {"pairs8": C.b200_hgx(8), "solo4": C.b200_hgx(4, shared_pairs=False),
+             "fig5a": C.fig5a(), "one": C.b200_hgx(1)}[topo]
+    flags = G.D2H_MULTIPATH | (0 if multipath else G.NO_MULTIPATH)
+    with _plan_ctx(calib, flags=flags) as ctx:
+        for src in range(calib["n_gpus"]):
+            for size in SIZES:
+                st, got = ctx.plan(src, -1, size)
+                exp = osplit.plan_d2h(calib, src, size, multipath)
+                assert got == [(c["offset"], c["bytes"], c["path"], c["route_gpu"]) for c in exp]
+                assert ctx.plan(-1, src, size)[1] == _oracle_plan(calib, -1, src, size, multipath=multipath)
+
+
+def test_fig5a_gfn_host_routes():
+    """Fig. 5(a) (L178): "data from GPU1 is first routed via NVLink to peer
+    GPUs (GPU3, GPU5, and GPU7), which concurrently stage it to host memory";
+    GPU2 shares GPU1's PCIe switch and is excluded (0-based: GPU0 -> 2, 4, 6)."""
+    calib = C.fig5a()
+    p = osplit.plan_d2h(calib, 0, 1 << 30)
+    assert sorted({c["route_gpu"] for c in p}) == [0, 2, 4, 6]
