@@ -125,3 +125,40 @@ def dump(c: dict, path: str) -> None:
 def load(path: str) -> dict:
     with open(path) as f:
         return json.load(f)
+
+
+# NVLink topologies for Alg. 1; capacities in B/s per direction.
+NVL_LINK_Bps = 24_000_000_000        # L242 "24 GB/s or 48 GB/s per link" (V100 NVLink2)
+# DGX-V100 hybrid cube-mesh, numbered so that the paper's examples hold
+# (0-based index = paper "GPUk" - 1): GPU1-GPU4 has one link (half bandwidth,
+# L131), GPU1-GPU5 none, and Fig. 9(b)'s GPU4->GPU6->GPU7->GPU1 path exists.
+DGX_V100_LINKS = {(0, 1): 1, (0, 2): 2, (0, 3): 1, (0, 6): 2, (1, 2): 1, (1, 3): 2, (1, 4): 2,
+                  (2, 3): 2, (2, 7): 1, (3, 5): 1, (4, 5): 2, (4, 6): 1, (4, 7): 1, (5, 6): 1,
+                  (5, 7): 2, (6, 7): 2}
+
+
+def dgx_v100_topo() -> list:
+    """8x8 directed capacity matrix of the DGX-V100 NVLink mesh (Fig. 6a)."""
+    t = [[0] * 8 for _ in range(8)]
+    for (a, b), k in DGX_V100_LINKS.items():
+        t[a][b] = t[b][a] = k * NVL_LINK_Bps
+    return t
+
+
+def nvswitch_topo(n: int = 8, port_Bps: int = 900_000_000_000) -> list:
+    """HGX B200: n GPUs and one NVSwitch node (index n); every GPU has one
+    port of port_Bps per direction to the switch fabric."""
+    t = [[0] * (n + 1) for _ in range(n + 1)]
+    for g in range(n):
+        t[g][n] = t[n][g] = port_Bps
+    return t
+
+
+def random_topo(rng: random.Random, n: int) -> list:
+    """Random symmetric NVLink mesh (0-3 links per pair) for fuzzing."""
+    t = [[0] * n for _ in range(n)]
+    for a in range(n):
+        for b in range(a + 1, n):
+            k = rng.choice([0, 0, 1, 2, 3])
+            t[a][b] = t[b][a] = k * NVL_LINK_Bps
+    return t
