@@ -312,6 +312,46 @@ grouter_status grouter_restored(grouter_ctx *ctx, grouter_oid *out, uint64_t cap
 grouter_status grouter_dispatch_log(grouter_ctx *ctx, grouter_dispatch *out, uint64_t cap,
                                     uint64_t *n_out);
 
+/* ------------------------------------------------------------ NVLink path planner
+ * Contention-aware path selection, Algorithm 1 in full (§4.3.3
+ * L199-L242; R11, R46).  Host-only planner state, no GPU needed.
+ * The graph has n_nodes nodes: GPUs 0..n_gpus-1, then switch nodes (an
+ * NVSwitch is one node every GPU links to); topo is row-major n_nodes x
+ * n_nodes, topo[u*n_nodes+v] = capacity u -> v in B/s (0 = no link; the
+ * diagonal is ignored).  Paths are simple, <= max_edges edges.  On an
+ * NVSwitch topology every pair receives exactly its direct path. */
+#define GROUTER_MAX_PATH_NODES 8
+#define GROUTER_MAX_PATH_GRAPH 32
+typedef struct {
+  uint64_t bw_Bps;                         /* b_min(path) when it was taken  */
+  uint32_t func;                           /* owning function                */
+  uint32_t n_nodes;                        /* path length in nodes (edges+1) */
+  int32_t nodes[GROUTER_MAX_PATH_NODES];   /* g_s, ..., g_d                  */
+} grouter_path;
+typedef struct grouter_paths grouter_paths;
+/* NULL on bad arguments (n_nodes > GROUTER_MAX_PATH_GRAPH, max_edges + 1 >
+ * GROUTER_MAX_PATH_NODES, n_gpus > n_nodes).  Caller owns; free with
+ * grouter_paths_free. */
+grouter_paths *grouter_paths_new(uint32_t n_nodes, uint32_t n_gpus, const uint64_t *topo, uint32_t max_edges);
+void grouter_paths_free(grouter_paths *t);
+/* Alg. 1 for func moving data g_s -> g_d (GPUs): may move other functions'
+ * allocations (direct priority, balancing; they re-run the free phase).
+ * Writes func's paths (allocation order) to out[0..cap); *n_out = count
+ * (EINVAL if > cap).  ESTATE if func already holds paths (release first). */
+grouter_status grouter_paths_select(grouter_paths *t, uint32_t func, int32_t gs, int32_t gd, grouter_path *out,
+                                    uint32_t cap, uint32_t *n_out);
+/* The function finished: its bandwidth returns to BW. */
+grouter_status grouter_paths_release(grouter_paths *t, uint32_t func);
+/* Every active allocation in allocation order (EINVAL if cap is short). */
+grouter_status grouter_paths_table(grouter_paths *t, grouter_path *out, uint32_t cap, uint32_t *n_out);
+/* Chunk plan of n bytes over func's current paths (L182, L242, O6 split):
+ * path p -> grouter_chunk.path = p (allocation order), beta = its bw, alpha 0,
+ * phi = (GPU relays on p) * relay_phi_ps; route_gpu = first relay GPU (the
+ * source for a direct or switch-only path). */
+grouter_status grouter_paths_plan(grouter_paths *t, uint32_t func, uint64_t n, uint64_t chunk_bytes,
+                                  uint64_t granule, uint64_t relay_phi_ps, grouter_chunk *out, uint64_t cap,
+                                  uint64_t *n_out);
+
 /* ------------------------------------------------------------ stride scheduler
  * The tenant-share scheduler used by every server (L229 batches, stride
  * order), exposed standalone for host-side tests; needs no GPU. */

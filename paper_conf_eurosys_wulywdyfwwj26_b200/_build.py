@@ -16,7 +16,7 @@ CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgrouter.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["api.cpp", "engine.cpp", "ipc.cpp", "plan.cpp", "pool.cpp", "probe.cpp", "kernels.cu"]
+SOURCES = ["api.cpp", "engine.cpp", "ipc.cpp", "paths.cpp", "plan.cpp", "pool.cpp", "probe.cpp", "kernels.cu"]
 HEADERS = ["common.h", "ctx.h", "kernels.h", "plan.h", "stride.h"]
 
 

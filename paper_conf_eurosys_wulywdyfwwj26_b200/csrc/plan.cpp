@@ -114,11 +114,11 @@ static uint64_t path_cap(u128 T, uint64_t N, const PathModel &p, uint64_t g) {
   return lo;
 }
 
-void Planner::plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const {
+// O6 split of n bytes over paths P (route order): exact min-makespan shares,
+// canonical fill, interleaved layout with C_p-sized chunks.
+void split_plan(const std::vector<PathModel> &P, uint64_t n, uint64_t g, std::vector<grouter_chunk> &out) {
   out.clear();
-  if (n == 0) return;
-  const auto &P = paths[d];
-  const uint64_t g = cfg.granule;
+  if (n == 0 || P.empty()) return;
   const uint64_t N = ceil_div(n, g);
   // 1. T* = min { T : sum_p cap_p(T) >= N }  (bisection on integer ps)
   u128 lo = 0, hi = path_time(N, P[0], g);
@@ -151,6 +151,20 @@ void Planner::plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const
     }
   }
   out.back().bytes = n - out.back().offset;  // clip the final chunk to n
+}
+
+// C_p = max(g, floor(C * beta_p / beta_max / g) * g)  (L242, R2)
+void size_chunks(std::vector<PathModel> &P, uint64_t C, uint64_t g) {
+  uint64_t bmax = 0;
+  for (auto &p : P) bmax = std::max(bmax, p.beta_Bps);
+  for (auto &p : P) {
+    uint64_t cp = (uint64_t)(((u128)C * p.beta_Bps) / ((u128)bmax * g)) * g;
+    p.chunk = std::max(g, cp);
+  }
+}
+
+void Planner::plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const {
+  split_plan(paths[d], n, cfg.granule, out);
 }
 
 void Planner::plan_single(uint64_t n, int route_gpu, std::vector<grouter_chunk> &out) const {

@@ -23,6 +23,10 @@ struct PathModel {
   uint64_t chunk;     // C_p
 };
 
+// O6 split over arbitrary paths (shared by host<->GPU plans and NVLink plans)
+void split_plan(const std::vector<PathModel> &P, uint64_t n, uint64_t g, std::vector<grouter_chunk> &out);
+void size_chunks(std::vector<PathModel> &P, uint64_t C, uint64_t g);
+
 struct Planner {
   grouter_config cfg;
   std::vector<std::vector<int>> groups;          // uplink groups, each sorted

@@ -78,6 +78,14 @@ class grouter_stats_t(C.Structure):
     ]
 
 
+MAX_PATH_NODES = 8
+
+
+class grouter_path(C.Structure):
+    _fields_ = [("bw_Bps", C.c_uint64), ("func", C.c_uint32), ("n_nodes", C.c_uint32),
+                ("nodes", C.c_int32 * MAX_PATH_NODES)]
+
+
 IPC_MAX_SEGS = 8
 
 
@@ -125,6 +133,14 @@ SIGNATURES = {
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
+    "grouter_paths_new": (C.c_void_p, [C.c_uint32, C.c_uint32, C.POINTER(_U64), C.c_uint32]),
+    "grouter_paths_free": (None, [C.c_void_p]),
+    "grouter_paths_select": (_ST, [C.c_void_p, C.c_uint32, C.c_int32, C.c_int32, C.POINTER(grouter_path),
+                                   C.c_uint32, C.POINTER(C.c_uint32)]),
+    "grouter_paths_release": (_ST, [C.c_void_p, C.c_uint32]),
+    "grouter_paths_table": (_ST, [C.c_void_p, C.POINTER(grouter_path), C.c_uint32, C.POINTER(C.c_uint32)]),
+    "grouter_paths_plan": (_ST, [C.c_void_p, C.c_uint32, _U64, _U64, _U64, _U64, C.POINTER(grouter_chunk),
+                                 _U64, C.POINTER(_U64)]),
     "grouter_pool_target": (_ST, [_CTX, C.c_int32, C.POINTER(_U64)]),
     "grouter_test_set_clock": (_ST, [_CTX, C.c_int32, _U64]),
     "grouter_set_tenant_slo": (_ST, [_CTX, C.c_uint32, _U64, _U64, _U64]),
@@ -410,6 +426,54 @@ class Ctx:
 
 
 # ------------------------------------------------------------------ test kernels (K9)
+class Paths:
+    """grouter_paths_*: the Alg. 1 NVLink path planner (host only)."""
+
+    def __init__(self, topo, n_gpus, max_edges=3):
+        self.lib = load()
+        n = len(topo)
+        flat = (C.c_uint64 * (n * n))(*[topo[u][v] for u in range(n) for v in range(n)])
+        self.h = self.lib.grouter_paths_new(n, n_gpus, flat, max_edges)
+        if not self.h:
+            raise GrouterError(EINVAL, "grouter_paths_new")
+
+    @staticmethod
+    def _conv(p):
+        return (p.func, p.bw_Bps, tuple(p.nodes[:p.n_nodes]))
+
+    def select(self, func, gs, gd):
+        arr, cnt = (grouter_path * 64)(), C.c_uint32(0)
+        st = self.lib.grouter_paths_select(self.h, func, gs, gd, arr, 64, C.byref(cnt))
+        return st, [(list(x[2]), x[1]) for x in map(self._conv, arr[:cnt.value])]
+
+    def release(self, func):
+        return self.lib.grouter_paths_release(self.h, func)
+
+    def table(self):
+        arr, cnt = (grouter_path * 1024)(), C.c_uint32(0)
+        check(self.lib.grouter_paths_table(self.h, arr, 1024, C.byref(cnt)), "paths_table")
+        return [self._conv(p) for p in arr[:cnt.value]]
+
+    def plan(self, func, n, chunk_bytes, relay_phi_ps, granule=4096):
+        cnt = C.c_uint64(0)
+        self.lib.grouter_paths_plan(self.h, func, n, chunk_bytes, granule, relay_phi_ps, None, 0, C.byref(cnt))
+        arr = (grouter_chunk * max(cnt.value, 1))()
+        check(self.lib.grouter_paths_plan(self.h, func, n, chunk_bytes, granule, relay_phi_ps, arr, cnt.value,
+                                          C.byref(cnt)), "paths_plan")
+        return [(c.offset, c.bytes, c.path, c.route_gpu) for c in arr[:cnt.value]]
+
+    def close(self):
+        if self.h:
+            self.lib.grouter_paths_free(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 def slo_weights(slos: dict, bw_all: int) -> dict:
     """grouter_slo_weights: {wf: (data_bytes, slo_ns, infer_ns)} -> {wf: weight}."""
     lib = load()

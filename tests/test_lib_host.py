@@ -191,3 +191,71 @@ def test_fig5a_gfn_host_routes():
     calib = C.fig5a()
     p = osplit.plan_d2h(calib, 0, 1 << 30)
     assert sorted({c["route_gpu"] for c in p}) == [0, 2, 4, 6]
+
+
+# ------------------------------------------------------------------ Alg. 1 planner parity
+def _alg1_ops(rng, n_gpus, steps=40):
+    ops, live, nxt = [], [], 1
+    for _ in range(steps):
+        if live and rng.random() < 0.3:
+            f = live.pop(rng.randrange(len(live)))
+            ops.append(("release", f))
+        else:
+            gs, gd = rng.sample(range(n_gpus), 2)
+            ops.append(("select", nxt, gs, gd))
+            live.append(nxt)
+            nxt += 1
+    return ops
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_alg1_planner_parity(seed):
+    """grouter_paths_* (C++) == oracle.alg1.PathTable op by op: each selected
+    path list, the full allocation table after every op, and the NVLink chunk
+    plan of every live function."""
+    import random
+    from oracle import alg1
+    rng = random.Random(seed)
+    kind = seed % 4
+    if kind == 0:
+        topo, ng = C.dgx_v100_topo(), 8
+    elif kind == 1:
+        topo, ng = C.nvswitch_topo(8), 8
+    else:
+        ng = rng.choice([3, 4, 5, 6, 8])
+        topo = C.random_topo(rng, ng)
+    H = rng.choice([2, 3, 4])
+    orc, lib = alg1.PathTable(topo, ng, max_edges=H), G.Paths(topo, ng, max_edges=H)
+    try:
+        for op in _alg1_ops(rng, ng):
+            if op[0] == "release":
+                orc.release(op[1])
+                assert lib.release(op[1]) == G.OK
+            else:
+                _, f, gs, gd = op
+                exp, _ = orc.select(f, gs, gd)
+                st, got = lib.select(f, gs, gd)
+                assert st == G.OK and got == exp, (op, got, exp)
+            assert lib.table() == orc.table()
+            for f in sorted({a[0] for a in orc.alloc}):
+                n = rng.choice([1, 4096, 38_535_168, 1 << 30])
+                exp = alg1.nvl_plan([(a[1], a[2]) for a in orc.paths_of(f)], n, ng, 20_000_000, 2 << 20)
+                got = lib.plan(f, n, 2 << 20, 20_000_000)
+                assert got == [(c["offset"], c["bytes"], c["path"], c["route_gpu"]) for c in exp]
+    finally:
+        lib.close()
+
+
+def test_alg1_planner_bad_arguments():
+    t = C.dgx_v100_topo()
+    p = G.Paths(t, 8)
+    try:
+        assert p.select(1, 0, 0)[0] == G.EINVAL
+        assert p.select(1, 0, 9)[0] == G.EINVAL
+        assert p.select(1, 0, 3)[0] == G.OK
+        assert p.select(1, 0, 2)[0] == G.ESTATE        # release first
+        assert p.release(1) == G.OK and p.table() == []
+    finally:
+        p.close()
+    with pytest.raises(G.GrouterError):
+        G.Paths([[0] * 40 for _ in range(40)], 8)
