@@ -30,4 +30,30 @@ r = LibRunner(calib, replay=True, keep_bytes=True)
 out = r(ops)
 r.close()
 compare(orun.run(ops, calib, keep_bytes=True), out)
+# real-time mode with proactive restore and gFn-host striping: direct
+# launches (event completion, PDL), server rounds, spills, restores
+rng = random.Random(7)
+ops = T.random_trace(rng, 2, n_ops=60, max_n=3 * MiB, run_seed=7)
+r = LibRunner(calib, replay=False, keep_bytes=True, flags=G.RESTORE | G.D2H_MULTIPATH,
+              host_store_bytes=64 * MiB, pool_cap=[8 * MiB, 16 * MiB])
+out = r(ops)
+r.close()
+compare(orun.run(ops, calib, keep_bytes=True, restore=True, d2h_multipath=True,
+                 host_store_bytes=64 * MiB, pool_cap=[8 * MiB, 16 * MiB]), out, check_dispatch=False)
+# back-to-back direct get_into on one stream (the bench's pattern)
+c1 = dict(C.b200_hgx(1), device_map=[0])
+ctx = G.Ctx(G.config_from_calib(c1, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED], pool_floor_bytes=64 * MiB))
+n = 3 * MiB + 5
+src = torch.empty(n, dtype=torch.uint8, device="cuda")
+G.check(G.test_fill(src.data_ptr(), n, 11, 0, 0))
+torch.cuda.synchronize()
+st, oid = ctx.put(G.fn(1, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+s = torch.cuda.Stream()
+dsts = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(3)]
+for i in range(12):
+    G.check(ctx.get_into(G.fn(1, 2, 0), oid, dsts[i % 3].data_ptr(), n, s.cuda_stream)[0])
+s.synchronize()
+for d in dsts:
+    assert G.test_verify(d.data_ptr(), n, 11, 0, 0)[1] == 0
+ctx.close()
 print("sanitize workload OK", os.environ.get("GR_COPY", "default"))
