@@ -115,6 +115,99 @@ def cfg4_isolation(seconds=2.0):
             "weighted_GBps": part["GBps"][0], "unweighted_GBps": flat["GBps"][0]}
 
 
+def cfg2(seconds=3.0, outstanding=4):
+    """Config 2 (Traffic) at N = 1, data plane only: per request
+    a decode cFn puts a 39,321,600 B frame (hint GPU0, PCIe H2D), the YOLO gFn
+    gets it (zero copy: co-located), allocs + seals person and vehicle crops
+    (K x 602,112 B, K ~ Poisson(4) clipped to [0, 32]), the recognition gFns get
+    them (zero copy) and everyone releases.  `outstanding` closed-loop client
+    threads (Q = 4 N); req/s, per-request latency, and the PCIe roofline of the
+    frame put (39.3 MB per request at the probed link rate)."""
+    import math
+    import random
+    FRAME, CROP = 39_321_600, 602_112
+    ctx = mkctx(host_store_bytes=256 * MiB, pool_cap=[G.UNLIMITED])
+    frames = [torch.empty(FRAME, dtype=torch.uint8, pin_memory=True) for _ in range(outstanding)]
+    streams = [torch.cuda.Stream() for _ in range(outstanding)]
+    lat = [[] for _ in range(outstanding)]
+    done = [0] * outstanding
+    stop = [False]
+    start = threading.Barrier(outstanding + 1)
+
+    def poisson(rng, lam=4.0):
+        L, k, p = math.exp(-lam), 0, 1.0
+        while True:
+            p *= rng.random()
+            if p <= L:
+                return min(k, 32)
+            k += 1
+
+    def worker(t):
+        rng = random.Random(2000 + t)
+        s = streams[t].cuda_stream
+        start.wait()
+        i = 0
+        while not stop[0]:
+            wf = 10 + t * 100000 + i
+            dec, yolo, rp, rv = G.fn(wf, 1, G.HOST), G.fn(wf, 2, 0), G.fn(wf, 3, 0), G.fn(wf, 4, 0)
+            t0 = time.perf_counter()
+            st, o = ctx.put(dec, frames[t].data_ptr(), FRAME, 0, 1)
+            G.check(st, "put")
+            st, fp, _ = ctx.get(yolo, o, s)
+            G.check(st, "get")
+            outs = []
+            for k in (poisson(rng), poisson(rng)):
+                st, buf, a = ctx.alloc(yolo, k * CROP, G.NOHINT, 1)
+                G.check(st, "alloc")
+                G.check(ctx.seal(yolo, a, s), "seal")
+                outs.append(a)
+            gets = [(rp, outs[0]), (rv, outs[1])]
+            ptrs = []
+            for f, a in gets:
+                st, ptr, _ = ctx.get(f, a, s)
+                G.check(st, "get crops")
+                ptrs.append(ptr)
+            G.check(ctx.release(yolo, o, fp, s), "release")
+            for (f, a), ptr in zip(gets, ptrs):
+                if ptr:                              # K = 0: an empty object has no lease (R36)
+                    G.check(ctx.release(f, a, ptr, s), "release crops")
+            streams[t].synchronize()
+            lat[t].append(time.perf_counter() - t0)
+            done[t] += 1
+            i += 1
+
+    ths = [threading.Thread(target=worker, args=(t,)) for t in range(outstanding)]
+    for th in ths:
+        th.start()
+    start.wait()
+    t0 = time.perf_counter()
+    time.sleep(seconds)
+    stop[0] = True
+    for th in ths:
+        th.join()
+    dt = time.perf_counter() - t0
+    all_lat = [x for l in lat for x in l]
+    probe = G.probe([0], 256 * MiB)
+    link = probe["h2d_Bps"][0]
+    req_s = sum(done) / dt
+    ctx.close()
+    # the oracle on the same request structure (1 core)
+    from oracle import runner as orun
+    from synth import traces as TT
+    from synth.calib import b200_hgx as hgx
+    ops = TT.cfg2(1, requests=8)
+    t1 = time.perf_counter()
+    orun.run(ops, hgx(1))
+    o_req_s = 8 / (time.perf_counter() - t1)
+    return {"outstanding": outstanding, "seconds": round(dt, 3), "requests": sum(done),
+            "req_per_s": round(req_s, 1), "p50_ms": round(pct(all_lat, 50) * 1e3, 3),
+            "p99_ms": round(pct(all_lat, 99) * 1e3, 3),
+            "roofline": {"bound": "pcie", "achieved_GBps": round(req_s * FRAME / 1e9, 2),
+                         "peak_GBps": round(link / 1e9, 2), "frac": round(req_s * FRAME / link, 3),
+                         "peak_source": "grouter_probe solo pinned H2D of this GPU"},
+            "oracle_req_per_s": round(o_req_s, 1)}
+
+
 def cfg5(requests=4, limit_frac=0.1, hints=True, layers=32):
     KV, HID = 33_554_432, 67_108_864
     page = 2 * MiB
@@ -240,6 +333,11 @@ def main():
 
     def save():
         json.dump(res, open(out, "w"), indent=1)
+    if len(sys.argv) > 2 and sys.argv[2] == "cfg2":
+        res["cfg2"] = cfg2(3.0)
+        print("cfg2", json.dumps(res["cfg2"]), flush=True)
+        save()
+        return
     if len(sys.argv) > 2 and sys.argv[2] == "slo":
         res["cfg4_slo"] = cfg4_slo(3.0)
         print("cfg4_slo", json.dumps(res["cfg4_slo"]), flush=True)
