@@ -577,7 +577,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
     Fences done;
     done_fences(x, done);
     if (o.readers.size() > 8) prune(o.readers);
-    for (auto &w : done) o.readers.push_back(w);
+    for (auto &w : done) push_fence(o.readers, w);
     Lease L{oid, o.wf, d, lease, n, done};
     c->leases[(uintptr_t)lease] = std::move(L);
     result = lease;
@@ -632,7 +632,7 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
       Fences done;
       done_fences(x, done);
       if (o.readers.size() > 8) prune(o.readers);
-      for (auto &w : done) o.readers.push_back(w);
+      for (auto &w : done) push_fence(o.readers, w);
       if (!direct) wait = done;
     }
   }

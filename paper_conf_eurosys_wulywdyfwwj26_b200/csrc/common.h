@@ -120,12 +120,28 @@ struct Waitable {
   // already submitted (events, caller-stream signals).  A wait is never
   // enqueued before its producer is submitted (see engine.cpp).
   std::shared_ptr<Xfer> producer;
+  // stream the event was recorded on (events only): fences of one stream
+  // complete in order, so a newer one stands for the older ones
+  cudaStream_t origin = nullptr;
+  mutable bool fired = false;  // memo: an event query costs ~1.4 us of host time
   bool done() const {
     if (word) return (int32_t)(*word - target) >= 0;
-    if (ev) return cudaEventQuery(ev->ev) == cudaSuccess;
+    if (ev) {
+      if (!fired) fired = cudaEventQuery(ev->ev) == cudaSuccess;
+      return fired;
+    }
     return true;
   }
 };
+
+// Appends w to a fence list, replacing the last entry when both are events of
+// the same stream (the newer completes after the older).
+inline void push_fence(std::vector<Waitable> &f, const Waitable &w) {
+  if (!f.empty() && w.ev && !w.word && f.back().ev && !f.back().word && w.origin && f.back().origin == w.origin)
+    f.back() = w;
+  else
+    f.push_back(w);
+}
 using Fences = std::vector<Waitable>;
 
 // Drops completed fences (keeps long-lived objects' reader lists short).

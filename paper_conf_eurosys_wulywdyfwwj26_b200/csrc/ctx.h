@@ -106,6 +106,8 @@ struct Xfer {
   // caller stream after a direct launch that moved the whole transfer (its
   // completion slot is handed back at once)
   EventRef done_ev;
+  cudaStream_t done_stream = nullptr;      // stream done_ev was recorded on
+  mutable bool done_fired = false;
   bool done() const;
 };
 using XferRef = std::shared_ptr<Xfer>;

@@ -136,6 +136,8 @@ void done_fences(const XferRef &x, Fences &f) {
     Waitable w;
     w.ev = x->done_ev;
     w.epoch = x->epoch;
+    w.origin = x->done_stream;
+    w.fired = x->done_fired;
     f.push_back(w);
     return;
   }
@@ -151,7 +153,10 @@ void done_fences(const XferRef &x, Fences &f) {
 }
 
 bool Xfer::done() const {
-  if (done_ev) return cudaEventQuery(done_ev->ev) == cudaSuccess;
+  if (done_ev) {
+    if (!done_fired) done_fired = cudaEventQuery(done_ev->ev) == cudaSuccess;
+    return done_fired;
+  }
   for (uint32_t p = 0; p < npath; ++p)
     if (total[p] && (int32_t)(words[p] - target[p]) < 0) return false;
   return true;
@@ -667,9 +672,15 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
   Server &s = c->dev[server_logical].copy;
   if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty()) return false;
   if (s.sched.backlog_items != x->nchunks) return false;  // only this transfer is queued
-  retire(s);
-  for (auto &f : s.inflight)
-    if (f.direct != caller) return false;  // server-stream work in flight: keep order there
+  // server-stream or other-stream work in flight: keep order there (retire
+  // only when needed: an event query costs host time)
+  bool foreign = false;
+  for (auto &f : s.inflight) foreign |= f.direct != caller;
+  if (foreign) {
+    retire(s);
+    for (auto &f : s.inflight)
+      if (f.direct != caller) return false;
+  }
   for (auto &w : x->deps)
     if (!is_submitted(w)) return false;
   PhysDev &pd = *c->phys.at(s.phys);
@@ -689,6 +700,7 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     pd.next_scratch = (k + 1) % pd.n_scratch;
     for (auto &w : pd.scratch_busy[k])
       if (!w.done()) host_wait(Fences{w});
+    pd.scratch_busy[k].clear();
     // one launch moves the whole transfer: complete it by an event, not words
     static const bool ev_done = !getenv("GR_NO_EVDONE");
     const bool whole = ev_done && x->submitted_chunks == 0 && items.size() == x->nchunks && x->waiters.empty();
@@ -696,6 +708,7 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     launch_round(c, s, caller, pd.scratch + 2 * k, items, nullptr, whole ? &deferred : nullptr);
     if (deferred) {
       x->done_ev = record(c, caller, s.phys);
+      x->done_stream = caller;
       for (uint32_t p = 0; p < x->npath; ++p) c->slot_final[x->slot][p] -= x->total[p];  // slot back
     }
     for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
@@ -703,8 +716,13 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     after_submit(c, items);
     Fences done;
     done_fences(x, done);
-    pd.scratch_busy[k] = done;
-    s.inflight.push_back({done.empty() ? Waitable{} : done.front(), caller});
+    if (!deferred) pd.scratch_busy[k] = done;  // an in-kernel publish used the pair
+    // one entry per caller stream: its newest launch stands for the older ones
+    Waitable w = done.empty() ? Waitable{} : done.front();
+    if (!s.inflight.empty() && s.inflight.back().direct == caller && deferred && s.inflight.back().w.origin == caller)
+      s.inflight.back().w = w;
+    else
+      s.inflight.push_back({w, caller});
   }
   return true;
 }

@@ -839,11 +839,29 @@ extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, 
   cudaStream_t s = (cudaStream_t)stream;
   static SmallParams sp;
   static CopyParams bp;
+  // kinds 3/4: small block via cudaLaunchKernelEx with / without the PDL
+  // attribute; 5: cudaEventRecord only; 6: cudaEventQuery of a recorded event
+  static cudaEvent_t ev = nullptr;
+  if (!ev) cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(blocks);
+  cfg.blockDim = dim3(256);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  if (kind == 6) cudaEventRecord(ev, s);
   auto t0 = std::chrono::steady_clock::now();
   for (int i = 0; i < n; ++i) {
     if (kind == 0) gr_empty_kernel_tiny<<<blocks, 256, 0, s>>>(i);
     else if (kind == 1) gr_empty_kernel<<<blocks, 256, 0, s>>>(sp);
-    else gr_empty_kernel_big<<<blocks, 256, 0, s>>>(bp);
+    else if (kind == 2) gr_empty_kernel_big<<<blocks, 256, 0, s>>>(bp);
+    else if (kind == 3 || kind == 4) {
+      cfg.numAttrs = kind == 3 ? 1 : 0;
+      cudaLaunchKernelEx(&cfg, gr_empty_kernel, sp);
+    } else if (kind == 5) cudaEventRecord(ev, s);
+    else (void)cudaEventQuery(ev);
   }
   auto t1 = std::chrono::steady_clock::now();
   cudaStreamSynchronize(s);

@@ -29,3 +29,22 @@ for flags in (0, G.PROFILE):
         ctx.where(oid)
     print("ctypes where() us/call", round((time.perf_counter() - t) * 1e6 / 2000, 2))
     ctx.close()
+
+# latency mode: one get_into at a time on an idle GPU (host time of the call only)
+ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED]))
+h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+st, oid = ctx.put(G.fn(1, 1, -1), h.data_ptr(), n, 0, 0)
+s = torch.cuda.Stream()
+b = torch.empty(n, dtype=torch.uint8, device="cuda")
+f = G.fn(1, 2, 0)
+ts = []
+for i in range(300):
+    s.synchronize()
+    t = time.perf_counter()
+    ctx.get_into(f, oid, b.data_ptr(), n, s.cuda_stream)
+    ts.append((time.perf_counter() - t) * 1e6)
+ts.sort()
+print("latency mode: host us/call p50", round(ts[150], 2), "p10", round(ts[30], 2), flush=True)
+# raw ctypes call of the same entry point (no Python wrapper)
+fnp = G.grouter_fn(1, 2, 0) if hasattr(G, "grouter_fn") else None
+ctx.close()

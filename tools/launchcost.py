@@ -6,8 +6,8 @@ from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G
 lib = G.load()
 s = torch.cuda.Stream()
 for stream_name, st in (("torch stream", s.cuda_stream), ("legacy default", 0)):
-    for kind in (0, 1, 2):
-        for blocks in (1, 592):
+    for kind in (0, 1, 2, 3, 4, 5, 6):
+        for blocks in (592,):
             for rep in range(2):
                 v = C.c_double(0)
                 G.check(lib.grouter_test_launch_cost(kind, 2000, blocks, st or None, C.byref(v)))

@@ -63,10 +63,32 @@ def host_timed(fn, reps):
     return out
 
 
+def oracle_get_into(n, budget_s=0.4):
+    """The oracle's get_into of an n-byte GPU object (np.copyto between
+    simulated buffers), single-threaded, on this box's host."""
+    import numpy as np
+    from oracle.model import Oracle
+    from synth.calib import b200_hgx as hgx
+    orc = Oracle(hgx(1))
+    src = np.zeros(n, np.uint8)
+    st, out = orc.put({"wf": 1, "fid": 1, "dev": 0}, src, n, -2, 0)
+    oid = out["oid"]
+    dst = np.empty(n, np.uint8)
+    f = {"wf": 1, "fid": 2, "dev": 0}
+    lat = []
+    t_end = time.perf_counter() + budget_s
+    while len(lat) < 3 or (time.perf_counter() < t_end and len(lat) < 200):
+        t = time.perf_counter()
+        orc.get_into(f, oid, dst, n)
+        lat.append((time.perf_counter() - t) * 1e6)
+    return summarize(n, lat)
+
+
 def main():
     _build.build()
     G.load()
-    res = {"gpu": torch.cuda.get_device_name(0), "patterns": {}}
+    import os
+    res = {"gpu": torch.cuda.get_device_name(0), "patterns": {}, "host_cores": len(os.sched_getaffinity(0))}
     res["probe"] = G.probe([0], 256 * MiB)
     calib = b200_hgx(1)
     calib["device_map"] = [0]
@@ -119,6 +141,7 @@ def main():
             pats["base_memcpy_d2d"].append(summarize(n, dev_timed(s, lambda: dst.copy_(src), reps)))
             pats["base_h2d_pinned"].append(summarize(n, dev_timed(s, lambda: dst.copy_(hb, non_blocking=True), reps)))
             pats["base_d2h_pinned"].append(summarize(n, dev_timed(s, lambda: hb.copy_(dst, non_blocking=True), reps)))
+        pats.setdefault("oracle_get_into", []).append(oracle_get_into(n))
         print(n, {k: v[-1]["p50_us"] for k, v in pats.items()}, flush=True)
     res["patterns"] = pats
     ctx.close()
