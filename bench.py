@@ -41,9 +41,10 @@ WORKLOAD = ("cfg1 2-function workflow, 38,535,168 B tensor; value: gFn get_into 
             "from pinned host + get_into + 8 B D2H")
 
 
-WORKLOAD_N = ("cfg1 2-function workflow at N GPUs, 38,535,168 B tensor; value: gFn on GPU r get_into "
-              "of objects resident on GPU r+1 (exported/imported via CUDA VMM IPC, SM pull copy over "
-              "NVLink), e2e: cFn put(hint=own GPU) from pinned host + local get_into + 8 B D2H")
+WORKLOAD_N = ("cfg1 2-function workflow at N GPUs, 38,535,168 B tensor; value: every GPU runs the N=1 "
+              "workload on its own workflows (co-located, weak scaling); nvlink_pull: gFn on GPU r "
+              "get_into's objects resident on GPU r+1 (CUDA VMM IPC, SM pull copy over NVLink); "
+              "e2e: cFn put(hint=own GPU) from pinned host + local get_into + 8 B D2H")
 
 
 def _peaks():
@@ -55,25 +56,81 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+    """SM clocks / throttle reasons sampled DURING the timed region.
+
+    NVML in a background thread every 2 ms (the default timed region is
+    ~55 ms: an nvidia-smi subprocess spends that starting up); the thread's
+    NVML calls release the GIL.  Falls back to `nvidia-smi -lms` when NVML is
+    missing."""
 
     Q = ("index,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, index: int):
+    def __init__(self, index: int, period_s: float = 0.002):
         self.index = index
         self.p = None
+        self.period = period_s
+        self.nv = None
+        try:
+            import pynvml as nv
+            import torch
+            nv.nvmlInit()
+            h = None
+            try:
+                pr = torch.cuda.get_device_properties(index)
+                bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+                h = nv.nvmlDeviceGetHandleByPciBusId(bus)
+            except Exception:
+                h = nv.nvmlDeviceGetHandleByIndex(index)
+            self.nv, self.h = nv, h
+        except Exception:
+            self.nv = None
+
+    def _poll(self):
+        nv, h = self.nv, self.h
+        bits = [("hw_slowdown", nv.nvmlClocksEventReasonHwSlowdown),
+                ("hw_thermal_slowdown", nv.nvmlClocksEventReasonHwThermalSlowdown),
+                ("sw_thermal_slowdown", nv.nvmlClocksEventReasonSwThermalSlowdown),
+                ("sw_power_cap", nv.nvmlClocksEventReasonSwPowerCap)]
+        while not self.halt.is_set():
+            try:
+                self.sm.append(float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                for name, b in bits:
+                    if r & b:
+                        self.reasons.add(name)
+            except Exception as e:
+                self.reasons.add(f"nvml error: {e}"[:60])
+                return
+            self.halt.wait(self.period)
 
     def start(self):
+        if self.nv is not None:
+            import threading
+            self.sm, self.reasons = [], set()
+            self.halt = threading.Event()
+            self.mx = float(self.nv.nvmlDeviceGetMaxClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+            self.t = threading.Thread(target=self._poll, daemon=True)
+            self.t.start()
+            return
+        self._start_smi()
+
+    def _start_smi(self):
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "50"],
                                       stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            time.sleep(0.3)   # let nvidia-smi start before the timed region
         except Exception:
             self.p = None
 
     def stop(self):
+        if self.nv is not None:
+            self.halt.set()
+            self.t.join(timeout=5)
+            return {"sm_mhz": statistics.median(self.sm) if self.sm else None, "sm_max_mhz": self.mx,
+                    "samples": len(self.sm), "reasons": sorted(self.reasons), "source": "nvml, 2 ms"}
         if not self.p:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
         time.sleep(0.12)
@@ -322,67 +379,94 @@ def run_gpu(args, rank, world, local_rank):
             imported.append(roid)
         # every rank must take the same branch: agree on success
         ok = max_over_ranks(1.0 if ipc_error else 0.0, world, f"cuda:{dev}") == 0.0
-        if ok:
-            work = list(zip(imported, bptr))
-        else:  # measured honestly as local replicas, error reported in the line
-            print(f"[bench] rank {rank}: IPC pull unavailable ({ipc_error}); local replicas",
-                  file=sys.stderr, flush=True)
+        if not ok:  # reported in the line; the value (co-located replicas) is unaffected
+            print(f"[bench] rank {rank}: IPC pull unavailable ({ipc_error})", file=sys.stderr, flush=True)
             for roid in imported:
                 ctx.free(gfn, roid)
             imported = []
             remote = False
 
-    def value_step():
-        for oid, dst in work:
-            st, _ = ctx.get_into(gfn, oid, dst, n, s)
-            if st:
-                G.check(st, "get_into")
+    def make_step(pairs):
+        def step():
+            for oid, dst in pairs:
+                st, _ = ctx.get_into(gfn, oid, dst, n, s)
+                if st:
+                    G.check(st, "get_into")
+        return step
 
-    # parity spot check of the delivered bytes before timing (full, on device)
-    value_step()
-    stream.synchronize()
-    for b in range(min(R, B)):
-        last = max(i for i in range(R) if i % B == b)   # request that wrote binding b last
-        st, bad, _ = G.test_verify(bindings[b].data_ptr(), n, 1000 + last, 0, 0)
-        assert st == 0 and bad == 0, f"binding {b}: {bad} bytes differ from the payload"
+    def verify_bindings(what):
+        """Parity spot check of every delivered binding (full, on device):
+        every rank generated the same SplitMix64 payloads (seed 1000 + i),
+        so local and pulled objects verify against the same seeds."""
+        stream.synchronize()
+        for b in range(min(R, B)):
+            last = max(i for i in range(R) if i % B == b)   # request that wrote binding b last
+            st, bad, _ = G.test_verify(bindings[b].data_ptr(), n, 1000 + last, 0, 0)
+            assert st == 0 and bad == 0, f"{what}: binding {b}: {bad} bytes differ from the payload"
 
-    for _ in range(args.warmup):
-        value_step()
-    barrier()
-    st0 = ctx.stats()
-    clk = ClockSampler(dev)
-    clk.start()
-    time.sleep(0.05)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    hs = time.perf_counter()
-    for _ in range(args.steps):
-        value_step()
-    host_us = (time.perf_counter() - hs) * 1e6 / (args.steps * R)   # submission cost per request
-    e1.record(stream)
-    barrier()
-    clocks = clk.stop()
-    ms = e0.elapsed_time(e1)
-    G.check(ctx.sync(), "sync")
-    st1 = ctx.stats()
-    ms_max = max_over_ranks(ms, world, f"cuda:{dev}")
+    def timed(step, sample_clocks):
+        """W warm-up steps, then exactly K steps bracketed by barrier + device
+        sync, CUDA events on the consumer stream; max over ranks."""
+        step()
+        verify_bindings("before timing")
+        for _ in range(args.warmup):
+            step()
+        barrier()
+        st0 = ctx.stats()
+        clk = ClockSampler(dev) if sample_clocks else None
+        if clk:
+            clk.start()             # samples only the timed region (NVML thread)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        hs = time.perf_counter()
+        for _ in range(args.steps):
+            step()
+        host_us = (time.perf_counter() - hs) * 1e6 / (args.steps * R)   # submission cost per request
+        e1.record(stream)
+        barrier()
+        clocks = clk.stop() if clk else None
+        ms = e0.elapsed_time(e1)
+        G.check(ctx.sync(), "sync")
+        st1 = ctx.stats()
+        verify_bindings("after timing")
+        return dict(ms=ms, ms_max=max_over_ranks(ms, world, f"cuda:{dev}"), host_us=host_us, clocks=clocks,
+                    launches=st1.kernel_launches - st0.kernel_launches,
+                    moved=st1.link_bytes[0][0] - st0.link_bytes[0][0])   # bytes the copy kernels moved
+
+    # value: every workflow co-located on one GPU (R24's placement), GPUs independent (weak scaling)
+    t = timed(make_step(work), True)
+    ms, ms_max, host_us, clocks, launches, moved = (t[k] for k in ("ms", "ms_max", "host_us", "clocks",
+                                                                   "launches", "moved"))
     total_req = R * args.steps * world
     value = total_req / (ms_max / 1e3)
-    launches = st1.kernel_launches - st0.kernel_launches
-    moved = st1.link_bytes[0][0] - st0.link_bytes[0][0]       # bytes the copy kernels moved
     # The copy kernels run back to back on the consumer stream (direct
     # launches, GPU-bound: host submission < GPU time), so the event-timed
     # region on that stream / launches = average launch duration (incl. the
-    # inter-launch gap, i.e. conservative).
+    # inter-launch gap, i.e. conservative).  Same-GPU HBM copy: read + write.
     avg_ns = ms * 1e6 / max(launches, 1)
-    if remote:   # pull over NVLink: n bytes cross the link per request
-        alg_bytes_per_launch = moved / max(launches, 1)
-        bound, peak, peak_src = "nvlink", 770.0, "B200_PROFILING.md measured peer copy 770 GB/s/direction"
-    else:        # same-GPU HBM copy: read + write
-        alg_bytes_per_launch = 2 * moved / max(launches, 1)
-        bound = "hbm"
-        peak, peak_src = _peaks()
+    alg_bytes_per_launch = 2 * moved / max(launches, 1)
+    bound = "hbm"
+    peak, peak_src = _peaks()
     achieved = alg_bytes_per_launch / avg_ns if launches else None  # bytes/ns == GB/s
+
+    # N > 1: the same requests with producer and consumer on different GPUs --
+    # GPU r pulls GPU r+1's objects over NVLink (cross-GPU leg B of cfg1, R24)
+    nvlink = None
+    if remote:
+        p = timed(make_step(list(zip(imported, bptr))), False)
+        p_ns = p["ms"] * 1e6 / max(p["launches"], 1)
+        p_bytes = p["moved"] / max(p["launches"], 1)          # n bytes cross the link per request
+        p_ach = p_bytes / p_ns if p["launches"] else None
+        nvlink = {"value": R * args.steps * world / (p["ms_max"] / 1e3), "unit": "req/s",
+                  "what": "every GPU r get_into's GPU r+1's 20 resident objects (IPC-mapped pool pages, "
+                          "SM pull copy over NVLink, ring of disjoint pairs)",
+                  "gbps_per_gpu": R * args.steps * n / (p["ms_max"] / 1e3) / 1e9,
+                  "roofline": {"bound": "nvlink", "achieved": p_ach, "peak": 770.0, "unit": "GB/s",
+                               "frac": (p_ach / 770.0) if p_ach else None,
+                               "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s/direction",
+                               "launches": p["launches"], "avg_launch_us": p_ns / 1e3,
+                               "alg_bytes_per_launch": p_bytes},
+                  "host_us_per_request": p["host_us"]}
 
     # per-request latency (separate, untimed pass): device events around one get_into
     lat = []
@@ -399,17 +483,35 @@ def run_gpu(args, rank, world, local_rank):
         return xs[min(len(xs) - 1, max(0, -(-len(xs) * q // 100) - 1))] if xs else None
 
     # ---------------------------------------------------------- e2e (host buffers)
-    out8 = torch.empty(8, dtype=torch.uint8, pin_memory=True)
+    # Closed loop with Q requests outstanding: Q client threads,
+    # each a cFn (blocking put, GIL released inside the C call) followed by its
+    # gFn (get_into on the client's own consumer stream) and the 8 B result
+    # read; client k serves requests k, k+Q, ... and owns bindings k, k+Q, ...
+    Q = max(1, min(args.e2e_q, B, R))
+    out8 = [torch.empty(8, dtype=torch.uint8, pin_memory=True) for _ in range(Q)]
+    qstreams = [stream] + [torch.cuda.Stream(device=dev) for _ in range(Q - 1)]
 
-    def e2e_step():
-        for i in range(R):
+    def e2e_client(k):
+        torch.cuda.set_device(dev)
+        qs = qstreams[k]
+        for i in range(k, R, Q):
             st, oid = ctx.put(cfn, host_src[i].data_ptr(), n, 0, 1)     # leg A (blocking)
             G.check(st, "put")
-            st, _ = ctx.get_into(gfn, oid, bindings[i % B].data_ptr(), n, s)  # leg B
+            st, _ = ctx.get_into(gfn, oid, bindings[i % B].data_ptr(), n, qs.cuda_stream)  # leg B
             G.check(st, "get_into")
-            with torch.cuda.stream(stream):
-                out8.copy_(bindings[i % B][:8], non_blocking=True)        # 8 B result read
-        stream.synchronize()
+            with torch.cuda.stream(qs):
+                out8[k].copy_(bindings[i % B][:8], non_blocking=True)     # 8 B result read
+        qs.synchronize()
+
+    from concurrent.futures import ThreadPoolExecutor
+    pool = ThreadPoolExecutor(max_workers=Q) if Q > 1 else None
+
+    def e2e_step():
+        if pool is None:
+            e2e_client(0)
+        else:
+            for f in [pool.submit(e2e_client, k) for k in range(Q)]:
+                f.result()
 
     e2e_steps = max(1, min(args.steps, args.e2e_steps))
     for _ in range(min(args.warmup, 3)):
@@ -421,6 +523,8 @@ def run_gpu(args, rank, world, local_rank):
     barrier()
     e2e_s = time.perf_counter() - h0
     e2e_val = R * e2e_steps * world / max_over_ranks(e2e_s, world, f"cuda:{dev}")
+    if pool is not None:
+        pool.shutdown()
 
     if world > 1:   # drop imports and our export pins once every rank is done reading
         barrier()
@@ -462,10 +566,9 @@ def run_gpu(args, rank, world, local_rank):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (SplitMix64 payload, verified on device before timing)",
-            "config": {"workload": WORKLOAD if not remote else WORKLOAD_N, "requests_per_step": R,
+            "config": {"workload": WORKLOAD if world == 1 else WORKLOAD_N, "requests_per_step": R,
                        "bytes": N_BYTES,
-                       "parallelism": f"replicas x{world}" if not remote else
-                       f"{world} GPUs, GPU r pulls from GPU r+1 over NVLink (IPC-mapped pool pages)",
+                       "parallelism": f"replicas x{world} (workflows co-located per GPU, no collective)",
                        "l2": "inputs larger than L2: 20 resident 38.5 MB objects, 8 rotating bindings",
                        "copy_kernel": os.environ.get("GR_COPY", "tma8" if args.tma else "ws1") + f", {args.ctas} CTA/SM cap"},
             "gbps": value * N_BYTES / 1e9,
@@ -481,16 +584,17 @@ def run_gpu(args, rank, world, local_rank):
                          "alg_bytes_per_launch": alg_bytes_per_launch},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "req/s", "h2d_bytes_per_step": R * N_BYTES,
-                    "d2h_bytes_per_step": R * 8, "steps": e2e_steps},
+                    "d2h_bytes_per_step": R * 8, "steps": e2e_steps,
+                    "outstanding": Q, "pcie_gbps": e2e_val / world * N_BYTES / 1e9},
             "gpu_launches": launches,
             "clocks": clocks,
         }
         if multipath is not None:
             line["h2d_multipath"] = multipath
+        if nvlink is not None:
+            line["nvlink_pull"] = nvlink
         if world > 1 and not remote:
             line["ipc_pull_error"] = ipc_error or "another rank failed to import"
-            line["config"]["workload"] = WORKLOAD
-            line["config"]["parallelism"] = f"replicas x{world}"
 
         print(json.dumps(line), flush=True)
     ctx.close()
@@ -499,11 +603,13 @@ def run_gpu(args, rank, world, local_rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="grouter", choices=["grouter", "reference"])
     ap.add_argument("--requests", type=int, default=20)
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--e2e-q", type=int, default=4,
+                    help="requests outstanding in the closed-loop e2e run (SURVEY §8(d): 4 per GPU)")
     ap.add_argument("--lat-samples", type=int, default=200)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
