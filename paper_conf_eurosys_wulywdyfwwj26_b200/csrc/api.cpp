@@ -292,6 +292,7 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   XferRef x = new_xfer(c, tenant, plan);
   x->deps = std::move(deps);
   x->pageable_src = pageable_src;
+  x->local_src = pool_src && src_loc >= 0;  // a GPU pool object, copied by that GPU's SMs
   const int kind = server_kind_for(src_loc, dst_loc);
   enqueue_plan(c, x, plan, kind, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, dst_loc);
   if (hprof().on) hprof().t[4] += now_ns() - tst;

@@ -95,6 +95,7 @@ struct Xfer {
   uint64_t deps_waited = 0;                 // bitmask of servers that already waited
   uint64_t epoch = 0;
   bool pageable_src = false;
+  bool local_src = false;                   // source = pool pages of the copying GPU (L2 prefetch safe)
   uint32_t nchunks = 0, submitted_chunks = 0;
   bool submitted() const { return submitted_chunks == nchunks; }
   struct Waiter {

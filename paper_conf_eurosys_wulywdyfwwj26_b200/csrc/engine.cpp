@@ -366,9 +366,12 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
   bool local = true;  // every destination in the launching GPU's memory -> GPU-scope fences
   for (auto &it : items)
     local &= it.dst_logical >= 0 && c->dev[it.dst_logical].phys == s.phys;
+  bool local_src = true;  // relay forwards read this GPU's staging ring
+  if (!src_override)
+    for (auto &it : items) local_src &= it.x->local_src;
   while (i < items.size()) {
     const uint64_t tparams = hprof().on ? now_ns() : 0;
-    p->flags = local ? kFlagLocalDst : 0;
+    p->flags = (local ? kFlagLocalDst : 0) | (local_src ? kFlagLocalSrc : 0);
     p->n_chunks = 0;
     p->n_pub = 0;
     p->scratch = scratch;

@@ -1,6 +1,8 @@
 // kernels.cu -- sm_100a data-movement kernels (no tensor cores: pure bytes).
 //
-// gr_copy: see kernels.h.  Two tile engines:
+// gr_copy: see kernels.h.  Default engines: wv8 (warp-strided, 256-bit
+// LDG/STG, L2 prefetch of each warp's first unit before the PDL wait) below
+// 256 MiB, the TMA bulk ring above.  Tile engines:
 //   * LD/ST: 256 threads, 128-bit vector loads/stores, 4 in flight per
 //     thread before the first store (coalesced, L1 no-allocate), with
 //     co-aligned and shifted (funnel-shift) paths for misaligned user
@@ -54,6 +56,9 @@ __device__ __forceinline__ void pdl_wait_raw() { asm volatile("griddepcontrol.wa
     if (p.flags & kFlagPdl) pdl_wait_raw(); \
   } while (0)
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void prefetch_l2(uint64_t addr, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
+}
 
 __device__ __forceinline__ void st_release_sys(uint64_t addr, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(addr), "r"(v) : "memory");
@@ -322,6 +327,27 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
   finish_round(p);
 }
 
+// Before waiting on the predecessor grid (PDL), a warp may pull the first
+// units of its OWN source into L2 with bulk prefetches: L2 is the point of
+// coherence for this GPU's memory, so a prefetch can never return stale
+// data (a line the predecessor still writes is updated in L2), and the
+// DRAM read ramp of this launch overlaps the predecessor's tail.  Only for
+// rounds whose sources are all in this GPU's memory (kFlagLocalSrc).
+template <int LG, class KP>
+__device__ __forceinline__ void prefetch_units(const KP &p, uint32_t w0, uint32_t W, uint32_t total,
+                                               uint32_t lane) {
+  const uint32_t n = (p.flags >> kPfShift) & 0xffu;
+  if (!n || !(p.flags & kFlagLocalSrc) || lane != 0) return;
+  for (uint32_t k = 0, id = w0; k < n && id < total; ++k, id += W) {
+    const int c = find_chunk(p, id);
+    const KChunk &ch = p.chunk[c];
+    const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << LG;
+    const uint64_t src = ch.src + off;
+    const uint32_t len = (uint32_t)umin64(ch.bytes - off, 1ull << LG);
+    if (((src | len) & 15) == 0) prefetch_l2(src, len);
+  }
+}
+
 // Warp-strided streaming copy: the round is cut into 4 KiB units; warp w of
 // W takes units w, w+W, w+2W ... and keeps U units (U x 8 x 16 B per lane)
 // in flight before storing.  No tile claims, no CTA barriers on the hot
@@ -330,11 +356,13 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
 // byte path.
 template <bool COUNT, int U, class KP>
 __global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ KP p) {
-  pdl_wait();
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   const uint32_t lane = threadIdx.x & 31;
   const uint32_t W = gridDim.x * (kThreads / 32);
   const uint32_t w0 = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+  prefetch_units<12>(p, w0, W, total, lane);
+  pdl_wait();
+  if (p.flags & kFlagEarlyTrigger) pdl_trigger();
   for (uint32_t base = w0; base < total; base += W * U) {
     int4 v[U][8];
     uint64_t dsts[U];
@@ -390,7 +418,116 @@ __global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ K
       }
     }
   }
-  pdl_trigger();
+  if (!(p.flags & kFlagEarlyTrigger)) pdl_trigger();
+  finish_round(p);
+}
+
+// 256-bit global accesses (sm_100: LDG.256 / STG.256).  H selects L2
+// eviction priorities (bit0: loads evict_first -- a source is read once;
+// bit1: stores evict_first; bit2: stores evict_last -- the consumer reads
+// the destination next).  The .L2::evict_* qualifiers exist only for the
+// 256-bit forms.
+struct alignas(32) V8 {
+  uint32_t x[8];
+};
+template <int H>
+__device__ __forceinline__ V8 ld256(const V8 *p) {
+  V8 r;
+  if (H & 1)
+    asm volatile("ld.global.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.x[0]), "=r"(r.x[1]), "=r"(r.x[2]), "=r"(r.x[3]), "=r"(r.x[4]), "=r"(r.x[5]),
+                   "=r"(r.x[6]), "=r"(r.x[7])
+                 : "l"(p));
+  else
+    asm volatile("ld.global.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(r.x[0]), "=r"(r.x[1]), "=r"(r.x[2]), "=r"(r.x[3]), "=r"(r.x[4]), "=r"(r.x[5]),
+                   "=r"(r.x[6]), "=r"(r.x[7])
+                 : "l"(p));
+  return r;
+}
+template <int H>
+__device__ __forceinline__ void st256(V8 *p, const V8 &v) {
+  if (H & 2)
+    asm volatile("st.global.L1::no_allocate.L2::evict_first.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p),
+                 "r"(v.x[0]), "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]),
+                 "r"(v.x[7])
+                 : "memory");
+  else if (H & 4)
+    asm volatile("st.global.L1::no_allocate.L2::evict_last.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p),
+                 "r"(v.x[0]), "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]),
+                 "r"(v.x[7])
+                 : "memory");
+  else
+    asm volatile("st.global.L1::no_allocate.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.x[0]),
+                 "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]), "r"(v.x[7])
+                 : "memory");
+}
+
+// Warp-strided copy with 256-bit accesses: units of 2^LG bytes (4 or 8 KiB),
+// warp w of W takes units w, w+W, ...; each lane keeps 2^LG / 1 KiB 32-byte
+// loads in flight per unit.  32 B aligned full units take the 256-bit path;
+// anything else the 16 B / byte fallback of the ws engine.
+template <bool COUNT, int LG, int H, class KP>
+__global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ KP p) {
+  constexpr uint32_t kUnit = 1u << LG;
+  constexpr int kPer = (int)(kUnit / (32 * 32));  // 32 B loads per lane per unit
+  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t W = gridDim.x * (kThreads / 32);
+  prefetch_units<LG>(p, blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5), W, total, lane);
+  pdl_wait();
+  if (p.flags & kFlagEarlyTrigger) pdl_trigger();
+  const uint32_t ahead = (p.flags & kFlagPfLoop) ? ((p.flags >> kPfShift) & 0xffu) * W : 0u;
+  for (uint32_t id = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5); id < total; id += W) {
+    if (ahead && lane == 0 && id + ahead < total && (p.flags & kFlagLocalSrc)) {
+      const uint32_t a = id + ahead;
+      const int ca = find_chunk(p, a);
+      const uint64_t oa = (uint64_t)(a - (uint32_t)p.tile_prefix[ca]) << LG;
+      const uint64_t sa = p.chunk[ca].src + oa;
+      const uint32_t la = (uint32_t)umin64(p.chunk[ca].bytes - oa, kUnit);
+      if (((sa | la) & 15) == 0) prefetch_l2(sa, la);
+    }
+    const int c = find_chunk(p, id);
+    const KChunk &ch = p.chunk[c];
+    const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << LG;
+    const uint64_t src = ch.src + off, dst = ch.dst + off;
+    const uint32_t len = (uint32_t)umin64(ch.bytes - off, kUnit);
+    if (len == kUnit && ((src | dst) & 31) == 0) {
+      const V8 *sv = reinterpret_cast<const V8 *>(src);
+      V8 *dv = reinterpret_cast<V8 *>(dst);
+      V8 v[kPer];
+#pragma unroll
+      for (int j = 0; j < kPer; ++j) v[j] = ld256<H>(sv + j * 32 + lane);
+#pragma unroll
+      for (int j = 0; j < kPer; ++j) {
+        st256<H>(dv + j * 32 + lane, v[j]);
+        count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
+        count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane) + 16, 16);
+      }
+    } else if (((src | dst) & 15) == 0) {
+      const uint32_t nv = len >> 4;
+      const int4 *sv = reinterpret_cast<const int4 *>(src);
+      int4 *dv = reinterpret_cast<int4 *>(dst);
+      for (uint32_t i = lane; i < nv; i += 32) {
+        st_stream(dv + i, ld_stream(sv + i));
+        count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
+      }
+      uint8_t *d = reinterpret_cast<uint8_t *>(dst);
+      const uint8_t *sp = reinterpret_cast<const uint8_t *>(src);
+      for (uint32_t i = (nv << 4) + lane; i < len; i += 32) {
+        d[i] = sp[i];
+        count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
+      }
+    } else {
+      uint8_t *d = reinterpret_cast<uint8_t *>(dst);
+      const uint8_t *sp = reinterpret_cast<const uint8_t *>(src);
+      for (uint32_t i = lane; i < len; i += 32) {
+        d[i] = sp[i];
+        count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
+      }
+    }
+  }
+  if (!(p.flags & kFlagEarlyTrigger)) pdl_trigger();
   finish_round(p);
 }
 
@@ -589,7 +726,7 @@ static int variant_from_env() {
       std::string s(e);
       v = s == "ldst8" ? 0 : s == "ldst16" ? 1 : s == "tma4" ? 2 : s == "tma8" ? 3 : s == "tma12" ? 4
         : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : s == "wd1" ? 8 : s == "wd2" ? 9
-        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : -1;
+        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : s == "wv4" ? 13 : s == "wv8" ? 14 : -1;
     }
   }
   return v;
@@ -652,6 +789,51 @@ static void launch_ws(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   else launch_pdl(gr_copy_ws<false, U, KP>, grid, kThreads, 0, s, p);
 }
 
+static int hint_from_env() {
+  static int h = -1;
+  if (h < 0) {
+    const char *e = getenv("GR_HINT");
+    h = e ? atoi(e) : 0;
+    if (h < 0 || h > 5) h = 0;
+  }
+  return h;
+}
+
+template <int LG, int H, class KP>
+static void launch_wv_h(KP &p, uint64_t grid, cudaStream_t s) {
+  if (p.counts) launch_pdl(gr_copy_wv<true, LG, H, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_wv<false, LG, H, KP>, grid, kThreads, 0, s, p);
+}
+
+template <int LG, class KP>
+static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  static int occ = 0;
+  if (!occ) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, LG, 0, KP>, kThreads, 0);
+    if (occ <= 0) occ = 1;
+  }
+  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
+  p.tile_log2 = LG;
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += (p.chunk[i].bytes + (1ull << LG) - 1) >> LG;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+  uint64_t grid = (t + (kThreads / 32) - 1) / (kThreads / 32);
+  const uint64_t cap = (uint64_t)sm_count * per_sm;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  switch (hint_from_env()) {
+    case 1: launch_wv_h<LG, 1>(p, grid, s); break;
+    case 2: launch_wv_h<LG, 2>(p, grid, s); break;
+    case 3: launch_wv_h<LG, 3>(p, grid, s); break;
+    case 4: launch_wv_h<LG, 4>(p, grid, s); break;
+    case 5: launch_wv_h<LG, 5>(p, grid, s); break;
+    default: launch_wv_h<LG, 0>(p, grid, s); break;
+  }
+}
+
 template <int U, class KP>
 static void launch_wd(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   static int occ = 0;
@@ -696,6 +878,8 @@ static void launch_gs(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
 template <class KP>
 static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
   switch (v) {
+    case 13: launch_wv<12>(p, sm_count, ctas_per_sm, s); break;
+    case 14: launch_wv<13>(p, sm_count, ctas_per_sm, s); break;
     case 10: launch_gs<8>(p, sm_count, ctas_per_sm, s); break;
     case 11: launch_gs<4>(p, sm_count, ctas_per_sm, s); break;
     case 12: launch_gs<16>(p, sm_count, ctas_per_sm, s); break;
@@ -740,14 +924,32 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
   int v = variant_from_env();
   // default: the 8-stage TMA bulk ring for large aligned rounds (best at
-  // >= 64 MiB), the warp-strided LD/ST engine otherwise; GROUTER_COPY_TMA
-  // forces the bulk ring for every aligned round
-  if (v < 0) v = (tma || (aligned && total >= (64ull << 20))) ? 3 : 5;
-  if (((v >= 2 && v <= 4) || v >= 10) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
+  // >= 256 MiB: 6.47 TB/s at 1 GiB; tools/engine_sizes.py), otherwise the warp-strided 256-bit engine over 8 KiB units
+  // (wv8) whose warps prefetch their first unit into L2 before the PDL wait
+  // (38.5 MB get_into back to back: 13.2 us with ws1, 11.8 us with wv8 +
+  // prefetch); GROUTER_COPY_TMA forces the bulk ring for every aligned round
+  if (v < 0) v = (tma || (aligned && total >= (256ull << 20))) ? 3 : 14;
+  if (((v >= 2 && v <= 4) || (v >= 10 && v <= 12)) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
   // static-assignment engines (ws, gs) need no scratch: their completion can
   // be published by a stream write after the launch, which costs the GPU
   // ~2 us less than the in-kernel fence + counter + last-CTA protocol
-  const bool is_static = (v >= 5 && v <= 7) || v >= 10;
+  const bool is_static = (v >= 5 && v <= 7) || v >= 10;  // ws, gs, wv
+  p.flags &= ~(kFlagEarlyTrigger | kFlagPfLoop | (0xffu << kPfShift));
+  if ((v >= 5 && v <= 7) || v == 13 || v == 14) {  // ws / wv: L2 prefetch + early trigger
+    static int pf = -1, early = -1, loop = -1;
+    if (pf < 0) {
+      const char *e = getenv("GR_PF");
+      pf = e ? atoi(e) : 1;  // measured best: one unit per warp (tools/exp_hints.sh)
+      if (pf < 0 || pf > 255) pf = 0;
+      const char *t = getenv("GR_EARLY");
+      early = t ? atoi(t) : 0;
+      const char *l = getenv("GR_PFLOOP");
+      loop = l ? atoi(l) : 0;
+    }
+    p.flags |= (uint32_t)pf << kPfShift;
+    if (early) p.flags |= kFlagEarlyTrigger;
+    if (loop && v >= 13) p.flags |= kFlagPfLoop;
+  }
   p.flags &= ~kFlagNoPublish;
   if (host_publish && is_static && !p.counts) {
     p.flags |= kFlagNoPublish;
@@ -914,7 +1116,7 @@ extern "C" grouter_status grouter_test_copy(void *dst_base, const void *src_base
     cudaMemset(scratch[dev], 0, 2 * sizeof(uint32_t));
   }
   CopyParams *p = new CopyParams();
-  p->flags = kFlagLocalDst;  // test copies stay on the current device
+  p->flags = kFlagLocalDst | kFlagLocalSrc;  // test copies stay on the current device
   p->n_chunks = n_chunks;
   p->scratch = scratch[dev];
   p->counts = counts;

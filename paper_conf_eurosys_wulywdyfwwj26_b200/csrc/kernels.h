@@ -30,6 +30,10 @@ struct KPublish {
 constexpr uint32_t kFlagPdl = 1;        // launched with programmatic stream serialization
 constexpr uint32_t kFlagLocalDst = 2;   // every destination is in this GPU's memory
 constexpr uint32_t kFlagNoPublish = 4;  // completion written by the host after the launch
+constexpr uint32_t kFlagLocalSrc = 8;   // every source is in this GPU's memory (L2 prefetch is safe)
+constexpr uint32_t kFlagEarlyTrigger = 16;  // let the successor launch right after our own wait
+constexpr uint32_t kPfShift = 8;        // flags >> kPfShift & 0xff: units per warp prefetched to L2
+constexpr uint32_t kFlagPfLoop = 1u << 16;  // keep prefetching that many units ahead inside the loop
 
 // Kernel parameters (passed by value, __grid_constant__).  Two capacities:
 // the large one for rounds with many distinct chunks, a small one (a few

@@ -68,19 +68,25 @@ def test_copy_kernel_exactly_once(tma, src_off, dst_off):
     _copy_exactly_once(tma, src_off, dst_off)
 
 
-VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4", "wd1", "wd2", "gs4", "gs8", "gs16"]
+VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4", "wd1", "wd2", "gs4", "gs8", "gs16",
+            "wv4", "wv8", "wv4:GR_HINT=3", "wv8:GR_HINT=5", "wv4:GR_PF=2:GR_EARLY=1", "ws1:GR_PF=1:GR_EARLY=1",
+            "wv8:GR_PF=1", "wv8:GR_PF=2:GR_PFLOOP=1"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
 def test_copy_kernel_variants(variant):
-    """Every engine variant (GR_COPY) in a subprocess: byte-exact over aligned
-    and misaligned chunk lists, exactly-once counts where it can count."""
+    """Every engine variant (GR_COPY[:ENV=VAL...]: cache hints, L2 prefetch,
+    early PDL trigger) in a subprocess: byte-exact over aligned and
+    misaligned chunk lists, exactly-once counts where it can count."""
     import os
     import subprocess
     import sys
+    name, *extra = variant.split(":")
+    env = dict(os.environ, GR_COPY=name)
+    env.update(kv.split("=", 1) for kv in extra)
     code = ("import sys; sys.path.insert(0, '.'); from tests.test_gpu_parity import _copy_exactly_once as f; "
-            "[f(t, a, b) for t in (False, True) for a, b in ((0, 0), (3, 3), (1, 0), (7, 13))]")
-    r = subprocess.run([sys.executable, "-c", code], env=dict(os.environ, GR_COPY=variant),
+            "[f(t, a, b) for t in (False, True) for a, b in ((0, 0), (3, 3), (1, 0), (7, 13), (32, 64))]")
+    r = subprocess.run([sys.executable, "-c", code], env=env,
                        capture_output=True, text=True, timeout=240)
     assert r.returncode == 0, r.stderr[-2000:]
 
