@@ -18,6 +18,7 @@
 #include <cstdio>
 #include <sstream>
 #include "ctx.h"
+#include "kernels.h"
 
 using namespace gr;
 
@@ -239,10 +240,13 @@ void block_on(grouter_ctx *c, Guard &g, const Fences &f) {
     host_wait(f);
     return;
   }
-  pump(c, false);
-  c->cv.notify_one();
+  const uint64_t t0 = hprof().on ? now_ns() : 0;
+  pump(c, false);  // wakes the daemon itself when work stays queued (a futex wake costs ~2.6 us)
   g.lk.unlock();
+  if (hprof().on) hprof().t[13] += now_ns() - t0;  // pump + daemon notify
+  const uint64_t t1 = hprof().on ? now_ns() : 0;
   host_wait(f);
+  if (hprof().on) hprof().t[15] += now_ns() - t1;
 }
 
 // Stream-ordered completion for device callers: work enqueued on `s` after
@@ -397,12 +401,29 @@ grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
 
 grouter_status grouter_finalize(grouter_ctx *c) {
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
-  if (hprof().on && hprof().calls) {
+  if (hprof().on && (hprof().calls || hprof().put_calls)) {
     HostProf &h = hprof();
     fprintf(stderr, "[grouter host profile] get_into calls %llu: lock+lookup %.2f us, transfer+launch %.2f us, "
                     "fences+consume %.2f us, ordering %.2f us\n",
             (unsigned long long)h.calls, h.t[0] / h.calls / 1e3, h.t[1] / h.calls / 1e3,
             h.t[2] / h.calls / 1e3, h.t[3] / h.calls / 1e3);
+    if (g_launch_prof_n) {
+      double q10, q50, q90;
+      launch_prof_percentiles(&q10, &q50, &q90);
+      fprintf(stderr, "[grouter host profile] launch_copy x%llu: prepare %.2f us, launch call %.2f us "
+                      "(p10/p50/p90 %.2f/%.2f/%.2f), cudaGetLastError %.2f us\n",
+              (unsigned long long)g_launch_prof_n, g_launch_prof[0] / g_launch_prof_n / 1e3,
+              g_launch_prof[1] / g_launch_prof_n / 1e3, q10, q50, q90, g_launch_prof[2] / g_launch_prof_n / 1e3);
+    }
+    if (h.put_calls)
+      fprintf(stderr, "[grouter host profile] blocking put calls %llu: reserve %.2f us, pageable check %.2f us, "
+                      "transfer+dispatch %.2f us, observe %.2f us, block_on %.2f us (of it pump+notify %.2f us)\n",
+              (unsigned long long)h.put_calls, h.t[8] / h.put_calls / 1e3, h.t[9] / h.put_calls / 1e3,
+              h.t[10] / h.put_calls / 1e3, h.t[11] / h.put_calls / 1e3, h.t[12] / h.put_calls / 1e3,
+              h.t[13] / h.put_calls / 1e3);
+    if (h.put_calls)
+      fprintf(stderr, "[grouter host profile] put call -> first H2D copy submitted %.2f us, host wait %.2f us\n",
+              h.t[14] / h.put_calls / 1e3, h.t[15] / h.put_calls / 1e3);
     if (h.t[4] > 0)
       fprintf(stderr, "[grouter host profile] inside transfer: plan+xfer+enqueue %.2f us, take %.2f us, "
                       "params %.2f us, launch %.2f us\n",
@@ -433,6 +454,9 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
   if (!fn || !out || !valid_loc(c, fn->device) ||
       !(hint == GROUTER_NOHINT || hint == GROUTER_HOST || valid_gpu(c, hint)) || (!src && n))
     return fail(GROUTER_EINVAL, "put: bad argument");
+  HostProf &hp = hprof();
+  uint64_t p0 = hp.on ? now_ns() : 0, p1 = 0, p2 = 0, p3 = 0, p4 = 0;
+  if (hp.on) tl_put_t0 = p0;
   const int from = fn->device;
   const bool blocking = !stream || from == GROUTER_HOST;
   int home = from != GROUTER_HOST ? from : (hint >= 0 ? hint : GROUTER_HOST);  // L165, R23
@@ -440,6 +464,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
   if (home != GROUTER_HOST && !reserve(c, home, ch)) home = GROUTER_HOST;    // R16
   if (home == GROUTER_HOST && !host_reserve(c, ch)) return fail(GROUTER_ENOMEM, "host store full");
   uint8_t *ptr = storage(c, home, ch);
+  if (hp.on) p1 = p2 = now_ns();
   Obj o;
   o.oid = c->next_oid++;
   o.wf = fn->workflow_id;
@@ -456,6 +481,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
       std::memcpy(ptr, src, n);  // cFn -> host store: plain memcpy
     } else {
       bool pageable = from == GROUTER_HOST && is_pageable(src);
+      if (hp.on) p2 = now_ns();
       bool direct = false;
       XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr, Fences{},
                                  pageable, blocking ? nullptr : (cudaStream_t)stream, from, true,
@@ -465,10 +491,21 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
       if (!blocking && !direct) order_after(c, g, (cudaStream_t)stream, done);
     }
   }
+  if (hp.on) p3 = now_ns();
   *out = o.oid;
   observe(c, o);
   c->objects.emplace(o.oid, std::move(o));
+  if (hp.on) p4 = now_ns();
   if (blocking && (c->replay || !done.empty())) block_on(c, g, done);
+  if (hp.on && blocking) {
+    const uint64_t p5 = now_ns();
+    hp.put_calls++;
+    hp.t[8] += p1 - p0;   // reserve + storage
+    hp.t[9] += p2 - p1;   // pageable check
+    hp.t[10] += p3 - p2;  // plan + transfer + dispatch
+    hp.t[11] += p4 - p3;  // observe + object table
+    hp.t[12] += p5 - p4;  // block_on (pump, notify, wait)
+  }
   return GROUTER_OK;
   API_CATCH(c)
 }

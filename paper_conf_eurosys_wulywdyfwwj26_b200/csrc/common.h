@@ -159,10 +159,11 @@ inline void prune(Fences &f) {
 // printed to stderr at grouter_finalize (tuning aid).
 struct HostProf {
   bool on = false;
-  uint64_t calls = 0;
-  double t[8] = {};
+  uint64_t calls = 0, put_calls = 0;
+  double t[16] = {};  // [0..7] get_into stages, [8..15] blocking put stages
 };
 HostProf &hprof();
 uint64_t now_ns();
+extern thread_local uint64_t tl_put_t0;  // profiling: start of the current blocking put
 
 }  // namespace gr

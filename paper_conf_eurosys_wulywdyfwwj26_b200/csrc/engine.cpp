@@ -517,9 +517,14 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   // (per-copy engine overhead ~3.6 us measured by the probe)
   uint64_t run_src = 0, run_dst = 0, run_len = 0;
   auto flush_run = [&]() {
-    if (run_len)
+    if (run_len) {
       GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyHostToDevice,
                               s.stream));
+      if (tl_put_t0) {  // profiling: put call -> its first H2D copy submitted
+        hprof().t[14] += now_ns() - tl_put_t0;
+        tl_put_t0 = 0;
+      }
+    }
     run_len = 0;
   };
   auto end_segment = [&]() {

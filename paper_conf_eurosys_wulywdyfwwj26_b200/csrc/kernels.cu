@@ -18,6 +18,8 @@
 #include <chrono>
 #include <cstdlib>
 #include <string>
+#include <vector>
+#include <algorithm>
 
 #include "../../include/grouter.h"
 #include "../../include/grouter_testing.h"
@@ -896,7 +898,30 @@ static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStre
   }
 }
 
+double g_launch_prof[3] = {};
+uint64_t g_launch_prof_n = 0;
+bool g_launch_prof_on = [] {
+  const char *e = getenv("GROUTER_HOST_PROFILE");
+  return e && e[0] == '1';
+}();
+static std::vector<uint32_t> g_launch_ns;
+void launch_prof_percentiles(double *p10, double *p50, double *p90) {
+  std::vector<uint32_t> v = g_launch_ns;
+  std::sort(v.begin(), v.end());
+  auto at = [&](double q) { return v.empty() ? 0.0 : v[(size_t)(q * (v.size() - 1))] / 1e3; };
+  *p10 = at(0.1);
+  *p50 = at(0.5);
+  *p90 = at(0.9);
+}
+static inline uint64_t lp_now() {
+  return (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
 int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream, bool *host_publish) {
+  const uint64_t lp0 = g_launch_prof_on ? lp_now() : 0;
+  uint64_t lp1 = 0, lp2 = 0;
   if (host_publish) *host_publish = false;
   if (p.n_chunks == 0) return (int)cudaSuccess;
   static int ctas_env = -1;
@@ -965,11 +990,22 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
     q.count_base = p.count_base;
     for (uint32_t i = 0; i < p.n_chunks; ++i) q.chunk[i] = p.chunk[i];
     for (uint32_t i = 0; i < p.n_pub; ++i) q.pub[i] = p.pub[i];
+    if (g_launch_prof_on) lp1 = lp_now();
     launch_variant(q, v, sm_count, ctas_per_sm, s);
   } else {
+    if (g_launch_prof_on) lp1 = lp_now();
     launch_variant(p, v, sm_count, ctas_per_sm, s);
   }
-  return (int)cudaGetLastError();
+  if (g_launch_prof_on) lp2 = lp_now();
+  const int err = (int)cudaGetLastError();
+  if (g_launch_prof_on) {
+    g_launch_prof[0] += lp1 - lp0;
+    g_launch_prof[1] += lp2 - lp1;
+    if (g_launch_ns.size() < (1u << 20)) g_launch_ns.push_back((uint32_t)(lp2 - lp1));
+    g_launch_prof[2] += lp_now() - lp2;
+    g_launch_prof_n++;
+  }
+  return err;
 }
 
 // ------------------------------------------------------------------ test kernels (K9)
@@ -1054,8 +1090,25 @@ extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, 
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   if (kind == 6) cudaEventRecord(ev, s);
+  // kind >= 100: latency mode -- the stream is drained before every launch
+  // and only the launch call itself is timed
+  // kind >= 200: like 100 plus a 50 us host spin after the drain (GPU and
+  // link left idle as between latency-mode requests)
+  const bool spin = kind >= 200;
+  if (spin) kind -= 100;
+  const bool idle = kind >= 100;
+  if (idle) kind -= 100;
+  double idle_us = 0;
   auto t0 = std::chrono::steady_clock::now();
   for (int i = 0; i < n; ++i) {
+    auto ti = std::chrono::steady_clock::now();
+    if (idle) {
+      cudaStreamSynchronize(s);
+      if (spin)
+        while (std::chrono::steady_clock::now() - ti < std::chrono::microseconds(50)) {
+        }
+      ti = std::chrono::steady_clock::now();
+    }
     if (kind == 0) gr_empty_kernel_tiny<<<blocks, 256, 0, s>>>(i);
     else if (kind == 1) gr_empty_kernel<<<blocks, 256, 0, s>>>(sp);
     else if (kind == 2) gr_empty_kernel_big<<<blocks, 256, 0, s>>>(bp);
@@ -1063,11 +1116,31 @@ extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, 
       cfg.numAttrs = kind == 3 ? 1 : 0;
       cudaLaunchKernelEx(&cfg, gr_empty_kernel, sp);
     } else if (kind == 5) cudaEventRecord(ev, s);
-    else (void)cudaEventQuery(ev);
+    else if (kind == 6) (void)cudaEventQuery(ev);
+    else {  // 7: launch_copy of 4 KiB, 8: of 38.5 MB (the production launch path), 9: event + 8
+      static uint8_t *buf = nullptr;
+      static uint32_t *scr = nullptr;
+      if (!buf) {
+        cudaMalloc(&buf, 2 * 38535168ull);
+        cudaMalloc(&scr, 64);
+        cudaMemset(scr, 0, 64);
+      }
+      if (kind == 9) cudaEventRecord(ev, s);
+      CopyParams &q = bp;
+      q.flags = kFlagLocalDst | kFlagLocalSrc;
+      q.n_chunks = 1;
+      q.n_pub = 0;
+      q.scratch = scr;
+      q.counts = nullptr;
+      q.chunk[0] = {(uint64_t)buf, (uint64_t)buf + 38535168ull, kind == 7 ? 4096ull : 38535168ull};
+      bool hp = false;
+      launch_copy(q, 148, 4, false, s, &hp);
+    }
+    if (idle) idle_us += std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - ti).count();
   }
   auto t1 = std::chrono::steady_clock::now();
   cudaStreamSynchronize(s);
-  *us_per_launch = std::chrono::duration<double, std::micro>(t1 - t0).count() / n;
+  *us_per_launch = idle ? idle_us / n : std::chrono::duration<double, std::micro>(t1 - t0).count() / n;
   return cudaGetLastError() == cudaSuccess ? GROUTER_OK : GROUTER_ECUDA;
 }
 

@@ -61,6 +61,13 @@ using SmallParams = KParams<8, 8>;
 // assignment (no ticket scratch to reset), the kernel skips its completion
 // protocol and *host_publish = true: the CALLER must publish p.pub with
 // stream writes right after the launch on the same stream.
+// GROUTER_HOST_PROFILE tuning aid: host ns inside launch_copy
+// [0] before the launch call, [1] the launch call, [2] cudaGetLastError.
+extern double g_launch_prof[3];
+extern uint64_t g_launch_prof_n;
+extern bool g_launch_prof_on;
+void launch_prof_percentiles(double *p10, double *p50, double *p90);  // us, launch call
+
 int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *stream,
                 bool *host_publish = nullptr);
 

@@ -48,6 +48,7 @@ static int bt_init = [] {
   return 0;
 }();
 
+thread_local uint64_t tl_put_t0 = 0;
 HostProf &hprof() {
   static HostProf h = [] {
     HostProf x;

@@ -5,19 +5,14 @@ import torch
 from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G
 lib = G.load()
 s = torch.cuda.Stream()
-for stream_name, st in (("torch stream", s.cuda_stream), ("legacy default", 0)):
-    for kind in (0, 1, 2, 3, 4, 5, 6):
-        for blocks in (592,):
-            for rep in range(2):
+names = {0: "<<<>>> int arg", 1: "<<<>>> SmallParams", 2: "<<<>>> CopyParams (5 KB)", 3: "LaunchKernelEx PDL",
+         4: "LaunchKernelEx", 5: "EventRecord", 6: "EventQuery", 7: "launch_copy 4 KiB (wv8)",
+         8: "launch_copy 38.5 MB (wv8)", 9: "event record + launch_copy 38.5 MB"}
+for mode, off in (("back-to-back", 0), ("idle stream (sync before each)", 100)):
+    for stream_name, st in (("torch stream", s.cuda_stream), ("legacy default", 0)):
+        for kind in (0, 1, 2, 3, 4, 5, 6, 7, 8, 9):
+            for blocks in ((1, 592) if kind < 7 else (0,)):
                 v = C.c_double(0)
-                G.check(lib.grouter_test_launch_cost(kind, 2000, blocks, st or None, C.byref(v)))
-            print(stream_name, "kind", kind, "blocks", blocks, "us/launch", round(v.value, 2), flush=True)
-# torch's own launch cost for comparison
-x = torch.empty(1, device="cuda")
-import time
-with torch.cuda.stream(s):
-    for _ in range(100): x.add_(1)
-    torch.cuda.synchronize()
-    t = time.perf_counter()
-    for _ in range(2000): x.add_(1)
-    print("torch add_ us/launch", round((time.perf_counter() - t) * 1e6 / 2000, 2))
+                for rep in range(2):
+                    G.check(lib.grouter_test_launch_cost(kind + off, 500, blocks, st or None, C.byref(v)))
+                print(mode, stream_name, names[kind], "blocks", blocks, "us/call", round(v.value, 2), flush=True)
