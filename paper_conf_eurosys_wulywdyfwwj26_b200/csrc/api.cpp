@@ -15,6 +15,7 @@
 #include "../../include/grouter.h"
 #include "../../include/grouter_testing.h"
 
+#include <chrono>
 #include <cstdio>
 #include <sstream>
 #include "ctx.h"
@@ -242,6 +243,8 @@ void block_on(grouter_ctx *c, Guard &g, const Fences &f) {
   }
   const uint64_t t0 = hprof().on ? now_ns() : 0;
   pump(c, false);  // wakes the daemon itself when work stays queued (a futex wake costs ~2.6 us)
+  static const bool always_notify = getenv("GR_BLOCK_NOTIFY") != nullptr;
+  if (always_notify) c->cv.notify_one();
   g.lk.unlock();
   if (hprof().on) hprof().t[13] += now_ns() - t0;  // pump + daemon notify
   const uint64_t t1 = hprof().on ? now_ns() : 0;
@@ -266,7 +269,34 @@ void order_after(grouter_ctx *c, Guard &g, cudaStream_t s, const Fences &f) {
     if (!all_submitted()) {
       pump(c, false);
       c->cv.notify_one();
-      c->submit_cv.wait(g.lk, all_submitted);
+      static const bool diag = getenv("GR_DIAG") != nullptr;
+      if (!diag) {
+        c->submit_cv.wait(g.lk, all_submitted);
+      } else {  // diagnostics: report the servers' state when a submission stalls
+        const uint64_t t0 = now_ns();
+        while (!c->submit_cv.wait_for(g.lk, std::chrono::milliseconds(50), all_submitted)) {
+          fprintf(stderr, "[grouter diag] order_after: transfer unsubmitted for %.0f ms\n", (now_ns() - t0) / 1e6);
+          const char *kn[] = {"copy", "h2d", "d2h"};
+          for (size_t i = 0; i < c->dev.size(); ++i) {
+            Server *sv[] = {&c->dev[i].copy, &c->dev[i].h2d, &c->dev[i].d2h};
+            for (int k = 0; k < 3; ++k) {
+              Server &q = *sv[k];
+              std::string inf;
+              for (auto &f : q.inflight) {
+                inf += f.w.done() ? "D" : "p";
+                if (f.w.word) inf += "(w " + std::to_string(*f.w.word) + "/" + std::to_string(f.w.target) + ")";
+              }
+              fprintf(stderr, "  dev %zu %s: sched %llu carry %zu urgent %zu inflight [%s]\n", i, kn[k],
+                      (unsigned long long)q.sched.backlog_items, q.carry.size(), q.urgent.size(), inf.c_str());
+            }
+          }
+          for (auto &w : f)
+            if (w.producer)
+              fprintf(stderr, "  waiting on xfer %llu: %u/%u chunks submitted, %zu deps\n",
+                      (unsigned long long)w.producer->id, w.producer->submitted_chunks, w.producer->nchunks,
+                      w.producer->deps.size());
+        }
+      }
     }
   }
   caller_wait(c, s, f);

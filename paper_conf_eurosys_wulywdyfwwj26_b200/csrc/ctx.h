@@ -46,7 +46,11 @@ struct PageHeap {
 struct DevicePool {
   int logical = -1, phys = -1;
   CUdeviceptr base = 0;
-  uint64_t va_size = 0, mapped = 0;
+  // mapped: physical bytes mapped; va_top: VA offset where the next segment
+  // maps (> mapped only while detached segments are being unmapped, or after
+  // a grow raced an unmap and left a hole that is never handed out)
+  uint64_t va_size = 0, mapped = 0, va_top = 0;
+  uint64_t excess_since = 0;  // ns since mapped first exceeded the trim mark (0 = not over)
   struct Seg {
     uint64_t off, size;
     CUmemGenericAllocationHandle h;
@@ -56,7 +60,14 @@ struct DevicePool {
   std::vector<int> access;  // physical devices that may access the pages
   void init(int logical, int phys, uint64_t va, const std::vector<int> &access, uint64_t prewarm);
   void grow(uint64_t need);
-  void trim(uint64_t keep);
+  // trim in two steps so the (slow, up to ~0.8 s measured) cuMemUnmap runs
+  // without the context lock: detach() takes trailing free segments out of
+  // the heap (lock held), unmap() releases them (lock NOT held), settle()
+  // lowers va_top again when nothing mapped above them meanwhile (lock held)
+  std::vector<Seg> detach(uint64_t keep);
+  static void unmap(CUdeviceptr base, const std::vector<Seg> &segs);
+  void settle(const std::vector<Seg> &segs);
+  void trim(uint64_t keep);  // all three steps with the lock held (tests, shutdown)
   void destroy();
 };
 

@@ -26,6 +26,7 @@
 //    pushes it over NVLink into the lease on d and publishes the word; the
 //    slot is reused after the forward round's event.
 #include <algorithm>
+#include <cstdio>
 #include <chrono>
 #include <cstring>
 #include <thread>
@@ -784,6 +785,8 @@ void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst) {
 }
 
 // ------------------------------------------------------------------ lifecycle
+static constexpr uint64_t kTrimDelayNs = 1000000000ull;  // 1 s of sustained excess before a trim
+
 static void daemon_main(grouter_ctx *c) {
   std::unique_lock<std::mutex> lk(c->mu);
   auto last_trim = std::chrono::steady_clock::now();
@@ -803,6 +806,7 @@ static void daemon_main(grouter_ctx *c) {
       auto now = std::chrono::steady_clock::now();
       if (now - last_trim > std::chrono::milliseconds(50)) {  // I/O thread: reclaim (L269)
         last_trim = now;
+        static const bool diag = getenv("GR_DIAG") != nullptr;
         for (size_t i = 0; i < c->dev.size(); ++i) {
           LogicalDev &d = c->dev[i];
           DeviceGuard g(d.phys);
@@ -810,6 +814,7 @@ static void daemon_main(grouter_ctx *c) {
           // histogram-driven size (L250-L256, R44): pre-warm one segment per
           // tick toward the target, trim back to max(used, target)
           const uint64_t tgt = pool_target(c, (int)i);
+          const uint64_t t0 = diag ? now_ns() : 0, m0 = d.pool.mapped;
           if (d.pool.mapped < tgt) {
             try {
               d.pool.grow(std::min<uint64_t>(tgt - d.pool.mapped, 64ull << 20));
@@ -817,7 +822,34 @@ static void daemon_main(grouter_ctx *c) {
               // HBM short: pre-warming is best effort
             }
           }
-          d.pool.trim(std::max<uint64_t>(d.used, tgt) + (64ull << 20));
+          const uint64_t t1 = diag ? now_ns() : 0, m1 = d.pool.mapped;
+          // trim only once the excess has lasted kTrimDelay and this GPU's
+          // servers are idle, and unmap WITHOUT the context lock: cuMemUnmap
+          // of a few hundred MiB took up to ~0.8 s under load (it drains the
+          // GPU), which stalled every API call behind the lock
+          const uint64_t keep = std::max<uint64_t>(d.used, tgt) + (64ull << 20);
+          const uint64_t tnow = now_ns();
+          if (d.pool.mapped <= keep) d.pool.excess_since = 0;
+          else if (!d.pool.excess_since) d.pool.excess_since = tnow;
+          const bool idle = d.copy.inflight.empty() && d.h2d.inflight.empty() && d.d2h.inflight.empty() &&
+                            !has_work(d.copy) && !has_work(d.h2d) && !has_work(d.d2h);
+          if (d.pool.excess_since && tnow - d.pool.excess_since >= kTrimDelayNs && idle) {
+            std::vector<DevicePool::Seg> v = d.pool.detach(keep);
+            if (!v.empty()) {
+              const CUdeviceptr base = d.pool.base;
+              lk.unlock();
+              DevicePool::unmap(base, v);
+              lk.lock();
+              d.pool.settle(v);
+            }
+            d.pool.excess_since = 0;
+          }
+          if (diag && now_ns() - t0 > 5000000)
+            fprintf(stderr, "[grouter diag] pool tick dev %zu: grow %.1f ms (%llu -> %llu MiB), trim %.1f ms "
+                            "(-> %llu MiB), used %llu MiB, target %llu MiB\n",
+                    i, (t1 - t0) / 1e6, (unsigned long long)(m0 >> 20), (unsigned long long)(m1 >> 20),
+                    (now_ns() - t1) / 1e6, (unsigned long long)(d.pool.mapped >> 20),
+                    (unsigned long long)(d.used >> 20), (unsigned long long)(tgt >> 20));
         }
         c->host.heap.reclaim();
       }

@@ -253,8 +253,8 @@ void DevicePool::init(int lg, int ph, uint64_t va, const std::vector<int> &acc, 
 void DevicePool::grow(uint64_t need) {
   need = charge(need);
   uint64_t seg = std::max<uint64_t>(need, 64ull << 20);
-  if (mapped + seg > va_size) seg = need;
-  if (mapped + seg > va_size) throw Error(GROUTER_ENOMEM, "pool VA range exhausted");
+  if (va_top + seg > va_size) seg = need;
+  if (va_top + seg > va_size) throw Error(GROUTER_ENOMEM, "pool VA range exhausted");
   CUmemAllocationProp prop = {};
   prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
@@ -267,7 +267,7 @@ void DevicePool::grow(uint64_t need) {
     r = drv().memCreate(&h, seg, &prop, 0);
   }
   if (r != CUDA_SUCCESS) throw Error(GROUTER_ENOMEM, "cuMemCreate failed (HBM exhausted)");
-  GR_CU(drv().memMap(base + mapped, seg, 0, h, 0));
+  GR_CU(drv().memMap(base + va_top, seg, 0, h, 0));
   std::vector<CUmemAccessDesc> ad;
   for (int p : access) {
     CUmemAccessDesc a = {};
@@ -276,29 +276,54 @@ void DevicePool::grow(uint64_t need) {
     a.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
     ad.push_back(a);
   }
-  GR_CU(drv().memSetAccess(base + mapped, seg, ad.data(), ad.size()));
-  segs.push_back({mapped, seg, h});
-  heap.give(mapped, seg);
+  GR_CU(drv().memSetAccess(base + va_top, seg, ad.data(), ad.size()));
+  segs.push_back({va_top, seg, h});
+  heap.give(va_top, seg);
+  va_top += seg;
   mapped += seg;
 }
 
-// Unmaps trailing segments that are entirely free while the mapping stays >= keep.
-void DevicePool::trim(uint64_t keep) {
+// Detaches trailing segments that are entirely free while the mapping stays
+// >= keep; their pages leave the heap at once (never handed out again).
+std::vector<DevicePool::Seg> DevicePool::detach(uint64_t keep) {
   heap.reclaim();
+  std::vector<Seg> out;
+  uint64_t end = va_top;
   while (!segs.empty()) {
     Seg s = segs.back();
     if (mapped - s.size < keep) break;
-    if (heap.tail_free(mapped) < s.size) break;
+    if (s.off + s.size != end || heap.tail_free(end) < s.size) break;  // (a hole above: stop)
     // carve the segment out of the trailing free run
     auto it = std::prev(heap.free_runs.end());
     uint64_t run_off = it->first;
     heap.free_runs.erase(it);
     if (s.off > run_off) heap.free_runs[run_off] = s.off - run_off;
-    drv().memUnmap(base + s.off, s.size);
-    drv().memRelease(s.h);
     mapped -= s.size;
     segs.pop_back();
+    out.push_back(s);
+    end = s.off;
   }
+  return out;
+}
+
+void DevicePool::unmap(CUdeviceptr base, const std::vector<Seg> &v) {
+  for (auto &s : v) {
+    drv().memUnmap(base + s.off, s.size);
+    drv().memRelease(s.h);
+  }
+}
+
+// out is in descending VA order; lower va_top only if nothing grew above it
+void DevicePool::settle(const std::vector<Seg> &v) {
+  if (v.empty()) return;
+  const uint64_t hi = v.front().off + v.front().size, lo = v.back().off;
+  if (va_top == hi) va_top = lo;
+}
+
+void DevicePool::trim(uint64_t keep) {
+  auto v = detach(keep);
+  unmap(base, v);
+  settle(v);
 }
 
 void DevicePool::destroy() {
@@ -310,6 +335,7 @@ void DevicePool::destroy() {
   if (base) drv().memAddressFree(base, va_size);
   base = 0;
   mapped = 0;
+  va_top = 0;
 }
 
 static bool all_grounded(const grouter_ctx *c, const Quarantined &q) {
@@ -333,7 +359,7 @@ uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
     P.heap.reclaim();
     if (P.heap.take(len, &off)) return (uint8_t *)(P.base + off);
   }
-  P.grow(len - std::min(len, P.heap.tail_free(P.mapped)));
+  P.grow(len - std::min(len, P.heap.tail_free(P.va_top)));
   if (!P.heap.take(len, &off)) throw Error(GROUTER_ENOMEM, "pool fragmentation");
   return (uint8_t *)(P.base + off);
 }

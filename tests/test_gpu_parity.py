@@ -329,3 +329,19 @@ def test_full_size_cfg1_sampled():
     for o, l in zip(orc["records"], recs):
         if o["op"] == "get":
             assert o["digest"] == l["digest"]
+
+
+def test_full_size_cfg2_cfg5():
+    """cfg2 and cfg5 at their real sizes (39,321,600 B frames + 602,112 B crops;
+    32 x 33,554,432 B KV objects + a 67,108,864 B hidden state per request) on
+    two logical GPUs, cfg5 under a 10% pool limit (queue-aware spill to pinned
+    host, later gets fetched from the host store): statuses, placements,
+    victims, pool accounting and full-byte digests equal the oracle's."""
+    calib = C.virtual(2)
+    for ops, kw in [(T.cfg2(2, requests=3), {}),
+                    (T.cfg5(2, requests=2, limit_frac=0.1), {"host_store_bytes": 3 << 30})]:
+        orc, lib_out = _both(ops, calib, replay=False, keep=False, **kw)
+        spilled = sum(len(r["victims"]) for r in orc["records"])
+        assert compare(orc, lib_out, check_dispatch=False) > 0
+        if kw:
+            assert spilled > 0, "the 10% limit should force spills"

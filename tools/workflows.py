@@ -245,11 +245,19 @@ def cfg5(requests=4, limit_frac=0.1, hints=True, layers=32):
     for r in range(requests):
         B = G.fn(500 + r, 2, 0)
         t0 = time.perf_counter()
-        for oid, nb in objs[r]:
+        slow = []
+        for j, (oid, nb) in enumerate(objs[r]):
+            tc = time.perf_counter()
             st, n = ctx.get_into(B, oid, dst.data_ptr(), nb, s.cuda_stream)
             G.check(st, "get_into")
+            if time.perf_counter() - tc > 2e-3:
+                slow.append((j, round((time.perf_counter() - tc) * 1e3, 1)))
+        ts = time.perf_counter()
         s.synchronize()
         lat.append(time.perf_counter() - t0)
+        if slow or lat[-1] > 0.1:
+            print(f"[cfg5 diag] request {r}: {lat[-1] * 1e3:.1f} ms, submit {1e3 * (ts - t0):.1f} ms, "
+                  f"slow get_into calls (idx, ms) {slow}", file=sys.stderr, flush=True)
     total = time.perf_counter() - t_start
     stt = ctx.stats()
     out = {"requests": requests, "limit_frac": limit_frac, "queue_aware": hints,
