@@ -305,6 +305,82 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
         ctx.free(g0, oid)
         ctx.close()
     out["d2h_speedup"] = round(out["d2h_striped"]["GBps"] / out["d2h_direct"]["GBps"], 2)
+    out.update(measure_d2d_push(world, G, calib, devs))
+    return out
+
+
+def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
+    """cfg1 leg B at N >= 2 inside ONE GROUTER context spanning the node (the
+    paper's deployment: one service per node): a gFn on GPU1 get_into's
+    objects resident on GPU0 -- GPU0's copy server pushes them over NVLink
+    with the SM copy kernel (K2', L167 (1)); the consumer stream waits on the
+    completion words.  Then every GPU i pulls from its ring successor at once
+    (cfg3 (ii), disjoint pairs): aggregate GB/s.  Device-timed with CUDA
+    events on the consumer streams."""
+    import torch
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED] * world,
+                                    pool_floor_bytes=64 << 20))
+    out = {}
+    try:
+        src = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[0]}")
+        resident = {}   # logical GPU -> oids
+        for g in range(world):
+            s0 = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[g]}")
+            for i in range(objs):
+                G.check(G.test_fill(s0.data_ptr(), n, 7000 + i, 0, 0))
+                torch.cuda.synchronize(devs[g])
+                st, oid = ctx.put(G.fn(9, 1, g), s0.data_ptr(), n, G.NOHINT, 0, 0)
+                G.check(st, "put")
+                resident.setdefault(g, []).append(oid)
+        del src
+        ctx.sync()
+
+        def run(pairs):
+            """pairs: [(consumer logical GPU, producer logical GPU)]; returns GB/s aggregate, us/get."""
+            streams = {c: torch.cuda.Stream(device=f"cuda:{devs[c]}") for c, _ in pairs}
+            dst = {c: [torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[c]}") for _ in range(2)]
+                   for c, _ in pairs}
+
+            def one_pass():
+                for i in range(objs):
+                    for c, p in pairs:
+                        st, _ = ctx.get_into(G.fn(9, 2, c), resident[p][i], dst[c][i % 2].data_ptr(), n,
+                                             streams[c].cuda_stream)
+                        G.check(st, "get_into")
+            one_pass()
+            for c, p in pairs:
+                streams[c].synchronize()
+                for b in range(2):   # the last object that wrote binding b
+                    last = max(i for i in range(objs) if i % 2 == b)
+                    st, bad, _ = G.test_verify(dst[c][b].data_ptr(), n, 7000 + last, 0, 0)
+                    assert st == 0 and bad == 0, f"d2d push {p}->{c}: {bad} bytes differ"
+            ev = {c: (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                  for c, _ in pairs}
+            for c, _ in pairs:
+                ev[c][0].record(streams[c])
+            for _ in range(reps):
+                one_pass()
+            for c, _ in pairs:
+                ev[c][1].record(streams[c])
+            for c, _ in pairs:
+                ev[c][1].synchronize()
+            ms = max(ev[c][0].elapsed_time(ev[c][1]) for c, _ in pairs)
+            gets = reps * objs
+            return gets * len(pairs) * n / (ms / 1e3) / 1e9, ms * 1e3 / gets
+
+        gbps, us = run([(1, 0)])
+        out["d2d_push"] = {"what": "GPU1 gFn get_into of GPU0-resident 38.5 MB objects (GPU0 SM push over "
+                                   "NVLink, one context)", "GBps": round(gbps, 1), "us_per_get": round(us, 2),
+                           "frac_of_770": round(gbps / 770.0, 3)}
+        ring = [(c, (c + 1) % world) for c in range(world)]
+        gbps, us = run(ring)
+        out["d2d_ring"] = {"what": f"all {world} GPUs get_into their ring successor's objects at once",
+                           "aggregate_GBps": round(gbps, 1), "per_gpu_GBps": round(gbps / world, 1),
+                           "us_per_get": round(us, 2)}
+    except Exception as e:  # reported, never fatal for the line
+        out["d2d_error"] = f"{type(e).__name__}: {e}"[:300]
+    finally:
+        ctx.close()
     return out
 
 
