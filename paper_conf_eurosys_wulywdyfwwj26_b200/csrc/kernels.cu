@@ -115,8 +115,7 @@ __device__ void tile_ldst(const KP &p, uint8_t *dst, const uint8_t *src, uint64_
     const uint32_t r = (uint32_t)(s & 15);
     const uint32_t q = r >> 2, b = (r & 3) * 8;
     const uint4 *as = reinterpret_cast<const uint4 *>(s - r);
-    for (uint64_t i = tid; i < nvec; i += kThreads) {
-      uint4 lo = as[i], hi = as[i + 1];
+    auto shift = [&](const uint4 &lo, const uint4 &hi) {
       uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
       uint32_t o[4];
 #pragma unroll
@@ -130,8 +129,25 @@ __device__ void tile_ldst(const KP &p, uint8_t *dst, const uint8_t *src, uint64_
         }
         o[k] = b ? __funnelshift_r(a0, a1, b) : a0;
       }
-      int4 v = make_int4((int)o[0], (int)o[1], (int)o[2], (int)o[3]);
-      st_stream(vd + i, v);
+      return make_int4((int)o[0], (int)o[1], (int)o[2], (int)o[3]);
+    };
+    uint64_t i = tid;
+    // 4 output vectors (8 aligned loads) in flight per thread
+    for (; i + 3 * kThreads < nvec; i += 4 * kThreads) {
+      uint4 lo[4], hi[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        lo[u] = as[i + u * kThreads];
+        hi[u] = as[i + u * kThreads + 1];
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        st_stream(vd + i + u * kThreads, shift(lo[u], hi[u]));
+        count_bytes<COUNT>(p, (uint64_t)(vd + i + u * kThreads), 16);
+      }
+    }
+    for (; i < nvec; i += kThreads) {
+      st_stream(vd + i, shift(as[i], as[i + 1]));
       count_bytes<COUNT>(p, (uint64_t)(vd + i), 16);
     }
   }
@@ -510,7 +526,19 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
       const uint32_t nv = len >> 4;
       const int4 *sv = reinterpret_cast<const int4 *>(src);
       int4 *dv = reinterpret_cast<int4 *>(dst);
-      for (uint32_t i = lane; i < nv; i += 32) {
+      uint32_t i = lane;
+      // 16 B co-aligned (not 32 B): 8 x 16 B loads in flight per lane
+      for (; i + 7 * 32 < nv; i += 8 * 32) {
+        int4 w[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) w[j] = ld_stream(sv + i + j * 32);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          st_stream(dv + i + j * 32, w[j]);
+          count_bytes<COUNT>(p, (uint64_t)(dv + i + j * 32), 16);
+        }
+      }
+      for (; i < nv; i += 32) {
         st_stream(dv + i, ld_stream(sv + i));
         count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
       }
@@ -942,9 +970,11 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
       p.chunk[w++] = p.chunk[i];
   }
   p.n_chunks = w;
-  bool aligned = true;
-  for (uint32_t i = 0; i < p.n_chunks; ++i)
+  bool aligned = true, addr_aligned = true;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
     aligned &= ((p.chunk[i].src | p.chunk[i].dst | p.chunk[i].bytes) & 15) == 0;
+    addr_aligned &= ((p.chunk[i].src | p.chunk[i].dst) & 15) == 0;
+  }
   uint64_t total = 0;
   for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
   int v = variant_from_env();
@@ -954,6 +984,11 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   // (38.5 MB get_into back to back: 13.2 us with ws1, 11.8 us with wv8 +
   // prefetch); GROUTER_COPY_TMA forces the bulk ring for every aligned round
   if (v < 0) v = (tma || (aligned && total >= (256ull << 20))) ? 3 : 14;
+  // a user buffer at an odd address (a tensor view, a by-copy put of a host
+  // structure): the warp-strided engines would fall back to byte copies;
+  // the tiled LD/ST engine keeps 16 B accesses with its co-aligned and
+  // funnel-shift paths
+  if (!addr_aligned && variant_from_env() < 0) v = 0;
   if (((v >= 2 && v <= 4) || (v >= 10 && v <= 12)) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
   // static-assignment engines (ws, gs) need no scratch: their completion can
   // be published by a stream write after the launch, which costs the GPU
