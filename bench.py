@@ -372,6 +372,21 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
         out["d2d_push"] = {"what": "GPU1 gFn get_into of GPU0-resident 38.5 MB objects (GPU0 SM push over "
                                    "NVLink, one context)", "GBps": round(gbps, 1), "us_per_get": round(us, 2),
                            "frac_of_770": round(gbps / 770.0, 3)}
+        # baseline on the same devices and sizes: cudaMemcpyPeerAsync (copy engine)
+        a0 = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[0]}")
+        b1 = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[1]}") for _ in range(2)]
+        sp = torch.cuda.Stream(device=f"cuda:{devs[1]}")
+        with torch.cuda.stream(sp):
+            for i in range(3):
+                b1[i % 2].copy_(a0, non_blocking=True)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(sp)
+            for i in range(reps * objs):
+                b1[i % 2].copy_(a0, non_blocking=True)
+            e1.record(sp)
+        e1.synchronize()
+        us_b = e0.elapsed_time(e1) * 1e3 / (reps * objs)
+        out["d2d_memcpy_peer_baseline"] = {"GBps": round(n / us_b / 1e3, 1), "us_per_copy": round(us_b, 2)}
         ring = [(c, (c + 1) % world) for c in range(world)]
         gbps, us = run(ring)
         out["d2d_ring"] = {"what": f"all {world} GPUs get_into their ring successor's objects at once",
@@ -382,6 +397,38 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
     finally:
         ctx.close()
     return out
+
+
+def nccl_ring_baseline(world, rank, dev, n, per_step, steps):
+    """The library-free baseline for the same exchange: every rank receives
+    n-byte tensors from rank+1 (and sends to rank-1) with NCCL send/recv,
+    per_step per step; device-timed on the NCCL stream's caller stream, max
+    over ranks.  GB/s per GPU received."""
+    import torch
+    import torch.distributed as dist
+    src = torch.empty(n, dtype=torch.uint8, device=f"cuda:{dev}")
+    dst = torch.empty(n, dtype=torch.uint8, device=f"cuda:{dev}")
+    to, frm = (rank - 1) % world, (rank + 1) % world
+
+    def step():
+        for _ in range(per_step):
+            ops = [dist.P2POp(dist.isend, src, to), dist.P2POp(dist.irecv, dst, frm)]
+            for w in dist.batch_isend_irecv(ops):
+                w.wait()
+    for _ in range(3):
+        step()
+    torch.cuda.synchronize(dev)
+    dist.barrier()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(steps):
+        step()
+    b.record()
+    b.synchronize()
+    ms = max_over_ranks(a.elapsed_time(b), world, f"cuda:{dev}")
+    return {"what": "NCCL send/recv ring (torch.distributed batch_isend_irecv), same bytes and pairing",
+            "gbps_per_gpu": round(steps * per_step * n / (ms / 1e3) / 1e9, 1),
+            "us_per_transfer": round(ms * 1e3 / (steps * per_step), 2)}
 
 
 # ------------------------------------------------------------------ GPU arm
@@ -543,6 +590,9 @@ def run_gpu(args, rank, world, local_rank):
                                "launches": p["launches"], "avg_launch_us": p_ns / 1e3,
                                "alg_bytes_per_launch": p_bytes},
                   "host_us_per_request": p["host_us"]}
+        if dist.get_backend() == "nccl":
+            nvlink["nccl_p2p_baseline"] = nccl_ring_baseline(world, rank, dev, n, R, args.steps // 10 or 1)
+
 
     # per-request latency (separate, untimed pass): device events around one get_into
     lat = []
