@@ -678,11 +678,13 @@ def run_gpu(args, rank, world, local_rank):
         cpu = {"value": v, "unit": "req/s", "cores": 1, "kind": "oracle",
                "sample": f"{done} oracle get_into of {N_BYTES} B in {dt:.1f} s (numpy memcpy)"}
 
-    traffic = None
+    traffic = traffic_steady = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
         try:
-            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+            tj = json.load(open(tp))
+            traffic = tj.get("dram_bytes_per_launch")
+            traffic_steady = tj.get("steady_dram_bytes_per_launch")
         except Exception:
             traffic = None
 
@@ -705,6 +707,11 @@ def run_gpu(args, rank, world, local_rank):
                            "what": "one get_into of 38,535,168 B, CUDA events on the consumer stream"},
             "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+                         "traffic_note": "ncu --set full (caches flushed per replay: the 38.5 MB of writes stay "
+                                         "in L2, so this is the read half); without flushing, 20 consecutive "
+                                         "launches average traffic_steady = read + write-back ~= 0.98 x the "
+                                         "algorithmic bytes (profiles/r01_ncu_steady_traffic.json)",
+                         "traffic_steady": traffic_steady,
                          "kernel": "gr_copy (K2')", "peak_source": peak_src,
                          "launches": launches, "avg_launch_us": avg_ns / 1e3,
                          "timing": "CUDA events over the timed region on the stream the kernels "
