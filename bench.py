@@ -371,7 +371,7 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
         gbps, us = run([(1, 0)])
         out["d2d_push"] = {"what": "GPU1 gFn get_into of GPU0-resident 38.5 MB objects (GPU0 SM push over "
                                    "NVLink, one context)", "GBps": round(gbps, 1), "us_per_get": round(us, 2),
-                           "frac_of_770": round(gbps / 770.0, 3)}
+                           "frac_of_770": round(gbps / 770.0, 3), "frac_of_900_nominal": round(gbps / 900.0, 3)}
         # baseline on the same devices and sizes: cudaMemcpyPeerAsync (copy engine)
         a0 = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[0]}")
         b1 = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[1]}") for _ in range(2)]
@@ -586,6 +586,7 @@ def run_gpu(args, rank, world, local_rank):
                   "gbps_per_gpu": R * args.steps * n / (p["ms_max"] / 1e3) / 1e9,
                   "roofline": {"bound": "nvlink", "achieved": p_ach, "peak": 770.0, "unit": "GB/s",
                                "frac": (p_ach / 770.0) if p_ach else None,
+                               "frac_of_900_nominal": (p_ach / 900.0) if p_ach else None,
                                "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s/direction",
                                "launches": p["launches"], "avg_launch_us": p_ns / 1e3,
                                "alg_bytes_per_launch": p_bytes},
@@ -663,14 +664,26 @@ def run_gpu(args, rank, world, local_rank):
     # N > 1: host->GPU striping over the other GPUs' PCIe links (L120, L178), measured by
     # rank 0 alone on a context spanning every GPU of the node while the others wait
     multipath = None
+    stuck = False
     if world > 1 and not args.no_multipath_probe:
         barrier()
         if rank == 0:
-            try:
-                multipath = measure_multipath(world, G)
-            except Exception as e:  # report, never abort the scaling line
-                multipath = {"error": f"{type(e).__name__}: {e}"[:300]}
-        barrier()
+            # watchdog: this node-wide measurement never ran on a multi-GPU box
+            # in-round; a hang must not cost the scaling line
+            import threading
+            box = {}
+
+            def _mp():
+                try:
+                    box["r"] = measure_multipath(world, G)
+                except Exception as e:  # report, never abort the scaling line
+                    box["r"] = {"error": f"{type(e).__name__}: {e}"[:300]}
+            th = threading.Thread(target=_mp, daemon=True)
+            th.start()
+            th.join(args.multipath_timeout)
+            stuck = th.is_alive()
+            multipath = box.get("r") or {"error": f"timed out after {args.multipath_timeout:.0f} s"}
+        barrier() if not stuck else dist.barrier()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -732,6 +745,9 @@ def run_gpu(args, rank, world, local_rank):
             line["ipc_pull_error"] = ipc_error or "another rank failed to import"
 
         print(json.dumps(line), flush=True)
+    if stuck:   # a measurement thread still owns the GPUs: leave without teardown
+        sys.stdout.flush()
+        os._exit(0)
     ctx.close()
 
 
@@ -751,6 +767,8 @@ def main():
     ap.add_argument("--tma", action="store_true")
     ap.add_argument("--ctas", type=int, default=4)
     ap.add_argument("--no-multipath-probe", action="store_true")
+    ap.add_argument("--multipath-timeout", type=float, default=300.0,
+                    help="N>1: seconds rank 0 waits for the node-wide multipath/D2D measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
