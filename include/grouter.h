@@ -65,6 +65,10 @@ extern "C" {
 #define GROUTER_RESTORE       0x40u/* proactive restore (L260-L262): when pool storage is released
                                       or a cap is raised, objects migrated away from that GPU come
                                       back while they fit (R42)                      */
+#define GROUTER_STRIPED_MIGRATION 0x100u /* spills leave over R(src) on the route GPUs' D2H
+                                      engines (the gFn-host plan, L178), restores come back over
+                                      R(d) with relays like a fetch (L178, L366 "parallel PCIe
+                                      transfers ... mitigate the overhead"); R47      */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;

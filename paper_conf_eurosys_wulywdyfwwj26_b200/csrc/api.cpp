@@ -452,8 +452,10 @@ grouter_status grouter_finalize(grouter_ctx *c) {
               h.t[10] / h.put_calls / 1e3, h.t[11] / h.put_calls / 1e3, h.t[12] / h.put_calls / 1e3,
               h.t[13] / h.put_calls / 1e3);
     if (h.put_calls)
-      fprintf(stderr, "[grouter host profile] put call -> first H2D copy submitted %.2f us, host wait %.2f us\n",
-              h.t[14] / h.put_calls / 1e3, h.t[15] / h.put_calls / 1e3);
+      fprintf(stderr, "[grouter host profile] put call -> first H2D copy submitted %.2f us (to round %.2f, "
+                      "take+guard %.2f, memcpy call %.2f), host wait %.2f us\n",
+              h.t[14] / h.put_calls / 1e3, h.t[16] / h.put_calls / 1e3, h.t[17] / h.put_calls / 1e3,
+              h.t[18] / h.put_calls / 1e3, h.t[15] / h.put_calls / 1e3);
     if (h.t[4] > 0)
       fprintf(stderr, "[grouter host profile] inside transfer: plan+xfer+enqueue %.2f us, take %.2f us, "
                       "params %.2f us, launch %.2f us\n",
@@ -603,6 +605,10 @@ static grouter_status get_common(grouter_ctx *c, const grouter_fn *fn, grouter_o
   if (it == c->objects.end() || dead(it->second)) return fail(GROUTER_ENOENT, "get: unknown oid");
   if (it->second.wf != fn->workflow_id) return fail(GROUTER_EPERM, "get: workflow mismatch (L394)");
   if (it->second.state == OBJ_OPEN) return fail(GROUTER_ENOENT, "get: object not sealed");
+  // completed producer fences are dropped once: an event fence is re-queried
+  // (~1 us of host time) by every later get otherwise (copies of a fence do
+  // not share its completion memo)
+  if (!it->second.ready.empty()) prune(it->second.ready);
   *out = &it->second;
   return GROUTER_OK;
 }

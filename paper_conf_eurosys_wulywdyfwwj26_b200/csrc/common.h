@@ -160,7 +160,7 @@ inline void prune(Fences &f) {
 struct HostProf {
   bool on = false;
   uint64_t calls = 0, put_calls = 0;
-  double t[16] = {};  // [0..7] get_into stages, [8..15] blocking put stages
+  double t[24] = {};  // [0..7] get_into stages, [8..15] blocking put stages, [16..18] put -> H2D copy
 };
 HostProf &hprof();
 uint64_t now_ns();

@@ -117,7 +117,11 @@ void host_wait(const Fences &f, double timeout_s) {
   auto t0 = std::chrono::steady_clock::now();
   for (auto &w : f) {
     if (w.ev && !w.word) {
-      GR_CUDA(cudaEventSynchronize(w.ev->ev));
+      // event fence (a direct launch or a whole CE round): spin on the query
+      // for a short transfer's worth of time, then block in the driver
+      bool ok = false;
+      for (int k = 0; k < 24 && !ok; ++k) ok = w.done();
+      if (!ok) GR_CUDA(cudaEventSynchronize(w.ev->ev));
       continue;
     }
     uint32_t spins = 0;
@@ -142,6 +146,7 @@ void done_fences(const XferRef &x, Fences &f) {
     f.push_back(w);
     return;
   }
+  x->word_fenced = true;
   for (uint32_t p = 0; p < x->npath; ++p) {
     if (!x->total[p]) continue;
     Waitable w;
@@ -493,7 +498,48 @@ static uint64_t bounce(grouter_ctx *c, uint64_t src, uint64_t bytes, uint32_t *s
   return (uint64_t)slot;
 }
 
-static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg) {
+// Transfers a CE round moves WHOLE (every chunk in this round, none relayed,
+// no word fences handed out yet, no deferred stream waits) complete by the
+// round's closing event instead of stream-written words: a
+// cuStreamWriteValue32 costs ~0.8 us of host time and ~1-2 us of latency
+// per round (tools/celat.cu), the dominant cost of small blocking cFn puts
+// and gets.  Real-time mode only (replay hands out word fences first).
+static std::vector<Xfer *> whole_in_round(grouter_ctx *c, const Server &s, const std::vector<ChunkItem> &items) {
+  std::vector<Xfer *> out;
+  static const bool ev_done = !getenv("GR_NO_EVDONE");
+  if (!ev_done || c->replay) return out;
+  std::unordered_map<Xfer *, uint32_t> n;
+  for (auto &it : items) {
+    Xfer *x = it.x;
+    if (x->word_fenced || x->submitted_chunks || !x->waiters.empty()) continue;
+    if (s.kind == SK_H2D && it.dst_logical != s.logical) {
+      n[x] = UINT32_MAX;  // a relayed chunk: the forward kernel publishes
+      continue;
+    }
+    uint32_t &k = n[x];
+    if (k != UINT32_MAX) ++k;
+  }
+  for (auto &kv : n)
+    if (kv.second == kv.first->nchunks) out.push_back(kv.first);
+  return out;
+}
+
+static void complete_by_event(grouter_ctx *c, const std::vector<Xfer *> &xs, const EventRef &e, cudaStream_t st) {
+  for (Xfer *x : xs) {
+    x->done_ev = e;
+    x->done_stream = st;
+    for (uint32_t p = 0; p < x->npath; ++p) c->slot_final[x->slot][p] -= x->total[p];  // slot back
+  }
+}
+
+static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
+                       const std::vector<Xfer *> &evented) {
+  if (!evented.empty())
+    seg.erase(std::remove_if(seg.begin(), seg.end(),
+                             [&](const ChunkItem &it) {
+                               return std::find(evented.begin(), evented.end(), it.x) != evented.end();
+                             }),
+              seg.end());
   for (auto &p : issue(seg))
     GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
                                    p.x->value_after(p.path), 0));
@@ -505,11 +551,13 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg) {
 // and a forward round kernel on r pushes them to their destination.
 static size_t round_h2d(grouter_ctx *c, Server &s) {
   const uint64_t budget = 2ull * s.sched.batch * c->cfg.chunk_bytes;
+  const uint64_t tr0 = tl_put_t0 ? now_ns() : 0;
   refill(c, s, 2, budget);
   std::vector<ChunkItem> items, direct, relay;
   std::vector<char> cut;
   take(s, budget, items, cut);
   if (items.empty()) return 0;
+  const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
   std::vector<uint64_t> slot_src;
   std::vector<uint32_t> slots_used;
@@ -519,10 +567,15 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   uint64_t run_src = 0, run_dst = 0, run_len = 0;
   auto flush_run = [&]() {
     if (run_len) {
+      const uint64_t tm = tl_put_t0 ? now_ns() : 0;
       GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyHostToDevice,
                               s.stream));
       if (tl_put_t0) {  // profiling: put call -> its first H2D copy submitted
-        hprof().t[14] += now_ns() - tl_put_t0;
+        const uint64_t te = now_ns();
+        hprof().t[14] += te - tl_put_t0;
+        hprof().t[16] += tr0 - tl_put_t0;  // put call -> round (after refill)
+        hprof().t[17] += tm - tr0;         // take + DeviceGuard -> memcpy call
+        hprof().t[18] += te - tm;          // the memcpy call
         tl_put_t0 = 0;
       }
     }
@@ -530,7 +583,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   };
   auto end_segment = [&]() {
     flush_run();
-    publish_ce(c, s, direct);
+    publish_ce(c, s, direct, evented);
     if (!relay.empty()) {
       EventRef ce = record(c, s.stream, s.phys);
       GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
@@ -578,6 +631,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   }
   end_segment();
   EventRef ce_end = record(c, s.stream, s.phys);
+  complete_by_event(c, evented, ce_end, s.stream);
   if (last_fwd) {  // one in-flight marker covering both the CE and the forward stream
     GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce_end->ev, 0));
     s.inflight.push_back({ev_wait(c, record(c, s.fwd_stream, s.phys)), nullptr});
@@ -598,6 +652,7 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
   std::vector<char> cut;
   take(s, UINT64_MAX, items, cut);
   if (items.empty()) return 0;
+  const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
   uint64_t run_src = 0, run_dst = 0, run_len = 0;
   auto flush_run = [&]() {
@@ -610,7 +665,7 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
     const ChunkItem &it = items[i];
     if (cut[i]) {
       flush_run();
-      publish_ce(c, s, seg);
+      publish_ce(c, s, seg, evented);
       stream_wait(c, s.stream, s.phys, it.x->deps);
     }
     if (run_len && run_src + run_len == it.src && run_dst + run_len == it.dst) {
@@ -625,8 +680,10 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
     c->stats.link_bytes[2][s.logical] += it.bytes;
   }
   flush_run();
-  publish_ce(c, s, seg);
-  s.inflight.push_back({ev_wait(c, record(c, s.stream, s.phys)), nullptr});
+  publish_ce(c, s, seg, evented);
+  EventRef ce_end = record(c, s.stream, s.phys);
+  complete_by_event(c, evented, ce_end, s.stream);
+  s.inflight.push_back({ev_wait(c, ce_end), nullptr});
   c->stats.rounds++;
   after_submit(c, items);
   return items.size();
@@ -641,10 +698,13 @@ static bool has_work(const Server &s) {
 }
 
 static size_t pump_server(grouter_ctx *c, Server &s, bool force) {
-  if (!s.stream) return 0;
-  retire(s);
+  if (!s.stream || !has_work(s)) return 0;
+  // retire only when the in-flight limit would hold the round back: every
+  // completed-round check is an event query (~1 us of host time), and pump
+  // runs on every call for every server of the node
+  if (!force && s.inflight.size() >= 2) retire(s);
   size_t total = 0;
-  while (has_work(s) && (force || s.inflight.size() < 2)) {
+  while (has_work(s) && (force || s.inflight.size() < 2 || (retire(s), s.inflight.size() < 2))) {
     size_t n = s.kind == SK_COPY ? round_copy(c, s) : s.kind == SK_H2D ? round_h2d(c, s) : round_d2h(c, s);
     if (!n) break;  // blocked on another server's submission
     total += n;
@@ -738,15 +798,18 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
 
 // D2H of an eviction victim (L258-L262; the per-GPU I/O path of L269): an
 // urgent, unscheduled transfer on the victim GPU's D2H engine.
+// GROUTER_STRIPED_MIGRATION (R47): the victim leaves over R(src), each route
+// GPU's copy engine reading its share straight from the source pool pages
+// (mapped for every GPU) -- the gFn-host plan of L178 / R45.
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
   std::vector<grouter_chunk> plan;
-  c->planner.plan_single(o.n, o.loc, plan);
+  if (c->cfg.flags & GROUTER_STRIPED_MIGRATION) c->planner.plan_h2d(o.loc, o.n, plan);
+  else c->planner.plan_single(o.n, o.loc, plan);
   XferRef x = new_xfer_slot(c, plan);
   x->deps = o.ready;
-  Server &s = c->dev[o.loc].d2h;
   for (uint32_t i = 0; i < plan.size(); ++i)
-    s.urgent.push_back(make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)host_dst,
-                                 GROUTER_HOST));
+    c->dev[plan[i].route_gpu].d2h.urgent.push_back(
+        make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)host_dst, GROUTER_HOST));
   Fences done;
   done_fences(x, done);
   Fences old = std::move(o.readers);
@@ -761,16 +824,17 @@ void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
 }
 
 // H2D of a proactively restored object (L260-L262) back to its home GPU d: an
-// urgent, unscheduled single-path transfer on d's own H2D engine (no relay:
-// restores are background work, they should not load other GPUs' links).
+// urgent, unscheduled transfer, single-path on d's own H2D engine (R42), or
+// striped over R(d) with relays under GROUTER_STRIPED_MIGRATION (R47).
 void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst) {
   std::vector<grouter_chunk> plan;
-  c->planner.plan_single(o.n, d, plan);
+  if (c->cfg.flags & GROUTER_STRIPED_MIGRATION) c->planner.plan_h2d(d, o.n, plan);
+  else c->planner.plan_single(o.n, d, plan);
   XferRef x = new_xfer_slot(c, plan);
   x->deps = o.ready;
-  Server &s = c->dev[d].h2d;
   for (uint32_t i = 0; i < plan.size(); ++i)
-    s.urgent.push_back(make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)dev_dst, d));
+    c->dev[plan[i].route_gpu].h2d.urgent.push_back(
+        make_item(x, i, plan[i], (uint64_t)(uintptr_t)o.ptr, (uint64_t)(uintptr_t)dev_dst, d));
   Fences done;
   done_fences(x, done);
   Fences old = std::move(o.readers);
@@ -944,7 +1008,12 @@ void engine_init(grouter_ctx *c) {
       s.sched.batch = c->cfg.batch_chunks;
       int lo = 0, hi = 0;
       cudaDeviceGetStreamPriorityRange(&lo, &hi);
-      GR_CUDA(cudaStreamCreateWithPriority(&s.stream, cudaStreamNonBlocking, hi));
+      // SM-copy rounds run at the highest priority (they share SMs with the
+      // functions' kernels); copy-engine streams at the default one: a memcpy
+      // on a high-priority stream costs ~2.2 us more host time and ~2 us more
+      // latency per call (tools/celat.cu), and priority buys a CE nothing
+      static const bool ce_hi = getenv("GR_CE_PRIO_HI") != nullptr;
+      GR_CUDA(cudaStreamCreateWithPriority(&s.stream, cudaStreamNonBlocking, (k == SK_COPY || ce_hi) ? hi : lo));
     }
     GR_CUDA(cudaMalloc(&d.copy.scratch, 64));
     GR_CUDA(cudaMemset(d.copy.scratch, 0, 64));

@@ -122,15 +122,17 @@ def _copy_exactly_once(tma, src_off, dst_off):
 
 
 # ------------------------------------------------------------------ trace parity
-def _both(ops, calib, replay=True, keep=True, restore=False, d2h=False, **kw):
+def _both(ops, calib, replay=True, keep=True, restore=False, d2h=False, striped=False, **kw):
     orc = orun.run(ops, calib, host_store_bytes=kw.get("host_store_bytes", 1 << 30),
                    pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore,
                    pool_floor=kw.get("pool_floor", 64 << 20), targets=kw.get("targets", False),
-                   d2h_multipath=d2h)
+                   d2h_multipath=d2h, striped_migration=striped)
     if restore:
         kw["flags"] = kw.get("flags", 0) | G.RESTORE
     if d2h:
         kw["flags"] = kw.get("flags", 0) | G.D2H_MULTIPATH
+    if striped:
+        kw["flags"] = kw.get("flags", 0) | G.STRIPED_MIGRATION
     r = LibRunner(calib, replay=replay, keep_bytes=keep, **kw)
     try:
         lib_out = r(ops)
@@ -345,3 +347,52 @@ def test_full_size_cfg2_cfg5():
         assert compare(orc, lib_out, check_dispatch=False) > 0
         if kw:
             assert spilled > 0, "the 10% limit should force spills"
+
+
+def _link_bytes_equal(orc, lib_out, n):
+    """Per-engine byte totals: the library's link_bytes[1] (H2D) and [2]
+    (D2H) per logical GPU equal the oracle's scheduled + migration plans."""
+    lb = orc["oracle"].link_bytes
+    st = lib_out["stats"]
+    for kind, row in (("h2d", 1), ("d2h", 2)):
+        got = [st.link_bytes[row][g] for g in range(n)]
+        exp = [lb.get((kind, g), 0) for g in range(n)]
+        assert got == exp, (kind, got, exp)
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_striped_migration(seed, replay):
+    """GROUTER_STRIPED_MIGRATION (R47) with proactive restore on virtual
+    topologies: statuses, victims, restores, placements and bytes equal the
+    oracle's, and every copy engine moved exactly the oracle's bytes."""
+    rng = random.Random(7000 + seed)
+    k = rng.choice([2, 3, 4])
+    calib = C.virtual(k)
+    ops = T.random_trace(rng, k, n_ops=120, max_n=9 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, restore=True, striped=True,
+                         host_store_bytes=64 * MiB, pool_cap=caps)
+    compare(orc, lib_out, check_dispatch=replay)
+    _link_bytes_equal(orc, lib_out, k)
+    assert lib_out["stats"].spill_count > 0 or seed % 2
+
+
+def test_fig5a_striped_spill_and_restore():
+    """The L178 worked example on 8 logical GPUs of one B200: GPU1's object
+    spills over GPU1/3/5/7's D2H engines and comes back over their H2D
+    engines with relays; bytes identical, engine totals equal the oracle's."""
+    calib = C.fig5a()
+    calib["device_map"] = [0] * 8
+    b = T.Builder(11)
+    f = T.fn(1, 1, 0)
+    o = b.put(f, 64 * MiB)
+    b.pool_limit(0, 0)
+    b.pool_limit(0, 1 << 40)
+    g = b.get_into(T.fn(1, 2, 0), o)
+    orc, lib_out = _both(b.ops, calib, replay=False, restore=True, striped=True, pool_floor=8 << 20)
+    assert compare(orc, lib_out, check_dispatch=False) == 1
+    _link_bytes_equal(orc, lib_out, 8)
+    st = lib_out["stats"]
+    assert [st.link_bytes[2][g] > 0 for g in range(8)] == [True, False, True, False, True, False, True, False]
+    del g
