@@ -84,6 +84,48 @@ def oracle_get_into(n, budget_s=0.4):
     return summarize(n, lat)
 
 
+def oracle_put_h2d(n, striped, budget_s=0.4):
+    """The oracle's cFn put with a GPU0 hint on the 8-GPU HGX calibration
+    (R(0) = 4 uplink groups): single-threaded (`Oracle.put` as it stands:
+    plan + one np.copyto), or the same O6 plan executed with one thread per
+    route path (SURVEY §8(d) striped variant, T = |R(0)| capped at the cores)."""
+    import os
+    from concurrent.futures import ThreadPoolExecutor
+
+    import numpy as np
+    from oracle.model import Oracle
+    from oracle.splitter import CHUNK, plan_h2d
+    from synth.calib import b200_hgx as hgx
+    calib = hgx(8)
+    src = np.zeros(n, np.uint8)
+    lat = []
+    t_end = time.perf_counter() + budget_s
+    if not striped:
+        orc = Oracle(calib)
+        f = {"wf": 1, "fid": 1, "dev": -1}
+        while len(lat) < 3 or (time.perf_counter() < t_end and len(lat) < 200):
+            t = time.perf_counter()
+            st, out = orc.put(f, src, n, 0, 0)
+            lat.append((time.perf_counter() - t) * 1e6)
+            orc.free(f, out["oid"])
+        return dict(summarize(n, lat), threads=1)
+    dst = np.empty(n, np.uint8)
+    by = {}
+    for c in plan_h2d(calib, 0, n, True, CHUNK):
+        by.setdefault(c["route_gpu"], []).append((c["offset"], c["offset"] + c["bytes"]))
+    T = max(1, min(len(by), len(os.sched_getaffinity(0))))
+
+    def work(spans):
+        for a, b in spans:
+            np.copyto(dst[a:b], src[a:b])
+    with ThreadPoolExecutor(T) as ex:
+        while len(lat) < 3 or (time.perf_counter() < t_end and len(lat) < 200):
+            t = time.perf_counter()
+            list(ex.map(work, by.values()))
+            lat.append((time.perf_counter() - t) * 1e6)
+    return dict(summarize(n, lat), threads=T)
+
+
 def main():
     _build.build()
     G.load()
@@ -142,6 +184,8 @@ def main():
             pats["base_h2d_pinned"].append(summarize(n, dev_timed(s, lambda: dst.copy_(hb, non_blocking=True), reps)))
             pats["base_d2h_pinned"].append(summarize(n, dev_timed(s, lambda: hb.copy_(dst, non_blocking=True), reps)))
         pats.setdefault("oracle_get_into", []).append(oracle_get_into(n))
+        pats.setdefault("oracle_put_h2d", []).append(oracle_put_h2d(n, False))
+        pats.setdefault("oracle_put_striped", []).append(oracle_put_h2d(n, True))
         print(n, {k: v[-1]["p50_us"] for k, v in pats.items()}, flush=True)
     res["patterns"] = pats
     ctx.close()

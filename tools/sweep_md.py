@@ -28,10 +28,13 @@ print("`python tools/sweep.py` (device-event timing for get_into / baselines on 
       "GPU, so every number includes the library's host path. GB/s = payload bytes / p50. Probe of this GPU: "
       f"{json.dumps(d['probe'])}\n")
 print("| bytes | get_into same-GPU p50/p99 µs (GB/s) | cudaMemcpy D2D p50 µs | zero-copy get µs | put H2D (hint GPU0) "
-      "p50 µs (GB/s) | pinned H2D p50 µs | get D2H p50 µs (GB/s) | pinned D2H p50 µs | oracle get_into µs |")
-print("|---|---|---|---|---|---|---|---|---|")
+      "p50 µs (GB/s) | pinned H2D p50 µs | get D2H p50 µs (GB/s) | pinned D2H p50 µs | oracle get_into µs | "
+      "oracle put H2D µs (1 thread / striped, threads) |")
+print("|---|---|---|---|---|---|---|---|---|---|")
 for r in P["get_into_same"]:
     n = r["n"]
     print(f"| {n:,} | {cell('get_into_same', n, True, True)} | {cell('base_memcpy_d2d', n, False)} | "
           f"{cell('zero_copy_get', n, False)} | {cell('put_h2d', n)} | {cell('base_h2d_pinned', n, False)} | "
-          f"{cell('get_d2h', n)} | {cell('base_d2h_pinned', n, False)} | {cell('oracle_get_into', n, False)} |")
+          f"{cell('get_d2h', n)} | {cell('base_d2h_pinned', n, False)} | {cell('oracle_get_into', n, False)} | "
+          f"{cell('oracle_put_h2d', n, False)} / {cell('oracle_put_striped', n, False)}"
+          f"{', T=' + str(row('oracle_put_striped', n)['threads']) if row('oracle_put_striped', n) else ''} |")
