@@ -396,3 +396,55 @@ def test_fig5a_striped_spill_and_restore():
     st = lib_out["stats"]
     assert [st.link_bytes[2][g] > 0 for g in range(8)] == [True, False, True, False, True, False, True, False]
     del g
+
+
+@pytest.mark.parametrize("n", [1 << 30, (1 << 30) - 4097])
+def test_full_size_cfg3_max(n):
+    """cfg3's largest size (1 GiB, and a ragged 1 GiB - 4097 B) through every
+    pattern on two logical GPUs: a cFn put striped over R(0) = {0, 1} (the
+    relay hop through logical GPU1's staging ring), a D2D get_into on GPU1, a
+    same-GPU get_into on GPU0 (the TMA engine above 256 MiB) and a cFn get
+    back to host memory.  Device results are verified in full against the
+    O11 generator; the host copy is compared in full with the source
+    (get(put(x)) == x) and at sampled offsets with synth.payload."""
+    from synth import payload as P
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=3 << 30, pool_cap=[G.UNLIMITED] * 2,
+                                    pool_floor_bytes=64 << 20))
+    seed = 424242
+    try:
+        st, plan = ctx.plan(G.HOST, 0, n)
+        assert st == G.OK and {c[3] for c in plan} == {0, 1}
+        tmp = torch.empty(n, dtype=torch.uint8, device="cuda:0")
+        G.check(G.test_fill(tmp.data_ptr(), n, seed, 0, 0))
+        host = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        host.copy_(tmp)
+        del tmp
+        cfn = G.fn(5, 1, G.HOST)
+        st, oid = ctx.put(cfn, host.data_ptr(), n, 0, 0)
+        G.check(st, "put")
+        assert ctx.where(oid) == (G.OK, 0)
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda:0")
+        s = torch.cuda.Stream()
+        for g in (1, 0):                                  # D2D push to GPU1, then same-GPU copy
+            dst.zero_()
+            torch.cuda.synchronize()
+            st, nn = ctx.get_into(G.fn(5, 2 + g, g), oid, dst.data_ptr(), n, s.cuda_stream)
+            G.check(st, "get_into")
+            s.synchronize()
+            st, bad, first = G.test_verify(dst.data_ptr(), n, seed, 0, 0)
+            assert st == 0 and bad == 0, (g, bad, first)
+        del dst
+        st, ptr, nn = ctx.get(cfn, oid, 0)
+        G.check(st, "get")
+        import ctypes
+        back = np.ctypeslib.as_array((ctypes.c_uint8 * nn).from_address(ptr))
+        assert np.array_equal(back, host.numpy())
+        rng = np.random.default_rng(n)
+        for off in list(rng.integers(0, n - 64, size=16)) + [0, n - 64, (1 << 21) - 7]:
+            off = int(off)
+            assert np.array_equal(back[off:off + 64], P.payload(seed, 64, off)), off
+        ctx.release(cfn, oid, ptr, 0)
+        ctx.free(cfn, oid)
+    finally:
+        ctx.close()
