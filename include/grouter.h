@@ -305,6 +305,13 @@ grouter_status grouter_pool_target(grouter_ctx *ctx, int32_t dev, uint64_t *targ
 /* Current location of an object: GPU index or GROUTER_HOST. */
 grouter_status grouter_where(grouter_ctx *ctx, grouter_oid oid, int32_t *loc);
 grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
+/* Per-tenant share accounting (L193: "data chunks of each function are
+ * scheduled proportionally to their allocated bandwidth"; L227-L229):
+ * bytes[k] = bytes of workflow_id's chunks the servers of kind k dispatched
+ * so far (0 = SM-copy egress, 1 = H2D engines, 2 = D2H engines), summed over
+ * GPUs.  Scheduled transfers only: spills and restores are unscheduled
+ * (R41, R42).  An unknown tenant reads zeros.  EINVAL on null arguments. */
+grouter_status grouter_tenant_stats(grouter_ctx *ctx, uint32_t workflow_id, uint64_t bytes[3]);
 /* Takes (and clears) the objects spilled since the last call, in order. */
 grouter_status grouter_victims(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
 /* Takes (and clears) the objects proactively restored to a GPU pool since the

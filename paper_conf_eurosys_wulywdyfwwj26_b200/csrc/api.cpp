@@ -1055,6 +1055,14 @@ grouter_status grouter_where(grouter_ctx *c, grouter_oid oid, int32_t *loc) {
   return GROUTER_OK;
 }
 
+grouter_status grouter_tenant_stats(grouter_ctx *c, uint32_t workflow_id, uint64_t bytes[3]) {
+  if (!c || !bytes) return fail(GROUTER_EINVAL, "null argument");
+  Guard g(c);
+  auto it = c->tenant_bytes.find(workflow_id);
+  for (int k = 0; k < 3; ++k) bytes[k] = it == c->tenant_bytes.end() ? 0 : it->second[k];
+  return GROUTER_OK;
+}
+
 grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
   if (!c || !out) return fail(GROUTER_EINVAL, "null argument");
   Guard g(c);

@@ -248,6 +248,7 @@ struct grouter_ctx {
   std::unordered_map<grouter_oid, gr::Obj> objects;
   std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
   std::unordered_map<uint32_t, uint32_t> weights;
+  std::unordered_map<uint32_t, std::array<uint64_t, 3>> tenant_bytes;  // dispatched, per server kind
   std::map<uint32_t, std::array<uint64_t, 3>> slos;    // wf -> (data, slo_ns, infer_ns), R43
   // pool sizing (R44): per (wf, fid, gpu) histograms and resident counts
   std::map<std::tuple<uint32_t, uint32_t, int>, gr::FuncHist> hists;

@@ -268,6 +268,7 @@ static void refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max
     uint32_t t = s.sched.dispatch([&](uint32_t tn) { return weight_of(c, tn); }, b, &bb);
     if (t == UINT32_MAX) break;
     log_batch(c, s, t, b, bb);
+    c->tenant_bytes[t][s.kind] += bb;
     for (auto &it : b) s.carry.push_back(it);
     bytes += bb;
     ++nb;

@@ -132,6 +132,7 @@ SIGNATURES = {
     "grouter_route_set": (_ST, [_CTX, _I32, C.POINTER(_I32), _U32, C.POINTER(_U32)]),
     "grouter_where": (_ST, [_CTX, _U64, C.POINTER(_I32)]),
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
+    "grouter_tenant_stats": (_ST, [_CTX, C.c_uint32, C.POINTER(_U64)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_paths_new": (C.c_void_p, [C.c_uint32, C.c_uint32, C.POINTER(_U64), C.c_uint32]),
@@ -390,6 +391,12 @@ class Ctx:
         loc = C.c_int32(0)
         st = self.lib.grouter_where(self.h, oid, C.byref(loc))
         return st, loc.value
+
+    def tenant_stats(self, workflow_id: int):
+        """Bytes of this tenant's chunks dispatched per server kind [SM copy, H2D, D2H]."""
+        arr = (_U64 * 3)()
+        check(self.lib.grouter_tenant_stats(self.h, workflow_id, arr), "tenant_stats")
+        return list(arr)
 
     def stats(self) -> grouter_stats_t:
         s = grouter_stats_t()

@@ -246,7 +246,14 @@ class LibRunner:
                 rec["where"] = loc if stw == G.OK else None
             recs.append(rec)
         self._flush_and_verify()
-        return {"records": recs, "dispatch": ctx.dispatch_log(), "stats": ctx.stats()}
+        dispatch = ctx.dispatch_log()
+        # replay mode may leave transfers no later op waited for queued: the
+        # per-tenant totals count every enqueued chunk once dispatched
+        G.check(ctx.flush(), "flush")
+        G.check(ctx.sync(), "sync")
+        tenants = sorted({op["fn"]["wf"] for op in ops if isinstance(op.get("fn"), dict)})
+        return {"records": recs, "dispatch": dispatch, "stats": ctx.stats(),
+                "tenant_bytes": {wf: ctx.tenant_stats(wf) for wf in tenants}}
 
     _size_of: dict
 
@@ -284,6 +291,13 @@ def compare(orc_out, lib_out, check_dispatch=True):
                                          f"orc[:8]={o['bytes'][bad[0]:bad[0]+8]}")
             assert l["digest"] == o["digest"], ctx
             compared += 1
+    if "tenant_bytes" in lib_out and "oracle" in orc_out:
+        # per-tenant dispatched bytes per server kind (L193, grouter_tenant_stats):
+        # independent of dispatch timing, so real-time runs compare too
+        tb = orc_out["oracle"].tenant_bytes
+        for wf, got in lib_out["tenant_bytes"].items():
+            exp = [tb.get((wf, k), 0) for k in ("copy", "h2d", "d2h")]
+            assert got == exp, (wf, got, exp)
     if check_dispatch:
         olog = {}
         for r in o_recs:

@@ -297,3 +297,28 @@ def test_cfg5_interleaved_drains(restore, hints):
         for r in out["records"]:
             if r["op"] == "get_into" and r["restored"]:
                 assert all(by_oid[o] > ops[r["i"]]["fn"]["wf"] for o in r["restored"])
+
+
+def test_tenant_bytes_closed_form():
+    """Per-tenant scheduled bytes per server kind (L193; grouter_tenant_stats):
+    tenant 1 puts n1 from a CPU function toward GPU0 (H2D, striped over R(0))
+    and a GPU1 function reads it (one NVLink copy); tenant 2's GPU function
+    puts n2 by copy (an SM copy on its GPU) and a CPU function reads it (D2H).
+    Zero-copy gets and the host-store memcpy move nothing scheduled."""
+    n1, n2 = 5 * MiB + 123, 3 * MiB + 7
+    b = T.Builder(9)
+    o1 = b.put(T.fn(1, 1, model.HOST), n1, hint=0)
+    g1 = b.get_into(T.fn(1, 2, 1), o1)
+    z1 = b.get(T.fn(1, 3, 0), o1)                   # co-located: zero copy
+    b.release(T.fn(1, 3, 0), z1)
+    o2 = b.put(T.fn(2, 1, 1), n2)
+    g2 = b.get(T.fn(2, 2, model.HOST), o2)
+    b.release(T.fn(2, 2, model.HOST), g2)
+    o3 = b.put(T.fn(3, 1, model.HOST), MiB)          # cFn -> host store: memcpy only
+    b.get_into(T.fn(3, 2, model.HOST), o3)
+    orc = runner.run(b.ops, C.b200_hgx(2, shared_pairs=False))["oracle"]
+    assert orc.tenant_bytes == {(1, "h2d"): n1, (1, "copy"): n1, (2, "copy"): n2, (2, "d2h"): n2}
+    # the H2D share really was striped over both uplinks, and sums to n1
+    assert orc.link_bytes[("h2d", 0)] > 0 and orc.link_bytes[("h2d", 1)] > 0
+    assert orc.link_bytes[("h2d", 0)] + orc.link_bytes[("h2d", 1)] == n1
+    del g1
