@@ -65,6 +65,10 @@ extern "C" {
 #define GROUTER_RESTORE       0x40u/* proactive restore (L260-L262): when pool storage is released
                                       or a cap is raised, objects migrated away from that GPU come
                                       back while they fit (R42)                      */
+#define GROUTER_NO_POOL       0x200u/* ablation "ES off" (Fig. 16; L248 "cudaMalloc/cudaFree
+                                      ... millisecond-level"): every object / lease is its own
+                                      cudaMalloc, freed by cudaFree once its GPU work completed;
+                                      accounting, caps and eviction unchanged; no IPC export  */
 #define GROUTER_STRIPED_MIGRATION 0x100u /* spills leave over R(src) on the route GPUs' D2H
                                       engines (the gFn-host plan, L178), restores come back over
                                       R(d) with relays like a fetch (L178, L366 "parallel PCIe

@@ -801,6 +801,7 @@ grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_
   if (st) return st;
   Obj &o = *op;
   if (o.loc < 0) return fail(GROUTER_EINVAL, "export_ipc: object is not in a GPU pool");
+  if (c->cfg.flags & GROUTER_NO_POOL) return fail(GROUTER_EINVAL, "export_ipc: no pool segments (GROUTER_NO_POOL)");
   if (c->replay) flush_all(c);
   else pump(c, true);
   host_wait(o.ready);  // the importer sees finished bytes

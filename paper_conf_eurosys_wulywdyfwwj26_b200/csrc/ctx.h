@@ -249,6 +249,14 @@ struct grouter_ctx {
   std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
   std::unordered_map<uint32_t, uint32_t> weights;
   std::unordered_map<uint32_t, std::array<uint64_t, 3>> tenant_bytes;  // dispatched, per server kind
+  // GROUTER_NO_POOL (ablation): live cudaMalloc'ed buffers (ptr -> physical
+  // device) and frees waiting for the buffer's GPU work to complete
+  struct NoPoolFree {
+    uint8_t *p;
+    gr::Fences f;
+  };
+  std::unordered_map<uint8_t *, int> nopool_live;
+  std::vector<NoPoolFree> nopool_pending;
   std::map<uint32_t, std::array<uint64_t, 3>> slos;    // wf -> (data, slo_ns, infer_ns), R43
   // pool sizing (R44): per (wf, fid, gpu) histograms and resident counts
   std::map<std::tuple<uint32_t, uint32_t, int>, gr::FuncHist> hists;
@@ -291,6 +299,7 @@ void enqueue_plan(grouter_ctx *c, const XferRef &x, const std::vector<grouter_ch
                   int kind, uint64_t src_base, uint64_t dst_base, int dst_logical);
 void pump(grouter_ctx *c, bool force_all);            // dispatch rounds (caller holds mu)
 void flush_all(grouter_ctx *c);                        // replay flush
+void nopool_sweep(grouter_ctx *c, bool wait);            // GROUTER_NO_POOL deferred cudaFree
 void harvest_profile(grouter_ctx *c, bool wait);       // completed timed launches -> stats
 // Same-GPU SM copy run directly on the caller's stream when its copy server
 // is idle (or only busy with direct launches on that same stream).  Returns

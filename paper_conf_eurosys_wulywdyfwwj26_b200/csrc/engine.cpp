@@ -876,11 +876,12 @@ static void daemon_main(grouter_ctx *c) {
           LogicalDev &d = c->dev[i];
           DeviceGuard g(d.phys);
           d.pool.heap.reclaim();
+          if (i == 0 && !c->nopool_pending.empty()) nopool_sweep(c, false);
           // histogram-driven size (L250-L256, R44): pre-warm one segment per
           // tick toward the target, trim back to max(used, target)
           const uint64_t tgt = pool_target(c, (int)i);
           const uint64_t t0 = diag ? now_ns() : 0, m0 = d.pool.mapped;
-          if (d.pool.mapped < tgt) {
+          if (d.pool.mapped < tgt && !(c->cfg.flags & GROUTER_NO_POOL)) {
             try {
               d.pool.grow(std::min<uint64_t>(tgt - d.pool.mapped, 64ull << 20));
             } catch (const Error &) {
@@ -999,6 +1000,7 @@ void engine_init(grouter_ctx *c) {
     if (c->cfg.pool_cap_bytes[i]) d.cap = c->cfg.pool_cap_bytes[i];
     else d.cap = (uint64_t)((unsigned __int128)fr * c->cfg.pool_cap_permille / 1000) / kPage * kPage;
     uint64_t prewarm = std::min<uint64_t>(c->cfg.pool_floor_bytes, d.cap == GROUTER_UNLIMITED ? c->cfg.pool_floor_bytes : d.cap);
+    if (c->cfg.flags & GROUTER_NO_POOL) prewarm = 0;  // ablation: nothing pooled
     d.pool.init(i, d.phys, (uint64_t)tot * 2 / kPage * kPage, phys_list, prewarm / kPage * kPage);
     Server *ss[3] = {&d.copy, &d.h2d, &d.d2h};
     for (int k = 0; k < 3; ++k) {
@@ -1052,6 +1054,19 @@ void engine_shutdown(grouter_ctx *c) {
                std::chrono::steady_clock::now() - t0 < std::chrono::seconds(10))
           std::this_thread::sleep_for(std::chrono::microseconds(100));
   }
+  try {  // GROUTER_NO_POOL: every buffer still allocated goes back
+    if (!c->sticky_error && !c->nopool_pending.empty()) {
+      pump(c, true);  // replay: submit what the pending buffers wait for
+      nopool_sweep(c, true);
+    }
+  } catch (const Error &) {
+  }
+  for (auto &kv : c->nopool_live) {
+    DeviceGuard g(kv.second);
+    cudaFree(kv.first);
+  }
+  c->nopool_live.clear();
+  c->nopool_pending.clear();
   for (auto &d : c->dev) {
     DeviceGuard g(d.phys);
     Server *ss[3] = {&d.copy, &d.h2d, &d.d2h};

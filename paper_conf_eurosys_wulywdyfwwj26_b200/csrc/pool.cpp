@@ -346,6 +346,17 @@ static bool all_grounded(const grouter_ctx *c, const Quarantined &q) {
 // Order: free runs; reclaimed quarantine; wait for grounded quarantine (after
 // draining queued work so no wait depends on the caller); grow the mapping.
 uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
+  if (c->cfg.flags & GROUTER_NO_POOL) {  // ablation: no pool (Fig. 16 "ES" off)
+    nopool_sweep(c, false);
+    DeviceGuard g(c->dev[logical].phys);
+    void *p = nullptr;
+    if (cudaMalloc(&p, len) != cudaSuccess) {
+      cudaGetLastError();
+      throw Error(GROUTER_ENOMEM, "cudaMalloc failed (GROUTER_NO_POOL)");
+    }
+    c->nopool_live[(uint8_t *)p] = c->dev[logical].phys;
+    return (uint8_t *)p;
+  }
   DevicePool &P = c->dev[logical].pool;
   uint64_t off;
   P.heap.reclaim();
@@ -366,12 +377,43 @@ uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
 
 void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f) {
   if (!len) return;
+  if (c->cfg.flags & GROUTER_NO_POOL) {  // ablation: cudaFree once the buffer's GPU work completed
+    c->nopool_pending.push_back({p, std::move(f)});
+    nopool_sweep(c, false);
+    return;
+  }
   DevicePool &P = c->dev[logical].pool;
   uint64_t off = (uint64_t)p - P.base;
   bool done = true;
   for (auto &w : f) done &= w.done();
   if (done) P.heap.give(off, len);
   else P.heap.quarantine.push_back({off, len, std::move(f)});
+}
+
+// GROUTER_NO_POOL: cudaFree (which synchronizes the device -- the cost the
+// pool exists to avoid, L248) every pending buffer whose fences completed;
+// wait: first wait for all of them (shutdown).
+void nopool_sweep(grouter_ctx *c, bool wait) {
+  size_t k = 0;
+  for (size_t i = 0; i < c->nopool_pending.size(); ++i) {
+    auto &e = c->nopool_pending[i];
+    bool done = true;
+    if (wait) host_wait(e.f);
+    else
+      for (auto &w : e.f) done &= w.done();
+    if (!done) {
+      if (k != i) c->nopool_pending[k] = std::move(e);
+      ++k;
+      continue;
+    }
+    auto it = c->nopool_live.find(e.p);
+    if (it != c->nopool_live.end()) {
+      DeviceGuard g(it->second);
+      GR_CUDA(cudaFree(e.p));
+      c->nopool_live.erase(it);
+    }
+  }
+  c->nopool_pending.resize(k);
 }
 
 uint8_t *host_alloc(grouter_ctx *c, uint64_t len) {

@@ -448,3 +448,20 @@ def test_full_size_cfg3_max(n):
         ctx.free(cfn, oid)
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_no_pool(seed, replay):
+    """Ablation "ES off" (GROUTER_NO_POOL, Fig. 16): every object and lease
+    its own cudaMalloc; decisions, accounting and bytes are those of the
+    pooled library, i.e. the oracle's (the pool is a mechanism, not a policy)."""
+    rng = random.Random(9100 + seed)
+    k = rng.choice([1, 2, 3])
+    calib = C.virtual(k)
+    ops = T.random_trace(rng, k, n_ops=100, max_n=9 * MiB, run_seed=seed)
+    caps = [rng.choice([16, 64]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, host_store_bytes=64 * MiB, pool_cap=caps,
+                         flags=G.NO_POOL)
+    compare(orc, lib_out, check_dispatch=replay)
+    assert all(lib_out["stats"].mapped[g] == 0 for g in range(k))   # nothing pooled

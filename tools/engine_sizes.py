@@ -47,8 +47,19 @@ def child():
         reps = 40 if n <= 64 * MiB else 10
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(s)
+        ce = os.environ.get("GR_SIZES_CE") == "1"     # baseline: cudaMemcpyAsync D2D (copy engine)
+        srcs = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(k)] if ce else None
+        if ce:
+            with torch.cuda.stream(s):
+                for i in range(3):
+                    dsts[(i + 1) % k].copy_(srcs[i % k])
+            a.record(s)
         for i in range(reps):
-            ctx.get_into(f, objs[i % k], dsts[(i + 1) % k].data_ptr(), n, s.cuda_stream)
+            if ce:
+                with torch.cuda.stream(s):
+                    dsts[(i + 1) % k].copy_(srcs[i % k])
+            else:
+                ctx.get_into(f, objs[i % k], dsts[(i + 1) % k].data_ptr(), n, s.cuda_stream)
         b.record(s)
         b.synchronize()
         us = a.elapsed_time(b) * 1e3 / reps
@@ -58,7 +69,7 @@ def child():
         del dsts
         torch.cuda.empty_cache()
     ctx.close()
-    print(json.dumps({"engine": os.environ.get("GR_COPY", "default"), "pf": os.environ.get("GR_PF", "1"),
+    print(json.dumps({"engine": "ce" if os.environ.get("GR_SIZES_CE") == "1" else os.environ.get("GR_COPY", "default"), "pf": os.environ.get("GR_PF", "1"),
                       "res": out}), flush=True)
 
 
@@ -69,7 +80,9 @@ if __name__ == "__main__":
         for e in sys.argv[1:] or ["default", "wv8", "tma8"]:
             env = dict(os.environ)
             name, _, pf = e.partition("@")
-            if name != "default":
+            if name == "ce":
+                env["GR_SIZES_CE"] = "1"
+            elif name != "default":
                 env["GR_COPY"] = name
             if pf:
                 env["GR_PF"] = pf
