@@ -49,7 +49,7 @@ def run(flags, workload, reqs):
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=512 << 20, pool_cap=[G.UNLIMITED] * 2,
                                     flags=flags))
     s = torch.cuda.Stream()
-    lat, mapped, used = [], [], []
+    lat, mapped = [], []
     mid = []            # demand while the request's objects are live
 
     def sample():
