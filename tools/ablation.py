@@ -22,7 +22,10 @@ Workloads per request (full sizes of BASELINE.json configs 1 and 5):
 Reported: request latency p50/p99 (host clock, request issue -> consumer
 stream drained), req/s, and pool footprint: peak/mean `mapped` (physical
 pool pages) against the peak demand (`used` while a request's objects are
-live); -ES maps nothing (its cudaMalloc buffers are the demand itself).
+live); -ES maps nothing (its cudaMalloc buffers are the demand itself);
+and the process CPU time over wall time while requests run (Fig. 20b
+analog: the caller thread spins while it waits for its bytes, so ~1 core
+is the floor for a blocking client).
 usage: python tools/ablation.py OUT.json"""
 import json
 import sys
@@ -87,12 +90,14 @@ def run(flags, workload, reqs):
                 s.synchronize()
         for _ in range(3):
             request()
+        c0, w0 = time.process_time(), time.perf_counter()
         for _ in range(reqs):
             t = time.perf_counter()
             request()
             lat.append((time.perf_counter() - t) * 1e6)
             st = ctx.stats()
             mapped.append(st.mapped[0] + st.mapped[1])
+        cpu = (time.process_time() - c0) / (time.perf_counter() - w0)
         G.check(ctx.sync(), "sync")
     finally:
         ctx.close()
@@ -101,7 +106,8 @@ def run(flags, workload, reqs):
             "req_s": round(reqs / tot, 1), "mapped_peak_MiB": max(mapped) >> 20,
             "mapped_mean_MiB": round(sum(mapped) / len(mapped) / MiB, 1),
             "demand_peak_MiB": max(mid) >> 20, "requests": reqs,
-            "overhead_x": round(max(mapped) / max(1, max(mid)), 2)}
+            "overhead_x": round(max(mapped) / max(1, max(mid)), 2),
+            "cpu_cores": round(cpu, 2)}
 
 
 def main():
