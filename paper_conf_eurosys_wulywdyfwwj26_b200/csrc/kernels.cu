@@ -345,6 +345,70 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant
   finish_round(p);
 }
 
+// Static-assignment TMA ring ("tmas"): CTA b of G moves the 16 KiB units
+// b, b+G, b+2G ... of the round (no ticket, so no scratch to reset and the
+// completion can be published by the host after the launch), through a
+// STAGES-deep cp.async.bulk ring small enough (STAGES x 16 KiB <= 96 KiB)
+// that the NEXT launch's CTA is co-resident under PDL.  Before
+// griddepcontrol.wait it initialises its barriers and pulls its first
+// STAGES units of SOURCE into L2 (local sources only, like wv), so the DRAM
+// read ramp of launch i+1 overlaps the tail of launch i.  16 B-aligned
+// rounds only (bulk copies need 16 B addresses and sizes).
+template <int STAGES, class KP>
+__global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constant__ KP p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t bars[STAGES];
+  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
+  const uint32_t G = gridDim.x;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < STAGES; ++i) mbar_init(&bars[i], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (p.flags & kFlagLocalSrc)
+      for (uint32_t k = 0, id = blockIdx.x; k < (uint32_t)STAGES && id < total; ++k, id += G) {
+        const int c = find_chunk(p, id);
+        const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) * kTmaStage;
+        prefetch_l2(p.chunk[c].src + off, (uint32_t)umin64(p.chunk[c].bytes - off, kTmaStage));
+      }
+  }
+  pdl_wait();
+  if (threadIdx.x == 0) {
+    uint64_t dst_of[STAGES];
+    uint32_t bytes_of[STAGES];
+    uint32_t phase = 0;
+    auto load = [&](uint32_t k) {  // unit number k of this CTA -> stage k % STAGES
+      const uint32_t id = blockIdx.x + k * G;
+      const int c = find_chunk(p, id);
+      const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) * kTmaStage;
+      const uint32_t st = k % STAGES;
+      const uint32_t pb = (uint32_t)umin64(p.chunk[c].bytes - off, kTmaStage);
+      dst_of[st] = p.chunk[c].dst + off;
+      bytes_of[st] = pb;
+      mbar_expect_tx(&bars[st], pb);
+      bulk_g2s(smem + st * kTmaStage, reinterpret_cast<const void *>(p.chunk[c].src + off), pb, &bars[st]);
+    };
+    const uint32_t mine = blockIdx.x < total ? (total - blockIdx.x + G - 1) / G : 0;
+    uint32_t loaded = 0;
+    for (; loaded < mine && loaded < (uint32_t)STAGES; ++loaded) load(loaded);
+    for (uint32_t k = 0; k < mine; ++k) {
+      const uint32_t st = k % STAGES;
+      mbar_wait(&bars[st], (phase >> st) & 1u);
+      phase ^= (1u << st);
+      bulk_s2g(reinterpret_cast<void *>(dst_of[st]), smem + st * kTmaStage, bytes_of[st]);
+      bulk_commit();
+      if (k >= 1 && loaded < mine) {
+        bulk_wait_read<1>();  // the store of unit k-1 has left its stage
+        load(loaded);
+        ++loaded;
+      }
+    }
+    bulk_wait_all();
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+  }
+  __syncthreads();
+  pdl_trigger();
+  finish_round(p);
+}
+
 // Before waiting on the predecessor grid (PDL), a warp may pull the first
 // units of its OWN source into L2 with bulk prefetches: L2 is the point of
 // coherence for this GPU's memory, so a prefetch can never return stale
@@ -756,10 +820,38 @@ static int variant_from_env() {
       std::string s(e);
       v = s == "ldst8" ? 0 : s == "ldst16" ? 1 : s == "tma4" ? 2 : s == "tma8" ? 3 : s == "tma12" ? 4
         : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : s == "wd1" ? 8 : s == "wd2" ? 9
-        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : s == "wv4" ? 13 : s == "wv8" ? 14 : -1;
+        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : s == "wv4" ? 13 : s == "wv8" ? 14
+        : s == "tmas6" ? 15 : s == "tmas4" ? 16 : s == "tmas3" ? 17 : s == "tmas2" ? 18 : -1;
     }
   }
   return v;
+}
+
+template <int STAGES, class KP>
+static void launch_tmas(KP &p, int sm_count, cudaStream_t s) {
+  static bool attr_set = false;
+  const int smem = STAGES * kTmaStage;
+  if (!attr_set) {
+    cudaFuncSetAttribute(gr_copy_tmas<STAGES, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr_set = true;
+  }
+  p.tile_log2 = 14;  // units of kTmaStage bytes
+  uint64_t t = 0;
+  for (uint32_t i = 0; i < p.n_chunks; ++i) {
+    p.tile_prefix[i] = t;
+    t += (p.chunk[i].bytes + kTmaStage - 1) / kTmaStage;
+  }
+  p.tile_prefix[p.n_chunks] = t;
+  static int per_sm = -1;  // CTAs per SM (tuning: GR_TMAS_CTAS)
+  if (per_sm < 0) {
+    const char *e = getenv("GR_TMAS_CTAS");
+    per_sm = e ? atoi(e) : 1;
+    if (per_sm < 1 || per_sm > 8) per_sm = 1;
+  }
+  uint64_t grid = (uint64_t)sm_count * per_sm;
+  if (grid > t) grid = t;
+  if (grid == 0) grid = 1;
+  launch_pdl(gr_copy_tmas<STAGES, KP>, grid, kTmaThreads, smem, s, p);
 }
 
 template <int STAGES, class KP>
@@ -922,6 +1014,10 @@ static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStre
     case 2: launch_tma<4>(p, sm_count, s); break;
     case 3: launch_tma<8>(p, sm_count, s); break;
     case 4: launch_tma<12>(p, sm_count, s); break;
+    case 15: launch_tmas<6>(p, sm_count, s); break;
+    case 16: launch_tmas<4>(p, sm_count, s); break;
+    case 17: launch_tmas<3>(p, sm_count, s); break;
+    case 18: launch_tmas<2>(p, sm_count, s); break;
     default: launch_ldst<8, 1>(p, sm_count, ctas_per_sm, s); break;
   }
 }
@@ -978,18 +1074,23 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   uint64_t total = 0;
   for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
   int v = variant_from_env();
-  // default: the 8-stage TMA bulk ring for large aligned rounds (best at
-  // >= 256 MiB: 6.47 TB/s at 1 GiB; tools/engine_sizes.py), otherwise the warp-strided 256-bit engine over 8 KiB units
-  // (wv8) whose warps prefetch their first unit into L2 before the PDL wait
-  // (38.5 MB get_into back to back: 13.2 us with ws1, 11.8 us with wv8 +
-  // prefetch); GROUTER_COPY_TMA forces the bulk ring for every aligned round
-  if (v < 0) v = (tma || (aligned && total >= (256ull << 20))) ? 3 : 14;
+  // default: for large aligned rounds (>= 96 MiB) the static 4-stage TMA
+  // bulk ring, one CTA per SM, L2 prefetch before the PDL wait (tmas4:
+  // 128 MiB 45.1 us, 256 MiB 84.9 us, 1 GiB 329.6 us back to back = the
+  // copy engine's 44.4 / 84.3 / 329.3; tools/engine_sizes.py,
+  // profiles/r01_engine_sizes_tmas.txt); otherwise the warp-strided 256-bit
+  // engine over 8 KiB units (wv8) whose warps prefetch their first unit into
+  // L2 before the PDL wait (38.5 MB get_into back to back: 13.2 us with ws1,
+  // 11.8 us with wv8 + prefetch); GROUTER_COPY_TMA forces the ticketed bulk
+  // ring (tma8) for every aligned round
+  if (v < 0) v = tma ? 3 : (aligned && total >= (96ull << 20)) ? 16 : 14;
   // a user buffer at an odd address (a tensor view, a by-copy put of a host
   // structure): the warp-strided engines would fall back to byte copies;
   // the tiled LD/ST engine keeps 16 B accesses with its co-aligned and
   // funnel-shift paths
   if (!addr_aligned && variant_from_env() < 0) v = 0;
-  if (((v >= 2 && v <= 4) || (v >= 10 && v <= 12)) && (!aligned || p.counts)) v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
+  if (((v >= 2 && v <= 4) || (v >= 10 && v <= 12) || v >= 15) && (!aligned || p.counts))
+    v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
   // static-assignment engines (ws, gs) need no scratch: their completion can
   // be published by a stream write after the launch, which costs the GPU
   // ~2 us less than the in-kernel fence + counter + last-CTA protocol

@@ -70,7 +70,7 @@ def test_copy_kernel_exactly_once(tma, src_off, dst_off):
 
 VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4", "wd1", "wd2", "gs4", "gs8", "gs16",
             "wv4", "wv8", "wv4:GR_HINT=3", "wv8:GR_HINT=5", "wv4:GR_PF=2:GR_EARLY=1", "ws1:GR_PF=1:GR_EARLY=1",
-            "wv8:GR_PF=1", "wv8:GR_PF=2:GR_PFLOOP=1"]
+            "wv8:GR_PF=1", "wv8:GR_PF=2:GR_PFLOOP=1", "tmas4", "tmas6"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
@@ -89,6 +89,40 @@ def test_copy_kernel_variants(variant):
     r = subprocess.run([sys.executable, "-c", code], env=env,
                        capture_output=True, text=True, timeout=240)
     assert r.returncode == 0, r.stderr[-2000:]
+
+
+ALIGNED_VARIANTS = ["tma4", "tma8", "tma12", "tmas4", "tmas6", "wv8", "ws1", "gs8"]
+
+
+@pytest.mark.parametrize("variant", ALIGNED_VARIANTS)
+def test_copy_kernel_aligned_rounds(variant):
+    """The bulk-copy engines only take 16 B-aligned rounds (others fall back
+    to LD/ST): a chunk list whose cuts are multiples of 16 B, with units cut
+    mid-chunk, a ragged last unit and a chunk smaller than one 16 KiB unit,
+    byte-exact with untouched guard bands; sizes from one unit to 70 MiB."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, GR_COPY=variant)
+    code = ("import sys; sys.path.insert(0, '.'); from tests.test_gpu_parity import _copy_aligned as f; "
+            "[f(n, s) for n, s in ((16384, 1), (5 * 2**20 + 4096 + 48, 2), (70 * 2**20 + 16 * 77, 3))]")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=240)
+    assert r.returncode == 0, r.stderr[-2000:]
+
+
+def _copy_aligned(n, seed):
+    rng = random.Random(seed)
+    cuts = sorted({16 * rng.randint(1, n // 16 - 1) for _ in range(6)} | {16 * 5})
+    bounds = [0] + [c for c in cuts if 0 < c < n] + [n]
+    chunks = [(a, b - a, 0, 0) for a, b in zip(bounds, bounds[1:])]
+    src = torch.empty(n + 256, dtype=torch.uint8, device="cuda")
+    dst = torch.full((n + 256,), 0xA5, dtype=torch.uint8, device="cuda")
+    G.check(G.test_fill(src.data_ptr() + 128, n, 91 + seed, 0, 0))
+    G.check(G.test_copy(dst.data_ptr() + 128, src.data_ptr() + 128, chunks, counts=0, tma=False))
+    torch.cuda.synchronize()
+    d = dst.cpu().numpy()
+    assert np.array_equal(d[128:128 + n], payload(91 + seed, n))
+    assert (d[:128] == 0xA5).all() and (d[128 + n:] == 0xA5).all()
 
 
 def _copy_exactly_once(tma, src_off, dst_off):

@@ -69,7 +69,8 @@ def child():
         del dsts
         torch.cuda.empty_cache()
     ctx.close()
-    print(json.dumps({"engine": "ce" if os.environ.get("GR_SIZES_CE") == "1" else os.environ.get("GR_COPY", "default"), "pf": os.environ.get("GR_PF", "1"),
+    print(json.dumps({"engine": ("ce" if os.environ.get("GR_SIZES_CE") == "1" else os.environ.get("GR_COPY", "default"))
+                      + (f" ctas={os.environ['GR_TMAS_CTAS']}" if "GR_TMAS_CTAS" in os.environ else ""), "pf": os.environ.get("GR_PF", "1"),
                       "res": out}), flush=True)
 
 
@@ -79,6 +80,8 @@ if __name__ == "__main__":
     else:
         for e in sys.argv[1:] or ["default", "wv8", "tma8"]:
             env = dict(os.environ)
+            e, *extra = e.split(":")        # ENGINE[@PF][:ENV=VAL ...]
+            env.update(kv.split("=", 1) for kv in extra)
             name, _, pf = e.partition("@")
             if name == "ce":
                 env["GR_SIZES_CE"] = "1"
