@@ -21,6 +21,19 @@ for tma in (False, True):
         torch.cuda.synchronize()
         st, bad, _ = G.test_verify(dst.data_ptr() + do, n, 5, 0, 0)
         assert bad == 0
+# 16 B-aligned chunk lists (the bulk-copy engines only take these)
+for seed in (1, 2):
+    n = 3 * MiB + 48 * seed
+    rng = random.Random(seed)
+    cuts = sorted({16 * rng.randint(1, n // 16 - 1) for _ in range(5)})
+    b = [0] + cuts + [n]
+    src = torch.empty(n, dtype=torch.uint8, device="cuda")
+    dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+    G.check(G.test_fill(src.data_ptr(), n, 9, 0, 0))
+    G.check(G.test_copy(dst.data_ptr(), src.data_ptr(), [(x, y - x, 0, 0) for x, y in zip(b, b[1:])]))
+    torch.cuda.synchronize()
+    st, bad, _ = G.test_verify(dst.data_ptr(), n, 9, 0, 0)
+    assert bad == 0
 from tests.lib_runner import LibRunner
 from oracle import runner as orun
 from tests.lib_runner import compare
