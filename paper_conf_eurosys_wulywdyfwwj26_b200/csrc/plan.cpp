@@ -103,9 +103,23 @@ static u128 path_time(uint64_t m, const PathModel &p, uint64_t g) {
   return (u128)p.phi_ps + chunks * p.alpha_ps + xfer;
 }
 
-// Largest m <= N with T_p(m) <= T (T_p is non-decreasing in m).
+// Largest m <= N with T_p(m) <= T (T_p is non-decreasing in m).  The
+// ceilings put T_p(m) between L(m) = phi + m*r and L(m) + alpha + 1 ps, with
+// r = g*alpha/C + g*1e12/beta per granule, so the answer lies in a window of
+// about (alpha + 1)/r granules around (T - phi)/r; the window is verified
+// (and widened if rounding misplaced it) with the exact T_p before the
+// bisection, so the result is the exact one.
 static uint64_t path_cap(u128 T, uint64_t N, const PathModel &p, uint64_t g) {
-  uint64_t lo = 0, hi = N;
+  if (path_time(N, p, g) <= T) return N;
+  if (T < (u128)p.phi_ps) return 0;
+  const double r = (double)g * (double)p.alpha_ps / (double)p.chunk + (double)g * 1e12 / (double)p.beta_Bps;
+  const double span = (double)(T - (u128)p.phi_ps);
+  const double a = (span - (double)p.alpha_ps - 1.0) / r, b = span / r;
+  uint64_t lo = a <= 1.0 ? 0 : (uint64_t)a - 1, hi = b >= (double)N ? N : (uint64_t)b + 1;
+  if (hi > N) hi = N;
+  if (lo > hi) lo = hi;
+  while (lo > 0 && path_time(lo, p, g) > T) lo = lo > 64 ? lo - 64 : 0;  // lo must be feasible
+  while (hi < N && path_time(hi + 1, p, g) <= T) hi = std::min<uint64_t>(N, hi + 64);  // hi+1 infeasible
   while (lo < hi) {
     uint64_t mid = lo + (hi - lo + 1) / 2;
     if (path_time(mid, p, g) <= T) lo = mid;
@@ -120,6 +134,11 @@ void split_plan(const std::vector<PathModel> &P, uint64_t n, uint64_t g, std::ve
   out.clear();
   if (n == 0 || P.empty()) return;
   const uint64_t N = ceil_div(n, g);
+  if (P.size() == 1) {  // one path carries every granule: chunks of C_p
+    for (uint64_t off = 0; off < n; off += P[0].chunk)
+      out.push_back({off, std::min<uint64_t>(P[0].chunk, n - off), 0, (int32_t)P[0].route_gpu});
+    return;
+  }
   // 1. T* = min { T : sum_p cap_p(T) >= N }  (bisection on integer ps)
   u128 lo = 0, hi = path_time(N, P[0], g);
   while (lo < hi) {
@@ -164,7 +183,16 @@ void size_chunks(std::vector<PathModel> &P, uint64_t C, uint64_t g) {
 }
 
 void Planner::plan_h2d(int d, uint64_t n, std::vector<grouter_chunk> &out) const {
+  std::lock_guard<std::mutex> lk(cache_mu);
+  auto &m = cache[d];
+  auto it = m.find(n);
+  if (it != m.end()) {
+    out = it->second;
+    return;
+  }
   split_plan(paths[d], n, cfg.granule, out);
+  if (m.size() >= 256) m.clear();  // bounded; sizes in a workload repeat
+  m.emplace(n, out);
 }
 
 void Planner::plan_single(uint64_t n, int route_gpu, std::vector<grouter_chunk> &out) const {

@@ -9,6 +9,8 @@
 #pragma once
 
 #include <cstdint>
+#include <mutex>
+#include <unordered_map>
 #include <vector>
 
 #include "../../include/grouter.h"
@@ -32,6 +34,12 @@ struct Planner {
   std::vector<std::vector<int>> groups;          // uplink groups, each sorted
   std::vector<std::vector<int>> routes;          // R(d) per destination
   std::vector<std::vector<PathModel>> paths;     // per destination, in route order
+
+  // plan_h2d results by (d, n): the O6 split is a pure function of the
+  // calibration, d and n, and workloads repeat sizes (the exact split costs
+  // a bisection over makespans: ~40 us for 38.5 MB over 4 routes)
+  mutable std::mutex cache_mu;
+  mutable std::unordered_map<uint64_t, std::vector<grouter_chunk>> cache[GROUTER_MAX_GPUS];
 
   void build(const grouter_config &c);
   // host -> d striped plan (O6); D2D/same-GPU/D2H single-path plan.
