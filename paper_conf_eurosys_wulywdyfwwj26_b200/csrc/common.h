@@ -6,6 +6,8 @@
 // grouter_init().
 #pragma once
 
+#include <atomic>
+
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -95,6 +97,9 @@ struct Event {
   cudaEvent_t ev = nullptr;
   int phys = -1;
   EventPool *pool = nullptr;
+  // completion memo shared by every fence holding this event (an event query
+  // costs ~1 us of host time); reset when the pool hands the event out again
+  std::atomic<bool> fired{false};
 };
 using EventRef = std::shared_ptr<Event>;
 
@@ -123,12 +128,13 @@ struct Waitable {
   // stream the event was recorded on (events only): fences of one stream
   // complete in order, so a newer one stands for the older ones
   cudaStream_t origin = nullptr;
-  mutable bool fired = false;  // memo: an event query costs ~1.4 us of host time
   bool done() const {
     if (word) return (int32_t)(*word - target) >= 0;
     if (ev) {
-      if (!fired) fired = cudaEventQuery(ev->ev) == cudaSuccess;
-      return fired;
+      if (ev->fired.load(std::memory_order_relaxed)) return true;
+      if (cudaEventQuery(ev->ev) != cudaSuccess) return false;
+      ev->fired.store(true, std::memory_order_relaxed);
+      return true;
     }
     return true;
   }

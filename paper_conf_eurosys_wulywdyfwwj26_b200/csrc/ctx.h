@@ -119,7 +119,6 @@ struct Xfer {
   // completion slot is handed back at once)
   EventRef done_ev;
   cudaStream_t done_stream = nullptr;      // stream done_ev was recorded on
-  mutable bool done_fired = false;
   // word fences were handed out (done_fences before the transfer's rounds
   // ran): its words must be published, an event may not stand in for them
   mutable bool word_fenced = false;

@@ -142,7 +142,6 @@ void done_fences(const XferRef &x, Fences &f) {
     w.ev = x->done_ev;
     w.epoch = x->epoch;
     w.origin = x->done_stream;
-    w.fired = x->done_fired;
     f.push_back(w);
     return;
   }
@@ -160,8 +159,10 @@ void done_fences(const XferRef &x, Fences &f) {
 
 bool Xfer::done() const {
   if (done_ev) {
-    if (!done_fired) done_fired = cudaEventQuery(done_ev->ev) == cudaSuccess;
-    return done_fired;
+    if (done_ev->fired.load(std::memory_order_relaxed)) return true;
+    if (cudaEventQuery(done_ev->ev) != cudaSuccess) return false;
+    done_ev->fired.store(true, std::memory_order_relaxed);
+    return true;
   }
   for (uint32_t p = 0; p < npath; ++p)
     if (total[p] && (int32_t)(words[p] - target[p]) < 0) return false;

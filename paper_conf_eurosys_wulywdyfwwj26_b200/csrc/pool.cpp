@@ -115,6 +115,7 @@ EventRef EventPool::get() {
       free_list.pop_back();
     }
   }
+  if (e) e->fired.store(false, std::memory_order_relaxed);
   if (!e) {
     e = new Event();
     e->phys = phys;
