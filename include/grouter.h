@@ -201,7 +201,7 @@ grouter_status grouter_alloc(grouter_ctx *ctx, const grouter_fn *fn, uint64_t n,
 grouter_status grouter_seal(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *stream);
 /* Get (L165, L167): read-only lease on fn->device.  Same location -> the
  * object's own address (zero copy, pins the object).  Otherwise a copy lease
- * (D2D over NVLink, striped H2D, or D2H for a CPU fn).  *ptr/*n out. */
+ * (D2D over NVLink, striped H2D, or D2H for a CPU fn).  *ptr, *n out. */
 grouter_status grouter_get(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *stream,
                            const void **ptr, uint64_t *n);
 /* Get into caller memory `dst` (device memory of fn->device, or host memory
