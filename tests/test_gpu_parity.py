@@ -499,3 +499,50 @@ def test_random_traces_no_pool(seed, replay):
                          flags=G.NO_POOL)
     compare(orc, lib_out, check_dispatch=replay)
     assert all(lib_out["stats"].mapped[g] == 0 for g in range(k))   # nothing pooled
+
+
+def test_bench_launch_configuration_parity():
+    """Parity in the launch configuration bench.py times (BASELINE.json cfg1
+    at full size): the bench's context (one B200, copy_ctas_per_sm=4, pool
+    auto-capped), 38,535,168 B objects put by a cFn from pinned host with hint
+    GPU0, then gFn get_into's on one stream back to back into two rotating
+    bindings (direct launches, wv8 + L2 prefetch + PDL) -- every delivered
+    binding compared in full with the oracle's get_into of the same payload."""
+    from oracle.model import Oracle
+    from synth.calib import b200_hgx
+    n = 38_535_168
+    calib = b200_hgx(1)
+    calib["device_map"] = [0]
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED],
+                                    copy_ctas_per_sm=4))
+    orc = Oracle(b200_hgx(1))
+    cfn, gfn = G.fn(1, 1, G.HOST), G.fn(1, 2, 0)
+    ocfn, ogfn = {"wf": 1, "fid": 1, "dev": -1}, {"wf": 1, "fid": 2, "dev": 0}
+    s = torch.cuda.Stream()
+    bindings = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    try:
+        oids, ooids = [], []
+        for i in range(4):
+            data = payload(1000 + i, n)
+            host = torch.from_numpy(data).pin_memory()
+            st, oid = ctx.put(cfn, host.data_ptr(), n, 0, 0)
+            G.check(st, "put")
+            oids.append(oid)
+            ost, out = orc.put(ocfn, data, n, 0, 0)
+            assert ost == 0
+            ooids.append(out["oid"])
+        expect = np.empty(n, np.uint8)
+        for rep in range(3):
+            for i in range(4):       # back to back on one stream, as timed by bench.py
+                G.check(ctx.get_into(gfn, oids[i], bindings[i % 2].data_ptr(), n, s.cuda_stream)[0], "get_into")
+            s.synchronize()
+            for b in range(2):       # the last request that wrote binding b
+                i = 2 + b
+                ost, _ = orc.get_into(ogfn, ooids[i], expect, n)
+                assert ost == 0
+                got = bindings[b].cpu().numpy()
+                assert np.array_equal(got, expect), (rep, b, int(np.count_nonzero(got != expect)))
+        st = ctx.stats()
+        assert st.kernel_launches >= 12
+    finally:
+        ctx.close()
