@@ -316,6 +316,17 @@ grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
  * GPUs.  Scheduled transfers only: spills and restores are unscheduled
  * (R41, R42).  An unknown tenant reads zeros.  EINVAL on null arguments. */
 grouter_status grouter_tenant_stats(grouter_ctx *ctx, uint32_t workflow_id, uint64_t bytes[3]);
+/* Real-time rate monitor (L197: GROUTER "monitors the transfer rate of each
+ * function in real time, ensuring that it does not fall below Rate_least"):
+ * *rate_Bps = bytes of workflow_id's chunks dispatched by every server in
+ * the last window_ns nanoseconds (1 ms <= window_ns <= 10 s, else EINVAL),
+ * times 1e9 / window_ns (integer, rounded down); *rate_least_Bps =
+ * ceil(data * 1e9 / (slo - infer)) from grouter_set_tenant_slo, 0 without an
+ * SLO; *backlogged = 1 if chunks of the tenant are queued and not yet
+ * dispatched (a tenant below Rate_least only misses it while backlogged).
+ * Dispatch times use the library clock (grouter_test_set_clock fixes it). */
+grouter_status grouter_tenant_rate(grouter_ctx *ctx, uint32_t workflow_id, uint64_t window_ns, uint64_t *rate_Bps,
+                                   uint64_t *rate_least_Bps, int32_t *backlogged);
 /* Takes (and clears) the objects spilled since the last call, in order. */
 grouter_status grouter_victims(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
 /* Takes (and clears) the objects proactively restored to a GPU pool since the

@@ -1064,6 +1064,35 @@ grouter_status grouter_tenant_stats(grouter_ctx *c, uint32_t workflow_id, uint64
   return GROUTER_OK;
 }
 
+grouter_status grouter_tenant_rate(grouter_ctx *c, uint32_t wf, uint64_t window_ns, uint64_t *rate_Bps,
+                                   uint64_t *rate_least_Bps, int32_t *backlogged) {
+  if (!c || !rate_Bps || !rate_least_Bps || !backlogged) return fail(GROUTER_EINVAL, "null argument");
+  if (window_ns < 1000000ull || window_ns > 10000000000ull) return fail(GROUTER_EINVAL, "tenant_rate: window");
+  Guard g(c);
+  const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
+  unsigned __int128 bytes = 0;
+  auto it = c->tenant_log.find(wf);
+  if (it != c->tenant_log.end())
+    for (auto r = it->second.rbegin(); r != it->second.rend() && r->first + window_ns > now; ++r) bytes += r->second;
+  *rate_Bps = (uint64_t)(bytes * 1000000000u / window_ns);
+  uint64_t least = 0;
+  auto s = c->slos.find(wf);
+  if (s != c->slos.end()) {
+    const unsigned __int128 num = (unsigned __int128)s->second[0] * 1000000000u, den = s->second[1] - s->second[2];
+    least = (uint64_t)((num + den - 1) / den);
+  }
+  *rate_least_Bps = least;
+  int32_t bl = 0;
+  for (auto &d : c->dev)
+    for (Server *sv : {&d.copy, &d.h2d, &d.d2h}) {
+      auto t = sv->sched.tenants.find(wf);
+      if (t != sv->sched.tenants.end() && !t->second.q.empty()) bl = 1;
+      for (auto &ci : sv->carry) bl |= ci.x->tenant == wf;
+    }
+  *backlogged = bl;
+  return GROUTER_OK;
+}
+
 grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
   if (!c || !out) return fail(GROUTER_EINVAL, "null argument");
   Guard g(c);

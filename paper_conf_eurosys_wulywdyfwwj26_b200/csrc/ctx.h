@@ -248,6 +248,8 @@ struct grouter_ctx {
   std::unordered_map<uintptr_t, gr::Lease> leases;     // copy leases by address
   std::unordered_map<uint32_t, uint32_t> weights;
   std::unordered_map<uint32_t, std::array<uint64_t, 3>> tenant_bytes;  // dispatched, per server kind
+  // rate monitor (L197): (dispatch time ns, bytes) per dispatched batch, last 10 s
+  std::unordered_map<uint32_t, std::deque<std::pair<uint64_t, uint64_t>>> tenant_log;
   // GROUTER_NO_POOL (ablation): live cudaMalloc'ed buffers (ptr -> physical
   // device) and frees waiting for the buffer's GPU work to complete
   struct NoPoolFree {

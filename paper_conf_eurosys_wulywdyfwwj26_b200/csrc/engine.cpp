@@ -270,6 +270,12 @@ static void refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max
     if (t == UINT32_MAX) break;
     log_batch(c, s, t, b, bb);
     c->tenant_bytes[t][s.kind] += bb;
+    {  // rate monitor (L197): keep 10 s of dispatch records per tenant
+      auto &lg = c->tenant_log[t];
+      const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
+      lg.emplace_back(now, bb);
+      while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
+    }
     for (auto &it : b) s.carry.push_back(it);
     bytes += bb;
     ++nb;

@@ -134,6 +134,7 @@ SIGNATURES = {
     "grouter_where": (_ST, [_CTX, _U64, C.POINTER(_I32)]),
     "grouter_stats": (_ST, [_CTX, C.POINTER(grouter_stats_t)]),
     "grouter_tenant_stats": (_ST, [_CTX, C.c_uint32, C.POINTER(_U64)]),
+    "grouter_tenant_rate": (_ST, [_CTX, C.c_uint32, _U64, C.POINTER(_U64), C.POINTER(_U64), C.POINTER(_I32)]),
     "grouter_victims": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_restored": (_ST, [_CTX, C.POINTER(_U64), _U64, C.POINTER(_U64)]),
     "grouter_paths_new": (C.c_void_p, [C.c_uint32, C.c_uint32, C.POINTER(_U64), C.c_uint32]),
@@ -398,6 +399,13 @@ class Ctx:
         arr = (_U64 * 3)()
         check(self.lib.grouter_tenant_stats(self.h, workflow_id, arr), "tenant_stats")
         return list(arr)
+
+    def tenant_rate(self, workflow_id: int, window_ns: int):
+        """(dispatched B/s over the window, Rate_least B/s (0 without SLO), backlogged)."""
+        r, least, bl = _U64(0), _U64(0), _I32(0)
+        check(self.lib.grouter_tenant_rate(self.h, workflow_id, window_ns, C.byref(r), C.byref(least),
+                                           C.byref(bl)), "tenant_rate")
+        return r.value, least.value, bool(bl.value)
 
     def stats(self) -> grouter_stats_t:
         s = grouter_stats_t()

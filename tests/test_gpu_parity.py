@@ -546,3 +546,31 @@ def test_bench_launch_configuration_parity():
         assert st.kernel_launches >= 12
     finally:
         ctx.close()
+
+
+def test_tenant_rate_monitor_fixed_clock():
+    """The real-time rate monitor (L197) on the device path with the library
+    clock fixed: a tenant's 8 MiB cFn put dispatched at t = 1 s is counted in
+    a 10 ms window read at t = 1.005 s -- exactly 8 MiB x 1e9 / 1e7 B/s -- and
+    is out of a 1 ms window; a second tenant's bytes never mix in; nothing is
+    backlogged after blocking calls; Rate_least from the declared SLO."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2))
+    try:
+        G.check(ctx.set_tenant_slo(5, 8 * MiB, 20_000_000, 0), "slo")
+        host = torch.empty(8 * MiB, dtype=torch.uint8, pin_memory=True)
+        ctx.set_clock(1_000_000_000)
+        st, oid = ctx.put(G.fn(5, 1, G.HOST), host.data_ptr(), 8 * MiB, 0, 0)
+        G.check(st, "put")
+        st, oid2 = ctx.put(G.fn(6, 1, G.HOST), host.data_ptr(), 2 * MiB, 1, 0)
+        G.check(st, "put")
+        ctx.set_clock(1_005_000_000)
+        assert ctx.tenant_rate(5, 10_000_000) == (8 * MiB * 100, (8 * MiB * 1000 + 19) // 20, False)
+        assert ctx.tenant_rate(5, 1_000_000)[0] == 0
+        assert ctx.tenant_rate(6, 10_000_000) == (2 * MiB * 100, 0, False)
+        assert ctx.tenant_stats(5) == [0, 8 * MiB, 0] and ctx.tenant_stats(6) == [0, 2 * MiB, 0]
+        ctx.set_clock(None)
+        ctx.free(G.fn(5, 1, G.HOST), oid)
+        ctx.free(G.fn(6, 1, G.HOST), oid2)
+    finally:
+        ctx.close()

@@ -259,3 +259,25 @@ def test_alg1_planner_bad_arguments():
         p.close()
     with pytest.raises(G.GrouterError):
         G.Paths([[0] * 40 for _ in range(40)], 8)
+
+
+def test_tenant_rate_monitor_host():
+    """grouter_tenant_rate (L197) on a planner-only context: no dispatch yet,
+    so rates are 0; Rate_least follows the closed form of L195 (R43) once an
+    SLO is declared (same arithmetic as the oracle's slo.rate_least);
+    windows outside [1 ms, 10 s] are rejected."""
+    from oracle import slo as oslo
+    ctx = G.Ctx(G.config_from_calib(C.b200_hgx(2), flags=G.PLAN_ONLY))
+    try:
+        assert ctx.tenant_rate(7, 10_000_000) == (0, 0, False)
+        G.check(ctx.set_tenant_slo(7, 38_535_168, 50_000_000, 0), "slo")
+        r, least, bl = ctx.tenant_rate(7, 10_000_000)
+        assert (r, bl) == (0, False)
+        assert least == oslo.rate_least(38_535_168, 50_000_000, 0) == 770_703_360
+        G.check(ctx.set_tenant_slo(8, 1000, 3_000_000_000, 1), "slo")
+        assert ctx.tenant_rate(8, 10_000_000)[1] == oslo.rate_least(1000, 3_000_000_000, 1) == 334
+        for bad in (999_999, 10_000_000_001):
+            with pytest.raises(G.GrouterError):
+                ctx.tenant_rate(7, bad)
+    finally:
+        ctx.close()

@@ -73,6 +73,8 @@ def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8), slos=None, h2d_Bps=None)
     start.wait()
     t0 = time.perf_counter()
     time.sleep(seconds)
+    # the library's real-time rate monitor (L197) over the last second, while backlogged
+    monitor = [ctx.tenant_rate(100 + t, 1_000_000_000) for t in range(T)]
     stop[0] = True
     for th in ths:
         th.join()
@@ -85,7 +87,10 @@ def cfg4(seconds=3.0, weights=(1, 1, 2, 2, 4, 4, 8, 8), slos=None, h2d_Bps=None)
             "aggregate_GBps": round(tot, 2), "share_error": [round(e, 3) for e in err],
             "max_share_error": round(max(err), 3) if err else None,
             "p50_ms": [round(pct(l, 50) * 1e3, 2) if l else None for l in lat],
-            "p99_ms": [round(pct(l, 99) * 1e3, 2) if l else None for l in lat]}
+            "p99_ms": [round(pct(l, 99) * 1e3, 2) if l else None for l in lat],
+            "monitor_GBps": [round(r / 1e9, 2) for r, _, _ in monitor],
+            "monitor_rate_least_GBps": [round(q / 1e9, 3) for _, q, _ in monitor],
+            "monitor_at_least": [r >= q for r, q, _ in monitor]}
 
 
 def cfg4_slo(seconds=3.0, bw=53e9):
@@ -182,6 +187,8 @@ def cfg2(seconds=3.0, outstanding=4):
     start.wait()
     t0 = time.perf_counter()
     time.sleep(seconds)
+    # the library's real-time rate monitor (L197) over the last second, while backlogged
+    monitor = [ctx.tenant_rate(100 + t, 1_000_000_000) for t in range(T)]
     stop[0] = True
     for th in ths:
         th.join()
