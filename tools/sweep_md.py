@@ -1,4 +1,4 @@
-"""Renders a tools/sweep.py JSON document as the profiles/<round>_sweep.md table.
+"""Renders a tests/harness/sweep.py JSON document as the profiles/<round>_sweep.md table.
 usage: python tools/sweep_md.py SWEEP_JSON > profiles/rNN_sweep.md"""
 import json
 import sys
@@ -23,7 +23,7 @@ def cell(name, n, gbps=True, p99=False):
 
 
 print(f"# cfg3 sweep ({d['gpu']}, host cores {d['host_cores']})\n")
-print("`python tools/sweep.py` (device-event timing for get_into / baselines on the consumer stream; host clock "
+print("`python tests/harness/sweep.py` (device-event timing for get_into / baselines on the consumer stream; host clock "
       "for blocking cFn calls and the zero-copy get+release pair). Latency mode: one call at a time on an idle "
       "GPU, so every number includes the library's host path. GB/s = payload bytes / p50. Probe of this GPU: "
       f"{json.dumps(d['probe'])}\n")
