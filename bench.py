@@ -266,7 +266,8 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
     host = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
     out = {"probe_h2d_GBps": [round(b / 1e9, 2) for b in calib["h2d_Bps"]],
            "probe_nvl_GBps": round(calib["nvl_Bps"] / 1e9, 1)}
-    for name, flags in (("direct", G.NO_MULTIPATH), ("striped", 0)):
+    # TA off (GROUTER_NO_TOPOLOGY, Fig. 16): GPUs behind one PCIe switch both stage (R48)
+    for name, flags in (("direct", G.NO_MULTIPATH), ("striped", 0), ("striped_no_topology", G.NO_TOPOLOGY)):
         ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, flags=flags,
                                         pool_cap=[G.UNLIMITED] * world, pool_floor_bytes=64 << 20))
         st, routes = ctx.route_set(0)
@@ -283,6 +284,7 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
         out[name] = {"routes": routes, "GBps": round(nbytes / min(ts) / 1e9, 2)}
         ctx.close()
     out["speedup"] = round(out["striped"]["GBps"] / out["direct"]["GBps"], 2)
+    out["topology_gain"] = round(out["striped"]["GBps"] / out["striped_no_topology"]["GBps"], 2)
     # gFn-host (L178, Fig. 5a): a GPU0 object read into host memory by a cFn,
     # direct D2H vs striped over R(0) (GROUTER_D2H_MULTIPATH)
     src = torch.empty(nbytes, dtype=torch.uint8, device="cuda:0")

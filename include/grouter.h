@@ -69,6 +69,9 @@ extern "C" {
                                       ... millisecond-level"): every object / lease is its own
                                       cudaMalloc, freed by cudaFree once its GPU work completed;
                                       accounting, caps and eviction unchanged; no IPC export  */
+#define GROUTER_NO_TOPOLOGY   0x400u/* ablation "TA off" (Fig. 16; L131, L178): route sets
+                                      ignore shared PCIe uplinks (every GPU its own uplink group,
+                                      DESIGN.md R48), so GPUs behind one switch both stage data */
 #define GROUTER_STRIPED_MIGRATION 0x100u /* spills leave over R(src) on the route GPUs' D2H
                                       engines (the gFn-host plan, L178), restores come back over
                                       R(d) with relays like a fetch (L178, L366 "parallel PCIe

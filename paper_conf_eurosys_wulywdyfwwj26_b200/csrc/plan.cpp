@@ -26,6 +26,11 @@ static std::vector<std::vector<int>> build_groups(const grouter_config &c) {
     a = find(a), b = find(b);
     if (a != b) parent[std::max(a, b)] = std::min(a, b);
   };
+  if (c.flags & GROUTER_NO_TOPOLOGY) {  // ablation "TA off" (R48): no shared uplinks assumed
+    std::vector<std::vector<int>> g(n);
+    for (int i = 0; i < n; ++i) g[i] = {i};
+    return g;
+  }
   bool explicit_ids = false;
   for (int i = 0; i < n; ++i) explicit_ids |= c.uplink_group[i] >= 0;
   for (int i = 0; i < n; ++i)

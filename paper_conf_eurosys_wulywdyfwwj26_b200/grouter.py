@@ -29,6 +29,7 @@ REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE, RESTORE, D2H_MULTIPATH 
     0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40, 0x80
 STRIPED_MIGRATION = 0x100   # spills over R(src), restores over R(d) (R47)
 NO_POOL = 0x200             # ablation "ES off" (Fig. 16): cudaMalloc/cudaFree per object
+NO_TOPOLOGY = 0x400         # ablation "TA off" (Fig. 16): route sets ignore shared PCIe uplinks (R48)
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]

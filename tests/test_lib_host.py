@@ -281,3 +281,22 @@ def test_tenant_rate_monitor_host():
                 ctx.tenant_rate(7, bad)
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("topo", ["pairs8", "fig5a"])
+def test_no_topology_flag(topo):
+    """Ablation "TA off" (GROUTER_NO_TOPOLOGY, Fig. 16; reading R48): the
+    library's route sets and plans equal the oracle's on the same calibration
+    with every GPU its own uplink group -- so on the L178 example GPU2 (the
+    switch partner of GPU1) becomes a route of GPU1, which TA excludes."""
+    calib = {"pairs8": C.b200_hgx(8), "fig5a": C.fig5a()}[topo]
+    n = calib["n_gpus"]
+    flat = dict(calib, uplink_groups=[[i] for i in range(n)])
+    with _plan_ctx(calib, flags=G.NO_TOPOLOGY) as ctx:
+        for d in range(n):
+            assert ctx.route_set(d)[1] == oroutes.route_set(flat, d) == list(range(n)[d:d + 1]) + \
+                [r for r in range(n) if r != d]
+            for size in (2**21 + 1, 38_535_168, 1 << 30):
+                assert ctx.plan(-1, d, size)[1] == _oracle_plan(flat, -1, d, size)
+    with _plan_ctx(calib) as ctx:                      # TA on: the switch partner is excluded
+        assert 1 not in ctx.route_set(0)[1]
