@@ -72,6 +72,10 @@ extern "C" {
 #define GROUTER_NO_TOPOLOGY   0x400u/* ablation "TA off" (Fig. 16; L131, L178): route sets
                                       ignore shared PCIe uplinks (every GPU its own uplink group,
                                       DESIGN.md R48), so GPUs behind one switch both stage data */
+#define GROUTER_HOST_CENTRIC  0x800u/* ablation "UF off" (Fig. 16) / the host-centric data
+                                      passing of L90: a GPU -> other-GPU copy goes through
+                                      pinned host memory (D2H on the source's engine, then H2D on
+                                      the destination's), one path each (R49)        */
 #define GROUTER_STRIPED_MIGRATION 0x100u /* spills leave over R(src) on the route GPUs' D2H
                                       engines (the gFn-host plan, L178), restores come back over
                                       R(d) with relays like a fetch (L178, L366 "parallel PCIe

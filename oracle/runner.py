@@ -29,10 +29,11 @@ def digest(b: np.ndarray) -> str:
 def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
         multipath: bool = True, keep_bytes: bool = False, restore: bool = False,
         pool_floor: int | None = None, targets: bool = False, d2h_multipath: bool = False,
-        striped_migration: bool = False) -> dict:
+        striped_migration: bool = False, host_centric: bool = False) -> dict:
     kw = {} if pool_floor is None else {"pool_floor": pool_floor}
     kw["d2h_multipath"] = d2h_multipath
     kw["striped_migration"] = striped_migration
+    kw["host_centric"] = host_centric
     orc = Oracle(calib, host_store_bytes=host_store_bytes, pool_cap=pool_cap,
                  multipath=multipath, restore=restore, **kw)
     recs = []

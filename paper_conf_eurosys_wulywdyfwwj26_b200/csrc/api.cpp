@@ -320,6 +320,29 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
                        cudaStream_t caller = nullptr, int caller_logical = -1, bool caller_dep = false,
                        bool *direct = nullptr, bool pool_src = true) {
   const uint64_t tst = hprof().on ? now_ns() : 0;
+  if ((c->cfg.flags & GROUTER_HOST_CENTRIC) && src_loc >= 0 && dst_loc >= 0 && src_loc != dst_loc && n &&
+      pool_src) {
+    // ablation "UF off" (R49): GPU -> pinned host bounce -> GPU, one engine per hop
+    const uint64_t ch = charge(n);
+    uint8_t *bounce = host_alloc(c, ch);  // library-internal: not charged to the host store (R49)
+    std::vector<grouter_chunk> p1, p2;
+    c->planner.plan_single(n, src_loc, p1);
+    XferRef x1 = new_xfer(c, tenant, p1);
+    x1->deps = std::move(deps);
+    enqueue_plan(c, x1, p1, SK_D2H, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)bounce, GROUTER_HOST);
+    c->planner.plan_single(n, dst_loc, p2);
+    XferRef x2 = new_xfer(c, tenant, p2);
+    done_fences(x1, x2->deps);
+    enqueue_plan(c, x2, p2, SK_H2D, (uint64_t)(uintptr_t)bounce, (uint64_t)(uintptr_t)dst, dst_loc);
+    if (caller && caller_dep) x2->deps.push_back(signal(c, caller, c->dev[caller_logical].phys));
+    Fences f;
+    done_fences(x2, f);
+    host_free(c, bounce, ch, std::move(f));
+    if (direct) *direct = false;
+    if (hprof().on) hprof().t[4] += now_ns() - tst;
+    pump(c, false);
+    return x2;
+  }
   std::vector<grouter_chunk> plan;
   if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
   else c->planner.plan(src_loc, dst_loc, n, plan, pool_src);

@@ -30,6 +30,7 @@ REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE, RESTORE, D2H_MULTIPATH 
 STRIPED_MIGRATION = 0x100   # spills over R(src), restores over R(d) (R47)
 NO_POOL = 0x200             # ablation "ES off" (Fig. 16): cudaMalloc/cudaFree per object
 NO_TOPOLOGY = 0x400         # ablation "TA off" (Fig. 16): route sets ignore shared PCIe uplinks (R48)
+HOST_CENTRIC = 0x800        # ablation "UF off" (Fig. 16): GPU -> GPU copies through host memory (R49)
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]

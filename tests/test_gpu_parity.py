@@ -156,11 +156,14 @@ def _copy_exactly_once(tma, src_off, dst_off):
 
 
 # ------------------------------------------------------------------ trace parity
-def _both(ops, calib, replay=True, keep=True, restore=False, d2h=False, striped=False, **kw):
+def _both(ops, calib, replay=True, keep=True, restore=False, d2h=False, striped=False, host_centric=False,
+          **kw):
     orc = orun.run(ops, calib, host_store_bytes=kw.get("host_store_bytes", 1 << 30),
                    pool_cap=kw.get("pool_cap"), keep_bytes=keep, restore=restore,
                    pool_floor=kw.get("pool_floor", 64 << 20), targets=kw.get("targets", False),
-                   d2h_multipath=d2h, striped_migration=striped)
+                   d2h_multipath=d2h, striped_migration=striped, host_centric=host_centric)
+    if host_centric:
+        kw["flags"] = kw.get("flags", 0) | G.HOST_CENTRIC
     if restore:
         kw["flags"] = kw.get("flags", 0) | G.RESTORE
     if d2h:
@@ -574,3 +577,22 @@ def test_tenant_rate_monitor_fixed_clock():
         ctx.free(G.fn(6, 1, G.HOST), oid2)
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_host_centric(seed, replay):
+    """Ablation "UF off" (GROUTER_HOST_CENTRIC, R49): every GPU -> other-GPU
+    copy goes D2H into a pinned bounce and H2D out of it; statuses,
+    placements, victims, accounting and bytes equal the oracle's, and so do
+    the per-engine and per-tenant byte totals (the D2D bytes now cross PCIe
+    twice)."""
+    rng = random.Random(9300 + seed)
+    k = rng.choice([2, 3])
+    calib = C.virtual(k)
+    ops = T.random_trace(rng, k, n_ops=100, max_n=9 * MiB, run_seed=seed)
+    caps = [rng.choice([16, 64]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, host_store_bytes=64 * MiB, pool_cap=caps,
+                         host_centric=True)
+    compare(orc, lib_out, check_dispatch=replay)
+    _link_bytes_equal(orc, lib_out, k)

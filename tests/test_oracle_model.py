@@ -322,3 +322,27 @@ def test_tenant_bytes_closed_form():
     assert orc.link_bytes[("h2d", 0)] > 0 and orc.link_bytes[("h2d", 1)] > 0
     assert orc.link_bytes[("h2d", 0)] + orc.link_bytes[("h2d", 1)] == n1
     del g1
+
+
+def test_host_centric_closed_form():
+    """Ablation "UF off" (host_centric, R49; the host-centric passing of L90):
+    a GPU0 object read by a GPU1 function crosses PCIe twice -- n bytes D2H
+    on GPU0's engine, n bytes H2D on GPU1's, no SM copy -- while a same-GPU
+    get stays zero copy and a same-GPU get_into stays an SM copy; bytes and
+    every decision are those of the GPU-centric run."""
+    n = 5 * MiB + 77
+    b = T.Builder(4)
+    o = b.put(T.fn(1, 1, 0), n)                       # gFn put by copy on GPU0 (SM copy)
+    g1 = b.get_into(T.fn(1, 2, 1), o)                  # GPU1 reads it
+    z = b.get(T.fn(1, 3, 0), o)                        # co-located: zero copy
+    b.release(T.fn(1, 3, 0), z)
+    b.get_into(T.fn(1, 4, 0), o)                       # same GPU into caller memory
+    calib = C.b200_hgx(2, shared_pairs=False)
+    hc = runner.run(b.ops, calib, host_centric=True, keep_bytes=True)
+    gc = runner.run(b.ops, calib, keep_bytes=True)
+    assert hc["oracle"].tenant_bytes == {(1, "copy"): 2 * n, (1, "d2h"): n, (1, "h2d"): n}
+    assert gc["oracle"].tenant_bytes == {(1, "copy"): 3 * n}
+    assert hc["oracle"].link_bytes == {("d2h", 0): n, ("h2d", 1): n}
+    for x, y in zip(hc["records"], gc["records"]):
+        assert (x["status"], x.get("digest"), x["used"]) == (y["status"], y.get("digest"), y["used"])
+    del g1

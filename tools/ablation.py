@@ -10,8 +10,12 @@ Configurations (flags of the same library):
                routes share the one physical link, so this isolates the
                relay hop's cost, not PCIe parallelism)
   -ES-BH    -- both
-(TA, topology-aware scheduling, is the identity on NVSwitch (R11); UF, the
-unified framework, is what the library is.)
+  -UF       -- unified framework off: GROUTER_HOST_CENTRIC, a GPU -> other-GPU
+               copy goes through pinned host memory (D2H then H2D, R49; the
+               host-centric passing of L90)
+  -ES-BH-UF -- all three
+(TA, topology-aware scheduling, only changes route sets where GPUs share a
+PCIe switch: measured by bench.py N>1 `striped_no_topology`.)
 
 Workloads per request (full sizes of BASELINE.json configs 1 and 5):
   cfg1: cFn put of 38,535,168 B from pinned host (hint GPU0, consumers=1) ->
@@ -112,7 +116,8 @@ def run(flags, workload, reqs):
 
 def main():
     G.load()
-    cfgs = {"full": 0, "-ES": G.NO_POOL, "-BH": G.NO_MULTIPATH, "-ES-BH": G.NO_POOL | G.NO_MULTIPATH}
+    cfgs = {"full": 0, "-ES": G.NO_POOL, "-BH": G.NO_MULTIPATH, "-ES-BH": G.NO_POOL | G.NO_MULTIPATH,
+            "-UF": G.HOST_CENTRIC, "-ES-BH-UF": G.NO_POOL | G.NO_MULTIPATH | G.HOST_CENTRIC}
     out = {"gpu": torch.cuda.get_device_name(0), "what": __doc__.split("\n")[0], "results": {}}
     for wl, reqs in (("cfg1", 100), ("cfg5", 12)):
         for name, fl in cfgs.items():
