@@ -387,11 +387,12 @@ def test_full_size_cfg2_cfg5():
 
 
 def _link_bytes_equal(orc, lib_out, n):
-    """Per-engine byte totals: the library's link_bytes[1] (H2D) and [2]
-    (D2H) per logical GPU equal the oracle's scheduled + migration plans."""
+    """Per-engine byte totals: the library's link_bytes[0] (SM-copy egress),
+    [1] (H2D) and [2] (D2H) per logical GPU equal the oracle's scheduled +
+    migration plans (each copy crosses exactly once: L165, Fig. 4)."""
     lb = orc["oracle"].link_bytes
     st = lib_out["stats"]
-    for kind, row in (("h2d", 1), ("d2h", 2)):
+    for kind, row in (("copy", 0), ("h2d", 1), ("d2h", 2)):
         got = [st.link_bytes[row][g] for g in range(n)]
         exp = [lb.get((kind, g), 0) for g in range(n)]
         assert got == exp, (kind, got, exp)

@@ -48,7 +48,7 @@ def test_fig5a_spill_uses_l178_routes():
     assert sum(d2h.values()) == n and sum(h2d.values()) == n
     # single path: everything on the GPU's own engines
     ref = _spill_and_restore(C.fig5a(), n, striped=False)["oracle"].link_bytes
-    assert ref == {("d2h", 0): n, ("h2d", 0): n}
+    assert ref == {("copy", 0): n, ("d2h", 0): n, ("h2d", 0): n}     # copy: the gFn's by-copy put
 
 
 def test_migration_plans_tile_the_object():
@@ -74,7 +74,7 @@ def test_one_route_reduces_to_single_path():
         b.pool_limit(0, 0)
         b.pool_limit(0, 1 << 40)
         lb = runner.run(b.ops, calib, restore=True, striped_migration=True, multipath=mp)["oracle"].link_bytes
-        assert lb == {("d2h", 0): 9 * MiB, ("h2d", 0): 9 * MiB}
+        assert lb == {("copy", 0): 9 * MiB, ("d2h", 0): 9 * MiB, ("h2d", 0): 9 * MiB}
 
 
 @pytest.mark.parametrize("seed", range(10))

@@ -342,7 +342,8 @@ def test_host_centric_closed_form():
     gc = runner.run(b.ops, calib, keep_bytes=True)
     assert hc["oracle"].tenant_bytes == {(1, "copy"): 2 * n, (1, "d2h"): n, (1, "h2d"): n}
     assert gc["oracle"].tenant_bytes == {(1, "copy"): 3 * n}
-    assert hc["oracle"].link_bytes == {("d2h", 0): n, ("h2d", 1): n}
+    assert hc["oracle"].link_bytes == {("copy", 0): 2 * n, ("d2h", 0): n, ("h2d", 1): n}
+    assert gc["oracle"].link_bytes == {("copy", 0): 3 * n}       # each copy crosses once (L165)
     for x, y in zip(hc["records"], gc["records"]):
         assert (x["status"], x.get("digest"), x["used"]) == (y["status"], y.get("digest"), y["used"])
     del g1
