@@ -669,8 +669,23 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
       return fail(GROUTER_ENOMEM, "get: lease does not fit after eviction");
     uint8_t *lease = storage(c, d, ch);
     bool direct = false;
-    XferRef x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false,
-                               blocking ? nullptr : (cudaStream_t)stream, d, false, &direct);
+    XferRef x;
+    try {
+      x = start_transfer(c, fn->workflow_id, o.loc, d, n, o.ptr, lease, o.ready, false,
+                         blocking ? nullptr : (cudaStream_t)stream, d, false, &direct);
+    } catch (const Error &e) {
+      if (e.st == GROUTER_ECUDA) throw;  // sticky: the context is unusable anyway
+      // nothing was enqueued: give the lease back before reporting (e.g. a
+      // host-centric bounce that does not fit, R49)
+      if (d == GROUTER_HOST) {
+        c->host_used -= ch;
+        host_free(c, lease, ch, Fences{});
+      } else {
+        c->dev[d].used -= ch;
+        dev_free(c, d, lease, ch, Fences{});
+      }
+      throw;
+    }
     Fences done;
     done_fences(x, done);
     if (o.readers.size() > 8) prune(o.readers);

@@ -597,3 +597,31 @@ def test_random_traces_host_centric(seed, replay):
                          host_centric=True)
     compare(orc, lib_out, check_dispatch=replay)
     _link_bytes_equal(orc, lib_out, k)
+
+
+def test_host_centric_bounce_too_large_is_enomem():
+    """UF off (R49) with an object larger than the pinned host arena: the
+    cross-GPU get fails with ENOMEM and gives its lease back (pool accounting
+    returns to the object alone); the same-GPU get still works."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=8 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    pool_floor_bytes=16 * MiB, flags=G.HOST_CENTRIC))
+    try:
+        n = 96 * MiB                     # > the 2 H + 64 MiB physical arena (80 MiB)
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 5, 0, 0))
+        torch.cuda.synchronize()
+        st, oid = ctx.put(G.fn(1, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        used0 = [ctx.stats().used[g] for g in range(2)]
+        st, ptr, nn = ctx.get(G.fn(1, 2, 1), oid, 0)
+        assert st == G.ENOMEM
+        assert [ctx.stats().used[g] for g in range(2)] == used0
+        st, ptr, nn = ctx.get(G.fn(1, 3, 0), oid, 0)       # co-located: zero copy
+        G.check(st, "get")
+        st, bad, _ = G.test_verify(ptr, n, 5, 0, 0)
+        assert bad == 0
+        G.check(ctx.release(G.fn(1, 3, 0), oid, ptr, 0), "release")
+        G.check(ctx.free(G.fn(1, 1, 0), oid), "free")
+    finally:
+        ctx.close()
