@@ -398,7 +398,77 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
         out["d2d_error"] = f"{type(e).__name__}: {e}"[:300]
     finally:
         ctx.close()
+    out["d2d_sweep"] = measure_d2d_sweep(world, G, calib, devs)
     return out
+
+
+def measure_d2d_sweep(world, G, calib, devs, sizes=(4096, 65536, 1 << 20, 16 << 20, 38_535_168, 64 << 20,
+                                                     256 << 20, 1 << 30)):
+    """cfg3 (i) at N >= 2 (the metric's "latency & GB/s vs size"): a gFn on
+    GPU1 get_into's an object resident on GPU0 (GPU0's SM copy pushes it over
+    NVLink), per size: p50/p99 of single calls on an idle pair (CUDA events on
+    the consumer stream, host path included) and back-to-back GB/s; beside it
+    cudaMemcpyPeerAsync on the same buffers.  Byte-verified per size."""
+    import torch
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * world,
+                                    pool_floor_bytes=64 << 20))
+    res = []
+    try:
+        s1 = torch.cuda.Stream(device=f"cuda:{devs[1]}")
+        for n in sizes:
+            reps = 40 if n <= (64 << 20) else 10
+            src = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[0]}")
+            G.check(G.test_fill(src.data_ptr(), n, 4242, 0, 0))
+            torch.cuda.synchronize(devs[0])
+            oids = []
+            for _ in range(2):
+                st, oid = ctx.put(G.fn(9, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+                G.check(st, "put")
+                oids.append(oid)
+            ctx.sync()
+            dst = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[1]}") for _ in range(2)]
+            f1 = G.fn(9, 2, 1)
+            for i in range(3):
+                G.check(ctx.get_into(f1, oids[i % 2], dst[i % 2].data_ptr(), n, s1.cuda_stream)[0], "get_into")
+            s1.synchronize()
+            st, bad, _ = G.test_verify(dst[0].data_ptr(), n, 4242, 0, 0)
+            assert st == 0 and bad == 0, f"d2d sweep {n}: {bad} bytes differ"
+            lat = []
+            for i in range(reps):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(s1)
+                ctx.get_into(f1, oids[i % 2], dst[i % 2].data_ptr(), n, s1.cuda_stream)
+                b.record(s1)
+                b.synchronize()
+                lat.append(a.elapsed_time(b) * 1e3)
+            lat.sort()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s1)
+            for i in range(reps):
+                ctx.get_into(f1, oids[i % 2], dst[i % 2].data_ptr(), n, s1.cuda_stream)
+            b.record(s1)
+            b.synchronize()
+            tput = n * reps / (a.elapsed_time(b) / 1e3) / 1e9
+            with torch.cuda.stream(s1):                    # baseline: cudaMemcpyPeerAsync (copy engine)
+                a.record(s1)
+                for i in range(reps):
+                    dst[i % 2].copy_(src, non_blocking=True)
+                b.record(s1)
+            b.synchronize()
+            base = n * reps / (a.elapsed_time(b) / 1e3) / 1e9
+            res.append({"bytes": n, "p50_us": round(lat[len(lat) // 2], 2),
+                        "p99_us": round(lat[min(len(lat) - 1, -(-len(lat) * 99 // 100) - 1)], 2),
+                        "GBps": round(tput, 1), "frac_of_770": round(tput / 770.0, 3),
+                        "memcpy_peer_GBps": round(base, 1)})
+            for oid in oids:
+                ctx.free(G.fn(9, 1, 0), oid)
+            del src, dst
+            torch.cuda.empty_cache()
+    except Exception as e:  # reported, never fatal for the line
+        res.append({"error": f"{type(e).__name__}: {e}"[:300]})
+    finally:
+        ctx.close()
+    return res
 
 
 def nccl_ring_baseline(world, rank, dev, n, per_step, steps):

@@ -538,9 +538,22 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
       bool pageable = from == GROUTER_HOST && is_pageable(src);
       if (hp.on) p2 = now_ns();
       bool direct = false;
-      XferRef x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr, Fences{},
-                                 pageable, blocking ? nullptr : (cudaStream_t)stream, from, true,
-                                 &direct, /*pool_src=*/false);  // the caller's buffer
+      XferRef x;
+      try {
+        x = start_transfer(c, fn->workflow_id, from, home, n, (const uint8_t *)src, ptr, Fences{}, pageable,
+                           blocking ? nullptr : (cudaStream_t)stream, from, true, &direct,
+                           /*pool_src=*/false);  // the caller's buffer
+      } catch (const Error &e) {
+        if (e.st == GROUTER_ECUDA) throw;  // sticky: the context is unusable anyway
+        if (home == GROUTER_HOST) {        // nothing was enqueued: give the storage back
+          c->host_used -= ch;
+          host_free(c, ptr, ch, Fences{});
+        } else {
+          c->dev[home].used -= ch;
+          dev_free(c, home, ptr, ch, Fences{});
+        }
+        throw;
+      }
       done_fences(x, done);
       o.ready = done;
       if (!blocking && !direct) order_after(c, g, (cudaStream_t)stream, done);
