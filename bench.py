@@ -155,6 +155,9 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ multi-rank plumbing (gloo-tested)
+CPU_GROUP = [None]   # gloo group for waits that must not occupy the GPUs (set in main)
+
+
 def peer_of(rank: int, world: int) -> int:
     """cfg1 at N GPUs: the object produced on GPU r+1 is consumed on GPU r
     (a ring of disjoint producer->consumer pairs: every GPU's NVLink egress
@@ -755,7 +758,10 @@ def run_gpu(args, rank, world, local_rank):
             th.join(args.multipath_timeout)
             stuck = th.is_alive()
             multipath = box.get("r") or {"error": f"timed out after {args.multipath_timeout:.0f} s"}
-        barrier() if not stuck else dist.barrier()
+        # the other ranks wait on a CPU (gloo) barrier: an NCCL barrier would keep
+        # a spinning all-reduce kernel resident on their GPUs, and rank 0's
+        # copies there would only run in time slices against it
+        dist.barrier(group=CPU_GROUP[0])
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -863,6 +869,7 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
         else:
             dist.init_process_group(backend)
+        CPU_GROUP[0] = dist.new_group(backend="gloo")   # GPU-free waits (rank 0's node-wide probe)
     run_gpu(args, rank, world, local_rank)
     if world > 1:
         import torch.distributed as dist
