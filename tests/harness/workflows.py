@@ -187,8 +187,6 @@ def cfg2(seconds=3.0, outstanding=4):
     start.wait()
     t0 = time.perf_counter()
     time.sleep(seconds)
-    # the library's real-time rate monitor (L197) over the last second, while backlogged
-    monitor = [ctx.tenant_rate(100 + t, 1_000_000_000) for t in range(T)]
     stop[0] = True
     for th in ths:
         th.join()
