@@ -27,7 +27,7 @@ from synth.payload import payload  # noqa: E402
 MiB = 1 << 20
 K = 3          # logical GPUs
 THREADS = 8
-OPS = 100
+OPS = int(__import__("os").environ.get("GR_STRESS_OPS", "100"))
 
 
 def _consume(ctx, t, wf, item, rng, streams, dev):
