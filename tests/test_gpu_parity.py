@@ -220,14 +220,18 @@ def test_random_traces_replay(seed):
     compare(orc, lib_out)
 
 
-@pytest.mark.parametrize("seed", range(4))
+SOAK = int(__import__("os").environ.get("GR_SOAK_SEEDS", "4"))   # more seeds / longer traces on demand
+
+
+@pytest.mark.parametrize("seed", range(SOAK))
 def test_random_traces_realtime(seed):
     """Real-time mode (daemon + inline dispatch, <= 2 rounds in flight): same
-    bytes, statuses, placements and victims; dispatch order is not compared."""
+    bytes, statuses, placements and victims; dispatch order is not compared.
+    GR_SOAK_SEEDS=N runs N seeds with traces 4x longer from seed 4 on."""
     rng = random.Random(2000 + seed)
     k = rng.choice([2, 3])
     calib = C.virtual(k)
-    ops = T.random_trace(rng, k, n_ops=120, max_n=5 * MiB, run_seed=seed)
+    ops = T.random_trace(rng, k, n_ops=120 if seed < 4 else 480, max_n=5 * MiB, run_seed=seed)
     caps = [rng.choice([8, 16, 64]) * MiB for _ in range(k)]
     orc, lib_out = _both(ops, calib, replay=False, host_store_bytes=48 * MiB, pool_cap=caps)
     compare(orc, lib_out, check_dispatch=False)
