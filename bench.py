@@ -826,7 +826,10 @@ def run_gpu(args, rank, world, local_rank):
     if stuck:   # a measurement thread still owns the GPUs: leave without teardown
         sys.stdout.flush()
         os._exit(0)
-    ctx.close()
+    try:
+        ctx.close()
+    except Exception as e:  # the line is out; a teardown failure must not fail the run
+        print(f"[bench] teardown: {e}", file=sys.stderr, flush=True)
 
 
 def main():
@@ -873,7 +876,10 @@ def main():
     run_gpu(args, rank, world, local_rank)
     if world > 1:
         import torch.distributed as dist
-        dist.destroy_process_group()
+        try:
+            dist.destroy_process_group()
+        except Exception as e:
+            print(f"[bench] destroy_process_group: {e}", file=sys.stderr, flush=True)
 
 
 if __name__ == "__main__":

@@ -1083,7 +1083,10 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   // L2 before the PDL wait (38.5 MB get_into back to back: 13.2 us with ws1,
   // 11.8 us with wv8 + prefetch); GROUTER_COPY_TMA forces the ticketed bulk
   // ring (tma8) for every aligned round
-  if (v < 0) v = tma ? 3 : (aligned && total >= (96ull << 20)) ? 16 : 14;
+  // (peer rounds -- NVLink push/pull -- keep the LD/ST engine: TMA bulk copies
+  // to and from peer mappings were never measured on a multi-GPU box here)
+  const bool local_round = (p.flags & kFlagLocalDst) && (p.flags & kFlagLocalSrc);
+  if (v < 0) v = tma ? 3 : (aligned && local_round && total >= (96ull << 20)) ? 16 : 14;
   // a user buffer at an odd address (a tensor view, a by-copy put of a host
   // structure): the warp-strided engines would fall back to byte copies;
   // the tiled LD/ST engine keeps 16 B accesses with its co-aligned and
