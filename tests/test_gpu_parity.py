@@ -629,3 +629,31 @@ def test_host_centric_bounce_too_large_is_enomem():
         G.check(ctx.free(G.fn(1, 1, 0), oid), "free")
     finally:
         ctx.close()
+
+
+def test_tenant_rate_backlog_flag():
+    """Replay mode holds dispatch until grouter_flush: a device caller's
+    transfer is queued, so its tenant reads backlogged with nothing dispatched
+    yet; after the flush the bytes are counted and the backlog is gone."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    flags=G.REPLAY))
+    try:
+        n = 6 * MiB
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        s = torch.cuda.Stream()
+        ctx.set_clock(2_000_000_000)
+        st, oid = ctx.put(G.fn(3, 1, 0), src.data_ptr(), n, G.NOHINT, 0, s.cuda_stream)
+        G.check(st, "put")
+        st, _ = ctx.get_into(G.fn(3, 2, 1), oid, src.data_ptr(), n, s.cuda_stream)
+        G.check(st, "get_into")
+        r, least, bl = ctx.tenant_rate(3, 10_000_000)
+        assert bl and r == 0
+        G.check(ctx.flush(), "flush")
+        r, least, bl = ctx.tenant_rate(3, 10_000_000)
+        assert not bl and r == 2 * n * 100          # put by copy + D2D copy, both SM copies
+        assert ctx.tenant_stats(3) == [2 * n, 0, 0]
+        ctx.set_clock(None)
+        G.check(ctx.sync(), "sync")
+    finally:
+        ctx.close()
