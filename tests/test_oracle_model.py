@@ -347,3 +347,29 @@ def test_host_centric_closed_form():
     for x, y in zip(hc["records"], gc["records"]):
         assert (x["status"], x.get("digest"), x["used"]) == (y["status"], y.get("digest"), y["used"])
     del g1
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_host_centric_changes_engines_only(seed):
+    """On random traces the host-centric ablation (R49) changes which engines
+    move the bytes and nothing else: statuses, placements, victims, pool
+    usage and every delivered byte equal the GPU-centric run; per tenant, the
+    SM-copy bytes it loses reappear exactly once on the D2H and once on the
+    H2D engines."""
+    rng = random.Random(800 + seed)
+    n = rng.choice([2, 3, 4])
+    calib = C.b200_hgx(n, shared_pairs=False)
+    ops = T.random_trace(rng, n, n_ops=150, max_n=7 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16, 64]) * MiB for _ in range(n)]
+    kw = dict(host_store_bytes=1 << 30, pool_cap=caps)
+    a = runner.run(ops, calib, **kw)
+    b = runner.run(ops, calib, host_centric=True, **kw)
+    for x, y in zip(a["records"], b["records"]):
+        for k in ("status", "oid", "where", "victims", "used", "host_used", "digest"):
+            assert x.get(k) == y.get(k), (x["i"], k)
+    ta, tb = a["oracle"].tenant_bytes, b["oracle"].tenant_bytes
+    for wf in {k[0] for k in list(ta) + list(tb)}:
+        moved = ta.get((wf, "copy"), 0) - tb.get((wf, "copy"), 0)
+        assert moved >= 0
+        assert tb.get((wf, "d2h"), 0) - ta.get((wf, "d2h"), 0) == moved
+        assert tb.get((wf, "h2d"), 0) - ta.get((wf, "h2d"), 0) == moved
