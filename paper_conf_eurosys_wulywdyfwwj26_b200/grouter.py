@@ -281,7 +281,6 @@ class Ctx:
         h = C.c_void_p()
         check(self.lib.grouter_init(C.byref(cfg), C.byref(h)), "grouter_init")
         self.h = h
-        self._n = C.c_uint64(0)
 
     def close(self):
         if self.h:
@@ -321,7 +320,7 @@ class Ctx:
         return st, (p.value or 0), n.value
 
     def get_into(self, f, oid: int, dst: int, cap: int, stream=0):
-        n = self._n
+        n = C.c_uint64(0)   # per call: one context serves several client threads
         st = self.lib.grouter_get_into(self.h, C.byref(f), oid, dst or None, cap, stream or None,
                                        C.byref(n))
         return st, n.value
