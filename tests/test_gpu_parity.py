@@ -657,3 +657,30 @@ def test_tenant_rate_backlog_flag():
         G.check(ctx.sync(), "sync")
     finally:
         ctx.close()
+
+
+def test_probe_calibration():
+    """grouter_probe (a5, L178/L131/L271): on one B200 the solo pinned H2D rate
+    is a PCIe Gen5 x16 figure, per-copy and first-chunk costs are positive,
+    and two logical GPUs on the same physical device are detected as ONE
+    uplink group (their concurrent H2D sum is not above the solo rate: the
+    L131 shared-switch test), so neither is a route of the other; a context
+    built from the probe moves bytes exactly."""
+    cal = G.probe([0, 0], 64 * MiB)
+    assert all(20e9 < b < 80e9 for b in cal["h2d_Bps"]), cal["h2d_Bps"]
+    assert all(a > 0 for a in cal["h2d_alpha_ps"]) and all(p > 0 for p in cal["h2d_phi_ps"])
+    pair = cal["h2d_pair_Bps"][0][1]
+    assert 100 * pair <= 115 * max(cal["h2d_Bps"]), (pair, cal["h2d_Bps"])
+    ctx = G.Ctx(G.config_from_calib(cal, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2))
+    try:
+        assert ctx.route_set(0)[1] == [0] and ctx.route_set(1)[1] == [1]
+        n = 3 * MiB + 5
+        host = torch.from_numpy(payload(31, n)).pin_memory()
+        st, oid = ctx.put(G.fn(1, 1, G.HOST), host.data_ptr(), n, 1, 0)
+        G.check(st, "put")
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(ctx.get_into(G.fn(1, 2, 0), oid, dst.data_ptr(), n, 0)[0], "get_into")
+        torch.cuda.synchronize()
+        assert np.array_equal(dst.cpu().numpy(), payload(31, n))
+    finally:
+        ctx.close()
