@@ -157,6 +157,8 @@ typedef struct {
   uint64_t timed_bytes;                  /* sum of the bytes they moved         */
   uint64_t restore_count, restore_bytes; /* host -> home GPU restores (L260)    */
   uint64_t pool_target[GROUTER_MAX_GPUS]; /* histogram-driven pool size (R44)    */
+  uint64_t tracked_functions;            /* pool-sizing histograms held (R50)   */
+  uint64_t tracked_tenants;              /* per-tenant counters held (R50)      */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
@@ -321,7 +323,9 @@ grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
  * bytes[k] = bytes of workflow_id's chunks the servers of kind k dispatched
  * so far (0 = SM-copy egress, 1 = H2D engines, 2 = D2H engines), summed over
  * GPUs.  Scheduled transfers only: spills and restores are unscheduled
- * (R41, R42).  An unknown tenant reads zeros.  EINVAL on null arguments. */
+ * (R41, R42).  An unknown tenant reads zeros.  EINVAL on null arguments.
+ * Once more than 65,536 tenants are tracked, tenants idle for over 10 s are
+ * forgotten (they read zeros again). */
 grouter_status grouter_tenant_stats(grouter_ctx *ctx, uint32_t workflow_id, uint64_t bytes[3]);
 /* Real-time rate monitor (L197: GROUTER "monitors the transfer rate of each
  * function in real time, ensuring that it does not fall below Rate_least"):

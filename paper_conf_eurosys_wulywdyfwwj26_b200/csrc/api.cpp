@@ -66,8 +66,10 @@ Obj *lookup_live(grouter_ctx *c, grouter_oid oid) {
 // placement (L250-L256, R44).
 static void resident_add(grouter_ctx *c, const Obj &o, int64_t delta) {
   if (o.loc < 0) return;
-  uint64_t &r = c->resident[std::make_tuple(o.wf, o.fid, o.loc)];
+  const auto key = std::make_tuple(o.wf, o.fid, o.loc);
+  uint64_t &r = c->resident[key];
   r += delta;
+  if (r == 0) c->resident.erase(key);  // an absent entry reads 0: bounded for short-lived workflows
 }
 
 static void observe(grouter_ctx *c, const Obj &o) {
@@ -1161,6 +1163,8 @@ grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
   }
   out->host_used = c->host_used;
   out->host_cap = c->host_cap;
+  out->tracked_functions = c->hists.size();
+  out->tracked_tenants = c->tenant_bytes.size();
   return GROUTER_OK;
 }
 

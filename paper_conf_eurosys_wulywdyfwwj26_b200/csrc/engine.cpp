@@ -884,6 +884,28 @@ static void daemon_main(grouter_ctx *c) {
           DeviceGuard g(d.phys);
           d.pool.heap.reclaim();
           if (i == 0 && !c->nopool_pending.empty()) nopool_sweep(c, false);
+          for (Server *sv : {&d.copy, &d.h2d, &d.d2h}) sv->sched.prune();  // idle tenants (no-op for dispatch)
+          if (i == 0) {  // rate-monitor records older than its 10 s horizon; bounded per-tenant counters
+            const uint64_t tn = c->clock_fixed ? c->clock_ns : now_ns();
+            for (auto it = c->tenant_log.begin(); it != c->tenant_log.end();)
+              if (it->second.empty() || it->second.back().first + 10000000000ull < tn) it = c->tenant_log.erase(it);
+              else ++it;
+            // pool-sizing histograms (R44, R50): with more than 4096 functions
+            // tracked, forget those whose window closed over 60 s ago (one
+            // workflow id per request would otherwise grow the table -- and
+            // this tick's pool_target scan -- without bound)
+            if (c->hists.size() > 4096)
+              for (auto it = c->hists.begin(); it != c->hists.end();) {
+                const FuncHist &h = it->second;
+                if (!h.arrivals.empty() && !h.active(tn) && h.arrivals.back() + h.r_window() + 60000000000ull < tn)
+                  it = c->hists.erase(it);
+                else ++it;
+              }
+            if (c->tenant_bytes.size() > (1u << 16))
+              for (auto it = c->tenant_bytes.begin(); it != c->tenant_bytes.end();)
+                if (!c->tenant_log.count(it->first)) it = c->tenant_bytes.erase(it);
+                else ++it;
+          }
           // histogram-driven size (L250-L256, R44): pre-warm one segment per
           // tick toward the target, trim back to max(used, target)
           const uint64_t tgt = pool_target(c, (int)i);

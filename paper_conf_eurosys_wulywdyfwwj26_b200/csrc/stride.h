@@ -36,6 +36,15 @@ struct Stride {
   }
   bool empty() const { return backlog_items == 0; }
 
+  // Forgets idle tenants whose pass is <= V: a tenant that re-joins later gets
+  // max(pass, V) = V either way, so this changes no dispatch decision; it
+  // bounds the table when workflows are short-lived (one id per request).
+  void prune() {
+    for (auto it = tenants.begin(); it != tenants.end();)
+      if (it->second.q.empty() && it->second.pass <= V) it = tenants.erase(it);
+      else ++it;
+  }
+
   // Pops the next batch into `out`; returns the tenant id, or UINT32_MAX if idle.
   template <class WeightFn>
   uint32_t dispatch(WeightFn weight_of, std::vector<Item> &out, uint64_t *bytes_out = nullptr,

@@ -78,7 +78,8 @@ class grouter_stats_t(C.Structure):
         ("link_bytes", (C.c_uint64 * MAX_GPUS) * 3), ("kernel_launches", C.c_uint64),
         ("rounds", C.c_uint64), ("timed_launches", C.c_uint64), ("timed_ns", C.c_uint64),
         ("timed_bytes", C.c_uint64), ("restore_count", C.c_uint64), ("restore_bytes", C.c_uint64),
-        ("pool_target", C.c_uint64 * MAX_GPUS),
+        ("pool_target", C.c_uint64 * MAX_GPUS), ("tracked_functions", C.c_uint64),
+        ("tracked_tenants", C.c_uint64),
     ]
 
 

@@ -684,3 +684,36 @@ def test_probe_calibration():
         assert np.array_equal(dst.cpu().numpy(), payload(31, n))
     finally:
         ctx.close()
+
+
+def test_short_lived_workflows_bounded_state():
+    """R50: one workflow id per request (as in the cfg2 harness) must not grow
+    the library's per-function state without bound: 5000 one-shot workflows
+    leave 5000 pool-sizing histograms; once their windows have been closed
+    for over 60 s (library clock fixed and advanced), the daemon's tick
+    forgets them -- and the pool-sizing target falls back to the floor."""
+    import time as _t
+    calib = C.virtual(1)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED],
+                                    pool_floor_bytes=16 * MiB))
+    try:
+        ctx.set_clock(1_000_000_000)
+        for wf in range(1000, 6000):
+            f = G.fn(wf, 1, 0)
+            st, buf, oid = ctx.alloc(f, 4096, G.NOHINT, 1)
+            G.check(st, "alloc")
+            G.check(ctx.seal(f, oid, 0), "seal")
+            st, ptr, n = ctx.get(f, oid, 0)
+            G.check(st, "get")
+            G.check(ctx.release(f, oid, ptr, 0), "release")
+        st = ctx.stats()
+        assert st.tracked_functions == 5000 and st.used[0] == 0
+        ctx.set_clock(1_000_000_000 + 120_000_000_000)
+        deadline = _t.time() + 5
+        while ctx.stats().tracked_functions and _t.time() < deadline:
+            _t.sleep(0.05)
+        assert ctx.stats().tracked_functions == 0
+        assert ctx.pool_target(0) == 16 * MiB
+        ctx.set_clock(None)
+    finally:
+        ctx.close()
