@@ -285,6 +285,20 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
             if r:
                 ts.append(dt)
         out[name] = {"routes": routes, "GBps": round(nbytes / min(ts) / 1e9, 2)}
+        # cfg3 (iii) vs size: blocking cFn put GB/s (best of 3) at 4 MiB .. 256 MiB
+        sweep = {}
+        for sz in (4 << 20, 38_535_168, 64 << 20, 256 << 20):
+            best = None
+            for r in range(4):
+                t0 = time.perf_counter()
+                st, oid = ctx.put(f, host.data_ptr(), sz, 0, 0)
+                G.check(st, "put")
+                dt = time.perf_counter() - t0
+                ctx.free(f, oid)
+                if r:
+                    best = dt if best is None else min(best, dt)
+            sweep[sz] = round(sz / best / 1e9, 2)
+        out[name]["GBps_by_size"] = sweep
         ctx.close()
     out["speedup"] = round(out["striped"]["GBps"] / out["direct"]["GBps"], 2)
     out["topology_gain"] = round(out["striped"]["GBps"] / out["striped_no_topology"]["GBps"], 2)
