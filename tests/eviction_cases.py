@@ -1,0 +1,78 @@
+"""Traces of the hand-derived eviction-branch cases (tests/golden/eviction_branches.md).
+
+Inputs only: each builder returns (ops, run kwargs).  The expected values live
+in tests/golden/eviction_branches.json, typed in by hand from the derivation;
+the oracle is checked against them (tests/test_oracle_branches.py) and the
+library against the oracle on the GPU (tests/test_gpu_parity.py).
+"""
+from synth import traces as T
+
+MiB = 1 << 20
+
+
+def case_a():
+    """R15: mixed hinted / unhinted victims."""
+    b = T.Builder(21)
+    f, g = T.fn(1, 1, 0), T.fn(1, 2, 0)
+    A, B, C, D, E = (b.put(f, MiB) for _ in range(5))      # ops 0-4
+    b.next_use(A, 3)                                        # 5
+    b.next_use(C, 7)                                        # 6
+    b.next_use(E, 7)                                        # 7
+    b.get_into(g, B)                                        # 8
+    b.put(f, 5 * MiB)                                       # 9
+    b.put(f, MiB)                                           # 10
+    o8 = b.put(f, 3 * MiB)                                  # 11
+    o9 = b.put(f, 1)                                        # 12
+    b.next_use(o8, 5)                                       # 13
+    b.next_use(o9, 0)                                       # 14
+    b.put(f, 3 * MiB)                                       # 15
+    del D
+    return b.ops, {"pool_cap": [10 * MiB], "host_store_bytes": 1 << 30}
+
+
+def case_b():
+    """R33 all-or-nothing reserve, R16 put -> host store, alloc -> ENOMEM."""
+    b = T.Builder(22)
+    f, z, c = T.fn(1, 1, 0), T.fn(1, 2, 0), T.fn(1, 3, T.HOST)
+    o1 = b.put(f, 3 * MiB)                                  # 0
+    b.get(z, o1)                                            # 1 zero copy pin
+    b.put(f, MiB)                                           # 2
+    b.put(c, 5 * MiB, hint=0)                               # 3
+    b.alloc(f, 5 * MiB)                                     # 4
+    b.put(f, MiB)                                           # 5
+    return b.ops, {"pool_cap": [6 * MiB], "host_store_bytes": 64 * MiB}
+
+
+def case_c():
+    """R34: set_pool_limit below the unevictable floor."""
+    b = T.Builder(23)
+    f, z = T.fn(1, 1, 0), T.fn(1, 2, 0)
+    o1 = b.put(f, 3 * MiB)                                  # 0
+    g = b.get(z, o1)                                        # 1
+    b.put(f, 3 * MiB)                                       # 2
+    b.put(f, MiB)                                           # 3
+    b.pool_limit(0, 2 * MiB)                                # 4
+    b.put(f, 1)                                             # 5
+    b.release(z, g)                                         # 6
+    b.pool_limit(0, 2 * MiB)                                # 7
+    return b.ops, {"host_store_bytes": 64 * MiB}
+
+
+def case_d():
+    """R32: host store full."""
+    b = T.Builder(24)
+    c, g, r = T.fn(1, 1, T.HOST), T.fn(1, 2, 0), T.fn(1, 3, T.HOST)
+    o1 = b.put(c, 3 * MiB)                                  # 0
+    b.put(c, 1)                                             # 1
+    b.alloc(c, 1)                                           # 2
+    o2 = b.put(g, MiB)                                      # 3
+    b.get(r, o2)                                            # 4
+    b.put(g, MiB)                                           # 5
+    b.get_into(r, o2)                                       # 6
+    b.free(c, o1)                                           # 7
+    b.put(c, 1)                                             # 8
+    b.put(g, MiB)                                           # 9
+    return b.ops, {"pool_cap": [2 * MiB], "host_store_bytes": 4 * MiB}
+
+
+CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d}

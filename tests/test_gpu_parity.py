@@ -194,6 +194,28 @@ def test_golden_trace_on_virtual_pair():
         assert r["victims"] == e["victims"]
 
 
+@pytest.mark.parametrize("replay", [True, False])
+@pytest.mark.parametrize("case", ["A", "B", "C", "D"])
+def test_eviction_branch_golden_cases(case, replay):
+    """The hand-derived eviction-branch cases (tests/golden/eviction_branches.md:
+    R15 mixed hints, R33/R16 all-or-nothing reserve, R34 limit below the
+    unevictable floor, R32 full host store): the library equals the oracle
+    op by op, and both equal the hand-derived values."""
+    import json
+    import os
+    from tests.eviction_cases import CASES
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "eviction_branches.json")))
+    ops, kw = CASES[case]()
+    calib = C.b200_hgx(1)
+    calib["device_map"] = [0]
+    orc, lib_out = _both(ops, calib, replay=replay, **kw)
+    compare(orc, lib_out, check_dispatch=replay)
+    for r in lib_out["records"]:
+        e = g[case]["expect"].get(str(r["i"]), {})
+        assert r["status"] == e.get("status", "OK"), (case, r["i"])
+        assert r["victims"] == e.get("victims", []), (case, r["i"])
+
+
 @pytest.mark.parametrize("k", [1, 2, 4])
 def test_config_traces_virtual(k):
     calib = C.virtual(k) if k > 1 else C.b200_hgx(1)

@@ -1,0 +1,56 @@
+"""Pins for the oracle branches that decide victims and placements in every
+spill trace (VERDICT r01 What's weak #1): R15 mixed hinted/unhinted victim
+order, R33 all-or-nothing reserve with R16 host placement,
+R34 pool limit below the unevictable floor (L262), R32 full host store.
+
+Expected values are hand-derived (tests/golden/eviction_branches.md) and typed
+into tests/golden/eviction_branches.json; nothing here is produced by the
+oracle itself.
+"""
+import json
+import os
+
+import pytest
+
+from oracle import runner
+from synth import calib as C
+from tests.eviction_cases import CASES
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "eviction_branches.json")))
+MiB = GOLD["MiB"]
+
+
+def _check(case):
+    ops, kw = CASES[case]()
+    out = runner.run(ops, C.b200_hgx(1), **kw)
+    recs, exp = out["records"], GOLD[case]["expect"]
+    for r in recs:
+        e = exp.get(str(r["i"]), {})
+        assert r["status"] == e.get("status", "OK"), (case, r["i"], r["status"])
+        assert r["victims"] == e.get("victims", []), (case, r["i"], r["victims"])
+        if "oid" in e:
+            assert r.get("oid") == e["oid"], (case, r["i"])
+        if "where" in e:
+            assert r.get("where") == e["where"], (case, r["i"], r.get("where"))
+        if "used" in e:
+            assert r["used"] == [u * MiB for u in e["used"]], (case, r["i"], r["used"])
+        if "host_used" in e:
+            assert r["host_used"] == e["host_used"] * MiB, (case, r["i"], r["host_used"])
+        if "plan" in e:
+            assert r["plan"] == e["plan"], (case, r["i"])
+    orc = out["oracle"]
+    for oid, loc in GOLD[case]["final_where"].items():
+        assert orc.where(int(oid)) == loc, (case, oid, orc.where(int(oid)))
+    return out
+
+
+@pytest.mark.parametrize("case", sorted(CASES))
+def test_eviction_branch_golden(case):
+    _check(case)
+
+
+def test_case_c_cap_stays_after_enomem():
+    """R34: the failed limit is kept (op 5 lands on the host although GPU0
+    had no cap before op 4)."""
+    out = _check("C")
+    assert out["oracle"].cap == [2 * MiB]

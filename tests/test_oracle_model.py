@@ -120,12 +120,33 @@ def test_config_traces_drain_to_zero(n_gpus):
 
 
 def test_cfg5_spills_under_limit():
-    out = runner.run(T.cfg5(2, requests=4, limit_frac=0.1, scale=64, layers=4), C.b200_hgx(2))
-    spilled = [v for r in out["records"] for v in r["victims"]]
-    assert spilled, "10% pool limit must force migration"
-    # queue-aware: nothing of request 0 (queue head, pos 0) is evicted while
-    # later requests' data is resident
+    """cfg5 at a 10% limit: migration happens, and it is queue-aware (L258):
+    no object of request q is evicted while an object of a later request
+    q' > q (further back in the queue) stays resident on stage A's GPU.
+    Checked by replaying each prefix of the trace and reading the oracle's
+    resident set right after every op that evicted something."""
+    ops = T.cfg5(2, requests=4, limit_frac=0.1, scale=64, layers=4)
+    calib = C.b200_hgx(2)
+    out = runner.run(ops, calib)
     assert out["records"][0]["op"] == "pool_limit"
+    req_of = {}                                     # oid -> request (queue position)
+    for r in out["records"]:
+        if r["op"] == "alloc" and r["status"] == "OK":
+            req_of[r["oid"]] = ops[r["i"]]["fn"]["wf"] - 500
+    evicting = [r for r in out["records"] if r["victims"]]
+    assert evicting, "10% pool limit must force migration"
+    later_seen = 0
+    for r in evicting:
+        orc = runner.run(ops[:r["i"] + 1], calib)["oracle"]
+        resident = [o for o in orc.objects.values() if o.loc == 0 and o.state == "SEALED"]
+        for v in r["victims"]:
+            q = req_of[v]
+            later = [o.oid for o in resident if req_of.get(o.oid, -1) > q]
+            assert not later, (r["i"], v, q, later)
+            later_seen += q > 0
+    # request 0's objects were spilled only while request 0 itself was being
+    # produced; once request 1 exists, spills come from the queue tail
+    assert later_seen > 0
 
 
 @pytest.mark.parametrize("seed", range(40))
@@ -159,7 +180,8 @@ def test_capacity_never_exceeded_by_reserve():
         res = runner.run(ops, C.b200_hgx(2), host_store_bytes=1 << 30, pool_cap=caps)
         for r in res["records"]:
             assert all(u <= c for u, c in zip(r["used"], caps)), r
-        assert any(r["victims"] for r in res["records"]) or True
+        # the caps are small enough that every trace really evicts (the bound is exercised)
+        assert any(r["victims"] for r in res["records"]), s
 
 
 # ---------------------------------------------------------------- proactive restore
