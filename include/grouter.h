@@ -16,7 +16,7 @@
  *                queue-aware migration to pinned host memory.
  *   L260         data no longer needed is removed promptly.
  *   L394 §7      every access is authenticated by function id + workflow id.
- * Readings of silent/ambiguous points (R1-R31) are listed in DESIGN.md.
+ * Readings of silent/ambiguous points (R1 onward) are listed in DESIGN.md §3.
  *
  * Conventions (all calls):
  *   - Every call returns a grouter_status; on error outputs are untouched
@@ -136,7 +136,7 @@ typedef struct {
   uint64_t pool_cap_bytes[GROUTER_MAX_GPUS]; /* explicit cap; 0 = auto         */
   uint64_t host_store_bytes;   /* pinned host store H, default 1 GiB          */
   uint64_t round_bytes;        /* SM-copy dispatch horizon, default 64 MiB    */
-  uint32_t copy_ctas_per_sm;   /* SM copy kernel CTAs per SM, default 2       */
+  uint32_t copy_ctas_per_sm;   /* SM copy kernel CTAs per SM cap, default 4   */
   uint32_t flags;              /* GROUTER_* flags                              */
 } grouter_config;
 
@@ -406,6 +406,9 @@ void grouter_sched_free(grouter_sched *s);
 const char *grouter_strerror(grouter_status st);
 /* Text of the last error seen by this thread (thread-local). */
 const char *grouter_last_error(void);
+/* SHA-256 (hex) of the sources this library was built from (static string);
+ * the Python binding refuses a library whose hash differs from the tree. */
+const char *grouter_build_hash(void);
 
 #ifdef __cplusplus
 }

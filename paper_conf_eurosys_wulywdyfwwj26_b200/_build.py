@@ -3,9 +3,16 @@
 cudart is linked statically and only ``grouter_*`` symbols are exported
 (linker version script), so the library never interposes on, or is
 interposed by, the CUDA runtime PyTorch ships.
+
+The library carries the SHA-256 of the sources it was built from (every
+input file's bytes, and the compile flags): ``grouter_build_hash()`` returns
+it and the marker ``GROUTER_SRC_HASH=<hex>`` is in the binary.  A build is
+reused only when that hash equals the current sources' (not by mtime), and
+``grouter.load()`` refuses a library whose hash differs from the tree.
 """
 from __future__ import annotations
 
+import hashlib
 import os
 import subprocess
 import sys
@@ -27,11 +34,33 @@ def _inputs():
     return files
 
 
+COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC"]
+
+
+def source_hash() -> str:
+    """SHA-256 over every input file (name + bytes) and the compile flags."""
+    h = hashlib.sha256()
+    h.update(" ".join(COMMON + ARCH).encode())
+    for f in _inputs():
+        h.update(os.path.basename(f).encode() + b"\0")
+        with open(f, "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
+
+
+def built_hash(path: str = LIB) -> str | None:
+    """The source hash embedded in a built library (marker scan, no dlopen)."""
+    if not os.path.exists(path):
+        return None
+    data = open(path, "rb").read()
+    k = data.find(b"GROUTER_SRC_HASH=")
+    if k < 0:
+        return None
+    return data[k + 17:k + 17 + 64].decode("ascii", "replace")
+
+
 def up_to_date() -> bool:
-    if not os.path.exists(LIB):
-        return False
-    t = os.path.getmtime(LIB)
-    return all(os.path.getmtime(f) <= t for f in _inputs())
+    return built_hash() == source_hash()
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -39,8 +68,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     objdir = os.path.join(HERE, "build")
     os.makedirs(objdir, exist_ok=True)
-    common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
-              "-I", os.path.join(ROOT, "include")] + ARCH
+    digest = source_hash()
+    common = COMMON + ["-I", os.path.join(ROOT, "include"), f"-DGROUTER_SRC_HASH=\"{digest}\""] + ARCH
     objs = []
     procs = []
     for src in SOURCES:

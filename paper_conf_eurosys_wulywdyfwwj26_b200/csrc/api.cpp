@@ -386,6 +386,13 @@ const char *grouter_strerror(grouter_status st) {
 
 const char *grouter_last_error(void) { return gr::last_error(); }
 
+#ifndef GROUTER_SRC_HASH
+#define GROUTER_SRC_HASH "unknown"
+#endif
+// the marker is found by a byte scan of the .so (_build.built_hash), no dlopen needed
+static const char kSrcHashMarker[] __attribute__((used)) = "GROUTER_SRC_HASH=" GROUTER_SRC_HASH;
+const char *grouter_build_hash(void) { return kSrcHashMarker + 17; }
+
 void grouter_config_default(grouter_config *cfg) {
   if (!cfg) return;
   std::memset(cfg, 0, sizeof(*cfg));

@@ -165,6 +165,7 @@ SIGNATURES = {
     "grouter_sched_free": (None, [_P]),
     "grouter_strerror": (C.c_char_p, [_ST]),
     "grouter_last_error": (C.c_char_p, []),
+    "grouter_build_hash": (C.c_char_p, []),
     "grouter_test_fill": (_ST, [_P, _U64, _U64, _U64, _P]),
     "grouter_test_verify": (_ST, [_P, _U64, _U64, _U64, _P, C.POINTER(_U64), C.POINTER(_U64)]),
     "grouter_test_launch_cost": (_ST, [C.c_int, C.c_int, C.c_int, _P, C.POINTER(C.c_double)]),
@@ -185,11 +186,21 @@ def load(build_if_missing: bool = False):
             raise ImportError(f"{LIB_PATH} not built; run __graft_entry__.build()")
         from . import _build
         _build.build()
+    from . import _build
+    want = _build.source_hash()
+    if _build.built_hash() != want:
+        if not build_if_missing:
+            raise ImportError(f"{LIB_PATH} was built from other sources (hash {_build.built_hash()} != "
+                              f"{want}); run __graft_entry__.build()")
+        _build.build()
     lib = C.CDLL(LIB_PATH)
     for name, (res, args) in SIGNATURES.items():
         f = getattr(lib, name)
         f.restype = res
         f.argtypes = args
+    got = lib.grouter_build_hash().decode()
+    if got != want:   # the file changed between the scan and dlopen
+        raise ImportError(f"{LIB_PATH}: grouter_build_hash() {got} != source hash {want}")
     _lib = lib
     return lib
 
