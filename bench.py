@@ -851,8 +851,8 @@ def run_gpu(args, rank, world, local_rank):
                        "bytes": N_BYTES,
                        "parallelism": f"replicas x{world} (workflows co-located per GPU, no collective)",
                        "l2": "inputs larger than L2: 20 resident 38.5 MB objects, 8 rotating bindings",
-                       "copy_kernel": os.environ.get("GR_COPY", "tma8" if args.tma else "wv8")
-                       + f" (256-bit LD/ST, L2 prefetch of {os.environ.get('GR_PF', '1')} unit/warp before the PDL wait)"
+                       "copy_kernel": os.environ.get("GR_COPY", "tmas4" if args.tma else "wv8")
+                       + " (256-bit LD/ST, L2 prefetch of 1 unit/warp before the PDL wait)"
                        + f", {args.ctas} CTA/SM cap"},
             "gbps": value * N_BYTES / 1e9,
             "host_us_per_request": host_us,

@@ -80,6 +80,11 @@ extern "C" {
                                       engines (the gFn-host plan, L178), restores come back over
                                       R(d) with relays like a fetch (L178, L366 "parallel PCIe
                                       transfers ... mitigate the overhead"); R47      */
+#define GROUTER_FORCE_REMOTE  0x1000u/* TEST ONLY: every copy-kernel round is launched as if its
+                                      sources and destinations were on another GPU (the NVLink
+                                      branch: system-scope fences, no L2 prefetch, no TMA bulk
+                                      engine, completion published in-kernel), so one-GPU test
+                                      boxes execute the code a physical peer transfer runs    */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;
@@ -159,6 +164,9 @@ typedef struct {
   uint64_t pool_target[GROUTER_MAX_GPUS]; /* histogram-driven pool size (R44)    */
   uint64_t tracked_functions;            /* pool-sizing histograms held (R50)   */
   uint64_t tracked_tenants;              /* per-tenant counters held (R50)      */
+  uint64_t peer_launches;                /* copy-kernel launches on the peer (NVLink) branch:
+                                            a destination or source outside the launching GPU,
+                                            or GROUTER_FORCE_REMOTE                         */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
@@ -227,13 +235,17 @@ grouter_status grouter_free(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid 
 
 /* ------------------------------------------------------------ cross-process handoff
  * L167 (1) / L269: GROUTER maps stored data into the address space of the
- * consuming function through CUDA IPC.  Pool pages are CUDA VMM allocations
- * exported as POSIX file descriptors; the descriptor below is plain bytes
- * that any channel can carry; the file descriptors themselves travel over
- * an abstract Unix socket served by the exporting context. */
-#define GROUTER_IPC_MAX_SEGS 8
+ * consuming function through CUDA IPC; L394: only pre-mapped storage is
+ * exposed, and access is authenticated.  An exported object lives in its own
+ * CUDA VMM allocation (exactly its 2 MiB pages; R52), so an importer
+ * maps that object and nothing else.  The descriptor below is plain bytes that
+ * any channel can carry; it is the capability: the exporting context serves
+ * the allocation's file descriptor over an abstract Unix socket only for a
+ * live export whose random nonce matches, and only to a process of the same
+ * uid (or root). */
+#define GROUTER_IPC_MAX_SEGS 8  /* unused since descriptor version 2 */
 typedef struct {
-  uint32_t magic, version;
+  uint32_t magic, version;        /* 0x47524f55, 2                               */
   int32_t pid;                    /* exporting process                          */
   uint32_t ctx_id;                /* exporting context (socket name)            */
   uint8_t gpu_uuid[16];           /* GPU holding the bytes                      */
@@ -242,16 +254,20 @@ typedef struct {
   grouter_oid oid;                /* exporter-side object id                    */
   uint64_t n;                     /* bytes                                      */
   uint64_t exporter_ptr;          /* object address in the exporter (release)   */
-  uint64_t first_offset;          /* object start within the first segment      */
-  uint32_t n_segs, pad;
-  uint64_t seg_off[GROUTER_IPC_MAX_SEGS];   /* segment offsets in the exporter's pool */
-  uint64_t seg_size[GROUTER_IPC_MAX_SEGS];
+  uint64_t export_id;             /* the exporter's export record               */
+  uint64_t nonce[2];              /* 128-bit random capability                  */
+  uint64_t alloc_bytes;           /* size of the object's own allocation        */
 } grouter_ipc_desc;
 
 /* Exports a sealed object resident on a GPU for use by another process.
- * Blocks until the object's bytes are in place, pins the object like a
- * zero-copy lease and consumes one consumer; the exporter drops the pin
- * with grouter_release(fn, oid, (void*)desc.exporter_ptr, stream). */
+ * Blocks until the object's bytes are in place.  The first export of an
+ * object moves it out of the shared pool into its own allocation (one
+ * same-GPU copy); EBUSY if the object still has zero-copy leases then (their
+ * pointers would dangle).  Pins the object like a zero-copy lease and
+ * consumes one consumer; the exporter drops the pin with
+ * grouter_release(fn, oid, (void*)desc.exporter_ptr, stream).  The export
+ * ends when the object is freed: later imports fail with ENOENT, existing
+ * importer mappings stay valid (the pages live until the importer unmaps). */
 grouter_status grouter_export_ipc(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid,
                                   grouter_ipc_desc *desc);
 /* Imports an exported object as a local, sealed, read-only object owned by
@@ -285,7 +301,10 @@ grouter_status grouter_slo_weights(uint32_t n, const uint32_t *ids, const uint64
                                    const uint64_t *slo_ns, const uint64_t *infer_ns, uint64_t bw_all_Bps,
                                    uint32_t *weights_out);
 
-/* Queue position of the object's next consumer (D8; L258 queue-aware eviction). */
+/* Queue position of the object's next consumer (D8; L258 queue-aware eviction).
+ * CONTROL PLANE: called by the function scheduler that owns the request
+ * queue, not by functions, so it takes no grouter_fn and performs no
+ * workflow check (L394 authenticates the data-path calls). */
 grouter_status grouter_set_next_use(grouter_ctx *ctx, grouter_oid oid, uint64_t queue_pos);
 /* Pool cap of a GPU (GROUTER_UNLIMITED = no cap); evicts at once until used <= cap
  * (L262).  ENOMEM if unevictable data keeps the pool above the cap. */
@@ -315,7 +334,8 @@ grouter_status grouter_route_set(grouter_ctx *ctx, int32_t dst_dev, int32_t *out
  * The background thread pre-maps the pool up to the target (pre-warming)
  * and trims it down to max(used, target) + one 64 MiB segment. */
 grouter_status grouter_pool_target(grouter_ctx *ctx, int32_t dev, uint64_t *target);
-/* Current location of an object: GPU index or GROUTER_HOST. */
+/* Current location of an object: GPU index or GROUTER_HOST.  CONTROL PLANE
+ * (scheduler / introspection): no workflow check, like grouter_set_next_use. */
 grouter_status grouter_where(grouter_ctx *ctx, grouter_oid oid, int32_t *loc);
 grouter_status grouter_stats(grouter_ctx *ctx, grouter_stats_t *out);
 /* Per-tenant share accounting (L193: "data chunks of each function are

@@ -41,7 +41,10 @@ grouter_status fail(grouter_status st, const char *msg) {
   }                                                                           \
   catch (const gr::Error &e) {                                                \
     gr::set_error(e.what());                                                  \
-    if (e.st == GROUTER_ECUDA && (ctx)) (ctx)->sticky_error = true;           \
+    if (e.st == GROUTER_ECUDA && (ctx)) {                                    \
+      (ctx)->sticky_error = true;                                             \
+      (ctx)->submit_cv.notify_all();                                          \
+    }                                                                         \
     return e.st;                                                              \
   }                                                                           \
   catch (const std::exception &e) {                                           \
@@ -268,15 +271,19 @@ void order_after(grouter_ctx *c, Guard &g, cudaStream_t s, const Fences &f) {
         if (!is_submitted(w)) return false;
       return true;
     };
+    // a failed round (sticky error) or a shutdown never submits the rest:
+    // wake up and fail instead of waiting forever (the daemon notifies)
+    auto settled = [&] { return c->sticky_error.load() || c->stop || all_submitted(); };
     if (!all_submitted()) {
       pump(c, false);
       c->cv.notify_one();
       static const bool diag = getenv("GR_DIAG") != nullptr;
       if (!diag) {
-        c->submit_cv.wait(g.lk, all_submitted);
+        if (!c->submit_cv.wait_for(g.lk, std::chrono::seconds(120), settled))
+          throw Error(GROUTER_ECUDA, "timeout waiting for a transfer's submission");
       } else {  // diagnostics: report the servers' state when a submission stalls
         const uint64_t t0 = now_ns();
-        while (!c->submit_cv.wait_for(g.lk, std::chrono::milliseconds(50), all_submitted)) {
+        while (!c->submit_cv.wait_for(g.lk, std::chrono::milliseconds(50), settled)) {
           fprintf(stderr, "[grouter diag] order_after: transfer unsubmitted for %.0f ms\n", (now_ns() - t0) / 1e6);
           const char *kn[] = {"copy", "h2d", "d2h"};
           for (size_t i = 0; i < c->dev.size(); ++i) {
@@ -299,6 +306,8 @@ void order_after(grouter_ctx *c, Guard &g, cudaStream_t s, const Fences &f) {
                       w.producer->deps.size());
         }
       }
+      if (!all_submitted())
+        throw Error(GROUTER_ECUDA, c->stop ? "context shutting down" : "sticky CUDA error; see the first failure");
     }
   }
   caller_wait(c, s, f);
@@ -865,10 +874,14 @@ grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_
   if (c->replay) flush_all(c);
   else pump(c, true);
   host_wait(o.ready);  // the importer sees finished bytes
+  const bool dedicated = !o.n || c->dedicated.count((uint64_t)(uintptr_t)o.ptr);
+  if (!dedicated && o.pins)
+    return fail(GROUTER_EBUSY, "export_ipc: the object has zero-copy leases (export before leasing it)");
+  if (!dedicated) ipc_dedicate(c, o);  // its own VMM allocation: the importer maps only this object (R52)
   ipc_serve_start(c);
   grouter_ipc_desc d{};
   d.magic = 0x47524f55u;
-  d.version = 1;
+  d.version = 2;
   d.pid = (int32_t)getpid();
   d.ctx_id = c->ctx_id;
   cudaDeviceProp prop;
@@ -879,15 +892,9 @@ grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_
   d.oid = oid;
   d.n = o.n;
   d.exporter_ptr = (uint64_t)(uintptr_t)o.ptr;
-  const DevicePool &P = c->dev[o.loc].pool;
-  const uint64_t lo = (uint64_t)(o.ptr - (uint8_t *)P.base), hi = lo + std::max<uint64_t>(o.n, 1);
-  for (auto &sg : P.segs) {
-    if (sg.off + sg.size <= lo || sg.off >= hi) continue;
-    if (d.n_segs == GROUTER_IPC_MAX_SEGS) return fail(GROUTER_EINVAL, "export_ipc: object spans too many segments");
-    if (d.n_segs == 0) d.first_offset = lo - sg.off;
-    d.seg_off[d.n_segs] = sg.off;
-    d.seg_size[d.n_segs] = sg.size;
-    d.n_segs++;
+  if (o.n) {
+    d.export_id = ipc_export_record(c, (uint64_t)(uintptr_t)o.ptr, d.nonce);
+    d.alloc_bytes = charge(o.n);
   }
   o.pins++;  // like a zero-copy lease: released with grouter_release(ptr = exporter_ptr)
   o.last_access = c->seq;
@@ -904,7 +911,7 @@ grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const gr
   c->victims.clear();
   c->restored.clear();
   API_TRY
-  if (!fn || !d || !out || d->magic != 0x47524f55u || d->version != 1 || d->n_segs > GROUTER_IPC_MAX_SEGS)
+  if (!fn || !d || !out || d->magic != 0x47524f55u || d->version != 2 || (d->n && d->alloc_bytes < d->n))
     return fail(GROUTER_EINVAL, "import_ipc: bad descriptor");
   if (!valid_loc(c, fn->device)) return fail(GROUTER_EINVAL, "import_ipc: bad function");
   if (d->workflow_id != fn->workflow_id) return fail(GROUTER_EPERM, "import_ipc: workflow mismatch (L394)");
@@ -937,7 +944,7 @@ grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const gr
   o.fid = fn->function_id;
   o.n = d->n;
   o.loc = GROUTER_REMOTE;
-  o.ptr = d->n ? (uint8_t *)(uintptr_t)(map->va + d->first_offset) : nullptr;
+  o.ptr = d->n ? (uint8_t *)(uintptr_t)map->va : nullptr;
   o.state = OBJ_SEALED;
   o.consumers_left = consumers;
   o.last_access = c->seq;

@@ -168,6 +168,25 @@ struct RemoteMap {
   int phys = -1;   // local CUDA ordinal holding the bytes, -1 if not visible
 };
 
+// An exported object's own VMM allocation (ipc.cpp, R52): the
+// importer can map it and nothing else; it never returns to the pool.
+struct Dedicated {
+  int logical = -1, phys = -1;
+  CUdeviceptr va = 0;
+  uint64_t size = 0;
+  CUmemGenericAllocationHandle h = 0;
+  int fd = -1;                        // POSIX fd of h, created at the first export
+  std::vector<uint64_t> export_ids;   // live exports (grouter_ctx::exports)
+};
+struct ExportRec {
+  uint64_t nonce[2];                  // 128-bit random capability carried by the descriptor
+  uint64_t va;                        // the Dedicated it serves
+};
+struct DedRetire {
+  Dedicated d;
+  Fences f;                           // unmapped once these complete
+};
+
 enum ObjState { OBJ_OPEN, OBJ_SEALED, OBJ_CONSUMED, OBJ_FREED };
 
 struct Obj {
@@ -284,7 +303,10 @@ struct grouter_ctx {
   uint32_t ctx_id = 0;
   int ipc_listen = -1;
   std::thread ipc_thread;
-  std::map<std::pair<int, uint64_t>, int> exported_fds;  // (logical, seg offset) -> fd
+  std::map<uint64_t, gr::Dedicated> dedicated;         // by VA: exported objects' own allocations
+  std::unordered_map<uint64_t, gr::ExportRec> exports;   // live exports by id
+  uint64_t next_export_id = 1;
+  std::vector<gr::DedRetire> ded_retire;                 // freed dedicated allocations
 };
 
 namespace gr {
@@ -323,6 +345,11 @@ void ipc_serve_start(grouter_ctx *c);
 void ipc_shutdown(grouter_ctx *c);
 std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, int local_phys);
 void ipc_unmap(RemoteMap &m);
+void ipc_dedicate(grouter_ctx *c, Obj &o);                       // move into an own allocation
+uint64_t ipc_export_record(grouter_ctx *c, uint64_t va, uint64_t nonce[2]);
+bool ded_free(grouter_ctx *c, uint8_t *p, Fences &&f);          // false: not dedicated
+void ded_sweep(grouter_ctx *c, std::unique_lock<std::mutex> *lk, bool wait);
+void ipc_release_all(grouter_ctx *c);
 // pool.cpp
 uint64_t pool_target(grouter_ctx *c, int logical);   // R44 target at the current clock
 uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len);   // may grow the pool

@@ -383,6 +383,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
   bool local_src = true;  // relay forwards read this GPU's staging ring
   if (!src_override)
     for (auto &it : items) local_src &= it.x->local_src;
+  if (c->cfg.flags & GROUTER_FORCE_REMOTE) local = local_src = false;  // test: the peer branch
   while (i < items.size()) {
     const uint64_t tparams = hprof().on ? now_ns() : 0;
     p->flags = (local ? kFlagLocalDst : 0) | (local_src ? kFlagLocalSrc : 0);
@@ -448,6 +449,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       c->prof.push_back(pr);
     }
     c->stats.kernel_launches++;
+    if (!local) c->stats.peer_launches++;
   }
 }
 
@@ -780,7 +782,8 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     pd.scratch_busy[k].clear();
     // one launch moves the whole transfer: complete it by an event, not words
     static const bool ev_done = !getenv("GR_NO_EVDONE");
-    const bool whole = ev_done && x->submitted_chunks == 0 && items.size() == x->nchunks && x->waiters.empty();
+    const bool whole = ev_done && x->submitted_chunks == 0 && items.size() == x->nchunks && x->waiters.empty() &&
+                       !(c->cfg.flags & GROUTER_FORCE_REMOTE);  // forced remote: in-kernel publish
     bool deferred = false;
     launch_round(c, s, caller, pd.scratch + 2 * k, items, nullptr, whole ? &deferred : nullptr);
     if (deferred) {
@@ -947,10 +950,12 @@ static void daemon_main(grouter_ctx *c) {
                     (unsigned long long)(d.used >> 20), (unsigned long long)(tgt >> 20));
         }
         c->host.heap.reclaim();
+        if (!c->ded_retire.empty()) ded_sweep(c, &lk, false);  // exported objects' own allocations
       }
     } catch (const Error &e) {
       set_error(e.what());
       c->sticky_error = true;
+      c->submit_cv.notify_all();  // callers blocked in order_after fail with ECUDA
     }
     if (backlog && !c->replay) {
       lk.unlock();
@@ -1071,6 +1076,7 @@ void engine_shutdown(grouter_ctx *c) {
     c->stop = true;
   }
   c->cv.notify_all();
+  c->submit_cv.notify_all();
   if (c->daemon.joinable()) c->daemon.join();
   // drain the library's own streams (never the device: a caller stream may be
   // parked on a completion word that will not arrive after an error)
@@ -1117,6 +1123,7 @@ void engine_shutdown(grouter_ctx *c) {
     for (cudaEvent_t e : kv.second->timing_free) cudaEventDestroy(e);
     kv.second->scratch_busy.clear();
   }
+  ipc_release_all(c);  // dedicated (exported) allocations; their fences hold pooled events
   c->prof.clear();
   c->live.clear();
   delete c->params;

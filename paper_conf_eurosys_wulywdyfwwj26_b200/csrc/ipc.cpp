@@ -1,17 +1,26 @@
-// ipc.cpp -- cross-process zero-copy handoff of pool pages.
+// ipc.cpp -- cross-process zero-copy handoff of GPU objects.
 //
 // PAPER.md L167 (1): GROUTER "maps the address into the address space of
 // function via CUDA IPC"; L269: data is allocated "from the local pool and
 // mapped into the address space of functions using CUDA IPC"; L394: only
-// pre-mapped storage is exposed, authenticated by workflow.
+// pre-mapped storage is exposed to functions, and every access is
+// authenticated.
 //
-// Pool segments are CUDA VMM allocations created with
-// CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR.  An exporting context serves the
-// file descriptors of requested segments over an abstract Unix socket
-// ("\0grouter.<pid>.<ctx_id>", SCM_RIGHTS); the importer maps them into a
-// fresh virtual range with access for its GPU.  Same GPU: the importer's
-// pointer aliases the exporter's bytes (zero copy).  Other GPU: the mapping
-// is a peer mapping that the SM copy kernel reads over NVLink.
+// Isolation (R52).  An exported object lives in its OWN CUDA VMM
+// allocation ("dedicated", exactly charge(n) bytes, POSIX-FD exportable):
+// the first export of an object that still sits in a shared pool segment
+// moves its bytes there once (one same-GPU copy) and frees the pool pages;
+// later exports of the object reuse it.  An importer can therefore map the
+// object's pages and nothing else.  The exporting context serves a dedicated
+// allocation's file descriptor over an abstract Unix socket
+// ("\0grouter.<pid>.<ctx_id>", SCM_RIGHTS) only:
+//   * to a peer of the same uid (or root), checked with SO_PEERCRED, and
+//   * for a LIVE export whose 128-bit random nonce, carried in the
+//     descriptor, matches (the descriptor is the capability).
+// A dedicated allocation never returns to the pool: when the exporter frees
+// the object it unmaps its own view and releases its handle, and the physical
+// pages stay alive exactly as long as an importer maps them (VMM reference
+// counting) -- no page an importer still maps is ever reused for other data.
 #include <sys/socket.h>
 #include <sys/un.h>
 #include <unistd.h>
@@ -19,12 +28,14 @@
 #include <atomic>
 #include <cerrno>
 #include <cstring>
+#include <random>
 
 #include "ctx.h"
 
 namespace gr {
 
 static std::atomic<uint32_t> g_ctx_ids{1};
+static constexpr uint32_t kReqMagic = 0x47524958u;  // "GRIX"
 
 static void sock_name(sockaddr_un &a, socklen_t &len, int pid, uint32_t ctx_id) {
   std::memset(&a, 0, sizeof(a));
@@ -36,10 +47,13 @@ static void sock_name(sockaddr_un &a, socklen_t &len, int pid, uint32_t ctx_id) 
 }
 
 struct Req {
-  uint32_t magic, n;
-  int32_t logical;
-  uint32_t pad;
-  uint64_t seg_off[GROUTER_IPC_MAX_SEGS];
+  uint32_t magic, pad;
+  uint64_t export_id;
+  uint64_t nonce[2];
+};
+struct Rsp {
+  uint32_t ok, pad;
+  uint64_t size;
 };
 
 static bool read_full(int fd, void *p, size_t n) {
@@ -53,21 +67,123 @@ static bool read_full(int fd, void *p, size_t n) {
   return true;
 }
 
-// Returns the exported fd of a pool segment (cached); caller holds c->mu.
-static int segment_fd(grouter_ctx *c, int logical, uint64_t seg_off, uint64_t *size) {
-  DevicePool &P = c->dev[logical].pool;
-  for (auto &s : P.segs) {
-    if (s.off != seg_off) continue;
-    *size = s.size;
-    auto key = std::make_pair(logical, seg_off);
-    auto it = c->exported_fds.find(key);
-    if (it != c->exported_fds.end()) return it->second;
-    int fd = -1;
-    GR_CU(drv().memExportToShareableHandle(&fd, s.h, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0));
-    c->exported_fds[key] = fd;
-    return fd;
+static std::vector<CUmemAccessDesc> access_all(grouter_ctx *c) {
+  std::vector<CUmemAccessDesc> ad;
+  for (auto &kv : c->phys) {
+    CUmemAccessDesc x = {};
+    x.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    x.location.id = kv.first;
+    x.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+    ad.push_back(x);
   }
-  return -1;
+  return ad;
+}
+
+static void ded_release(Dedicated &d) {
+  if (d.fd >= 0) ::close(d.fd);
+  d.fd = -1;
+  if (d.va) {
+    drv().memUnmap(d.va, d.size);
+    drv().memAddressFree(d.va, d.size);
+    d.va = 0;
+  }
+  if (d.h) drv().memRelease(d.h);
+  d.h = 0;
+}
+
+// Moves a sealed pool object into its own exportable VMM allocation (once).
+// Caller holds c->mu; the object's bytes are in place (o.ready waited).
+void ipc_dedicate(grouter_ctx *c, Obj &o) {
+  const uint64_t len = charge(o.n);
+  if (!len || c->dedicated.count((uint64_t)(uintptr_t)o.ptr)) return;
+  LogicalDev &D = c->dev[o.loc];
+  DeviceGuard g(D.phys);
+  Dedicated d;
+  d.logical = o.loc;
+  d.phys = D.phys;
+  d.size = len;
+  CUmemAllocationProp prop = {};
+  prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  prop.location.id = D.phys;
+  prop.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  if (drv().memCreate(&d.h, len, &prop, 0) != CUDA_SUCCESS) throw Error(GROUTER_ENOMEM, "export: cuMemCreate failed");
+  try {
+    GR_CU(drv().memAddressReserve(&d.va, len, kPage, 0, 0));
+    GR_CU(drv().memMap(d.va, len, 0, d.h, 0));
+    const std::vector<CUmemAccessDesc> ad = access_all(c);
+    GR_CU(drv().memSetAccess(d.va, len, ad.data(), ad.size()));
+    // one same-GPU copy on the copy server's stream (ordered after its
+    // earlier rounds); export blocks until the bytes are in place anyway
+    GR_CUDA(cudaMemcpyAsync((void *)d.va, o.ptr, o.n, cudaMemcpyDeviceToDevice, D.copy.stream));
+    EventRef e = record(c, D.copy.stream, D.phys);
+    GR_CUDA(cudaEventSynchronize(e->ev));
+  } catch (...) {
+    ded_release(d);
+    throw;
+  }
+  Fences old = std::move(o.readers);
+  for (auto &w : o.ready) old.push_back(w);
+  dev_free(c, o.loc, o.ptr, len, std::move(old));  // the shared pool pages go back
+  o.ready.clear();
+  o.readers.clear();
+  o.ptr = (uint8_t *)(uintptr_t)d.va;
+  c->dedicated.emplace(d.va, d);
+}
+
+// Registers a live export of the dedicated allocation at `va`: returns its id
+// and a fresh 128-bit random nonce.  Caller holds c->mu.
+uint64_t ipc_export_record(grouter_ctx *c, uint64_t va, uint64_t nonce[2]) {
+  Dedicated &d = c->dedicated.at(va);
+  if (d.fd < 0) GR_CU(drv().memExportToShareableHandle(&d.fd, d.h, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0));
+  static thread_local std::random_device rd;  // /dev/urandom (getrandom) on Linux
+  for (int i = 0; i < 2; ++i) nonce[i] = ((uint64_t)rd() << 32) ^ (uint64_t)rd();
+  const uint64_t id = c->next_export_id++;
+  c->exports[id] = ExportRec{{nonce[0], nonce[1]}, va};
+  d.export_ids.push_back(id);
+  return id;
+}
+
+// dev_free for a dedicated allocation: its exports end now (no new imports),
+// its own mapping goes once the object's GPU work is done (ded_sweep).
+// Returns false if p is not a dedicated allocation.  Caller holds c->mu.
+bool ded_free(grouter_ctx *c, uint8_t *p, Fences &&f) {
+  auto it = c->dedicated.find((uint64_t)(uintptr_t)p);
+  if (it == c->dedicated.end()) return false;
+  for (uint64_t id : it->second.export_ids) c->exports.erase(id);
+  it->second.export_ids.clear();
+  c->ded_retire.push_back({it->second, std::move(f)});
+  c->dedicated.erase(it);
+  return true;
+}
+
+// Unmaps and releases retired dedicated allocations whose fences completed.
+// The driver calls run WITHOUT the context lock when `lk` is given (an unmap
+// drains the GPU; the pool trim does the same).
+void ded_sweep(grouter_ctx *c, std::unique_lock<std::mutex> *lk, bool wait) {
+  std::vector<Dedicated> done;
+  size_t w = 0;
+  for (size_t i = 0; i < c->ded_retire.size(); ++i) {
+    DedRetire &r = c->ded_retire[i];
+    bool ok = true;
+    if (wait) host_wait(r.f);
+    else
+      for (auto &x : r.f) ok &= x.done();
+    if (ok) {
+      done.push_back(r.d);
+    } else {
+      if (w != i) c->ded_retire[w] = std::move(c->ded_retire[i]);
+      ++w;
+    }
+  }
+  c->ded_retire.resize(w);
+  if (done.empty()) return;
+  if (lk) lk->unlock();
+  for (auto &d : done) {
+    DeviceGuard g(d.phys);
+    ded_release(d);
+  }
+  if (lk) lk->lock();
 }
 
 static void serve(grouter_ctx *c) {
@@ -78,43 +194,43 @@ static void serve(grouter_ctx *c) {
       return;  // listening socket closed: shutting down
     }
     Req rq;
-    if (read_full(cfd, &rq, sizeof(rq)) && rq.magic == 0x47524950u && rq.n <= GROUTER_IPC_MAX_SEGS) {
-      int fds[GROUTER_IPC_MAX_SEGS];
-      uint64_t sizes[GROUTER_IPC_MAX_SEGS] = {};
-      uint32_t ok = 1;
-      {
-        std::lock_guard<std::mutex> g(c->mu);
-        try {
-          if (rq.logical < 0 || rq.logical >= (int)c->dev.size()) ok = 0;
-          for (uint32_t i = 0; ok && i < rq.n; ++i) {
-            fds[i] = segment_fd(c, rq.logical, rq.seg_off[i], &sizes[i]);
-            if (fds[i] < 0) ok = 0;
-          }
-        } catch (...) {
-          ok = 0;
+    Rsp rsp{0, 0, 0};
+    int fd = -1;
+    ucred cr{};
+    socklen_t crl = sizeof(cr);
+    const bool peer_ok = ::getsockopt(cfd, SOL_SOCKET, SO_PEERCRED, &cr, &crl) == 0 &&
+                         (cr.uid == ::getuid() || cr.uid == 0);
+    if (peer_ok && read_full(cfd, &rq, sizeof(rq)) && rq.magic == kReqMagic) {
+      std::lock_guard<std::mutex> g(c->mu);
+      auto it = c->exports.find(rq.export_id);
+      if (it != c->exports.end()) {
+        const ExportRec &e = it->second;
+        const uint64_t diff = (e.nonce[0] ^ rq.nonce[0]) | (e.nonce[1] ^ rq.nonce[1]);
+        auto d = c->dedicated.find(e.va);
+        if (diff == 0 && d != c->dedicated.end() && d->second.fd >= 0) {
+          rsp.ok = 1;
+          rsp.size = d->second.size;
+          fd = ::dup(d->second.fd);  // sent while the allocation may be retired concurrently
+          if (fd < 0) rsp.ok = 0;
         }
       }
-      struct {
-        uint32_t ok, n;
-        uint64_t sizes[GROUTER_IPC_MAX_SEGS];
-      } rsp{ok, ok ? rq.n : 0, {}};
-      std::memcpy(rsp.sizes, sizes, sizeof(sizes));
-      iovec iov{&rsp, sizeof(rsp)};
-      msghdr m{};
-      m.msg_iov = &iov;
-      m.msg_iovlen = 1;
-      char cbuf[CMSG_SPACE(sizeof(int) * GROUTER_IPC_MAX_SEGS)];
-      if (ok && rq.n) {
-        m.msg_control = cbuf;
-        m.msg_controllen = CMSG_SPACE(sizeof(int) * rq.n);
-        cmsghdr *cm = CMSG_FIRSTHDR(&m);
-        cm->cmsg_level = SOL_SOCKET;
-        cm->cmsg_type = SCM_RIGHTS;
-        cm->cmsg_len = CMSG_LEN(sizeof(int) * rq.n);
-        std::memcpy(CMSG_DATA(cm), fds, sizeof(int) * rq.n);
-      }
-      (void)::sendmsg(cfd, &m, 0);
     }
+    iovec iov{&rsp, sizeof(rsp)};
+    msghdr m{};
+    m.msg_iov = &iov;
+    m.msg_iovlen = 1;
+    char cbuf[CMSG_SPACE(sizeof(int))];
+    if (rsp.ok) {
+      m.msg_control = cbuf;
+      m.msg_controllen = CMSG_SPACE(sizeof(int));
+      cmsghdr *cm = CMSG_FIRSTHDR(&m);
+      cm->cmsg_level = SOL_SOCKET;
+      cm->cmsg_type = SCM_RIGHTS;
+      cm->cmsg_len = CMSG_LEN(sizeof(int));
+      std::memcpy(CMSG_DATA(cm), &fd, sizeof(int));
+    }
+    (void)::sendmsg(cfd, &m, MSG_NOSIGNAL);
+    if (fd >= 0) ::close(fd);
     ::close(cfd);
   }
 }
@@ -135,6 +251,8 @@ void ipc_serve_start(grouter_ctx *c) {
   c->ipc_thread = std::thread(serve, c);
 }
 
+// Stops serving; the context's remaining dedicated allocations are released
+// by the caller's teardown (ipc_release_all).
 void ipc_shutdown(grouter_ctx *c) {
   if (c->ipc_listen >= 0) {
     ::shutdown(c->ipc_listen, SHUT_RDWR);
@@ -142,8 +260,20 @@ void ipc_shutdown(grouter_ctx *c) {
     c->ipc_listen = -1;
   }
   if (c->ipc_thread.joinable()) c->ipc_thread.join();
-  for (auto &kv : c->exported_fds) ::close(kv.second);
-  c->exported_fds.clear();
+  c->exports.clear();
+}
+
+void ipc_release_all(grouter_ctx *c) {
+  for (auto &kv : c->dedicated) {
+    DeviceGuard g(kv.second.phys);
+    ded_release(kv.second);
+  }
+  c->dedicated.clear();
+  for (auto &r : c->ded_retire) {
+    DeviceGuard g(r.d.phys);
+    ded_release(r.d);
+  }
+  c->ded_retire.clear();
 }
 
 std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, int local_phys) {
@@ -157,67 +287,51 @@ std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, in
     throw Error(GROUTER_EINVAL, "ipc: exporter not reachable (process gone or other namespace)");
   }
   Req rq{};
-  rq.magic = 0x47524950u;
-  rq.n = d.n_segs;
-  rq.logical = d.logical;
-  for (uint32_t i = 0; i < d.n_segs; ++i) rq.seg_off[i] = d.seg_off[i];
+  rq.magic = kReqMagic;
+  rq.export_id = d.export_id;
+  rq.nonce[0] = d.nonce[0];
+  rq.nonce[1] = d.nonce[1];
   if (::write(s, &rq, sizeof(rq)) != (ssize_t)sizeof(rq)) {
     ::close(s);
     throw Error(GROUTER_ECUDA, "ipc: request failed");
   }
-  struct {
-    uint32_t ok, n;
-    uint64_t sizes[GROUTER_IPC_MAX_SEGS];
-  } rsp{};
+  Rsp rsp{};
   iovec iov{&rsp, sizeof(rsp)};
   msghdr m{};
   m.msg_iov = &iov;
   m.msg_iovlen = 1;
-  char cbuf[CMSG_SPACE(sizeof(int) * GROUTER_IPC_MAX_SEGS)];
+  char cbuf[CMSG_SPACE(sizeof(int))];
   m.msg_control = cbuf;
   m.msg_controllen = sizeof(cbuf);
   ssize_t r = ::recvmsg(s, &m, MSG_WAITALL);
   ::close(s);
-  if (r != (ssize_t)sizeof(rsp) || !rsp.ok || rsp.n != d.n_segs)
-    throw Error(GROUTER_EINVAL, "ipc: exporter refused the segments");
-  int fds[GROUTER_IPC_MAX_SEGS];
-  cmsghdr *cm = CMSG_FIRSTHDR(&m);
-  if (!cm || cm->cmsg_type != SCM_RIGHTS) throw Error(GROUTER_ECUDA, "ipc: no descriptors received");
-  std::memcpy(fds, CMSG_DATA(cm), sizeof(int) * rsp.n);
+  cmsghdr *cm = (r == (ssize_t)sizeof(rsp) && rsp.ok) ? CMSG_FIRSTHDR(&m) : nullptr;
+  if (!cm || cm->cmsg_type != SCM_RIGHTS)
+    throw Error(GROUTER_ENOENT, "ipc: export refused (freed object, wrong nonce, or another user)");
+  int fd = -1;
+  std::memcpy(&fd, CMSG_DATA(cm), sizeof(int));
+  if (rsp.size != d.alloc_bytes || rsp.size < d.n) {
+    ::close(fd);
+    throw Error(GROUTER_EINVAL, "ipc: exporter's allocation does not match the descriptor");
+  }
   auto map = std::make_shared<RemoteMap>();
   map->phys = local_phys;
-  uint64_t total = 0;
-  for (uint32_t i = 0; i < rsp.n; ++i) total += rsp.sizes[i];
   try {
-    for (uint32_t i = 0; i < rsp.n; ++i) {
-      CUmemGenericAllocationHandle h;
-      GR_CU(drv().memImportFromShareableHandle(&h, (void *)(uintptr_t)fds[i],
-                                               CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR));
-      map->handles.push_back(h);
-      map->sizes.push_back(rsp.sizes[i]);
-    }
-    GR_CU(drv().memAddressReserve(&map->va, total, kPage, 0, 0));
-    map->size = total;
-    uint64_t off = 0;
-    for (size_t i = 0; i < map->handles.size(); ++i) {
-      GR_CU(drv().memMap(map->va + off, map->sizes[i], 0, map->handles[i], 0));
-      off += map->sizes[i];
-    }
-    std::vector<CUmemAccessDesc> ad;
-    for (auto &kv : c->phys) {
-      CUmemAccessDesc x = {};
-      x.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
-      x.location.id = kv.first;
-      x.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
-      ad.push_back(x);
-    }
-    GR_CU(drv().memSetAccess(map->va, total, ad.data(), ad.size()));
+    CUmemGenericAllocationHandle h;
+    GR_CU(drv().memImportFromShareableHandle(&h, (void *)(uintptr_t)fd, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR));
+    map->handles.push_back(h);
+    map->sizes.push_back(rsp.size);
+    GR_CU(drv().memAddressReserve(&map->va, rsp.size, kPage, 0, 0));
+    map->size = rsp.size;
+    GR_CU(drv().memMap(map->va, rsp.size, 0, h, 0));
+    const std::vector<CUmemAccessDesc> ad = access_all(c);
+    GR_CU(drv().memSetAccess(map->va, rsp.size, ad.data(), ad.size()));
   } catch (...) {
-    for (uint32_t i = 0; i < rsp.n; ++i) ::close(fds[i]);
+    ::close(fd);
     ipc_unmap(*map);
     throw;
   }
-  for (uint32_t i = 0; i < rsp.n; ++i) ::close(fds[i]);
+  ::close(fd);
   return map;
 }
 

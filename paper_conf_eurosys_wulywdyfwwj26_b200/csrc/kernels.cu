@@ -1,17 +1,18 @@
 // kernels.cu -- sm_100a data-movement kernels (no tensor cores: pure bytes).
 //
-// gr_copy: see kernels.h.  Default engines: wv8 (warp-strided, 256-bit
-// LDG/STG, L2 prefetch of each warp's first unit before the PDL wait) below
-// 256 MiB, the TMA bulk ring above.  Tile engines:
-//   * LD/ST: 256 threads, 128-bit vector loads/stores, 4 in flight per
-//     thread before the first store (coalesced, L1 no-allocate), with
-//     co-aligned and shifted (funnel-shift) paths for misaligned user
-//     buffers and byte head/tail;
-//   * TMA bulk: one elected thread streams the tile global -> shared ->
-//     global with cp.async.bulk through a 4-stage mbarrier ring (16 KiB per
-//     stage), used for 16-byte aligned tiles.
-// Both serve local HBM, peer (NVLink) and host-mapped addresses: the data
-// path never interprets bytes.
+// gr_copy (SURVEY K2'/K4', kernels.h) has three engines, chosen per launch
+// in launch_copy:
+//   * wv8   -- warp-strided, 256-bit LDG/STG over 8 KiB units, L2 prefetch
+//              of each warp's first unit before the PDL wait (default);
+//   * tmas4 -- static-assignment TMA bulk ring (cp.async.bulk global ->
+//              shared -> global, 4 x 16 KiB mbarrier stages, one elected
+//              thread per CTA) for large 16 B-aligned local rounds;
+//   * ldst8 -- 256-thread tiles claimed from a ticket, 128-bit LD/ST with
+//              co-aligned and funnel-shift paths for misaligned user buffers.
+// All serve local HBM, peer (NVLink) and host-mapped addresses: the data
+// path never interprets bytes.  The round-1 tuning variants (ws/wd/gs, the
+// ticketed TMA ring, L2 eviction hints, prefetch-ahead) were measured and
+// dropped; their numbers are in DESIGN.md §6 and profiles/r01_*.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -32,7 +33,6 @@ namespace gr {
 constexpr int kThreads = 256;
 constexpr int kTmaThreads = 32;
 constexpr uint32_t kTmaStage = 16384;
-constexpr int kTmaStages = 4;
 
 // ------------------------------------------------------------------ helpers
 __host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
@@ -262,89 +262,6 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
   finish_round(p);
 }
 
-// Continuous TMA stream: ONE elected thread per CTA claims tiles and keeps a
-// STAGES-deep ring of kTmaStage-byte pieces in flight across tile
-// boundaries -- bulk loads (global -> shared, mbarrier complete_tx) and bulk
-// stores (shared -> global, bulk groups); piece k+STAGES-1 is loaded into the
-// stage of piece k-1 once that piece's store has finished reading shared
-// memory.  Requires 16 B aligned chunks (checked by the launcher).
-template <int STAGES, class KP>
-__global__ void __launch_bounds__(kTmaThreads) gr_copy_tma(const __grid_constant__ KP p) {
-  pdl_wait();
-  extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ __align__(8) uint64_t bars[STAGES];
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < STAGES; ++i) mbar_init(&bars[i], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
-    // piece generator over claimed tiles
-    uint64_t cur_src = 0, cur_dst = 0, cur_left = 0;
-    auto next_piece = [&](uint64_t &ps, uint64_t &pd, uint32_t &pb) -> bool {
-      if (cur_left == 0) {
-        const uint32_t t = atomicAdd(&p.scratch[0], 1u);
-        if (t >= total) return false;
-        const int c = find_chunk(p, t);
-        const KChunk &ch = p.chunk[c];
-        const uint64_t off = (uint64_t)(t - (uint32_t)p.tile_prefix[c]) << p.tile_log2;
-        cur_src = ch.src + off;
-        cur_dst = ch.dst + off;
-        cur_left = umin64(ch.bytes - off, 1ull << p.tile_log2);
-      }
-      pb = (uint32_t)umin64(cur_left, kTmaStage);
-      ps = cur_src;
-      pd = cur_dst;
-      cur_src += pb;
-      cur_dst += pb;
-      cur_left -= pb;
-      return true;
-    };
-    uint64_t dst_of[STAGES];
-    uint32_t bytes_of[STAGES];
-    uint32_t phase = 0;
-    auto load = [&](uint32_t k, uint64_t ps, uint64_t pd, uint32_t pb) {
-      const uint32_t s = k % STAGES;
-      dst_of[s] = pd;
-      bytes_of[s] = pb;
-      mbar_expect_tx(&bars[s], pb);
-      bulk_g2s(smem + s * kTmaStage, reinterpret_cast<const void *>(ps), pb, &bars[s]);
-    };
-    uint32_t loaded = 0;
-    bool more = true;
-    for (; loaded < (uint32_t)STAGES; ++loaded) {
-      uint64_t ps, pd;
-      uint32_t pb;
-      if (!next_piece(ps, pd, pb)) {
-        more = false;
-        break;
-      }
-      load(loaded, ps, pd, pb);
-    }
-    for (uint32_t k = 0; k < loaded; ++k) {
-      const uint32_t s = k % STAGES;
-      mbar_wait(&bars[s], (phase >> s) & 1u);
-      phase ^= (1u << s);
-      bulk_s2g(reinterpret_cast<void *>(dst_of[s]), smem + s * kTmaStage, bytes_of[s]);
-      bulk_commit();
-      if (more && k >= 1) {
-        uint64_t ps, pd;
-        uint32_t pb;
-        if (next_piece(ps, pd, pb)) {
-          bulk_wait_read<1>();  // the store of piece k-1 has left its stage
-          load(loaded, ps, pd, pb);
-          ++loaded;
-        } else {
-          more = false;
-        }
-      }
-    }
-    bulk_wait_all();
-    asm volatile("fence.proxy.async.global;" ::: "memory");
-  }
-  __syncthreads();
-  pdl_trigger();
-  finish_round(p);
-}
-
 // Static-assignment TMA ring ("tmas"): CTA b of G moves the 16 KiB units
 // b, b+G, b+2G ... of the round (no ticket, so no scratch to reset and the
 // completion can be published by the host after the launch), through a
@@ -430,127 +347,34 @@ __device__ __forceinline__ void prefetch_units(const KP &p, uint32_t w0, uint32_
   }
 }
 
-// Warp-strided streaming copy: the round is cut into 4 KiB units; warp w of
-// W takes units w, w+W, w+2W ... and keeps U units (U x 8 x 16 B per lane)
-// in flight before storing.  No tile claims, no CTA barriers on the hot
-// loop; consecutive warps touch consecutive 4 KiB units (DRAM/L2-slice
-// friendly).  Partial or misaligned units fall back to the CTA-less warp
-// byte path.
-template <bool COUNT, int U, class KP>
-__global__ void __launch_bounds__(kThreads) gr_copy_ws(const __grid_constant__ KP p) {
-  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
-  const uint32_t lane = threadIdx.x & 31;
-  const uint32_t W = gridDim.x * (kThreads / 32);
-  const uint32_t w0 = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
-  prefetch_units<12>(p, w0, W, total, lane);
-  pdl_wait();
-  if (p.flags & kFlagEarlyTrigger) pdl_trigger();
-  for (uint32_t base = w0; base < total; base += W * U) {
-    int4 v[U][8];
-    uint64_t dsts[U];
-    uint32_t lens[U];
-    uint64_t srcs[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint32_t id = base + u * W;
-      lens[u] = 0;
-      if (id < total) {
-        const int c = find_chunk(p, id);
-        const KChunk &ch = p.chunk[c];
-        const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << 12;
-        srcs[u] = ch.src + off;
-        dsts[u] = ch.dst + off;
-        lens[u] = (uint32_t)umin64(ch.bytes - off, 4096);
-        if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
-          const int4 *sv = reinterpret_cast<const int4 *>(srcs[u]);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) v[u][j] = ld_stream(sv + j * 32 + lane);
-        }
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (!lens[u]) continue;
-      uint8_t *d = reinterpret_cast<uint8_t *>(dsts[u]);
-      const uint8_t *sp = reinterpret_cast<const uint8_t *>(srcs[u]);
-      if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
-        int4 *dv = reinterpret_cast<int4 *>(d);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          st_stream(dv + j * 32 + lane, v[u][j]);
-          count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
-        }
-      } else if (((srcs[u] | dsts[u]) & 15) == 0) {  // aligned partial unit: vectors + byte tail
-        const uint32_t nv = lens[u] >> 4;
-        const int4 *sv = reinterpret_cast<const int4 *>(sp);
-        int4 *dv = reinterpret_cast<int4 *>(d);
-        for (uint32_t i = lane; i < nv; i += 32) {
-          st_stream(dv + i, ld_stream(sv + i));
-          count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
-        }
-        for (uint32_t i = (nv << 4) + lane; i < lens[u]; i += 32) {
-          d[i] = sp[i];
-          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
-        }
-      } else {
-        for (uint32_t i = lane; i < lens[u]; i += 32) {
-          d[i] = sp[i];
-          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
-        }
-      }
-    }
-  }
-  if (!(p.flags & kFlagEarlyTrigger)) pdl_trigger();
-  finish_round(p);
-}
-
-// 256-bit global accesses (sm_100: LDG.256 / STG.256).  H selects L2
-// eviction priorities (bit0: loads evict_first -- a source is read once;
-// bit1: stores evict_first; bit2: stores evict_last -- the consumer reads
-// the destination next).  The .L2::evict_* qualifiers exist only for the
-// 256-bit forms.
+// 256-bit global accesses (sm_100: LDG.256 / STG.256; L1 no-allocate: a
+// source byte is read once).  L2 eviction hints measured no gain
+// and are not used.
 struct alignas(32) V8 {
   uint32_t x[8];
 };
-template <int H>
 __device__ __forceinline__ V8 ld256(const V8 *p) {
   V8 r;
-  if (H & 1)
-    asm volatile("ld.global.L1::no_allocate.L2::evict_first.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=r"(r.x[0]), "=r"(r.x[1]), "=r"(r.x[2]), "=r"(r.x[3]), "=r"(r.x[4]), "=r"(r.x[5]),
-                   "=r"(r.x[6]), "=r"(r.x[7])
-                 : "l"(p));
-  else
-    asm volatile("ld.global.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                 : "=r"(r.x[0]), "=r"(r.x[1]), "=r"(r.x[2]), "=r"(r.x[3]), "=r"(r.x[4]), "=r"(r.x[5]),
-                   "=r"(r.x[6]), "=r"(r.x[7])
-                 : "l"(p));
+  asm volatile("ld.global.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(r.x[0]), "=r"(r.x[1]), "=r"(r.x[2]), "=r"(r.x[3]), "=r"(r.x[4]), "=r"(r.x[5]),
+                 "=r"(r.x[6]), "=r"(r.x[7])
+               : "l"(p));
   return r;
 }
-template <int H>
 __device__ __forceinline__ void st256(V8 *p, const V8 &v) {
-  if (H & 2)
-    asm volatile("st.global.L1::no_allocate.L2::evict_first.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p),
-                 "r"(v.x[0]), "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]),
-                 "r"(v.x[7])
-                 : "memory");
-  else if (H & 4)
-    asm volatile("st.global.L1::no_allocate.L2::evict_last.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p),
-                 "r"(v.x[0]), "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]),
-                 "r"(v.x[7])
-                 : "memory");
-  else
-    asm volatile("st.global.L1::no_allocate.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.x[0]),
-                 "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]), "r"(v.x[7])
-                 : "memory");
+  asm volatile("st.global.L1::no_allocate.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.x[0]),
+               "r"(v.x[1]), "r"(v.x[2]), "r"(v.x[3]), "r"(v.x[4]), "r"(v.x[5]), "r"(v.x[6]), "r"(v.x[7])
+               : "memory");
 }
 
-// Warp-strided copy with 256-bit accesses: units of 2^LG bytes (4 or 8 KiB),
-// warp w of W takes units w, w+W, ...; each lane keeps 2^LG / 1 KiB 32-byte
-// loads in flight per unit.  32 B aligned full units take the 256-bit path;
-// anything else the 16 B / byte fallback of the ws engine.
-template <bool COUNT, int LG, int H, class KP>
+// wv8: warp-strided copy with 256-bit accesses over 8 KiB units; warp w of W
+// takes units w, w+W, ...; each lane keeps 8 x 32 B loads in flight per
+// unit.  32 B co-aligned full units take the 256-bit path, 16 B co-aligned
+// ones a 16 B path with 8 loads in flight per lane, anything else bytes
+// (misaligned rounds go to ldst8 instead, see launch_copy).
+template <bool COUNT, class KP>
 __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ KP p) {
+  constexpr int LG = 13;
   constexpr uint32_t kUnit = 1u << LG;
   constexpr int kPer = (int)(kUnit / (32 * 32));  // 32 B loads per lane per unit
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
@@ -558,17 +382,7 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
   const uint32_t W = gridDim.x * (kThreads / 32);
   prefetch_units<LG>(p, blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5), W, total, lane);
   pdl_wait();
-  if (p.flags & kFlagEarlyTrigger) pdl_trigger();
-  const uint32_t ahead = (p.flags & kFlagPfLoop) ? ((p.flags >> kPfShift) & 0xffu) * W : 0u;
   for (uint32_t id = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5); id < total; id += W) {
-    if (ahead && lane == 0 && id + ahead < total && (p.flags & kFlagLocalSrc)) {
-      const uint32_t a = id + ahead;
-      const int ca = find_chunk(p, a);
-      const uint64_t oa = (uint64_t)(a - (uint32_t)p.tile_prefix[ca]) << LG;
-      const uint64_t sa = p.chunk[ca].src + oa;
-      const uint32_t la = (uint32_t)umin64(p.chunk[ca].bytes - oa, kUnit);
-      if (((sa | la) & 15) == 0) prefetch_l2(sa, la);
-    }
     const int c = find_chunk(p, id);
     const KChunk &ch = p.chunk[c];
     const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << LG;
@@ -579,10 +393,10 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
       V8 *dv = reinterpret_cast<V8 *>(dst);
       V8 v[kPer];
 #pragma unroll
-      for (int j = 0; j < kPer; ++j) v[j] = ld256<H>(sv + j * 32 + lane);
+      for (int j = 0; j < kPer; ++j) v[j] = ld256(sv + j * 32 + lane);
 #pragma unroll
       for (int j = 0; j < kPer; ++j) {
-        st256<H>(dv + j * 32 + lane, v[j]);
+        st256(dv + j * 32 + lane, v[j]);
         count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
         count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane) + 16, 16);
       }
@@ -620,127 +434,6 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
         count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
       }
     }
-  }
-  if (!(p.flags & kFlagEarlyTrigger)) pdl_trigger();
-  finish_round(p);
-}
-
-// Warp-dynamic streaming copy: like ws, but each warp CLAIMS U consecutive
-// 4 KiB units from the round's ticket (lane 0, atomicAdd), and claims the
-// next batch while this batch's loads are in flight, so faster SMs take
-// more units (the per-SM latency spread no longer sets the launch length).
-template <bool COUNT, int U, class KP>
-__global__ void __launch_bounds__(kThreads) gr_copy_wd(const __grid_constant__ KP p) {
-  pdl_wait();
-  const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
-  const uint32_t lane = threadIdx.x & 31;
-  uint32_t next = 0;
-  if (lane == 0) next = atomicAdd(&p.scratch[0], (uint32_t)U);
-  next = __shfl_sync(0xffffffffu, next, 0);
-  while (next < total) {
-    const uint32_t base = next;
-    int4 v[U][8];
-    uint64_t dsts[U], srcs[U];
-    uint32_t lens[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint32_t id = base + u;
-      lens[u] = 0;
-      if (id < total) {
-        const int c = find_chunk(p, id);
-        const KChunk &ch = p.chunk[c];
-        const uint64_t off = (uint64_t)(id - (uint32_t)p.tile_prefix[c]) << 12;
-        srcs[u] = ch.src + off;
-        dsts[u] = ch.dst + off;
-        lens[u] = (uint32_t)umin64(ch.bytes - off, 4096);
-        if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
-          const int4 *sv = reinterpret_cast<const int4 *>(srcs[u]);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) v[u][j] = ld_stream(sv + j * 32 + lane);
-        }
-      }
-    }
-    if (lane == 0) next = atomicAdd(&p.scratch[0], (uint32_t)U);  // overlaps the loads
-    next = __shfl_sync(0xffffffffu, next, 0);
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      if (!lens[u]) continue;
-      uint8_t *d = reinterpret_cast<uint8_t *>(dsts[u]);
-      const uint8_t *sp = reinterpret_cast<const uint8_t *>(srcs[u]);
-      if (lens[u] == 4096 && ((srcs[u] | dsts[u]) & 15) == 0) {
-        int4 *dv = reinterpret_cast<int4 *>(d);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          st_stream(dv + j * 32 + lane, v[u][j]);
-          count_bytes<COUNT>(p, (uint64_t)(dv + j * 32 + lane), 16);
-        }
-      } else if (((srcs[u] | dsts[u]) & 15) == 0) {  // aligned partial unit: vectors + byte tail
-        const uint32_t nv = lens[u] >> 4;
-        const int4 *sv = reinterpret_cast<const int4 *>(sp);
-        int4 *dv = reinterpret_cast<int4 *>(d);
-        for (uint32_t i = lane; i < nv; i += 32) {
-          st_stream(dv + i, ld_stream(sv + i));
-          count_bytes<COUNT>(p, (uint64_t)(dv + i), 16);
-        }
-        for (uint32_t i = (nv << 4) + lane; i < lens[u]; i += 32) {
-          d[i] = sp[i];
-          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
-        }
-      } else {
-        for (uint32_t i = lane; i < lens[u]; i += 32) {
-          d[i] = sp[i];
-          count_bytes<COUNT>(p, (uint64_t)(d + i), 1);
-        }
-      }
-    }
-  }
-  pdl_trigger();
-  finish_round(p);
-}
-
-// Grid-stride streaming copy over the round's 16 B vectors: thread t moves
-// vectors t, t+S, t+2S, ... (S = grid threads), U loads in flight spread a
-// whole grid-width apart -- every DRAM channel/L2 slice is busy at once and
-// no two warps contend for the same lines.  Requires 16 B aligned chunks
-// (launcher checks); the flattened vector space maps to chunks through a
-// prefix (in vectors) -- a single coalesced chunk skips the search.
-template <int U, class KP>
-__global__ void __launch_bounds__(kThreads) gr_copy_gs(const __grid_constant__ KP p) {
-  pdl_wait();
-  const uint64_t total = p.tile_prefix[p.n_chunks];           // vectors
-  const uint64_t S = (uint64_t)gridDim.x * kThreads;
-  const bool one = p.n_chunks == 1;
-  const int4 *s0 = reinterpret_cast<const int4 *>(p.chunk[0].src);
-  int4 *d0 = reinterpret_cast<int4 *>(p.chunk[0].dst);
-  for (uint64_t i = (uint64_t)blockIdx.x * kThreads + threadIdx.x; i < total; i += S * U) {
-    int4 v[U];
-    int4 *dp[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint64_t j = i + (uint64_t)u * S;
-      dp[u] = nullptr;
-      if (j < total) {
-        const int4 *sp;
-        if (one) {
-          sp = s0 + j;
-          dp[u] = d0 + j;
-        } else {
-          int lo = 0, hi = (int)p.n_chunks - 1;
-          while (lo < hi) {
-            int mid = (lo + hi + 1) >> 1;
-            if (p.tile_prefix[mid] <= j) lo = mid;
-            else hi = mid - 1;
-          }
-          const uint64_t o = j - p.tile_prefix[lo];
-          sp = reinterpret_cast<const int4 *>(p.chunk[lo].src) + o;
-          dp[u] = reinterpret_cast<int4 *>(p.chunk[lo].dst) + o;
-        }
-        v[u] = ld_stream(sp);
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (dp[u]) st_stream(dp[u], v[u]);
   }
   pdl_trigger();
   finish_round(p);
@@ -809,26 +502,27 @@ static void choose_tiles(KP &p, uint64_t grid_cap, uint32_t min_lg, uint32_t max
   p.tile_prefix[p.n_chunks] = t;
 }
 
-// Kernel variant: GR_COPY env (tuning) = ldst8 | ldst16 | tma4 | tma8 | tma12 |
-// ws1 | ws2 | ws4; default ws1, or tma8 for 16-B aligned rounds when `tma`.
-static int variant_from_env() {
+// Engine: GR_COPY env (tests / tuning) = wv8 | tmas4 | ldst8; unset = the
+// product choice in launch_copy.
+enum Engine { kEngDefault = -1, kEngLdst8 = 0, kEngTmas4 = 1, kEngWv8 = 2 };
+static int engine_from_env() {
   static int v = -2;
   if (v == -2) {
     const char *e = getenv("GR_COPY");
-    v = -1;
+    v = kEngDefault;
     if (e) {
       std::string s(e);
-      v = s == "ldst8" ? 0 : s == "ldst16" ? 1 : s == "tma4" ? 2 : s == "tma8" ? 3 : s == "tma12" ? 4
-        : s == "ws1" ? 5 : s == "ws2" ? 6 : s == "ws4" ? 7 : s == "wd1" ? 8 : s == "wd2" ? 9
-        : s == "gs8" ? 10 : s == "gs4" ? 11 : s == "gs16" ? 12 : s == "wv4" ? 13 : s == "wv8" ? 14
-        : s == "tmas6" ? 15 : s == "tmas4" ? 16 : s == "tmas3" ? 17 : s == "tmas2" ? 18 : -1;
+      v = s == "ldst8" ? kEngLdst8 : s == "tmas4" ? kEngTmas4 : s == "wv8" ? kEngWv8 : kEngDefault;
     }
   }
   return v;
 }
 
-template <int STAGES, class KP>
+// tmas4: one 32-thread CTA per SM, 4 x 16 KiB stages (64 KiB of shared
+// memory, so the next launch's CTA co-resides under PDL).
+template <class KP>
 static void launch_tmas(KP &p, int sm_count, cudaStream_t s) {
+  constexpr int STAGES = 4;
   static bool attr_set = false;
   const int smem = STAGES * kTmaStage;
   if (!attr_set) {
@@ -842,96 +536,36 @@ static void launch_tmas(KP &p, int sm_count, cudaStream_t s) {
     t += (p.chunk[i].bytes + kTmaStage - 1) / kTmaStage;
   }
   p.tile_prefix[p.n_chunks] = t;
-  static int per_sm = -1;  // CTAs per SM (tuning: GR_TMAS_CTAS)
-  if (per_sm < 0) {
-    const char *e = getenv("GR_TMAS_CTAS");
-    per_sm = e ? atoi(e) : 1;
-    if (per_sm < 1 || per_sm > 8) per_sm = 1;
-  }
-  uint64_t grid = (uint64_t)sm_count * per_sm;
+  uint64_t grid = (uint64_t)sm_count;
   if (grid > t) grid = t;
   if (grid == 0) grid = 1;
   launch_pdl(gr_copy_tmas<STAGES, KP>, grid, kTmaThreads, smem, s, p);
 }
 
-template <int STAGES, class KP>
-static void launch_tma(KP &p, int sm_count, cudaStream_t s) {
-  static bool attr_set = false;
-  const int smem = STAGES * kTmaStage;
-  if (!attr_set) {
-    cudaFuncSetAttribute(gr_copy_tma<STAGES, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    attr_set = true;
-  }
-  const int per_sm = STAGES <= 4 ? 3 : STAGES <= 8 ? 1 : 1;
-  const uint64_t cap = (uint64_t)sm_count * per_sm;
-  choose_tiles(p, cap, 16, 20);
-  uint64_t tiles = p.tile_prefix[p.n_chunks];
-  uint64_t grid = cap > tiles ? tiles : cap;
-  launch_pdl(gr_copy_tma<STAGES, KP>, grid, kTmaThreads, smem, s, p);
-}
-
-template <int U, int MINB, class KP>
+// ldst8: 256-thread CTAs claim 32-256 KiB tiles from a ticket, 8 x 16 B in
+// flight per thread; co-aligned and funnel-shift paths for misaligned rounds.
+template <class KP>
 static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ldst<false, U, MINB, KP>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ldst<false, 8, 1, KP>, kThreads, 0);
     if (occ <= 0) occ = 1;
   }
   const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
   const uint64_t cap = (uint64_t)sm_count * (uint64_t)per_sm;
-  choose_tiles(p, cap, U == 16 ? 16 : 15, 18);
+  choose_tiles(p, cap, 15, 18);
   uint64_t tiles = p.tile_prefix[p.n_chunks];
   uint64_t grid = cap > tiles ? tiles : cap;
-  if (p.counts) launch_pdl(gr_copy_ldst<true, U, MINB, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_ldst<false, U, MINB, KP>, grid, kThreads, 0, s, p);
+  if (p.counts) launch_pdl(gr_copy_ldst<true, 8, 1, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_ldst<false, 8, 1, KP>, grid, kThreads, 0, s, p);
 }
 
-template <int U, class KP>
-static void launch_ws(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
-  static int occ = 0;
-  if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ws<false, U, KP>, kThreads, 0);
-    if (occ <= 0) occ = 1;
-  }
-  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
-  p.tile_log2 = 12;
-  uint64_t t = 0;
-  for (uint32_t i = 0; i < p.n_chunks; ++i) {
-    p.tile_prefix[i] = t;
-    t += (p.chunk[i].bytes + 4095) >> 12;
-  }
-  p.tile_prefix[p.n_chunks] = t;
-  // enough warps that every warp has U units in flight at least once
-  uint64_t warps = (t + U - 1) / U;
-  uint64_t grid = (warps + (kThreads / 32) - 1) / (kThreads / 32);
-  const uint64_t cap = (uint64_t)sm_count * per_sm;
-  if (grid > cap) grid = cap;
-  if (grid == 0) grid = 1;
-  if (p.counts) launch_pdl(gr_copy_ws<true, U, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_ws<false, U, KP>, grid, kThreads, 0, s, p);
-}
-
-static int hint_from_env() {
-  static int h = -1;
-  if (h < 0) {
-    const char *e = getenv("GR_HINT");
-    h = e ? atoi(e) : 0;
-    if (h < 0 || h > 5) h = 0;
-  }
-  return h;
-}
-
-template <int LG, int H, class KP>
-static void launch_wv_h(KP &p, uint64_t grid, cudaStream_t s) {
-  if (p.counts) launch_pdl(gr_copy_wv<true, LG, H, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_wv<false, LG, H, KP>, grid, kThreads, 0, s, p);
-}
-
-template <int LG, class KP>
+template <class KP>
 static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
+  constexpr int LG = 13;
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, LG, 0, KP>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, KP>, kThreads, 0);
     if (occ <= 0) occ = 1;
   }
   const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
@@ -946,79 +580,16 @@ static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   const uint64_t cap = (uint64_t)sm_count * per_sm;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
-  switch (hint_from_env()) {
-    case 1: launch_wv_h<LG, 1>(p, grid, s); break;
-    case 2: launch_wv_h<LG, 2>(p, grid, s); break;
-    case 3: launch_wv_h<LG, 3>(p, grid, s); break;
-    case 4: launch_wv_h<LG, 4>(p, grid, s); break;
-    case 5: launch_wv_h<LG, 5>(p, grid, s); break;
-    default: launch_wv_h<LG, 0>(p, grid, s); break;
-  }
-}
-
-template <int U, class KP>
-static void launch_wd(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
-  static int occ = 0;
-  if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wd<false, U, KP>, kThreads, 0);
-    if (occ <= 0) occ = 1;
-  }
-  const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
-  p.tile_log2 = 12;
-  uint64_t t = 0;
-  for (uint32_t i = 0; i < p.n_chunks; ++i) {
-    p.tile_prefix[i] = t;
-    t += (p.chunk[i].bytes + 4095) >> 12;
-  }
-  p.tile_prefix[p.n_chunks] = t;
-  uint64_t warps = (t + U - 1) / U;
-  uint64_t grid = (warps + (kThreads / 32) - 1) / (kThreads / 32);
-  const uint64_t cap = (uint64_t)sm_count * per_sm;
-  if (grid > cap) grid = cap;
-  if (grid == 0) grid = 1;
-  if (p.counts) launch_pdl(gr_copy_wd<true, U, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_wd<false, U, KP>, grid, kThreads, 0, s, p);
-}
-
-template <int U, class KP>
-static void launch_gs(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
-  uint64_t t = 0;
-  for (uint32_t i = 0; i < p.n_chunks; ++i) {
-    p.tile_prefix[i] = t;
-    t += p.chunk[i].bytes >> 4;
-  }
-  p.tile_prefix[p.n_chunks] = t;
-  p.tile_log2 = 4;
-  // enough threads for U vectors each, capped at ctas_per_sm CTAs per SM
-  uint64_t grid = (t + (uint64_t)kThreads * U - 1) / ((uint64_t)kThreads * U);
-  const uint64_t cap = (uint64_t)sm_count * (uint64_t)ctas_per_sm;
-  if (grid > cap) grid = cap;
-  if (grid == 0) grid = 1;
-  launch_pdl(gr_copy_gs<U, KP>, grid, kThreads, 0, s, p);
+  if (p.counts) launch_pdl(gr_copy_wv<true, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_wv<false, KP>, grid, kThreads, 0, s, p);
 }
 
 template <class KP>
-static void launch_variant(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
+static void launch_engine(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
   switch (v) {
-    case 13: launch_wv<12>(p, sm_count, ctas_per_sm, s); break;
-    case 14: launch_wv<13>(p, sm_count, ctas_per_sm, s); break;
-    case 10: launch_gs<8>(p, sm_count, ctas_per_sm, s); break;
-    case 11: launch_gs<4>(p, sm_count, ctas_per_sm, s); break;
-    case 12: launch_gs<16>(p, sm_count, ctas_per_sm, s); break;
-    case 8: launch_wd<1>(p, sm_count, ctas_per_sm, s); break;
-    case 9: launch_wd<2>(p, sm_count, ctas_per_sm, s); break;
-    case 5: launch_ws<1>(p, sm_count, ctas_per_sm, s); break;
-    case 6: launch_ws<2>(p, sm_count, ctas_per_sm, s); break;
-    case 7: launch_ws<4>(p, sm_count, ctas_per_sm, s); break;
-    case 1: launch_ldst<16, 4>(p, sm_count, ctas_per_sm, s); break;
-    case 2: launch_tma<4>(p, sm_count, s); break;
-    case 3: launch_tma<8>(p, sm_count, s); break;
-    case 4: launch_tma<12>(p, sm_count, s); break;
-    case 15: launch_tmas<6>(p, sm_count, s); break;
-    case 16: launch_tmas<4>(p, sm_count, s); break;
-    case 17: launch_tmas<3>(p, sm_count, s); break;
-    case 18: launch_tmas<2>(p, sm_count, s); break;
-    default: launch_ldst<8, 1>(p, sm_count, ctas_per_sm, s); break;
+    case kEngTmas4: launch_tmas(p, sm_count, s); break;
+    case kEngWv8: launch_wv(p, sm_count, ctas_per_sm, s); break;
+    default: launch_ldst(p, sm_count, ctas_per_sm, s); break;
   }
 }
 
@@ -1048,12 +619,6 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   uint64_t lp1 = 0, lp2 = 0;
   if (host_publish) *host_publish = false;
   if (p.n_chunks == 0) return (int)cudaSuccess;
-  static int ctas_env = -1;
-  if (ctas_env < 0) {
-    const char *e = getenv("GR_CTAS");
-    ctas_env = e ? atoi(e) : 0;
-  }
-  if (ctas_env > 0) ctas_per_sm = ctas_env;
   cudaStream_t s = (cudaStream_t)stream;
   // coalesce chunks that are contiguous in both source and destination (the
   // plan's 2 MiB chunks of one transfer are): fewer, longer runs per launch
@@ -1073,47 +638,32 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   }
   uint64_t total = 0;
   for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
-  int v = variant_from_env();
-  // default: for large aligned rounds (>= 96 MiB) the static 4-stage TMA
-  // bulk ring, one CTA per SM, L2 prefetch before the PDL wait (tmas4:
-  // 128 MiB 45.1 us, 256 MiB 84.9 us, 1 GiB 329.6 us back to back = the
-  // copy engine's 44.4 / 84.3 / 329.3; tools/engine_sizes.py,
-  // profiles/r01_engine_sizes_tmas.txt); otherwise the warp-strided 256-bit
-  // engine over 8 KiB units (wv8) whose warps prefetch their first unit into
-  // L2 before the PDL wait (38.5 MB get_into back to back: 13.2 us with ws1,
-  // 11.8 us with wv8 + prefetch); GROUTER_COPY_TMA forces the ticketed bulk
-  // ring (tma8) for every aligned round
-  // (peer rounds -- NVLink push/pull -- keep the LD/ST engine: TMA bulk copies
-  // to and from peer mappings were never measured on a multi-GPU box here)
+  // Product choice (measured; tools/engine_sizes.py):
+  //  * tmas4 for 16 B-aligned rounds >= 96 MiB whose sources and destinations
+  //    are all in the launching GPU's memory (128 MiB 45.1 us, 256 MiB 84.9 us,
+  //    1 GiB 329.6 us back to back = the copy engine's 44.4 / 84.3 / 329.3);
+  //    GROUTER_COPY_TMA takes it for every aligned round;
+  //  * wv8 otherwise (38.5 MB get_into back to back 11.8 us, 0.997 of the
+  //    measured HBM copy peak); peer rounds (NVLink push/pull) stay on wv8;
+  //  * ldst8 for rounds with a source or destination not 16 B aligned (a
+  //    tensor view, a by-copy put of a host structure): co-aligned and
+  //    funnel-shift 16 B paths instead of the warp engines' byte fallback.
   const bool local_round = (p.flags & kFlagLocalDst) && (p.flags & kFlagLocalSrc);
-  if (v < 0) v = tma ? 3 : (aligned && local_round && total >= (96ull << 20)) ? 16 : 14;
-  // a user buffer at an odd address (a tensor view, a by-copy put of a host
-  // structure): the warp-strided engines would fall back to byte copies;
-  // the tiled LD/ST engine keeps 16 B accesses with its co-aligned and
-  // funnel-shift paths
-  if (!addr_aligned && variant_from_env() < 0) v = 0;
-  if (((v >= 2 && v <= 4) || (v >= 10 && v <= 12) || v >= 15) && (!aligned || p.counts))
-    v = 5;  // TMA/gs need 16 B alignment; counting is LD/ST
-  // static-assignment engines (ws, gs) need no scratch: their completion can
-  // be published by a stream write after the launch, which costs the GPU
-  // ~2 us less than the in-kernel fence + counter + last-CTA protocol
-  const bool is_static = (v >= 5 && v <= 7) || v >= 10;  // ws, gs, wv
-  p.flags &= ~(kFlagEarlyTrigger | kFlagPfLoop | (0xffu << kPfShift));
-  if ((v >= 5 && v <= 7) || v == 13 || v == 14) {  // ws / wv: L2 prefetch + early trigger
-    static int pf = -1, early = -1, loop = -1;
-    if (pf < 0) {
-      const char *e = getenv("GR_PF");
-      pf = e ? atoi(e) : 1;  // measured best: one unit per warp (tools/exp_hints.sh)
-      if (pf < 0 || pf > 255) pf = 0;
-      const char *t = getenv("GR_EARLY");
-      early = t ? atoi(t) : 0;
-      const char *l = getenv("GR_PFLOOP");
-      loop = l ? atoi(l) : 0;
-    }
-    p.flags |= (uint32_t)pf << kPfShift;
-    if (early) p.flags |= kFlagEarlyTrigger;
-    if (loop && v >= 13) p.flags |= kFlagPfLoop;
+  int v = engine_from_env();
+  if (v == kEngDefault) {
+    if (!addr_aligned) v = kEngLdst8;
+    else if (aligned && (tma || (local_round && total >= (96ull << 20)))) v = kEngTmas4;
+    else v = kEngWv8;
   }
+  if (v == kEngTmas4 && (!aligned || p.counts)) v = kEngWv8;  // bulk copies: 16 B only; counting is LD/ST
+  // L2 prefetch of each warp's first 8 KiB unit before the PDL wait (wv8;
+  // measured best at one unit, tools/exp_hints.sh in round 1)
+  p.flags &= ~(0xffu << kPfShift);
+  if (v == kEngWv8) p.flags |= 1u << kPfShift;
+  // static-assignment engines (wv8, tmas4) need no scratch: their completion
+  // can be published by the host after the launch (an event), which costs
+  // the GPU ~2 us less than the in-kernel fence + counter + last-CTA protocol
+  const bool is_static = v == kEngWv8 || v == kEngTmas4;
   p.flags &= ~kFlagNoPublish;
   if (host_publish && is_static && !p.counts) {
     p.flags |= kFlagNoPublish;
@@ -1130,10 +680,10 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
     for (uint32_t i = 0; i < p.n_chunks; ++i) q.chunk[i] = p.chunk[i];
     for (uint32_t i = 0; i < p.n_pub; ++i) q.pub[i] = p.pub[i];
     if (g_launch_prof_on) lp1 = lp_now();
-    launch_variant(q, v, sm_count, ctas_per_sm, s);
+    launch_engine(q, v, sm_count, ctas_per_sm, s);
   } else {
     if (g_launch_prof_on) lp1 = lp_now();
-    launch_variant(p, v, sm_count, ctas_per_sm, s);
+    launch_engine(p, v, sm_count, ctas_per_sm, s);
   }
   if (g_launch_prof_on) lp2 = lp_now();
   const int err = (int)cudaGetLastError();

@@ -1,8 +1,9 @@
 // kernels.h -- host-side launch interface of the sm_100a data-movement kernels.
 //
 // gr_copy (SURVEY K2'/K4'): one launch moves a whole dispatch ROUND -- a list
-// of chunks in stride order (L229) -- with a persistent grid whose CTAs claim
-// 64 KiB tiles from a ticket in device scratch, in round order.  The same
+// of chunks in stride order (L229) -- with one of three engines (kernels.cu:
+// wv8 / tmas4 split the round statically over warps / CTAs, ldst8 claims
+// tiles from a ticket in device scratch).  The same
 // kernel is the NVLink D2D push (dst = peer VA), the same-GPU HBM copy, and
 // the relay forward hop of striped host->GPU transfers (src = staging slot
 // on the route GPU, dst = lease on the destination).  When the last CTA
@@ -31,9 +32,7 @@ constexpr uint32_t kFlagPdl = 1;        // launched with programmatic stream ser
 constexpr uint32_t kFlagLocalDst = 2;   // every destination is in this GPU's memory
 constexpr uint32_t kFlagNoPublish = 4;  // completion written by the host after the launch
 constexpr uint32_t kFlagLocalSrc = 8;   // every source is in this GPU's memory (L2 prefetch is safe)
-constexpr uint32_t kFlagEarlyTrigger = 16;  // let the successor launch right after our own wait
 constexpr uint32_t kPfShift = 8;        // flags >> kPfShift & 0xff: units per warp prefetched to L2
-constexpr uint32_t kFlagPfLoop = 1u << 16;  // keep prefetching that many units ahead inside the loop
 
 // Kernel parameters (passed by value, __grid_constant__).  Two capacities:
 // the large one for rounds with many distinct chunks, a small one (a few

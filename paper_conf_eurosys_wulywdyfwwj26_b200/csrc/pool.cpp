@@ -383,6 +383,7 @@ void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f)
     nopool_sweep(c, false);
     return;
   }
+  if (!c->dedicated.empty() && ded_free(c, p, std::move(f))) return;  // an exported object's own allocation
   DevicePool &P = c->dev[logical].pool;
   uint64_t off = (uint64_t)p - P.base;
   bool done = true;

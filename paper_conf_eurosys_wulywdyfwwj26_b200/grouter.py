@@ -31,6 +31,7 @@ STRIPED_MIGRATION = 0x100   # spills over R(src), restores over R(d) (DESIGN.md 
 NO_POOL = 0x200             # ablation "ES off" (Fig. 16): cudaMalloc/cudaFree per object
 NO_TOPOLOGY = 0x400         # ablation "TA off" (Fig. 16): route sets ignore shared PCIe uplinks (R48)
 HOST_CENTRIC = 0x800        # ablation "UF off" (Fig. 16): GPU -> GPU copies through host memory (R49)
+FORCE_REMOTE = 0x1000       # test only: every copy-kernel round takes the peer (NVLink) branch
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]
@@ -79,7 +80,7 @@ class grouter_stats_t(C.Structure):
         ("rounds", C.c_uint64), ("timed_launches", C.c_uint64), ("timed_ns", C.c_uint64),
         ("timed_bytes", C.c_uint64), ("restore_count", C.c_uint64), ("restore_bytes", C.c_uint64),
         ("pool_target", C.c_uint64 * MAX_GPUS), ("tracked_functions", C.c_uint64),
-        ("tracked_tenants", C.c_uint64),
+        ("tracked_tenants", C.c_uint64), ("peer_launches", C.c_uint64),
     ]
 
 
@@ -98,9 +99,8 @@ class grouter_ipc_desc(C.Structure):
     _fields_ = [("magic", C.c_uint32), ("version", C.c_uint32), ("pid", C.c_int32),
                 ("ctx_id", C.c_uint32), ("gpu_uuid", C.c_uint8 * 16), ("workflow_id", C.c_uint32),
                 ("logical", C.c_int32), ("oid", C.c_uint64), ("n", C.c_uint64),
-                ("exporter_ptr", C.c_uint64), ("first_offset", C.c_uint64), ("n_segs", C.c_uint32),
-                ("pad", C.c_uint32), ("seg_off", C.c_uint64 * IPC_MAX_SEGS),
-                ("seg_size", C.c_uint64 * IPC_MAX_SEGS)]
+                ("exporter_ptr", C.c_uint64), ("export_id", C.c_uint64), ("nonce", C.c_uint64 * 2),
+                ("alloc_bytes", C.c_uint64)]
 
 
 class grouter_dispatch(C.Structure):

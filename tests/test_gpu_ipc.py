@@ -1,9 +1,12 @@
 """Cross-process zero-copy handoff (PAPER.md L167 (1), L269: pool pages mapped
 into the consuming function's address space via CUDA IPC; L394: workflow
-authentication).  On one B200: (a) two contexts of one process, (b) two
-processes.  Importers see the exporter's bytes without a copy (zero copy on
-the same GPU: a write through the exporter is visible through the import),
-get_into copies them with the SM kernel, other workflows get EPERM."""
+authentication, pre-mapped storage only).  On one B200: (a) two contexts of
+one process, (b) two processes.  Zero copy is proven by aliasing: a canary
+written through the exporter's pointer after the import is read through the
+importer's mapping, and the reverse -- a copy would fail both.  get_into
+copies with the SM kernel; other workflows get EPERM; a wrong nonce or a
+freed export is refused; an importer's mapping keeps the object's pages
+(never reused by the exporter's pool) after the exporter frees it."""
 import os
 import subprocess
 import sys
@@ -21,9 +24,17 @@ from paper_conf_eurosys_wulywdyfwwj26_b200 import _build          # noqa: E402
 from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G    # noqa: E402
 from synth.calib import b200_hgx                                   # noqa: E402
 from synth.payload import payload                                  # noqa: E402
-from tests.lib_runner import read_device                           # noqa: E402
+from tests.lib_runner import DevView, read_device                  # noqa: E402
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _poke(ptr, n, value):
+    """Writes `value` into n bytes at a raw device address (through a torch
+    alias of the address, no copy)."""
+    t = torch.as_tensor(DevView(ptr, n), device="cuda")
+    t.fill_(value)
+    torch.cuda.synchronize()
 
 
 def _ctx():
@@ -63,6 +74,17 @@ def test_two_contexts_one_process(n):
         assert np.array_equal(read_device(ptr, min(n, 1 << 20), 0), payload(321, min(n, 1 << 20)))
         exp_ptr = G.Ctx.desc_exporter_ptr(desc)
         assert ptr != exp_ptr                        # a different mapping of the same pages
+        # the import is exactly the object's own 2 MiB pages (R52), no neighbour's
+        dd = G.grouter_ipc_desc.from_buffer_copy(desc)
+        assert dd.alloc_bytes == -(-n // (2 << 20)) * (2 << 20) and dd.version == 2
+        # aliasing, both ways: a copy would see neither write
+        k = min(n, 4096)
+        _poke(exp_ptr, k, 0x3C)
+        assert (read_device(ptr, k, 0) == 0x3C).all()
+        _poke(ptr, k, 0xC3)
+        assert (read_device(exp_ptr, k, 0) == 0xC3).all()
+        G.check(G.test_fill(exp_ptr, k, 321, 0, 0))   # put the payload back
+        torch.cuda.synchronize()
         # get_into: the SM copy kernel reads the imported mapping
         dst = torch.full((n + 32,), 0xA5, dtype=torch.uint8, device="cuda")
         torch.cuda.synchronize()
@@ -90,6 +112,7 @@ EXPORTER = textwrap.dedent("""
     import torch
     from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G
     from synth.calib import b200_hgx
+    from tests.lib_runner import DevView
     c = b200_hgx(1); c["device_map"] = [0]
     ctx = G.Ctx(G.config_from_calib(c, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED],
                                     pool_floor_bytes=64 << 20))
@@ -100,39 +123,120 @@ EXPORTER = textwrap.dedent("""
     f = G.fn(5, 1, 0)
     st, oid = ctx.put(f, src.data_ptr(), n, G.NOHINT, 0, 0)
     st, desc = ctx.export_ipc(f, oid)
+    ptr = G.Ctx.desc_exporter_ptr(desc)
     print(desc.hex(), flush=True)
-    sys.stdin.readline()                      # importer done
-    print(ctx.release(f, oid, G.Ctx.desc_exporter_ptr(desc), 0), ctx.free(f, oid), flush=True)
-    ctx.sync()
-    print(ctx.stats().used[0], flush=True)
+    keep = []
+    for line in sys.stdin:
+        cmd = line.split()
+        if cmd[0] == "poke":            # write through the exporter's own pointer
+            torch.as_tensor(DevView(ptr, 4096), device="cuda").fill_(int(cmd[1]))
+            torch.cuda.synchronize()
+            print("ok", flush=True)
+        elif cmd[0] == "peek":          # read through the exporter's own pointer
+            print(int(torch.as_tensor(DevView(ptr, 4096), device="cuda")[:4096].min().item()),
+                  int(torch.as_tensor(DevView(ptr, 4096), device="cuda")[:4096].max().item()), flush=True)
+        elif cmd[0] == "free":          # end the export, then churn the pool with other data
+            r = (ctx.release(f, oid, ptr, 0), ctx.free(f, oid))
+            ctx.sync()
+            for i in range(8):
+                st, o2 = ctx.put(f, src.data_ptr(), n, G.NOHINT, 0, 0)
+                keep.append(o2)
+            junk = torch.full((n,), 0xEE, dtype=torch.uint8, device="cuda")
+            for o2 in keep:
+                ctx.get_into(f, o2, junk.data_ptr(), n, 0)
+            ctx.sync()
+            print(*r, flush=True)
+        elif cmd[0] == "done":
+            for o2 in keep:
+                ctx.free(f, o2)
+            ctx.sync()
+            print(ctx.stats().used[0], flush=True)
+            break
     ctx.close()
 """)
 
 
 def test_two_processes():
+    """Two processes: the importer's mapping aliases the exporter's pages
+    (canaries both ways), a forged nonce and a freed export are refused, and
+    the importer's view survives the exporter freeing the object and reusing
+    its pool (the pages are the object's own allocation, never recycled)."""
     n = 5 * (1 << 20) + 3
     p = subprocess.Popen([sys.executable, "-c", EXPORTER.format(root=ROOT, n=n)], stdin=subprocess.PIPE,
                          stdout=subprocess.PIPE, text=True)
+
+    def cmd(c):
+        p.stdin.write(c + "\n")
+        p.stdin.flush()
+        return p.stdout.readline().split()
     try:
         desc = bytes.fromhex(p.stdout.readline().strip())
         b = _ctx()
         try:
             f = G.fn(5, 2, 0)
-            st, roid = b.import_ipc(f, desc, consumers=1)
+            # a forged capability (wrong nonce) is refused by the exporter
+            forged = G.grouter_ipc_desc.from_buffer_copy(desc)
+            forged.nonce[1] ^= 1
+            assert b.import_ipc(f, bytes(forged))[0] == G.ENOENT
+            st, roid = b.import_ipc(f, desc, consumers=0)
             assert st == G.OK
             dst = torch.empty(n, dtype=torch.uint8, device="cuda")
             s = torch.cuda.Stream()
-            st, nn = b.get_into(f, roid, dst.data_ptr(), n, s.cuda_stream)   # consumes -> unmapped
+            st, nn = b.get_into(f, roid, dst.data_ptr(), n, s.cuda_stream)   # SM copy from the mapping
             assert st == G.OK and nn == n
             s.synchronize()
             st2, bad, _ = G.test_verify(dst.data_ptr(), n, 99, 0, 0)
             assert st2 == G.OK and bad == 0
+            st, ptr, nn = b.get(f, roid, s.cuda_stream)                      # zero copy: the mapping
+            assert st == G.OK
+            s.synchronize()
+            assert cmd("poke 90") == ["ok"]                                  # exporter writes ...
+            assert (read_device(ptr, 4096, 0) == 90).all()                   # ... importer sees it
+            _poke(ptr, 4096, 165)                                            # importer writes ...
+            assert cmd("peek") == ["165", "165"]                             # ... exporter sees it
+            assert cmd("free") == ["0", "0"]           # exporter frees the object and churns its pool
+            # the importer's mapping still holds the object's pages, untouched by the churn
+            assert (read_device(ptr, 4096, 0) == 165).all()
+            assert np.array_equal(read_device(ptr + 4096, n - 4096, 0), payload(99, n - 4096, 4096))
+            # the export is over: a new import of the same descriptor is refused
+            assert b.import_ipc(f, desc)[0] == G.ENOENT
+            assert b.release(f, roid, ptr, s.cuda_stream) == G.OK
+            assert b.free(f, roid) == G.OK
             assert b.where(roid)[0] == G.ENOENT
         finally:
             b.close()
-        p.stdin.write("done\n")
-        p.stdin.flush()
-        rel, used = p.stdout.readline().split(), p.stdout.readline().strip()
-        assert rel == ["0", "0"] and used == "0"
+        assert cmd("done") == ["0"]
     finally:
         p.wait(timeout=60)
+
+
+def test_export_requires_no_zero_copy_leases():
+    """The first export moves the object into its own allocation; an object a
+    zero-copy lease still aliases cannot move (EBUSY), once the lease is
+    released the export succeeds, and a second export reuses the allocation
+    (same exporter pointer, no second move)."""
+    a = _ctx()
+    try:
+        n = 3 << 20
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 5, 0, 0))
+        torch.cuda.synchronize()
+        f = G.fn(3, 1, 0)
+        st, oid = a.put(f, src.data_ptr(), n, G.NOHINT, 0, 0)
+        st, lp, nn = a.get(f, oid, 0)
+        assert st == G.OK
+        assert a.export_ipc(f, oid)[0] == G.EBUSY
+        assert a.release(f, oid, lp, 0) == G.OK
+        st, d1 = a.export_ipc(f, oid)
+        assert st == G.OK
+        st, d2 = a.export_ipc(f, oid)
+        assert st == G.OK and G.Ctx.desc_exporter_ptr(d1) == G.Ctx.desc_exporter_ptr(d2)
+        e = G.Ctx.desc_exporter_ptr(d1)
+        assert np.array_equal(read_device(e, n, 0), payload(5, n))   # the move kept the bytes
+        for _ in range(2):
+            assert a.release(f, oid, e, 0) == G.OK
+        assert a.free(f, oid) == G.OK
+        a.sync()
+        assert a.stats().used[0] == 0
+    finally:
+        a.close()

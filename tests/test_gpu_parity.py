@@ -68,16 +68,15 @@ def test_copy_kernel_exactly_once(tma, src_off, dst_off):
     _copy_exactly_once(tma, src_off, dst_off)
 
 
-VARIANTS = ["ldst8", "ldst16", "tma4", "tma8", "tma12", "ws1", "ws2", "ws4", "wd1", "wd2", "gs4", "gs8", "gs16",
-            "wv4", "wv8", "wv4:GR_HINT=3", "wv8:GR_HINT=5", "wv4:GR_PF=2:GR_EARLY=1", "ws1:GR_PF=1:GR_EARLY=1",
-            "wv8:GR_PF=1", "wv8:GR_PF=2:GR_PFLOOP=1", "tmas4", "tmas6"]
+VARIANTS = ["ldst8", "wv8", "tmas4"]
 
 
 @pytest.mark.parametrize("variant", VARIANTS)
 def test_copy_kernel_variants(variant):
-    """Every engine variant (GR_COPY[:ENV=VAL...]: cache hints, L2 prefetch,
-    early PDL trigger) in a subprocess: byte-exact over aligned and
-    misaligned chunk lists, exactly-once counts where it can count."""
+    """Every engine (GR_COPY = ldst8 | wv8 | tmas4, forced for every round) in
+    a subprocess: byte-exact over aligned and misaligned chunk lists
+    (tmas4 takes only 16 B-aligned rounds and hands the others to wv8),
+    exactly-once counts where it can count."""
     import os
     import subprocess
     import sys
@@ -91,7 +90,7 @@ def test_copy_kernel_variants(variant):
     assert r.returncode == 0, r.stderr[-2000:]
 
 
-ALIGNED_VARIANTS = ["tma4", "tma8", "tma12", "tmas4", "tmas6", "wv8", "ws1", "gs8"]
+ALIGNED_VARIANTS = ["tmas4", "wv8", "ldst8"]
 
 
 @pytest.mark.parametrize("variant", ALIGNED_VARIANTS)
@@ -257,6 +256,40 @@ def test_random_traces_realtime(seed):
     caps = [rng.choice([8, 16, 64]) * MiB for _ in range(k)]
     orc, lib_out = _both(ops, calib, replay=False, host_store_bytes=48 * MiB, pool_cap=caps)
     compare(orc, lib_out, check_dispatch=False)
+
+
+@pytest.mark.parametrize("seed", range(3))
+@pytest.mark.parametrize("replay", [True, False])
+def test_random_traces_forced_remote(seed, replay):
+    """GROUTER_FORCE_REMOTE: every copy-kernel round takes the branch a
+    physical peer (NVLink) transfer takes -- system-scope fences, no L2
+    prefetch of sources, no TMA bulk engine, completion published in-kernel
+    by the last CTA -- so the one-GPU box executes that code: D2D pushes,
+    relay forwards and same-GPU copies are byte-exact and every decision
+    equals the oracle's."""
+    rng = random.Random(3000 + seed)
+    k = rng.choice([2, 3, 4])
+    calib = C.virtual(k)
+    ops = T.random_trace(rng, k, n_ops=120, max_n=5 * MiB, run_seed=seed)
+    caps = [rng.choice([8, 16, 64]) * MiB for _ in range(k)]
+    orc, lib_out = _both(ops, calib, replay=replay, host_store_bytes=48 * MiB, pool_cap=caps,
+                         flags=G.FORCE_REMOTE)
+    compare(orc, lib_out, check_dispatch=replay)
+    st = lib_out["stats"]
+    assert st.kernel_launches > 0 and st.peer_launches == st.kernel_launches
+
+
+@pytest.mark.parametrize("replay", [True, False])
+def test_config_traces_forced_remote(replay):
+    """cfg1 (striped put over R(0) with relays through the route GPUs' staging
+    rings, then D2D gets) and cfg2 (fan-out of crops to two other GPUs) on four
+    logical GPUs with every kernel round on the peer branch."""
+    calib = C.virtual(4)
+    for ops in [T.cfg1(4, iters=3, scale=4), T.cfg2(4, requests=3, scale=16)]:
+        orc, lib_out = _both(ops, calib, replay=replay, flags=G.FORCE_REMOTE)
+        assert compare(orc, lib_out, check_dispatch=replay) > 0
+        st = lib_out["stats"]
+        assert st.peer_launches == st.kernel_launches > 0
 
 
 def test_fig11b_restore():
@@ -462,8 +495,9 @@ def test_fig5a_striped_spill_and_restore():
     del g
 
 
+@pytest.mark.parametrize("flags", [0, "FORCE_REMOTE"])
 @pytest.mark.parametrize("n", [1 << 30, (1 << 30) - 4097])
-def test_full_size_cfg3_max(n):
+def test_full_size_cfg3_max(n, flags):
     """cfg3's largest size (1 GiB, and a ragged 1 GiB - 4097 B) through every
     pattern on two logical GPUs: a cFn put striped over R(0) = {0, 1} (the
     relay hop through logical GPU1's staging ring), a D2D get_into on GPU1, a
@@ -474,7 +508,7 @@ def test_full_size_cfg3_max(n):
     from synth import payload as P
     calib = C.virtual(2)
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=3 << 30, pool_cap=[G.UNLIMITED] * 2,
-                                    pool_floor_bytes=64 << 20))
+                                    pool_floor_bytes=64 << 20, flags=getattr(G, flags) if flags else 0))
     seed = 424242
     try:
         st, plan = ctx.plan(G.HOST, 0, n)
@@ -510,6 +544,9 @@ def test_full_size_cfg3_max(n):
             assert np.array_equal(back[off:off + 64], P.payload(seed, 64, off)), off
         ctx.release(cfn, oid, ptr, 0)
         ctx.free(cfn, oid)
+        st = ctx.stats()
+        if flags:   # the relay forward, the D2D push and the same-GPU copy all on the peer branch
+            assert st.peer_launches == st.kernel_launches > 0
     finally:
         ctx.close()
 

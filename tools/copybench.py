@@ -51,7 +51,7 @@ if __name__ == "__main__":
     if len(sys.argv) > 1 and sys.argv[1] == "--child":
         child(sys.argv[2])
     else:
-        for v in (sys.argv[1:] or ["torch", "ldst8", "ldst16", "tma4", "tma8", "tma12"]):
+        for v in (sys.argv[1:] or ["torch", "ldst8", "wv8", "tmas4"]):
             name, _, ctas = v.partition("@")
             env = dict(os.environ, GR_COPY=name)
             if ctas:

@@ -78,7 +78,7 @@ if __name__ == "__main__":
     if len(sys.argv) > 1 and sys.argv[1] == "--child":
         child()
     else:
-        for e in sys.argv[1:] or ["default", "wv8", "tma8"]:
+        for e in sys.argv[1:] or ["default", "wv8", "tmas4"]:
             env = dict(os.environ)
             e, *extra = e.split(":")        # ENGINE[@PF][:ENV=VAL ...]
             env.update(kv.split("=", 1) for kv in extra)
