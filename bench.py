@@ -1,25 +1,44 @@
 #!/usr/bin/env python
 """bench.py -- GROUTER data-passing hot path on B200 (one JSON line).
 
-Workload (BASELINE.json configs[0], cfg1, reading R24 + DESIGN.md "Bench"):
-a 2-function workflow passes a 38,535,168 B fp32 tensor (64x3x224x224).
-A request = leg A: CPU function puts the tensor from a pinned host buffer
-with a placement hint for GPU0 (striped host->GPU over R(0)); leg B: the GPU
-function gets it INTO its fixed input binding (get_into: the consumer's input
-address is fixed, e.g. a captured CUDA graph), the SM copy kernel gr_copy
-(K2').  On one B200 leg B is a same-GPU HBM copy; on 2+ GPUs of one process
-it is the NVLink push.
+metric (BASELINE.json): "p50/p99 data-passing latency & GB/s vs size; workflow
+req/s at 1/2/4/8 B200".
 
-  value : leg B with the objects already resident in HBM (20 requests per
-          step, req/s, device-timed with CUDA events on the consumer stream)
-  e2e   : legs A+B through the C ABI with host buffers (H2D inside the timed
-          region) plus an 8-byte D2H read of the delivered tensor per request
-  roofline : gr_copy, algorithmic bytes = 2 x 38,535,168 per request (read +
-          write, HBM), timed per launch with CUDA events on the copy stream
-          (GROUTER_PROFILE), against MEASURED_PEAKS.json hbm_gbs
-  cpu_baseline : the oracle (numpy memcpy on simulated buffers), same op
-N>1 (torchrun): one process per GPU, each runs the same workload on its own
-GPU (replicas, weak scaling); value = all ranks' requests / max-rank time.
+value = workflow req/s of cfg1 (BASELINE configs[0]; reading R24): a CPU
+function (cFn) puts a 38,535,168 B fp32 tensor (64x3x224x224, R25) from its
+pinned host buffer with a placement hint for the producer GPU (striped H2D over
+R(d); at one GPU the direct PCIe link), and the GPU function (gFn) gets it into
+its fixed input binding (get_into: the consumer's input address is fixed,
+e.g. a captured CUDA graph -- reading R51; the object is consumed and freed).
+20 requests per step (the config's "20 puts/gets"), closed loop with Q = 4
+requests outstanding, one client thread each.  Device-timed:
+CUDA events on a timing stream that every consumer stream joins before and
+after the K steps.  At N GPUs (torchrun, one process per GPU) every rank runs
+the same flow with its consumer on the next GPU: put host -> GPU r (its own
+PCIe link: every link carries its own rank's traffic), get_into on GPU r+1
+(GPU r's SM copy kernel pushes the tensor over NVLink) -- a ring of disjoint
+producer -> consumer pairs, weak scaling, no collective.
+
+Also in the line:
+  e2e          the same loop host-timed (wall clock) plus an 8 B D2H read of
+               each delivered tensor (the step's result)
+  latency_us   p50/p99 of single cfg1 requests on an idle GPU (R22: put call
+               -> the consumer's data ready)
+  roofline     gr_copy (the only kernel on the path), per-launch CUDA events
+               on its stream inside the timed region (GROUTER_PROFILE);
+               algorithmic bytes = 2n (HBM read + write) at one GPU, n over
+               NVLink at N > 1; roofline_step: the PCIe link that bounds
+               the workflow (live-measured pinned H2D)
+  kernel_b2b   leg B alone, back to back on HBM-resident objects (the kernel's
+               own speed of light)
+  sweep        cfg3 (iii)/(iv) at one GPU: per size 4 KiB..1 GiB, p50/p99 and
+               GB/s of same-GPU get_into, cFn put (H2D), cFn get (D2H) and
+               zero-copy get, each beside a bare cudaMemcpyAsync on the same
+               buffers through the same binding, plus the oracle's get_into
+  cpu_baseline the oracle (oracle/, numpy memcpy on simulated buffers) on the
+               same cfg1 request, single-threaded as it stands, plus the
+               striped put variant (one thread per route of the 8-GPU HGX
+               calibration's R(0))
 """
 from __future__ import annotations
 
@@ -29,22 +48,52 @@ import os
 import statistics
 import subprocess
 import sys
+import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 N_BYTES = 64 * 3 * 224 * 224 * 4          # 38,535,168 (R25)
-METRIC = "workflow req/s (cfg1 data plane)"
-WORKLOAD = ("cfg1 2-function workflow, 38,535,168 B tensor; value: gFn get_into of "
-            "HBM-resident objects (same-GPU K2' copy on 1 B200), e2e: cFn put(hint=GPU0) "
-            "from pinned host + get_into + 8 B D2H")
+METRIC = "p50/p99 data-passing latency & GB/s vs size; workflow req/s at 1/2/4/8 B200"
+NVL_PEAK = 900.0                           # GB/s per direction per GPU (north star roofline)
+MiB = 1 << 20
+WORKLOAD = ("cfg1 2-function workflow (BASELINE configs[0], R24): cFn put of a 38,535,168 B fp32 tensor from "
+            "pinned host memory (hint GPU0: H2D) -> gFn on GPU0 get_into its fixed input binding (R51); "
+            "20 requests/step, 4 outstanding")
+WORKLOAD_N = ("cfg1 2-function workflow at N GPUs (R24): on every GPU r a cFn puts the 38,535,168 B tensor "
+              "from pinned host memory into GPU r (its own PCIe link) and a gFn on GPU r+1 get_into's it "
+              "(GPU r's SM kernel pushes it over NVLink); ring of disjoint pairs, 20 requests/step per GPU, "
+              "4 outstanding per GPU")
 
 
-WORKLOAD_N = ("cfg1 2-function workflow at N GPUs, 38,535,168 B tensor; value: every GPU runs the N=1 "
-              "workload on its own workflows (co-located, weak scaling); nvlink_pull: gFn on GPU r "
-              "get_into's objects resident on GPU r+1 (CUDA VMM IPC, SM pull copy over NVLink); "
-              "e2e: cFn put(hint=own GPU) from pinned host + local get_into + 8 B D2H")
+def pct(xs, q):
+    """Nearest-rank percentile (R26): the ceil(q/100 * m)-th smallest."""
+    xs = sorted(xs)
+    return xs[min(len(xs) - 1, max(0, -(-len(xs) * q // 100) - 1))] if xs else None
+
+
+def host_info():
+    """Host cores this process may use and the CPU model."""
+    cores = len(os.sched_getaffinity(0))
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.strip().startswith("Model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    if not model:
+        try:
+            for ln in open("/proc/cpuinfo"):
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+        except Exception:
+            model = None
+    return cores, model
 
 
 def _peaks():
@@ -198,7 +247,7 @@ CPU_GROUP = [None]   # gloo group for waits that must not occupy the GPUs (set i
 
 
 def peer_of(rank: int, world: int) -> int:
-    """cfg1 at N GPUs: the object produced on GPU r+1 is consumed on GPU r
+    """cfg1 at N GPUs: the object produced on GPU r is consumed on GPU r+1
     (a ring of disjoint producer->consumer pairs: every GPU's NVLink egress
     and ingress carry one stream, no link is shared)."""
     return (rank + 1) % world
@@ -216,21 +265,25 @@ def exchange(obj, world: int, group=None):
 
 
 def max_over_ranks(x: float, world: int, device=None) -> float:
+    """MAX of a host float over the ranks, on the CPU (gloo) group: no kernel
+    is left resident on the GPUs (device is accepted for old callers)."""
     if world == 1:
         return x
     import torch
     import torch.distributed as dist
-    if dist.get_backend() != "nccl":
-        device = None
-    t = torch.tensor([x], dtype=torch.float64, device=device)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    t = torch.tensor([x], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=CPU_GROUP[0])
     return float(t.item())
 
 
 # ------------------------------------------------------------------ reference / oracle arm
-class OracleLeg:
-    """The oracle as it stands on the same request: get_into of the
-    HBM-resident object (numpy memcpy between simulated buffers).  State is
+
+# ------------------------------------------------------------------ reference / oracle arm
+class OracleRequest:
+    """The oracle as it stands on the bench's cfg1 request: a cFn put of the
+    38.5 MB tensor with hint GPU0 (O1: plan + np.copyto into the simulated
+    GPU0 buffer), then the gFn's get_into of it (O4: np.copyto into the
+    binding; consumers = 1, so the object is consumed and freed).  State is
     built once; only the calls are timed."""
 
     def __init__(self):
@@ -243,25 +296,25 @@ class OracleLeg:
         self.np = np
         self.orc = Oracle(b200_hgx(1))
         self.src = payload(1000, N_BYTES)
-        st, out = self.orc.put({"wf": 1, "fid": 2, "dev": 0}, self.src, N_BYTES, -2, 0)
-        assert st == 0
-        self.oid = out["oid"]
         self.dst = np.empty(N_BYTES, np.uint8)
-        self.g = {"wf": 1, "fid": 3, "dev": 0}
+        self.c = {"wf": 1, "fid": 1, "dev": -1}
+        self.g = {"wf": 1, "fid": 2, "dev": 0}
 
     def run(self, requests: int):
         for _ in range(requests):
-            st, _ = self.orc.get_into(self.g, self.oid, self.dst, N_BYTES)
+            st, out = self.orc.put(self.c, self.src, N_BYTES, 0, 1)
+            assert st == 0
+            st, _ = self.orc.get_into(self.g, out["oid"], self.dst, N_BYTES)
             assert st == 0
         return requests
 
     def check(self):
-        assert self.np.array_equal(self.dst[:4096], self.src[:4096])
+        assert self.np.array_equal(self.dst[:4096], self.src[:4096]) and not self.orc.objects
 
 
-def oracle_rate(requests: int, budget_s: float):
-    """(req/s, requests, seconds) of the oracle over >= budget_s."""
-    leg = OracleLeg()
+def oracle_rate(budget_s: float, requests: int = 2):
+    """(req/s, requests, seconds) of the oracle over >= budget_s (1 thread)."""
+    leg = OracleRequest()
     done, t0 = 0, time.perf_counter()
     while True:
         done += leg.run(requests)
@@ -272,11 +325,59 @@ def oracle_rate(requests: int, budget_s: float):
     return done / dt, done, dt
 
 
+def oracle_striped_put_rate(budget_s: float):
+    """SURVEY §8(d) striped variant: the cFn put's O6 plan on the 8-GPU HGX
+    calibration (R(0) = one GPU per PCIe uplink group) executed with one
+    thread per route (T = |R(0)|, capped at the cores), each np.copyto-ing
+    its chunks.  Returns (puts/s, threads)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    import numpy as np
+
+    from oracle.splitter import CHUNK, plan_h2d
+    from synth.calib import b200_hgx
+    from synth.payload import payload
+    src = payload(1000, N_BYTES)
+    dst = np.empty(N_BYTES, np.uint8)
+    by = {}
+    for c in plan_h2d(b200_hgx(8), 0, N_BYTES, True, CHUNK):
+        by.setdefault(c["route_gpu"], []).append((c["offset"], c["offset"] + c["bytes"]))
+    T = max(1, min(len(by), len(os.sched_getaffinity(0))))
+
+    def work(spans):
+        for a, b in spans:
+            np.copyto(dst[a:b], src[a:b])
+    done = 0
+    with ThreadPoolExecutor(T) as ex:
+        t0 = time.perf_counter()
+        while True:
+            list(ex.map(work, by.values()))
+            done += 1
+            dt = time.perf_counter() - t0
+            if dt >= budget_s:
+                break
+    assert np.array_equal(dst, src)
+    return done / dt, T
+
+
+def cpu_baseline_obj(budget_s: float):
+    cores, model = host_info()
+    v, done, dt = oracle_rate(budget_s)
+    sv, T = oracle_striped_put_rate(max(1.0, budget_s / 4))
+    return {"value": v, "unit": "req/s", "cores": 1, "kind": "oracle", "host_cores": cores, "cpu_model": model,
+            "sample": f"{done} oracle cfg1 requests (put hint GPU0 + get_into, {N_BYTES} B, numpy memcpy "
+                      f"on simulated buffers) in {dt:.1f} s, 1 thread",
+            "striped_put": {"value": sv, "unit": "puts/s", "threads": T,
+                            "what": "the put's O6 plan on the 8-GPU HGX calibration, one thread per route"}}
+
+
 def run_reference(args, rank):
+    """--impl reference: the oracle as it stands on the bench's cfg1 request,
+    on this box's host cores (rank 0 only; other ranks exit without work)."""
     if rank != 0:
         return
     reqs = max(1, min(args.requests, 4))          # bounded sample per step
-    leg = OracleLeg()
+    leg = OracleRequest()
     for _ in range(args.warmup):
         leg.run(reqs)
     t0 = time.perf_counter()
@@ -286,16 +387,216 @@ def run_reference(args, rank):
     dt = time.perf_counter() - t0
     leg.check()
     v = done / dt
+    cores, model = host_info()
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "req/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": dt * 1e3 / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "u8", "data": "synthetic (SplitMix64 payload)",
             "config": {"workload": WORKLOAD, "requests_per_step": reqs, "bytes": N_BYTES,
-                       "parallelism": "replicas"},
-            "cpu_baseline": {"kind": "oracle", "value": v, "unit": "req/s", "cores": 1,
-                             "sample": f"{args.steps} steps x {reqs} oracle get_into of {N_BYTES} B"},
+                       "parallelism": "oracle, 1 thread"},
+            "cpu_baseline": {"kind": "oracle", "value": v, "unit": "req/s", "cores": 1, "host_cores": cores,
+                             "cpu_model": model,
+                             "sample": f"{args.steps} steps x {reqs} oracle cfg1 requests of {N_BYTES} B"},
             "e2e": {"value": v, "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+
+
+# ------------------------------------------------------------------ cfg3 size sweep (one GPU)
+SWEEP_SIZES = [4096 * 4 ** i for i in range(10)] + [2 * MiB - 1, 2 * MiB + 1, N_BYTES]
+
+
+def _samples(n):
+    return 200 if n <= 64 * MiB else (50 if n <= 256 * MiB else 30)
+
+
+def _stats(xs, n, rw=1):
+    p50, p99 = pct(xs, 50), pct(xs, 99)
+    return {"p50_us": round(p50, 2), "p99_us": round(p99, 2), "GBps": round(rw * n / p50 / 1e3, 2)}
+
+
+def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
+    """cfg3 (iii) and (iv) at one GPU, per size, each beside a bare
+    cudaMemcpyAsync on the same buffers called through the same binding
+    (grouter_test_memcpy), byte-verified:
+      get_into  gFn get_into of a GPU0-resident object: single calls on an idle
+                GPU (CUDA events around the call on the consumer stream, host
+                path included) and back to back (GB/s read + write, fraction
+                of the HBM copy peak); baseline cudaMemcpyAsync D2D
+      put_h2d   cFn put(hint GPU0) from pinned host memory, blocking, host
+                timed; baseline pinned H2D + wait
+      get_d2h   cFn get of a GPU0 object into a host lease (+ release),
+                blocking, host timed; baseline D2H + wait
+      zero_copy gFn get + release of a co-located object, host timed
+    Samples: 200 (<= 64 MiB), 50 (256 MiB), 30 (1 GiB); nearest-rank p50/p99."""
+    import torch
+    from synth.calib import b200_hgx
+    calib = b200_hgx(1)
+    calib["device_map"] = [dev]
+    maxn = max(sizes)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=maxn + (256 << 20), pool_cap=[G.UNLIMITED],
+                                    pool_floor_bytes=64 << 20))
+    out = []
+    try:
+        s = torch.cuda.Stream(device=dev)
+        host = torch.empty(maxn, dtype=torch.uint8, pin_memory=True)
+        tmp = torch.empty(maxn, dtype=torch.uint8, device=f"cuda:{dev}")
+        G.check(G.test_fill(tmp.data_ptr(), maxn, 31337, 0, 0))
+        host.copy_(tmp)
+        dsts = [torch.empty(maxn, dtype=torch.uint8, device=f"cuda:{dev}") for _ in range(2)]
+        del tmp
+        torch.cuda.synchronize(dev)
+        cfn, gfn, gfn2 = G.fn(7, 1, G.HOST), G.fn(7, 2, 0), G.fn(7, 3, 0)
+        hp, ss = host.data_ptr(), s.cuda_stream
+
+        def dev_single(call, reps):
+            xs = []
+            for _ in range(reps):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(s)
+                call()
+                b.record(s)
+                b.synchronize()
+                xs.append(a.elapsed_time(b) * 1e3)
+            return xs
+
+        def dev_b2b(call, reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            for _ in range(reps):
+                call()
+            b.record(s)
+            b.synchronize()
+            return a.elapsed_time(b) * 1e3 / reps
+
+        def host_single(call, reps):
+            xs = []
+            for _ in range(reps):
+                t = time.perf_counter()
+                call()
+                xs.append((time.perf_counter() - t) * 1e6)
+            return xs
+
+        for n in sizes:
+            reps = _samples(n)
+            row = {"bytes": n}
+            st, oid = ctx.put(cfn, hp, n, 0, 0)
+            G.check(st, "put")
+            # back to back: a working set above the 126 MB L2 where memory allows
+            # (m source objects, destinations rotating over the two 1 GiB buffers)
+            m = max(1, min(32, (256 * MiB) // max(n, 1)))
+            srcs = [oid]
+            for _ in range(m - 1):
+                st, o2 = ctx.put(cfn, hp, n, 0, 0)
+                G.check(st, "put")
+                srcs.append(o2)
+            slots = max(1, min(64, maxn // max(-(-n // 256) * 256, 1)))
+            G.check(ctx.sync(), "sync")
+            k = [0]
+
+            def dst_at(j):
+                return dsts[j & 1].data_ptr() + ((j >> 1) % slots) * (-(-n // 256) * 256)
+
+            def gi():
+                st, _ = ctx.get_into(gfn, srcs[k[0] % m], dst_at(k[0]), n, ss)
+                k[0] += 1
+                if st:
+                    G.check(st, "get_into")
+
+            def mc():
+                G.check(G.test_memcpy(dst_at(k[0]), dst_at(k[0] + 1), n, ss, False))
+                k[0] += 1
+            for _ in range(5):
+                gi()
+            s.synchronize()
+            st, bad, _ = G.test_verify(dst_at(4), n, 31337, 0, 0)
+            assert st == 0 and bad == 0, f"sweep get_into {n}: {bad} bytes differ"
+            lib1 = dev_single(gi, reps)
+            b2b = dev_b2b(gi, max(10, min(reps, 200)))
+            for _ in range(3):
+                mc()
+            base1 = dev_single(mc, reps)
+            bb2b = dev_b2b(mc, max(10, min(reps, 200)))
+            row["get_into"] = dict(_stats(lib1, n, 2), b2b_us=round(b2b, 2), b2b_GBps=round(2 * n / b2b / 1e3, 1),
+                                   b2b_frac_hbm=round(2 * n / b2b / 1e3 / hbm_peak, 3),
+                                   memcpy=dict(_stats(base1, n, 2), b2b_us=round(bb2b, 2)))
+            # cFn put (H2D) vs bare pinned H2D; the free of each put object is
+            # outside the timed call
+            def put_timed(reps):
+                xs = []
+                for _ in range(reps):
+                    t = time.perf_counter()
+                    st, o2 = ctx.put(cfn, hp, n, 0, 0)
+                    xs.append((time.perf_counter() - t) * 1e6)
+                    if st:
+                        G.check(st, "put")
+                    ctx.free(cfn, o2)
+                return xs
+
+            def h2d():
+                G.check(G.test_memcpy(dsts[0].data_ptr(), hp, n, 0, True))
+            put_timed(3)
+            for _ in range(3):
+                h2d()
+            lp = put_timed(reps)
+            bp = host_single(h2d, reps)
+            row["put_h2d"] = dict(_stats(lp, n), frac_link=round(n / pct(lp, 50) / 1e3 / h2d_peak, 3),
+                                  memcpy=_stats(bp, n))
+            # cFn get (D2H into a host lease) vs bare D2H; the lease's release
+            # is outside the timed call
+            def get_timed(reps):
+                xs = []
+                for _ in range(reps):
+                    t = time.perf_counter()
+                    st, ptr, nn = ctx.get(cfn, oid, 0)
+                    xs.append((time.perf_counter() - t) * 1e6)
+                    if st:
+                        G.check(st, "get")
+                    ctx.release(cfn, oid, ptr, 0)
+                return xs
+
+            def d2h():
+                G.check(G.test_memcpy(hp, dsts[0].data_ptr(), n, 0, True))
+            get_timed(3)
+            for _ in range(3):
+                d2h()
+            lg = get_timed(reps)
+            bg = host_single(d2h, reps)
+            row["get_d2h"] = dict(_stats(lg, n), memcpy=_stats(bg, n))
+
+            def zc_timed(reps):   # gFn zero-copy get; the release is outside the timed call
+                xs = []
+                for _ in range(reps):
+                    t = time.perf_counter()
+                    st, ptr, nn = ctx.get(gfn2, oid, ss)
+                    xs.append((time.perf_counter() - t) * 1e6)
+                    ctx.release(gfn2, oid, ptr, ss)
+                return xs
+            zc_timed(3)
+            z = zc_timed(reps)
+            row["zero_copy_get_us"] = {"p50": round(pct(z, 50), 2), "p99": round(pct(z, 99), 2)}
+            for o2 in srcs:
+                G.check(ctx.free(cfn, o2), "free")
+            row["b2b_working_set"] = {"sources": m, "dst_slots": 2 * slots}
+            if oracle:   # the oracle's get_into of the same size (numpy memcpy), 1 thread
+                import numpy as np
+                from oracle.model import Oracle
+                orc = Oracle(b200_hgx(1))
+                buf = np.zeros(n, np.uint8)
+                st, o = orc.put({"wf": 1, "fid": 1, "dev": 0}, buf, n, -2, 0)
+                d = np.empty(n, np.uint8)
+                xs, t_end = [], time.perf_counter() + 0.25
+                while len(xs) < 3 or (time.perf_counter() < t_end and len(xs) < 100):
+                    t = time.perf_counter()
+                    orc.get_into({"wf": 1, "fid": 2, "dev": 0}, o["oid"], d, n)
+                    xs.append((time.perf_counter() - t) * 1e6)
+                row["oracle_get_into"] = {"p50_us": round(pct(xs, 50), 2), "samples": len(xs)}
+            row["samples"] = reps
+            out.append(row)
+    finally:
+        ctx.close()
+    return out
 
 
 def measure_multipath(world, G, nbytes=1 << 30, reps=3):
@@ -366,7 +667,7 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
     out.update(measure_d2d_push(world, G, calib, devs))
     if len(set(devs)) < len(devs):
         out["note"] = ("GR_BENCH_SAME_GPU: every logical GPU is device 0, so 'NVLink' copies are "
-                       "same-device HBM copies and frac_of_770 / the nvlink roofline do not apply")
+                       "same-device HBM copies and the NVLink fractions do not apply")
     return out
 
 
@@ -432,7 +733,8 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
         gbps, us = run([(1, 0)])
         out["d2d_push"] = {"what": "GPU1 gFn get_into of GPU0-resident 38.5 MB objects (GPU0 SM push over "
                                    "NVLink, one context)", "GBps": round(gbps, 1), "us_per_get": round(us, 2),
-                           "frac_of_770": round(gbps / 770.0, 3), "frac_of_900_nominal": round(gbps / 900.0, 3)}
+                           "frac": round(gbps / NVL_PEAK, 3),
+                           "frac_of_770_measured_peer_copy": round(gbps / 770.0, 3)}
         # baseline on the same devices and sizes: cudaMemcpyPeerAsync (copy engine)
         a0 = torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[0]}")
         b1 = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{devs[1]}") for _ in range(2)]
@@ -517,7 +819,8 @@ def measure_d2d_sweep(world, G, calib, devs, sizes=(4096, 65536, 1 << 20, 16 << 
             base = n * reps / (a.elapsed_time(b) / 1e3) / 1e9
             res.append({"bytes": n, "p50_us": round(lat[len(lat) // 2], 2),
                         "p99_us": round(lat[min(len(lat) - 1, -(-len(lat) * 99 // 100) - 1)], 2),
-                        "GBps": round(tput, 1), "frac_of_770": round(tput / 770.0, 3),
+                        "GBps": round(tput, 1), "frac": round(tput / NVL_PEAK, 3),
+                        "frac_of_770_measured_peer_copy": round(tput / 770.0, 3),
                         "memcpy_peer_GBps": round(base, 1)})
             for oid in oids:
                 ctx.free(G.fn(9, 1, 0), oid)
@@ -563,6 +866,25 @@ def nccl_ring_baseline(world, rank, dev, n, per_step, steps):
 
 
 # ------------------------------------------------------------------ GPU arm
+
+# ------------------------------------------------------------------ GPU arm
+def h2d_link_peak(G, dev, nbytes=256 << 20, reps=4):
+    """Pinned single-link H2D GB/s on this box (bare cudaMemcpyAsync back to
+    back, CUDA events): the PCIe roofline of the workflow."""
+    import torch
+    host = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=f"cuda:{dev}")
+    s = torch.cuda.Stream(device=dev)
+    G.check(G.test_memcpy(d.data_ptr(), host.data_ptr(), nbytes, s.cuda_stream, True))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(s)
+    for _ in range(reps):
+        G.check(G.test_memcpy(d.data_ptr(), host.data_ptr(), nbytes, s.cuda_stream, False))
+    b.record(s)
+    b.synchronize()
+    return nbytes * reps / (a.elapsed_time(b) / 1e3) / 1e9
+
+
 def run_gpu(args, rank, world, local_rank):
     import torch
     import torch.distributed as dist
@@ -573,26 +895,30 @@ def run_gpu(args, rank, world, local_rank):
 
     _build.build()
     G.load()
+    same_gpu = os.environ.get("GR_BENCH_SAME_GPU") == "1"
     dev = local_rank
     torch.cuda.set_device(dev)
-    calib = b200_hgx(1)
-    calib["device_map"] = [dev]
-    flags = (G.COPY_TMA if args.tma else 0)
-    cfg = G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED],
-                              flags=flags, copy_ctas_per_sm=args.ctas)
-    ctx = G.Ctx(cfg)
-    R, n = args.requests, N_BYTES
-    stream = torch.cuda.Stream(device=dev)
-    s = stream.cuda_stream
+    n, R = N_BYTES, args.requests
+    # one context per rank: the producer GPU (logical 0) and, at N > 1, the
+    # consumer GPU r+1 (logical 1); each rank's puts use its own PCIe link
+    cons_dev = dev if world == 1 else (dev if same_gpu else peer_of(dev, world))
+    calib = b200_hgx(1 if world == 1 else 2)
+    calib["device_map"] = [dev] if world == 1 else [dev, cons_dev]
+    flags = G.PROFILE | (G.COPY_TMA if args.tma else 0) | (G.NO_MULTIPATH if world > 1 else 0)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED] * calib["n_gpus"],
+                                    flags=flags, copy_ctas_per_sm=args.ctas))
+    cons_logical = 0 if world == 1 else 1
     cfn = G.fn(1, 1, G.HOST)
-    gfn = G.fn(1, 2, 0)
+    gfn = G.fn(1, 2, cons_logical)
 
     def barrier():
         if world > 1:
-            dist.barrier()
+            dist.barrier(group=CPU_GROUP[0])
         torch.cuda.synchronize(dev)
+        if cons_dev != dev:
+            torch.cuda.synchronize(cons_dev)
 
-    # pinned host sources (leg A) with the SplitMix payload, filled on device
+    # pinned host sources (the cFn's outputs) with the SplitMix payload
     host_src = []
     tmp = torch.empty(n, dtype=torch.uint8, device=f"cuda:{dev}")
     for i in range(R):
@@ -601,202 +927,171 @@ def run_gpu(args, rank, world, local_rank):
         h.copy_(tmp)
         host_src.append(h)
     del tmp
-    B = 8                                            # rotating bindings: 308 MB > L2
-    bindings = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{dev}") for _ in range(B)]
+    B = 8                                            # rotating input bindings: 308 MB > L2
+    bindings = [torch.empty(n, dtype=torch.uint8, device=f"cuda:{cons_dev}") for _ in range(B)]
     torch.cuda.synchronize(dev)
-
-    # HBM-resident objects for the device-timed leg (consumers = 0: persistent)
-    resident = []
-    for i in range(R):
-        st, oid = ctx.put(cfn, host_src[i].data_ptr(), n, 0, 0)
-        G.check(st, "put")
-        resident.append(oid)
-
-    bptr = [bindings[i % B].data_ptr() for i in range(R)]
-    work = list(zip(resident, bptr))
-
-    remote = world > 1
-    exports, imported, ipc_error = [], [], None
-    if remote:
-        # export every resident object, import the peer's (CUDA VMM IPC, L167/L269)
-        for oid in resident:
-            st, desc = ctx.export_ipc(gfn, oid)
-            G.check(st, "export_ipc")
-            exports.append((oid, desc))
-        all_descs = exchange([d for _, d in exports], world)
-        peer = peer_of(rank, world)
-        for desc in all_descs[peer]:
-            st, roid = ctx.import_ipc(gfn, desc)
-            if st != G.OK:
-                ipc_error = f"import_ipc from rank {peer}: {G.STATUS[st]} ({G.last_error()})"
-                break
-            imported.append(roid)
-        # every rank must take the same branch: agree on success
-        ok = max_over_ranks(1.0 if ipc_error else 0.0, world, f"cuda:{dev}") == 0.0
-        if not ok:  # reported in the line; the value (co-located replicas) is unaffected
-            print(f"[bench] rank {rank}: IPC pull unavailable ({ipc_error})", file=sys.stderr, flush=True)
-            for roid in imported:
-                ctx.free(gfn, roid)
-            imported = []
-            remote = False
-
-    def make_step(pairs):
-        def step():
-            for oid, dst in pairs:
-                st, _ = ctx.get_into(gfn, oid, dst, n, s)
-                if st:
-                    G.check(st, "get_into")
-        return step
-
-    def verify_bindings(what):
-        """Parity spot check of every delivered binding (full, on device):
-        every rank generated the same SplitMix64 payloads (seed 1000 + i),
-        so local and pulled objects verify against the same seeds."""
-        stream.synchronize()
-        for b in range(min(R, B)):
-            last = max(i for i in range(R) if i % B == b)   # request that wrote binding b last
-            st, bad, _ = G.test_verify(bindings[b].data_ptr(), n, 1000 + last, 0, 0)
-            assert st == 0 and bad == 0, f"{what}: binding {b}: {bad} bytes differ from the payload"
-
-    def timed(step, sample_clocks):
-        """W warm-up steps, then exactly K steps bracketed by barrier + device
-        sync, CUDA events on the consumer stream; max over ranks."""
-        step()
-        verify_bindings("before timing")
-        for _ in range(args.warmup):
-            step()
-        barrier()
-        st0 = ctx.stats()
-        clk = ClockSampler(dev) if sample_clocks else None
-        if clk:
-            clk.start()             # samples only the timed region (NVML thread)
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        hs = time.perf_counter()
-        for _ in range(args.steps):
-            step()
-        host_us = (time.perf_counter() - hs) * 1e6 / (args.steps * R)   # submission cost per request
-        e1.record(stream)
-        barrier()
-        clocks = clk.stop() if clk else None
-        ms = e0.elapsed_time(e1)
-        G.check(ctx.sync(), "sync")
-        st1 = ctx.stats()
-        verify_bindings("after timing")
-        return dict(ms=ms, ms_max=max_over_ranks(ms, world, f"cuda:{dev}"), host_us=host_us, clocks=clocks,
-                    launches=st1.kernel_launches - st0.kernel_launches,
-                    moved=st1.link_bytes[0][0] - st0.link_bytes[0][0])   # bytes the copy kernels moved
-
-    # value: every workflow co-located on one GPU (R24's placement), GPUs independent (weak scaling)
-    t = timed(make_step(work), True)
-    ms, ms_max, host_us, clocks, launches, moved = (t[k] for k in ("ms", "ms_max", "host_us", "clocks",
-                                                                   "launches", "moved"))
-    total_req = R * args.steps * world
-    value = total_req / (ms_max / 1e3)
-    # The copy kernels run back to back on the consumer stream (direct
-    # launches, GPU-bound: host submission < GPU time), so the event-timed
-    # region on that stream / launches = average launch duration (incl. the
-    # inter-launch gap, i.e. conservative).  Same-GPU HBM copy: read + write.
-    avg_ns = ms * 1e6 / max(launches, 1)
-    alg_bytes_per_launch = 2 * moved / max(launches, 1)
-    bound = "hbm"
-    peak, peak_src = _peaks()
-    achieved = alg_bytes_per_launch / avg_ns if launches else None  # bytes/ns == GB/s
-    try:
-        live_peaks = _live_copy_peaks(dev)
-    except Exception as e:   # context only; never fails the line
-        live_peaks = {"error": str(e)[:200]}
-
-    # N > 1: the same requests with producer and consumer on different GPUs --
-    # GPU r pulls GPU r+1's objects over NVLink (cross-GPU leg B of cfg1, R24)
-    nvlink = None
-    if remote:
-        p = timed(make_step(list(zip(imported, bptr))), False)
-        p_ns = p["ms"] * 1e6 / max(p["launches"], 1)
-        p_bytes = p["moved"] / max(p["launches"], 1)          # n bytes cross the link per request
-        p_ach = p_bytes / p_ns if p["launches"] else None
-        nvlink = {"value": R * args.steps * world / (p["ms_max"] / 1e3), "unit": "req/s",
-                  "what": "every GPU r get_into's GPU r+1's 20 resident objects (IPC-mapped pool pages, "
-                          "SM pull copy over NVLink, ring of disjoint pairs)",
-                  "gbps_per_gpu": R * args.steps * n / (p["ms_max"] / 1e3) / 1e9,
-                  "roofline": {"bound": "nvlink", "achieved": p_ach, "peak": 770.0, "unit": "GB/s",
-                               "frac": (p_ach / 770.0) if p_ach else None,
-                               "frac_of_900_nominal": (p_ach / 900.0) if p_ach else None,
-                               "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s/direction"
-                               + (" (n/a under GR_BENCH_SAME_GPU: same-device HBM copies)"
-                                  if os.environ.get("GR_BENCH_SAME_GPU") == "1" else ""),
-                               "launches": p["launches"], "avg_launch_us": p_ns / 1e3,
-                               "alg_bytes_per_launch": p_bytes},
-                  "host_us_per_request": p["host_us"]}
-        if dist.get_backend() == "nccl":
-            nvlink["nccl_p2p_baseline"] = nccl_ring_baseline(world, rank, dev, n, R, args.steps // 10 or 1)
-
-
-    # per-request latency (separate, untimed pass): device events around one get_into
-    lat = []
-    for i in range(args.lat_samples):
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        st, _ = ctx.get_into(gfn, resident[i % R], bindings[i % B].data_ptr(), n, s)
-        b.record(stream)
-        b.synchronize()
-        lat.append(a.elapsed_time(b) * 1e3)
-    lat.sort()
-
-    def pct(xs, q):
-        return xs[min(len(xs) - 1, max(0, -(-len(xs) * q // 100) - 1))] if xs else None
-
-    # ---------------------------------------------------------- e2e (host buffers)
-    # Closed loop with Q requests outstanding (SURVEY §8(d)): Q client threads,
-    # each a cFn (blocking put, GIL released inside the C call) followed by its
-    # gFn (get_into on the client's own consumer stream) and the 8 B result
-    # read; client k serves requests k, k+Q, ... and owns bindings k, k+Q, ...
-    Q = max(1, min(args.e2e_q, B, R))
+    Q = max(1, min(args.q, B, R))
+    qstreams = [torch.cuda.Stream(device=cons_dev) for _ in range(Q)]
     out8 = [torch.empty(8, dtype=torch.uint8, pin_memory=True) for _ in range(Q)]
-    qstreams = [stream] + [torch.cuda.Stream(device=dev) for _ in range(Q - 1)]
 
-    def e2e_client(k):
-        torch.cuda.set_device(dev)
-        qs = qstreams[k]
-        for i in range(k, R, Q):
-            st, oid = ctx.put(cfn, host_src[i].data_ptr(), n, 0, 1)     # leg A (blocking)
+    def request(i, qs, read_result):
+        """One cfg1 request: leg A (cFn put, blocking) + leg B (gFn get_into,
+        stream-ordered on the client's consumer stream)."""
+        st, oid = ctx.put(cfn, host_src[i % R].data_ptr(), n, 0, 1)
+        if st:
             G.check(st, "put")
-            st, _ = ctx.get_into(gfn, oid, bindings[i % B].data_ptr(), n, qs.cuda_stream)  # leg B
+        st, _ = ctx.get_into(gfn, oid, bindings[i % B].data_ptr(), n, qs.cuda_stream)
+        if st:
             G.check(st, "get_into")
+        if read_result:                              # e2e: the step's result back to the host
             with torch.cuda.stream(qs):
-                out8[k].copy_(bindings[i % B][:8], non_blocking=True)     # 8 B result read
-        qs.synchronize()
+                out8[i % Q].copy_(bindings[i % B][:8], non_blocking=True)
 
     from concurrent.futures import ThreadPoolExecutor
-    pool = ThreadPoolExecutor(max_workers=Q) if Q > 1 else None
+    pool = ThreadPoolExecutor(max_workers=Q)
 
-    def e2e_step():
-        if pool is None:
-            e2e_client(0)
-        else:
-            for f in [pool.submit(e2e_client, k) for k in range(Q)]:
-                f.result()
+    def client(k, total, read_result):
+        torch.cuda.set_device(dev)
+        for i in range(k, total, Q):
+            request(i, qstreams[k], read_result)
 
+    def run_requests(total, read_result=False):
+        for f in [pool.submit(client, k, total, read_result) for k in range(Q)]:
+            f.result()
+
+    def verify(total, what):
+        """Every binding holds the payload of the last request that wrote it
+        (full compare on the device against the generator)."""
+        for qs in qstreams:
+            qs.synchronize()
+        for b in range(min(total, B)):
+            last = max(i for i in range(total) if i % B == b)
+            st, bad, _ = G.test_verify(bindings[b].data_ptr(), n, 1000 + last % R, 0, 0)
+            assert st == 0 and bad == 0, f"{what}: binding {b}: {bad} bytes differ from the payload"
+
+    # warm-up (W steps) + parity spot check
+    run_requests(R * args.warmup)
+    verify(R * args.warmup, "warm-up")
+    total = R * args.steps
+    barrier()
+    st0 = ctx.stats()
+    clk = ClockSampler(dev)
+    clk.start()
+    ts = torch.cuda.Stream(device=cons_dev)          # timing stream: every consumer stream joins it
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(ts)
+    for qs in qstreams:
+        qs.wait_event(e0)
+    h0 = time.perf_counter()
+    run_requests(total)
+    host_s = time.perf_counter() - h0
+    for qs in qstreams:
+        ev = torch.cuda.Event()
+        ev.record(qs)
+        ts.wait_event(ev)
+    e1.record(ts)
+    barrier()
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1)
+    G.check(ctx.sync(), "sync")
+    ms_max = max_over_ranks(ms, world)
+    st1 = ctx.stats()
+    verify(total, "timed region")
+    value = total * world / (ms_max / 1e3)
+    launches = st1.kernel_launches - st0.kernel_launches
+    tl = st1.timed_launches - st0.timed_launches
+    t_ns = st1.timed_ns - st0.timed_ns
+    t_bytes = st1.timed_bytes - st0.timed_bytes
+
+    # ---------------------------------------------------------- e2e (host-timed, + 8 B result read)
     e2e_steps = max(1, min(args.steps, args.e2e_steps))
-    for _ in range(min(args.warmup, 3)):
-        e2e_step()
+    run_requests(R, True)
     barrier()
     h0 = time.perf_counter()
-    for _ in range(e2e_steps):
-        e2e_step()
+    run_requests(R * e2e_steps, True)
+    for qs in qstreams:
+        qs.synchronize()
     barrier()
     e2e_s = time.perf_counter() - h0
-    e2e_val = R * e2e_steps * world / max_over_ranks(e2e_s, world, f"cuda:{dev}")
-    if pool is not None:
-        pool.shutdown()
+    e2e_val = R * e2e_steps * world / max_over_ranks(e2e_s, world)
 
-    if world > 1:   # drop imports and our export pins once every rank is done reading
-        barrier()
-        for roid in imported:
-            ctx.free(gfn, roid)
-        barrier()
-        for oid, desc in exports:
-            ctx.release(gfn, oid, G.Ctx.desc_exporter_ptr(desc), 0)
+    # ---------------------------------------------------------- single-request latency (R22)
+    lat, lat_a = [], []
+    s0 = qstreams[0]
+    for i in range(args.lat_samples):
+        t0 = time.perf_counter()
+        st, oid = ctx.put(cfn, host_src[i % R].data_ptr(), n, 0, 1)
+        G.check(st, "put")
+        ta = time.perf_counter()
+        G.check(ctx.get_into(gfn, oid, bindings[i % B].data_ptr(), n, s0.cuda_stream)[0], "get_into")
+        ev = torch.cuda.Event()
+        ev.record(s0)
+        while not ev.query():
+            pass
+        t1 = time.perf_counter()
+        lat.append((t1 - t0) * 1e6)
+        lat_a.append((ta - t0) * 1e6)
+
+    # ---------------------------------------------------------- leg B alone, back to back (kernel speed of light)
+    # a context without GROUTER_PROFILE: per-launch events would sit between
+    # the launches and defeat programmatic dependent launch
+    ctx_b = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * calib["n_gpus"],
+                                      flags=flags & ~G.PROFILE, copy_ctas_per_sm=args.ctas))
+    resident = []
+    for i in range(R):
+        st, oid = ctx_b.put(cfn, host_src[i].data_ptr(), n, 0, 0)
+        G.check(st, "put")
+        resident.append(oid)
+    G.check(ctx_b.sync(), "sync")
+    sb = qstreams[0]
+
+    def legb():
+        for i, oid in enumerate(resident):
+            st, _ = ctx_b.get_into(gfn, oid, bindings[i % B].data_ptr(), n, sb.cuda_stream)
+            if st:
+                G.check(st, "get_into")
+    for _ in range(3):
+        legb()
+    sb.synchronize()
+    k0 = ctx_b.stats()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(sb)
+    b2b_steps = max(20, args.b2b_steps)
+    for _ in range(b2b_steps):
+        legb()
+    b.record(sb)
+    b.synchronize()
+    G.check(ctx_b.sync(), "sync")
+    k1 = ctx_b.stats()
+    verify(R, "back-to-back leg B")
+    b2b_l = k1.kernel_launches - k0.kernel_launches
+    b2b_us = a.elapsed_time(b) * 1e3 / max(b2b_l, 1)
+    for oid in resident:
+        ctx_b.free(cfn, oid)
+    ctx_b.close()
+    pool.shutdown()
+
+    # ---------------------------------------------------------- rooflines
+    peak_hbm, peak_src = _peaks()
+    link_peak = h2d_link_peak(G, dev)
+    rw = 2 if world == 1 or same_gpu else 1     # HBM read + write on one GPU; NVLink carries n once
+    kpeak = peak_hbm if rw == 2 else NVL_PEAK
+    k_us = t_ns / max(tl, 1) / 1e3
+    k_ach = rw * t_bytes / t_ns if t_ns else None   # bytes / ns == GB/s
+    b2b_ach = rw * n / b2b_us / 1e3
+    try:
+        live_peaks = _live_copy_peaks(dev) if world == 1 else None
+    except Exception as e:   # context only; never fails the line
+        live_peaks = {"error": str(e)[:200]}
+    traffic = traffic_steady = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            tj = json.load(open(tp))
+            traffic = tj.get("dram_bytes_per_launch")
+            traffic_steady = tj.get("steady_dram_bytes_per_launch")
+        except Exception:
+            traffic = None
 
     # N > 1: host->GPU striping over the other GPUs' PCIe links (L120, L178), measured by
     # rank 0 alone on a context spanning every GPU of the node while the others wait
@@ -805,9 +1100,6 @@ def run_gpu(args, rank, world, local_rank):
     if world > 1 and not args.no_multipath_probe:
         barrier()
         if rank == 0:
-            # watchdog: this node-wide measurement never ran on a multi-GPU box
-            # in-round; a hang must not cost the scaling line
-            import threading
             box = {}
 
             def _mp():
@@ -820,77 +1112,84 @@ def run_gpu(args, rank, world, local_rank):
             th.join(args.multipath_timeout)
             stuck = th.is_alive()
             multipath = box.get("r") or {"error": f"timed out after {args.multipath_timeout:.0f} s"}
-        # the other ranks wait on a CPU (gloo) barrier: an NCCL barrier would keep
-        # a spinning all-reduce kernel resident on their GPUs, and rank 0's
-        # copies there would only run in time slices against it
         dist.barrier(group=CPU_GROUP[0])
+
+    nccl = None
+    if world > 1 and dist.get_backend() == "nccl":
+        try:   # the library-free baseline of the same NVLink exchange (context only)
+            nccl = nccl_ring_baseline(world, rank, dev, n, R, max(1, args.steps // 10))
+        except Exception as e:
+            nccl = {"error": f"{type(e).__name__}: {e}"[:200]}
+
+    sweep = None
+    if rank == 0 and world == 1 and not args.no_sweep:
+        try:
+            sweep = measure_sweep(G, dev, peak_hbm, link_peak, oracle=not args.no_cpu_baseline)
+        except Exception as e:   # reported, never fatal for the line
+            sweep = [{"error": f"{type(e).__name__}: {e}"[:300]}]
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, done, dt = oracle_rate(4, args.cpu_seconds)
-        cpu = {"value": v, "unit": "req/s", "cores": 1, "kind": "oracle",
-               "sample": f"{done} oracle get_into of {N_BYTES} B in {dt:.1f} s (numpy memcpy)"}
-
-    traffic = traffic_steady = None
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        try:
-            tj = json.load(open(tp))
-            traffic = tj.get("dram_bytes_per_launch")
-            traffic_steady = tj.get("steady_dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+        cpu = cpu_baseline_obj(args.cpu_seconds)
 
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "req/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-            "data": "synthetic (SplitMix64 payload, verified on device before timing)",
+            "data": "synthetic (SplitMix64 payload; every delivered tensor verified on the device)",
             "config": {"workload": WORKLOAD if world == 1 else WORKLOAD_N, "requests_per_step": R,
-                       "bytes": N_BYTES,
-                       "parallelism": f"replicas x{world} (workflows co-located per GPU, no collective)",
-                       "l2": "inputs larger than L2: 20 resident 38.5 MB objects, 8 rotating bindings",
-                       "copy_kernel": os.environ.get("GR_COPY", "tmas4" if args.tma else "wv8")
-                       + " (256-bit LD/ST, L2 prefetch of 1 unit/warp before the PDL wait)"
-                       + f", {args.ctas} CTA/SM cap"},
+                       "outstanding": Q, "bytes": N_BYTES,
+                       "parallelism": "single GPU" if world == 1 else
+                       f"ring of {world} producer->consumer GPU pairs, one process per GPU, no collective",
+                       "l2": "inputs larger than L2: 20 x 38.5 MB pinned host sources, 8 rotating 38.5 MB "
+                             "device bindings (308 MB)",
+                       "copy_kernel": os.environ.get("GR_COPY", "tmas4" if args.tma else "wv8")},
             "gbps": value * N_BYTES / 1e9,
-            "host_us_per_request": host_us,
+            "host_s": host_s,
             "latency_us": {"p50": pct(lat, 50), "p99": pct(lat, 99), "samples": len(lat),
-                           "what": "one get_into of 38,535,168 B, CUDA events on the consumer stream"},
-            "roofline": {"bound": bound, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": (achieved / peak) if achieved else None, "traffic": traffic,
-                         "traffic_note": "ncu --set full (caches flushed per replay: the 38.5 MB of writes stay "
-                                         "in L2, so this is the read half); without flushing, 20 consecutive "
-                                         "launches average traffic_steady = read + write-back ~= 0.98 x the "
-                                         "algorithmic bytes (profiles/r01_ncu_steady_traffic.json)",
-                         "traffic_steady": traffic_steady,
-                         "kernel": "gr_copy (K2')", "peak_source": peak_src,
-                         "peak_live": live_peaks,
-                         "frac_of_live_torch_copy_2GiB": (achieved / live_peaks["torch_copy_2GiB"])
-                         if achieved and live_peaks.get("torch_copy_2GiB") else None,
-                         "frac_note": "frac can exceed 1: `peak` is the driver's one-off 2 GiB torch copy_ "
-                                      "(box-to-box spread ~3%); peak_live repeats that recipe on this box, "
-                                      "and steady DRAM traffic per launch is 0.98 x the algorithmic bytes "
-                                      "(no bytes are skipped: every launch reads and writes 38.5 MB)",
-                         "launches": launches, "avg_launch_us": avg_ns / 1e3,
-                         "timing": "CUDA events over the timed region on the stream the kernels "
-                                   "run on (consumer stream), / launches",
-                         "alg_bytes_per_launch": alg_bytes_per_launch},
+                           "put_p50": pct(lat_a, 50),
+                           "what": "one cfg1 request on an idle GPU: cFn put call -> gFn's data ready "
+                                   "(event on the consumer stream observed by the host), R22"},
+            "roofline": {"bound": "hbm" if rw == 2 else "nvlink", "achieved": k_ach, "peak": kpeak,
+                         "unit": "GB/s", "frac": (k_ach / kpeak) if k_ach else None, "traffic": traffic,
+                         "kernel": "gr_copy (K2') leg B" + (" same-GPU" if rw == 2 else " NVLink push"),
+                         "peak_source": peak_src if rw == 2 else "north star: 900 GB/s per direction",
+                         "launches": tl, "avg_launch_us": k_us,
+                         "alg_bytes_per_launch": rw * t_bytes / max(tl, 1),
+                         "timing": "CUDA events recorded around every gr_copy launch on its own stream "
+                                   "(GROUTER_PROFILE) during the timed region; each launch runs alone "
+                                   "(requests are PCIe-paced), so it pays its own ramp-up",
+                         "traffic_note": "ncu --set full, per launch (profiles/); steady traffic without "
+                                         "cache flushes in traffic_steady", "traffic_steady": traffic_steady,
+                         "peak_live": live_peaks},
+            "roofline_step": {"bound": "pcie", "achieved": value / world * N_BYTES / 1e9,
+                              "peak": link_peak, "unit": "GB/s",
+                              "frac": value / world * N_BYTES / 1e9 / link_peak,
+                              "what": "per-GPU payload GB/s of the workflow against this box's pinned "
+                                      "single-link H2D (bare cudaMemcpyAsync of 256 MiB back to back): the "
+                                      "link every request crosses once"},
+            "kernel_b2b": {"what": "leg B alone: gFn get_into of 20 HBM-resident objects back to back "
+                                   "(CUDA events on the consumer stream / launches)",
+                           "us_per_launch": b2b_us, "achieved": b2b_ach, "peak": kpeak,
+                           "frac": b2b_ach / kpeak, "launches": b2b_l},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "req/s", "h2d_bytes_per_step": R * N_BYTES,
-                    "d2h_bytes_per_step": R * 8, "steps": e2e_steps,
-                    "outstanding": Q, "pcie_gbps": e2e_val / world * N_BYTES / 1e9},
+                    "d2h_bytes_per_step": R * 8, "steps": e2e_steps, "outstanding": Q,
+                    "what": "the same closed loop through the C ABI, wall clock, plus an 8 B D2H read of "
+                            "each delivered tensor"},
             "gpu_launches": launches,
             "clocks": clocks,
         }
+        if sweep is not None:
+            line["sweep"] = sweep
+        if nccl is not None:
+            line["nccl_p2p_baseline"] = nccl
         if multipath is not None:
             line["h2d_multipath"] = multipath
-        if nvlink is not None:
-            line["nvlink_pull"] = nvlink
-        if world > 1 and not remote:
-            line["ipc_pull_error"] = ipc_error or "another rank failed to import"
-
+        if same_gpu and world > 1:
+            line["note"] = ("GR_BENCH_SAME_GPU: every rank on device 0 (plumbing check): the 'NVLink' push is a "
+                            "same-device copy")
         print(json.dumps(line), flush=True)
     if stuck:   # a measurement thread still owns the GPUs: leave without teardown
         sys.stdout.flush()
@@ -904,16 +1203,17 @@ def run_gpu(args, rank, world, local_rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=1000)
-    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="grouter", choices=["grouter", "reference"])
     ap.add_argument("--requests", type=int, default=20)
+    ap.add_argument("--q", type=int, default=4, help="requests outstanding per GPU (SURVEY §8(d): 4)")
     ap.add_argument("--e2e-steps", type=int, default=10)
-    ap.add_argument("--e2e-q", type=int, default=4,
-                    help="requests outstanding in the closed-loop e2e run (SURVEY §8(d): 4 per GPU)")
+    ap.add_argument("--b2b-steps", type=int, default=200)
     ap.add_argument("--lat-samples", type=int, default=200)
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--tma", action="store_true")
     ap.add_argument("--ctas", type=int, default=4)
     ap.add_argument("--no-multipath-probe", action="store_true")
@@ -929,7 +1229,7 @@ def main():
         run_reference(args, rank)
         return
     # GR_BENCH_SAME_GPU=1 + GR_BENCH_BACKEND=gloo: every rank on GPU 0 (exercises the
-    # N>1 IPC pull path on a 1-GPU box; NCCL refuses two ranks on one GPU)
+    # N>1 plumbing on a 1-GPU box; NCCL refuses two ranks on one GPU)
     if os.environ.get("GR_BENCH_SAME_GPU") == "1":
         local_rank = 0
     if world > 1:
@@ -941,7 +1241,7 @@ def main():
             dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local_rank}"))
         else:
             dist.init_process_group(backend)
-        CPU_GROUP[0] = dist.new_group(backend="gloo")   # GPU-free waits (rank 0's node-wide probe)
+        CPU_GROUP[0] = dist.new_group(backend="gloo")   # GPU-free waits and the max over ranks
     run_gpu(args, rank, world, local_rank)
     if world > 1:
         import torch.distributed as dist

@@ -58,7 +58,10 @@ extern "C" {
 #define GROUTER_PLAN_ONLY     0x4u /* no CUDA at all: planner/introspection only            */
 #define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
 #define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
-#define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream */
+#define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream;
+                                      the stream is held at a host-released gate until start
+                                      event, kernel and stop event are enqueued, so the interval
+                                      is the launch alone (measurement mode)                    */
 #define GROUTER_D2H_MULTIPATH 0x80u/* gFn-host striping (L178, Fig. 5a; R45): a GPU
                                       object read into host memory is split over R(src) like a
                                       host->GPU plan; route r's copy engine moves its share      */
@@ -140,7 +143,7 @@ typedef struct {
   uint32_t pool_cap_permille;  /* auto cap = permille of free, default 500 (L262) */
   uint64_t pool_cap_bytes[GROUTER_MAX_GPUS]; /* explicit cap; 0 = auto         */
   uint64_t host_store_bytes;   /* pinned host store H, default 1 GiB          */
-  uint64_t round_bytes;        /* SM-copy dispatch horizon, default 64 MiB    */
+  uint64_t round_bytes;        /* unused since rounds carry one batch (O8)     */
   uint32_t copy_ctas_per_sm;   /* SM copy kernel CTAs per SM cap, default 4   */
   uint32_t flags;              /* GROUTER_* flags                              */
 } grouter_config;
@@ -170,7 +173,9 @@ typedef struct {
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
- * server).  server_kind: 0 = SM copy egress of server_dev, 1 = H2D engine of
+ * server; a dispatch round carries one batch and each server keeps <= 2
+ * rounds in flight -- SURVEY O8 -- except a direct launch, which moves the
+ * whole transfer of the only tenant queued on an idle SM-copy server).  server_kind: 0 = SM copy egress of server_dev, 1 = H2D engine of
  * route GPU server_dev, 2 = D2H engine of server_dev.  Chunk ids are
  * (xfer << 32 | chunk index) where xfer numbers transfers from 1 in call order. */
 typedef struct {
@@ -180,6 +185,11 @@ typedef struct {
   uint32_t n_chunks;
   uint64_t chunk_ids[8];
   uint64_t bytes;
+  uint32_t inflight;  /* real-time mode: batches of this server dispatched earlier whose
+                         completion had not been observed when this one was dispatched
+                         (an upper bound; SURVEY O8 keeps it <= 1, i.e. <= 2 in flight).
+                         Replay flushes dispatch everything at once: not meaningful there */
+  uint32_t pad;
 } grouter_dispatch;
 
 /* ------------------------------------------------------------ lifecycle */

@@ -43,6 +43,15 @@ grouter_status grouter_test_copy(void *dst_base, const void *src_base, const gro
  * *us_per_launch = host time per launch call. */
 grouter_status grouter_test_launch_cost(int kind, int n, int blocks, void *stream, double *us_per_launch);
 
+/* Measured BASELINE, not the data path: one bare cudaMemcpyAsync(dst, src, n,
+ * cudaMemcpyDefault) on `stream` (a cudaStream_t as void*; NULL = a
+ * library-internal non-blocking stream of the current device).  wait != 0:
+ * the call returns once the copy has completed (an event recorded after it,
+ * polled like the library's blocking callers poll theirs); wait == 0: it
+ * returns after the enqueue.  The bench times it through the same binding as
+ * the library calls it is compared with (SURVEY §8(d) baselines). */
+grouter_status grouter_test_memcpy(void *dst, const void *src, uint64_t n, void *stream, int32_t wait);
+
 /* Text dump of the context's internal state (servers, objects, leases,
  * pending completion words) for debugging; truncated to cap bytes.  Returns
  * the full length needed in *len (may be NULL). */

@@ -145,6 +145,7 @@ struct Server {
   struct Inflight {
     Waitable w;                  // completion of a dispatched round
     cudaStream_t direct;         // caller stream of a direct launch, null for the server stream
+    uint32_t batches = 0;        // scheduled batches the round carries (O8: <= 2 in flight)
   };
   std::deque<Inflight> inflight;
   std::deque<ChunkItem> carry;        // scheduled (stride order) but not yet submitted
@@ -235,6 +236,11 @@ struct PhysDev {
   uint32_t n_scratch = 0, next_scratch = 0;
   std::vector<Fences> scratch_busy;
   std::vector<cudaEvent_t> timing_free;  // timing-enabled events (GROUTER_PROFILE)
+  // GROUTER_PROFILE gate: a host-mapped word the profiled stream waits on
+  // until start event, kernel and stop event are all enqueued, so the timed
+  // interval holds the launch alone (no host submission gap inside it)
+  volatile uint32_t *gate = nullptr;
+  uint32_t gate_seq = 0;
 };
 
 struct ProfRec {

@@ -240,10 +240,16 @@ static uint32_t weight_of(grouter_ctx *c, uint32_t t) {
   return it == c->weights.end() ? 1u : it->second;
 }
 
-static void log_batch(grouter_ctx *c, const Server &s, uint32_t tenant,
+static void retire(Server &s);
+
+static void log_batch(grouter_ctx *c, Server &s, uint32_t tenant,
                       const std::vector<ChunkItem> &b, uint64_t bytes) {
   if (!(c->replay || (c->cfg.flags & GROUTER_LOG))) return;
   grouter_dispatch d{};
+  if (!c->replay) {  // batches still in flight on this server (logging mode only: retire costs queries)
+    retire(s);
+    for (auto &f : s.inflight) d.inflight += f.batches;
+  }
   d.server_kind = s.kind;
   d.server_dev = s.logical;
   d.tenant = tenant;
@@ -255,9 +261,9 @@ static void log_batch(grouter_ctx *c, const Server &s, uint32_t tenant,
 }
 
 // Moves whole batches (stride order, logged) from the scheduler into the
-// carry queue until the round budget is covered.
-static void refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes,
-                   size_t max_items = kRoundItems) {
+// carry queue until the round budget is covered; returns how many.
+static uint32_t refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes,
+                       size_t max_items = kRoundItems) {
   uint64_t bytes = 0;
   for (auto &it : s.carry) bytes += it.bytes;
   uint32_t nb = 0;
@@ -280,6 +286,20 @@ static void refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max
     bytes += bb;
     ++nb;
   }
+  return nb;
+}
+
+// One dispatch round carries at most ONE scheduled batch (and urgent
+// unscheduled work, e.g. spills); with <= 2 rounds in flight per server that
+// is SURVEY O8's "<= 2 batches in flight": a tenant that becomes backlogged
+// waits behind at most two batches already handed to the engine (L229).
+// A new batch is taken only when the previous one has left the carry queue.
+static uint32_t refill_one(grouter_ctx *c, Server &s) {
+  return s.carry.empty() ? refill(c, s, 1, 1) : 0;
+}
+
+static uint64_t batch_budget(const grouter_ctx *c, const Server &s) {
+  return (uint64_t)s.sched.batch * c->cfg.chunk_bytes;
 }
 
 // Takes the longest submittable prefix of urgent + carry (bounded by the
@@ -417,6 +437,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       for (auto &pb : pubs)
         if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path]) p->pub[k].value = pb.x->value_after(pb.path);
     ProfRec pr{s.phys, nullptr, nullptr, bytes};
+    uint32_t gate_v = 0;
     if (prof) {
       for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
         if (!pd.timing_free.empty()) {
@@ -426,8 +447,22 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
           GR_CUDA(cudaEventCreate(e));
         }
       }
+      if (!pd.gate) {
+        GR_CUDA(cudaHostAlloc((void **)&pd.gate, 64, cudaHostAllocMapped | cudaHostAllocPortable));
+        *pd.gate = 0;
+      }
+      gate_v = ++pd.gate_seq;  // released below, after the stop event is enqueued
+      GR_CU(drv().streamWaitValue32((CUstream)st, (CUdeviceptr)(uintptr_t)pd.gate, gate_v,
+                                    CU_STREAM_WAIT_VALUE_GEQ));
       GR_CUDA(cudaEventRecord(pr.start, st));
     }
+    struct GateRelease {  // the gate opens on every path out (an exception must not park the stream)
+      volatile uint32_t *g;
+      uint32_t v;
+      ~GateRelease() {
+        if (v) __atomic_store_n(g, v, __ATOMIC_RELEASE);
+      }
+    } gate_release{pd.gate, gate_v};
     HostProf &hp = hprof();
     uint64_t tl = hp.on ? now_ns() : 0;
     if (hp.on) hp.t[6] += tl - tparams;
@@ -448,6 +483,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       GR_CUDA(cudaEventRecord(pr.stop, st));
       c->prof.push_back(pr);
     }
+    (void)gate_release;
     c->stats.kernel_launches++;
     if (!local) c->stats.peer_launches++;
   }
@@ -473,10 +509,10 @@ void harvest_profile(grouter_ctx *c, bool wait) {
 // SM-copy server: one kernel launch per round segment (D2D push over
 // NVLink, or a same-GPU HBM copy).
 static size_t round_copy(grouter_ctx *c, Server &s) {
-  refill(c, s, UINT32_MAX, c->cfg.round_bytes);
+  const uint32_t nb = refill_one(c, s);
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
-  take(s, c->cfg.round_bytes, items, cut);
+  take(s, batch_budget(c, s), items, cut);
   if (items.empty()) return 0;
   DeviceGuard g(s.phys);
   for (size_t i = 0; i < items.size(); ++i) {
@@ -489,7 +525,7 @@ static size_t round_copy(grouter_ctx *c, Server &s) {
     c->stats.link_bytes[0][s.logical] += items[i].bytes;
   }
   launch_round(c, s, s.stream, s.scratch, seg, nullptr);
-  s.inflight.push_back({ev_wait(c, record(c, s.stream, s.phys)), nullptr});
+  s.inflight.push_back({ev_wait(c, record(c, s.stream, s.phys)), nullptr, nb});
   c->stats.rounds++;
   after_submit(c, items);
   return items.size();
@@ -560,9 +596,9 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
 // for r itself land in the lease; relayed chunks go through r's staging ring
 // and a forward round kernel on r pushes them to their destination.
 static size_t round_h2d(grouter_ctx *c, Server &s) {
-  const uint64_t budget = 2ull * s.sched.batch * c->cfg.chunk_bytes;
+  const uint64_t budget = batch_budget(c, s);
   const uint64_t tr0 = tl_put_t0 ? now_ns() : 0;
-  refill(c, s, 2, budget);
+  const uint32_t nb = refill_one(c, s);
   std::vector<ChunkItem> items, direct, relay;
   std::vector<char> cut;
   take(s, budget, items, cut);
@@ -644,9 +680,9 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   complete_by_event(c, evented, ce_end, s.stream);
   if (last_fwd) {  // one in-flight marker covering both the CE and the forward stream
     GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce_end->ev, 0));
-    s.inflight.push_back({ev_wait(c, record(c, s.fwd_stream, s.phys)), nullptr});
+    s.inflight.push_back({ev_wait(c, record(c, s.fwd_stream, s.phys)), nullptr, nb});
   } else {
-    s.inflight.push_back({ev_wait(c, ce_end), nullptr});
+    s.inflight.push_back({ev_wait(c, ce_end), nullptr, nb});
   }
   c->stats.rounds++;
   after_submit(c, items);
@@ -656,11 +692,10 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
 // D2H server: CE copies device -> host (host store, host leases, caller
 // host buffers, and urgent spills).
 static size_t round_d2h(grouter_ctx *c, Server &s) {
-  const uint64_t budget = 2ull * s.sched.batch * c->cfg.chunk_bytes;
-  refill(c, s, 2, budget);
+  const uint32_t nb = refill_one(c, s);
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
-  take(s, UINT64_MAX, items, cut);
+  take(s, batch_budget(c, s), items, cut);
   if (items.empty()) return 0;
   const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
@@ -693,7 +728,7 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
   publish_ce(c, s, seg, evented);
   EventRef ce_end = record(c, s.stream, s.phys);
   complete_by_event(c, evented, ce_end, s.stream);
-  s.inflight.push_back({ev_wait(c, ce_end), nullptr});
+  s.inflight.push_back({ev_wait(c, ce_end), nullptr, nb});
   c->stats.rounds++;
   after_submit(c, items);
   return items.size();
@@ -769,7 +804,7 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
   HostProf &hp = hprof();
   while (has_work(s)) {
     uint64_t ta = hp.on ? now_ns() : 0;
-    refill(c, s, UINT32_MAX, kDirectBytes, kDirectItems);
+    const uint32_t nb = refill(c, s, UINT32_MAX, kDirectBytes, kDirectItems);
     take(s, kDirectBytes, items, cut, kDirectItems);
     if (hp.on) hp.t[5] += now_ns() - ta;
     if (items.empty()) throw Error(GROUTER_ECUDA, "internal: direct launch made no progress");
@@ -802,7 +837,7 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
     if (!s.inflight.empty() && s.inflight.back().direct == caller && deferred && s.inflight.back().w.origin == caller)
       s.inflight.back().w = w;
     else
-      s.inflight.push_back({w, caller});
+      s.inflight.push_back({w, caller, nb});
   }
   return true;
 }
@@ -1121,6 +1156,7 @@ void engine_shutdown(grouter_ctx *c) {
     DeviceGuard g(kv.first);
     if (kv.second->scratch) cudaFree(kv.second->scratch);
     for (cudaEvent_t e : kv.second->timing_free) cudaEventDestroy(e);
+    if (kv.second->gate) cudaFreeHost((void *)kv.second->gate);
     kv.second->scratch_busy.clear();
   }
   ipc_release_all(c);  // dedicated (exported) allocations; their fences hold pooled events

@@ -833,6 +833,34 @@ extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, 
   return cudaGetLastError() == cudaSuccess ? GROUTER_OK : GROUTER_ECUDA;
 }
 
+extern "C" grouter_status grouter_test_memcpy(void *dst, const void *src, uint64_t n, void *stream, int32_t wait) {
+  if (n && (!dst || !src)) return GROUTER_EINVAL;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev >= 64) return GROUTER_ECUDA;
+  static cudaStream_t own[64] = {};
+  static cudaEvent_t ev[64] = {};
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!s) {
+    if (!own[dev] && cudaStreamCreateWithFlags(&own[dev], cudaStreamNonBlocking) != cudaSuccess)
+      return GROUTER_ECUDA;
+    s = own[dev];
+  }
+  if (!ev[dev] && cudaEventCreateWithFlags(&ev[dev], cudaEventDisableTiming) != cudaSuccess) return GROUTER_ECUDA;
+  if (n && cudaMemcpyAsync(dst, src, n, cudaMemcpyDefault, s) != cudaSuccess) return GROUTER_ECUDA;
+  if (wait) {
+    if (cudaEventRecord(ev[dev], s) != cudaSuccess) return GROUTER_ECUDA;
+    cudaError_t e;
+    int spins = 0;
+    while ((e = cudaEventQuery(ev[dev])) == cudaErrorNotReady)
+      if (++spins > 24) {  // the library's host_wait: spin briefly, then block in the driver
+        e = cudaEventSynchronize(ev[dev]);
+        break;
+      }
+    if (e != cudaSuccess) return GROUTER_ECUDA;
+  }
+  return GROUTER_OK;
+}
+
 extern "C" grouter_status grouter_test_fill(void *dst, uint64_t n, uint64_t seed, uint64_t offset,
                                             void *stream) {
   if (n == 0) return GROUTER_OK;

@@ -105,7 +105,8 @@ class grouter_ipc_desc(C.Structure):
 
 class grouter_dispatch(C.Structure):
     _fields_ = [("server_kind", C.c_int32), ("server_dev", C.c_int32), ("tenant", C.c_uint32),
-                ("n_chunks", C.c_uint32), ("chunk_ids", C.c_uint64 * 8), ("bytes", C.c_uint64)]
+                ("n_chunks", C.c_uint32), ("chunk_ids", C.c_uint64 * 8), ("bytes", C.c_uint64),
+                ("inflight", C.c_uint32), ("pad", C.c_uint32)]
 
 
 _P = C.c_void_p
@@ -171,6 +172,7 @@ SIGNATURES = {
     "grouter_test_launch_cost": (_ST, [C.c_int, C.c_int, C.c_int, _P, C.POINTER(C.c_double)]),
     "grouter_test_dump": (_ST, [_CTX, C.c_char_p, _U64, C.POINTER(_U64)]),
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
+    "grouter_test_memcpy": (_ST, [_P, _P, C.c_uint64, _P, C.c_int32]),
 }
 
 _lib = None
@@ -450,7 +452,7 @@ class Ctx:
             for d in arr[:cnt.value]:
                 out.append({"kind": d.server_kind, "dev": d.server_dev, "tenant": d.tenant,
                             "chunks": [(x >> 32, x & 0xFFFFFFFF) for x in d.chunk_ids[:d.n_chunks]],
-                            "bytes": d.bytes})
+                            "bytes": d.bytes, "inflight": d.inflight})
             if cnt.value < 4096:
                 return out
 
@@ -526,6 +528,11 @@ def test_verify(ptr: int, n: int, seed: int, offset: int = 0, stream: int = 0):
     st = load().grouter_test_verify(ptr or None, n, seed, offset, stream or None, C.byref(mism),
                                     C.byref(first))
     return st, mism.value, first.value
+
+
+def test_memcpy(dst: int, src: int, n: int, stream: int = 0, wait: bool = True):
+    """Measured baseline: one bare cudaMemcpyAsync (+ wait for completion)."""
+    return load().grouter_test_memcpy(dst or None, src or None, n, stream or None, 1 if wait else 0)
 
 
 def test_copy(dst: int, src: int, chunks, counts: int = 0, tma: bool = False, stream: int = 0):

@@ -1,6 +1,8 @@
 """Traces of the hand-derived eviction-branch cases (tests/golden/eviction_branches.md).
 
-Inputs only: each builder returns (ops, run kwargs).  The expected values live
+Inputs only: each builder returns (ops, run kwargs).  Every case ends with a
+flush (replay mode dispatches queued copies only there; it moves no
+placement, victim or accounting).  The expected values live
 in tests/golden/eviction_branches.json, typed in by hand from the derivation;
 the oracle is checked against them (tests/test_oracle_branches.py) and the
 library against the oracle on the GPU (tests/test_gpu_parity.py).
@@ -26,6 +28,7 @@ def case_a():
     b.next_use(o8, 5)                                       # 13
     b.next_use(o9, 0)                                       # 14
     b.put(f, 3 * MiB)                                       # 15
+    b.flush()                                               # 16 (replay: dispatch)
     del D
     return b.ops, {"pool_cap": [10 * MiB], "host_store_bytes": 1 << 30}
 
@@ -40,6 +43,7 @@ def case_b():
     b.put(c, 5 * MiB, hint=0)                               # 3
     b.alloc(f, 5 * MiB)                                     # 4
     b.put(f, MiB)                                           # 5
+    b.flush()                                               # 6 (replay: dispatch)
     return b.ops, {"pool_cap": [6 * MiB], "host_store_bytes": 64 * MiB}
 
 
@@ -55,6 +59,7 @@ def case_c():
     b.put(f, 1)                                             # 5
     b.release(z, g)                                         # 6
     b.pool_limit(0, 2 * MiB)                                # 7
+    b.flush()                                               # 8 (replay: dispatch)
     return b.ops, {"host_store_bytes": 64 * MiB}
 
 
@@ -72,6 +77,7 @@ def case_d():
     b.free(c, o1)                                           # 7
     b.put(c, 1)                                             # 8
     b.put(g, MiB)                                           # 9
+    b.flush()                                               # 10 (replay: dispatch)
     return b.ops, {"pool_cap": [2 * MiB], "host_store_bytes": 4 * MiB}
 
 

@@ -718,6 +718,75 @@ def test_tenant_rate_backlog_flag():
         ctx.close()
 
 
+def test_two_batches_in_flight_under_contention():
+    """SURVEY O8 / PAPER.md L229 in real time: a dispatch round carries one
+    batch (<= 5 chunks of one tenant) and a server keeps <= 2 rounds in
+    flight, so a tenant that becomes backlogged behind a saturating one waits
+    behind at most two batches already handed to the copy engine.  Tenant 1
+    keeps GPU0's H2D engine busy with 64 MiB cFn puts (7 batches each) from a
+    thread; tenant 2 issues 4 KiB cFn puts meanwhile.  The real-time dispatch
+    log (GROUTER_LOG) records, per batch, how many earlier batches of that
+    server were still in flight: never more than one.  Tenant 2's batches are
+    dispatched between tenant 1's (preemption at batch boundaries) and its
+    put latency stays within ~3 batch times of the link."""
+    import threading
+    import time
+    calib = dict(C.b200_hgx(1), device_map=[0])
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=512 * MiB, pool_cap=[G.UNLIMITED],
+                                    flags=G.LOG))
+    big = 64 * MiB
+    host = torch.empty(big, dtype=torch.uint8, pin_memory=True)
+    small = torch.empty(4096, dtype=torch.uint8, pin_memory=True)
+    stop = threading.Event()
+    errs = []
+
+    def saturate():
+        try:
+            f = G.fn(1, 1, G.HOST)
+            while not stop.is_set():
+                st, oid = ctx.put(f, host.data_ptr(), big, 0, 0)
+                G.check(st, "put")
+                G.check(ctx.free(f, oid), "free")
+        except Exception as e:   # surfaced below
+            errs.append(e)
+    th = threading.Thread(target=saturate)
+    try:
+        t0 = time.perf_counter()
+        st, oid = ctx.put(G.fn(1, 1, G.HOST), host.data_ptr(), big, 0, 0)
+        G.check(st, "put")
+        solo = time.perf_counter() - t0
+        ctx.free(G.fn(1, 1, G.HOST), oid)
+        batch_s = solo * 5 * 2 * MiB / big          # one 10 MiB batch on this link
+        th.start()
+        time.sleep(0.01)
+        lat = []
+        f2 = G.fn(2, 1, G.HOST)
+        for _ in range(20):
+            t = time.perf_counter()
+            st, o2 = ctx.put(f2, small.data_ptr(), 4096, 0, 0)
+            G.check(st, "put")
+            lat.append(time.perf_counter() - t)
+            ctx.free(f2, o2)
+            time.sleep(0.002)
+        stop.set()
+        th.join(timeout=60)
+        assert not errs, errs
+        log = [d for d in ctx.dispatch_log() if d["kind"] == 1]
+        assert log and max(d["inflight"] for d in log) <= 1, max(d["inflight"] for d in log)
+        assert all(d["bytes"] <= 5 * 2 * MiB for d in log)
+        ten = [d["tenant"] for d in log]
+        i2 = [i for i, t in enumerate(ten) if t == 2]
+        assert len(i2) == 20 and any(0 < i < len(ten) - 1 and ten[i - 1] == ten[i + 1] == 1 for i in i2)
+        lat.sort()
+        assert lat[len(lat) // 2] < 3.5 * batch_s, (lat[len(lat) // 2], batch_s)
+        print(f"4 KiB put p50 under contention {lat[len(lat) // 2] * 1e6:.0f} us, batch {batch_s * 1e6:.0f} us")
+    finally:
+        stop.set()
+        if th.is_alive():
+            th.join(timeout=60)
+        ctx.close()
+
+
 def test_probe_calibration():
     """grouter_probe (a5, L178/L131/L271): on one B200 the solo pinned H2D rate
     is a PCIe Gen5 x16 figure, per-copy and first-chunk costs are positive,
