@@ -52,6 +52,12 @@ grouter_status grouter_test_launch_cost(int kind, int n, int blocks, void *strea
  * the library calls it is compared with (SURVEY §8(d) baselines). */
 grouter_status grouter_test_memcpy(void *dst, const void *src, uint64_t n, void *stream, int32_t wait);
 
+/* Positive control for the race detector (sanitizer builds):
+ * two threads increment one plain int `iters` times each, unsynchronised --
+ * a ThreadSanitizer build must report exactly this data race.  Returns the
+ * final count in *out (any value; the race is the point). */
+grouter_status grouter_test_race(int32_t iters, int64_t *out);
+
 /* Text dump of the context's internal state (servers, objects, leases,
  * pending completion words) for debugging; truncated to cap bytes.  Returns
  * the full length needed in *len (may be NULL). */

@@ -63,13 +63,26 @@ def up_to_date() -> bool:
     return built_hash() == source_hash()
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
-        return LIB
-    objdir = os.path.join(HERE, "build")
+# Sanitizer builds of the host code (race detection): a separate
+# library selected at load time with GROUTER_LIB (run the process with the
+# sanitizer runtime preloaded, e.g. LD_PRELOAD=$(gcc -print-file-name=libtsan.so)).
+SANITIZERS = {"tsan": ["-fsanitize=thread"], "asan": ["-fsanitize=address"]}
+
+
+def lib_path(variant: str | None = None) -> str:
+    return LIB if not variant else os.path.join(HERE, f"libgrouter_{variant}.so")
+
+
+def build(force: bool = False, verbose: bool = False, variant: str | None = None) -> str:
+    target = lib_path(variant)
+    if not force and built_hash(target) == source_hash():
+        return target
+    objdir = os.path.join(HERE, "build" if not variant else f"build_{variant}")
     os.makedirs(objdir, exist_ok=True)
     digest = source_hash()
-    common = COMMON + ["-I", os.path.join(ROOT, "include"), f"-DGROUTER_SRC_HASH=\"{digest}\""] + ARCH
+    san = SANITIZERS[variant] if variant else []
+    san_cc = [x for f in san + (["-fno-omit-frame-pointer", "-g"] if san else []) for x in ("-Xcompiler", f)]
+    common = COMMON + san_cc + ["-I", os.path.join(ROOT, "include"), f"-DGROUTER_SRC_HASH=\"{digest}\""] + ARCH
     objs = []
     procs = []
     for src in SOURCES:
@@ -89,17 +102,18 @@ def build(force: bool = False, verbose: bool = False) -> str:
     vscript = os.path.join(objdir, "exports.map")
     with open(vscript, "w") as f:
         f.write("{ global: grouter_*; local: *; };\n")
-    tmp = LIB + ".tmp"
+    tmp = target + ".tmp"
     link = [NVCC] + ARCH + ["-shared", "-cudart=static", "-o", tmp] + objs + [
         "-Xlinker", "--version-script=" + vscript, "-Xlinker", "-Bsymbolic",
-        "-lpthread", "-ldl", "-lrt"]
+        "-lpthread", "-ldl", "-lrt"] + [x for f in san for x in ("-Xcompiler", f)]
     r = subprocess.run(link, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)
     if r.returncode != 0:
         sys.stderr.write(r.stdout.decode())
         raise RuntimeError("link failed")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    var = next((a[2:] for a in sys.argv[1:] if a[2:] in SANITIZERS), None)   # --tsan / --asan
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, variant=var))

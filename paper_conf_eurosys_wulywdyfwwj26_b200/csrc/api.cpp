@@ -10,6 +10,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <thread>
 #include <cstring>
 
 #include "../../include/grouter.h"
@@ -354,6 +355,16 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
     pump(c, false);
     return x2;
   }
+  if (caller && direct && n && server_kind_for(src_loc, dst_loc) == SK_COPY) {
+    const int server = src_loc == GROUTER_REMOTE ? dst_loc : src_loc;
+    XferRef fx = fast_direct(c, tenant, server, dst_loc, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, n,
+                             pool_src && src_loc >= 0, deps, caller, c->dev[caller_logical].phys);
+    if (fx) {
+      *direct = true;
+      if (hprof().on) hprof().t[4] += now_ns() - tst;
+      return fx;
+    }
+  }
   std::vector<grouter_chunk> plan;
   if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
   else c->planner.plan(src_loc, dst_loc, n, plan, pool_src);
@@ -401,6 +412,24 @@ const char *grouter_last_error(void) { return gr::last_error(); }
 // the marker is found by a byte scan of the .so (_build.built_hash), no dlopen needed
 static const char kSrcHashMarker[] __attribute__((used)) = "GROUTER_SRC_HASH=" GROUTER_SRC_HASH;
 const char *grouter_build_hash(void) { return kSrcHashMarker + 17; }
+
+static int64_t g_race_counter;  // deliberately unsynchronised (grouter_test_race)
+static void race_body(int32_t iters) {
+  for (int32_t i = 0; i < iters; ++i) {
+    int64_t v = g_race_counter;
+    asm volatile("" ::: "memory");
+    g_race_counter = v + 1;
+  }
+}
+grouter_status grouter_test_race(int32_t iters, int64_t *out) {
+  if (!out || iters < 0) return GROUTER_EINVAL;
+  g_race_counter = 0;
+  std::thread a(race_body, iters), b(race_body, iters);
+  a.join();
+  b.join();
+  *out = g_race_counter;
+  return GROUTER_OK;
+}
 
 void grouter_config_default(grouter_config *cfg) {
   if (!cfg) return;

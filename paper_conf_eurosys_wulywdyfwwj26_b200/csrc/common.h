@@ -69,6 +69,7 @@ struct Driver {
   CUresult (*memImportFromShareableHandle)(CUmemGenericAllocationHandle *, void *, CUmemAllocationHandleType);
   CUresult (*streamWaitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
   CUresult (*streamWriteValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+  CUresult (*launchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **);
 };
 const Driver &drv();
 

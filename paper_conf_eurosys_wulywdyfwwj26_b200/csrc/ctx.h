@@ -334,6 +334,9 @@ void harvest_profile(grouter_ctx *c, bool wait);       // completed timed launch
 // is idle (or only busy with direct launches on that same stream).  Returns
 // false (nothing done) when the server path must be used.
 bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys);
+XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
+                    uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
+                    int caller_phys);
 void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);  // submitted fences only
 // Waits on a CALLER stream: submitted fences now, the others as soon as their
 // producer transfer is submitted.

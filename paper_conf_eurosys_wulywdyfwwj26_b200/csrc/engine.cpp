@@ -17,14 +17,16 @@
 //    with cuStreamWaitValue32(GEQ) on their own stream, or poll from the
 //    host -- no host round trip on the data path, no partial visibility.
 //  * Each server (SM-copy egress of a GPU, H2D engine of a route GPU, D2H
-//    engine) owns a Stride scheduler; a ROUND = consecutive batches in
-//    stride order up to a byte horizon, executed by ONE kernel launch (SM
-//    copy) or one memcpy burst (CE).  <= 2 rounds in flight per server in
-//    real-time mode; replay mode dispatches only at grouter_flush().
+//    engine) owns a Stride scheduler; a ROUND = ONE batch in stride order
+//    (plus urgent unscheduled work), executed by one kernel launch (SM copy)
+//    or one memcpy burst (CE).  <= 2 rounds -- so <= 2 batches, SURVEY O8 --
+//    in flight per server in real-time mode; replay mode dispatches only at
+//    grouter_flush().
 //  * Host->GPU relay: CE copies a chunk into a staging slot on route GPU r,
-//    an event hands the slot to r's forward stream, the forward round kernel
-//    pushes it over NVLink into the lease on d and publishes the word; the
-//    slot is reused after the forward round's event.
+//    an event hands that chunk's slot to r's forward stream, a forward launch
+//    pushes it over NVLink into the lease on d and publishes the chunk's word
+//    (per chunk: the NVLink hop overlaps the next chunk's PCIe copy); the
+//    slot is reused after that launch's event.
 #include <algorithm>
 #include <cstdio>
 #include <chrono>
@@ -447,13 +449,16 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
           GR_CUDA(cudaEventCreate(e));
         }
       }
-      if (!pd.gate) {
+      static const bool no_gate = getenv("GR_NO_GATE") != nullptr;  // diagnostics
+      if (!pd.gate && !no_gate) {
         GR_CUDA(cudaHostAlloc((void **)&pd.gate, 64, cudaHostAllocMapped | cudaHostAllocPortable));
         *pd.gate = 0;
       }
-      gate_v = ++pd.gate_seq;  // released below, after the stop event is enqueued
-      GR_CU(drv().streamWaitValue32((CUstream)st, (CUdeviceptr)(uintptr_t)pd.gate, gate_v,
-                                    CU_STREAM_WAIT_VALUE_GEQ));
+      if (!no_gate) {
+        gate_v = ++pd.gate_seq;  // released below, after the stop event is enqueued
+        GR_CU(drv().streamWaitValue32((CUstream)st, (CUdeviceptr)(uintptr_t)pd.gate, gate_v,
+                                      CU_STREAM_WAIT_VALUE_GEQ));
+      }
       GR_CUDA(cudaEventRecord(pr.start, st));
     }
     struct GateRelease {  // the gate opens on every path out (an exception must not park the stream)
@@ -599,14 +604,12 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   const uint64_t budget = batch_budget(c, s);
   const uint64_t tr0 = tl_put_t0 ? now_ns() : 0;
   const uint32_t nb = refill_one(c, s);
-  std::vector<ChunkItem> items, direct, relay;
+  std::vector<ChunkItem> items, direct;
   std::vector<char> cut;
   take(s, budget, items, cut);
   if (items.empty()) return 0;
   const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
-  std::vector<uint64_t> slot_src;
-  std::vector<uint32_t> slots_used;
   EventRef last_fwd;
   // contiguous direct chunks of a round go to the copy engine as ONE copy
   // (per-copy engine overhead ~3.6 us measured by the probe)
@@ -627,19 +630,25 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
     }
     run_len = 0;
   };
+  // Relay forward, pipelined per chunk (K4', L182 "chunks are pipelined
+  // across GPU streams"): as soon as a relayed chunk's copy into the staging
+  // slot is enqueued, the forward stream waits for exactly that copy and a
+  // forward launch pushes that chunk to its destination and publishes its
+  // completion word -- the NVLink hop of chunk k overlaps the PCIe copy of
+  // chunk k+1, and the relay adds one chunk's forward to the tail instead of
+  // a whole round's.  The forward kernels run only while a chunk is moving
+  // (no SMs parked polling for PCIe arrivals).
+  auto forward_chunk = [&](const ChunkItem &it, uint64_t slot, uint32_t k) {
+    EventRef ce = record(c, s.stream, s.phys);
+    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
+    const std::vector<ChunkItem> one(1, it);
+    launch_round(c, s, s.fwd_stream, s.fwd_scratch, one, &slot);
+    last_fwd = record(c, s.fwd_stream, s.phys);
+    s.slot_free[k] = last_fwd;
+  };
   auto end_segment = [&]() {
     flush_run();
     publish_ce(c, s, direct, evented);
-    if (!relay.empty()) {
-      EventRef ce = record(c, s.stream, s.phys);
-      GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
-      launch_round(c, s, s.fwd_stream, s.fwd_scratch, relay, slot_src.data());
-      last_fwd = record(c, s.fwd_stream, s.phys);
-      for (uint32_t k : slots_used) s.slot_free[k] = last_fwd;
-      relay.clear();
-      slot_src.clear();
-      slots_used.clear();
-    }
   };
   for (size_t i = 0; i < items.size(); ++i) {
     const ChunkItem &it = items[i];
@@ -668,9 +677,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
       if (s.slot_free[k]) GR_CUDA(cudaStreamWaitEvent(s.stream, s.slot_free[k]->ev, 0));
       uint8_t *slot = s.staging + (uint64_t)k * s.slot_bytes;
       GR_CUDA(cudaMemcpyAsync(slot, (const void *)src, it.bytes, cudaMemcpyHostToDevice, s.stream));
-      relay.push_back(it);
-      slot_src.push_back((uint64_t)slot);
-      slots_used.push_back(k);
+      forward_chunk(it, (uint64_t)slot, k);
     }
     if (it.x->pageable_src) c->bounce_ev[bslot] = record(c, s.stream, s.phys);
     c->stats.link_bytes[1][s.logical] += it.bytes;
@@ -779,6 +786,86 @@ void pump(grouter_ctx *c, bool force_all) {
 void flush_all(grouter_ctx *c) {
   pump(c, true);
   c->epoch++;  // everything created before is now submitted (grounded)
+}
+
+// Direct launch without the queues: one same-GPU (or same-device logical
+// pair) SM copy of a contiguous single-path plan on an idle copy server, in
+// real-time mode.  Does exactly what enqueue + try_direct would -- the
+// tenant's stride passes advance as if its batches had been dispatched
+// (Stride::account_solo), tenant bytes, the rate monitor and the stats are
+// updated, the transfer completes by an event on the caller's stream -- but
+// skips building chunk items, the scheduler queues, round assembly and the
+// completion slot (~1.5 us of host time per call, tools/libcost.cpp).  Only
+// for static-assignment engines (16 B-aligned addresses: wv8 / tmas4, no
+// device scratch).  Returns null when the queued path must be used.
+XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
+                    uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
+                    int caller_phys) {
+  static const bool off = getenv("GR_NO_FAST") != nullptr || getenv("GR_COPY") != nullptr;
+  const uint32_t never = GROUTER_LOG | GROUTER_PROFILE | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
+  if (off || c->replay || !caller || (c->cfg.flags & never) || !n || ((src | dst) & 15)) return nullptr;
+  Server &s = c->dev[server_logical].copy;
+  if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
+  for (auto &f : s.inflight)
+    if (f.direct != caller) {
+      retire(s);
+      for (auto &g : s.inflight)
+        if (g.direct != caller) return nullptr;
+      break;
+    }
+  for (auto &w : deps)
+    if (!is_submitted(w)) return nullptr;
+  const uint64_t C = c->cfg.chunk_bytes;
+  auto x = std::make_shared<Xfer>();
+  x->id = ++c->xfer_seq;
+  x->tenant = tenant;
+  x->epoch = c->epoch;
+  x->npath = 1;
+  x->nchunks = x->submitted_chunks = (uint32_t)((n + C - 1) / C);
+  x->local_src = local_src;
+  c->stats.xfer_count++;
+  DeviceGuard g(s.phys);
+  stream_wait(c, caller, s.phys, deps);  // no-op for completed fences
+  if (!c->params) c->params = new CopyParamsHost();
+  CopyParams *p = &c->params->p;
+  const bool local = dst_logical >= 0 && c->dev[dst_logical].phys == s.phys;
+  p->flags = (local ? kFlagLocalDst : 0) | (local_src ? kFlagLocalSrc : 0);
+  p->n_chunks = 1;
+  p->n_pub = 0;
+  p->scratch = nullptr;
+  p->counts = nullptr;
+  p->count_base = 0;
+  p->chunk[0] = {src, dst, n};
+  bool host_pub = false;
+  PhysDev &pd = *c->phys.at(s.phys);
+  int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm, false, caller, &host_pub);
+  if (e != 0) throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
+  if (!host_pub) throw Error(GROUTER_ECUDA, "internal: fast direct launch needs a static engine");
+  x->done_ev = record(c, caller, s.phys);
+  x->done_stream = caller;
+  // the bookkeeping a queued dispatch would have done
+  s.sched.account_solo(tenant, n, C, weight_of(c, tenant));
+  c->tenant_bytes[tenant][SK_COPY] += n;
+  {
+    auto &lg = c->tenant_log[tenant];
+    const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
+    lg.emplace_back(now, n);
+    while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
+  }
+  c->stats.link_bytes[0][s.logical] += n;
+  c->stats.rounds++;
+  c->stats.kernel_launches++;
+  if (!local) c->stats.peer_launches++;
+  Waitable w;
+  w.ev = x->done_ev;
+  w.epoch = x->epoch;
+  w.origin = caller;
+  const uint32_t nb = (uint32_t)((x->nchunks + s.sched.batch - 1) / s.sched.batch);
+  if (!s.inflight.empty() && s.inflight.back().direct == caller && s.inflight.back().w.origin == caller)
+    s.inflight.back().w = w;
+  else
+    s.inflight.push_back({w, caller, nb});
+  return x;
 }
 
 bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys) {

@@ -25,6 +25,7 @@
 #include "../../include/grouter.h"
 #include "../../include/grouter_testing.h"
 #include "kernels.h"
+#include "common.h"
 
 typedef int CUresult_t;
 
@@ -804,6 +805,22 @@ extern "C" grouter_status grouter_test_launch_cost(int kind, int n, int blocks, 
     else if (kind == 3 || kind == 4) {
       cfg.numAttrs = kind == 3 ? 1 : 0;
       cudaLaunchKernelEx(&cfg, gr_empty_kernel, sp);
+    } else if (kind == 10 || kind == 11) {  // driver API cuLaunchKernelEx (with / without PDL)
+      static CUfunction f = nullptr;
+      if (!f) cudaGetFuncBySymbol(&f, (const void *)gr_empty_kernel);
+      CUlaunchAttribute at[1];
+      at[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+      at[0].value.programmaticStreamSerializationAllowed = 1;
+      CUlaunchConfig lc = {};
+      lc.gridDimX = blocks;
+      lc.gridDimY = lc.gridDimZ = 1;
+      lc.blockDimX = 256;
+      lc.blockDimY = lc.blockDimZ = 1;
+      lc.hStream = (CUstream)s;
+      lc.attrs = at;
+      lc.numAttrs = kind == 10 ? 1 : 0;
+      void *args[] = {(void *)&sp};
+      drv().launchKernelEx(&lc, f, args, nullptr);
     } else if (kind == 5) cudaEventRecord(ev, s);
     else if (kind == 6) (void)cudaEventQuery(ev);
     else {  // 7: launch_copy of 4 KiB, 8: of 38.5 MB (the production launch path), 9: event + 8

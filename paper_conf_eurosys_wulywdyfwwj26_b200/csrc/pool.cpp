@@ -97,6 +97,7 @@ const Driver &drv() {
       resolve("cuMemImportFromShareableHandle", d.memImportFromShareableHandle);
       resolve("cuStreamWaitValue32", d.streamWaitValue32);
       resolve("cuStreamWriteValue32", d.streamWriteValue32);
+      resolve("cuLaunchKernelEx", d.launchKernelEx);
     } catch (const Error &e) {
       err = e.what();
     }

@@ -45,6 +45,25 @@ struct Stride {
       else ++it;
   }
 
+  // The pass/V updates dispatch() makes when tenant t, alone on an idle
+  // server, has n bytes in chunks of `chunk` bytes (all full but the last)
+  // dispatched in batches -- for transfers that bypass the queues (a direct
+  // launch on an idle SM-copy server), so later contention sees the same
+  // passes as if the chunks had been queued.
+  void account_solo(uint32_t t, uint64_t n, uint64_t chunk, uint64_t w) {
+    Tenant &tn = tenants[t];
+    if (tn.q.empty()) tn.pass = tn.pass > V ? tn.pass : V;  // join rule
+    if (w == 0) w = 1;
+    const uint64_t per_batch = chunk * batch;
+    while (n) {
+      const uint64_t bytes = n < per_batch ? n : per_batch;
+      V = tn.pass;
+      unsigned __int128 s = ((unsigned __int128)bytes << 20);
+      tn.pass += (uint64_t)((s + w - 1) / w);
+      n -= bytes;
+    }
+  }
+
   // Pops the next batch into `out`; returns the tenant id, or UINT32_MAX if idle.
   template <class WeightFn>
   uint32_t dispatch(WeightFn weight_of, std::vector<Item> &out, uint64_t *bytes_out = nullptr,

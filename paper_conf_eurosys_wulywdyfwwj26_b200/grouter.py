@@ -173,6 +173,7 @@ SIGNATURES = {
     "grouter_test_dump": (_ST, [_CTX, C.c_char_p, _U64, C.POINTER(_U64)]),
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
     "grouter_test_memcpy": (_ST, [_P, _P, C.c_uint64, _P, C.c_int32]),
+    "grouter_test_race": (_ST, [C.c_int32, C.POINTER(C.c_int64)]),
 }
 
 _lib = None
@@ -183,26 +184,31 @@ def load(build_if_missing: bool = False):
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(LIB_PATH):
-        if not build_if_missing:
-            raise ImportError(f"{LIB_PATH} not built; run __graft_entry__.build()")
-        from . import _build
-        _build.build()
     from . import _build
-    want = _build.source_hash()
-    if _build.built_hash() != want:
+    # GROUTER_LIB selects a sanitizer build of the same sources (tsan / asan,
+    # _build.SANITIZERS); the default is the product library
+    variant = os.environ.get("GROUTER_LIB") or None
+    if variant and variant not in _build.SANITIZERS:
+        raise ImportError(f"GROUTER_LIB={variant!r}: expected one of {sorted(_build.SANITIZERS)}")
+    path = _build.lib_path(variant)
+    if not os.path.exists(path):
         if not build_if_missing:
-            raise ImportError(f"{LIB_PATH} was built from other sources (hash {_build.built_hash()} != "
+            raise ImportError(f"{path} not built; run __graft_entry__.build()")
+        _build.build(variant=variant)
+    want = _build.source_hash()
+    if _build.built_hash(path) != want:
+        if not build_if_missing:
+            raise ImportError(f"{path} was built from other sources (hash {_build.built_hash(path)} != "
                               f"{want}); run __graft_entry__.build()")
-        _build.build()
-    lib = C.CDLL(LIB_PATH)
+        _build.build(variant=variant)
+    lib = C.CDLL(path)
     for name, (res, args) in SIGNATURES.items():
         f = getattr(lib, name)
         f.restype = res
         f.argtypes = args
     got = lib.grouter_build_hash().decode()
     if got != want:   # the file changed between the scan and dlopen
-        raise ImportError(f"{LIB_PATH}: grouter_build_hash() {got} != source hash {want}")
+        raise ImportError(f"{path}: grouter_build_hash() {got} != source hash {want}")
     _lib = lib
     return lib
 
