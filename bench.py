@@ -24,13 +24,14 @@ Also in the line:
                each delivered tensor (the step's result)
   latency_us   p50/p99 of single cfg1 requests on an idle GPU (R22: put call
                -> the consumer's data ready)
-  roofline     gr_copy (the only kernel on the path), per-launch CUDA events
-               on its stream inside the timed region (GROUTER_PROFILE);
+  roofline     gr_copy (the only kernel on the path) in leg B's own timed
+               region: get_into of HBM-resident objects back to back, CUDA
+               events on the stream the kernels run on / launches;
                algorithmic bytes = 2n (HBM read + write) at one GPU, n over
-               NVLink at N > 1; roofline_step: the PCIe link that bounds
-               the workflow (live-measured pinned H2D)
-  kernel_b2b   leg B alone, back to back on HBM-resident objects (the kernel's
-               own speed of light)
+               NVLink at N > 1.  roofline.in_step: the same kernel timed per
+               launch inside the workflow's region (isolated launches).
+               roofline_step: the PCIe link that bounds the workflow
+               (live-measured pinned H2D)
   sweep        cfg3 (iii)/(iv) at one GPU: per size 4 KiB..1 GiB, p50/p99 and
                GB/s of same-GPU get_into, cFn put (H2D), cFn get (D2H) and
                zero-copy get, each beside a bare cudaMemcpyAsync on the same
@@ -1084,7 +1085,7 @@ def run_gpu(args, rank, world, local_rank):
     except Exception as e:   # context only; never fails the line
         live_peaks = {"error": str(e)[:200]}
     traffic = traffic_steady = None
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")   # per-launch DRAM bytes of the b2b region
     if os.path.exists(tp):
         try:
             tj = json.load(open(tp))
@@ -1151,28 +1152,31 @@ def run_gpu(args, rank, world, local_rank):
                            "put_p50": pct(lat_a, 50),
                            "what": "one cfg1 request on an idle GPU: cFn put call -> gFn's data ready "
                                    "(event on the consumer stream observed by the host), R22"},
-            "roofline": {"bound": "hbm" if rw == 2 else "nvlink", "achieved": k_ach, "peak": kpeak,
-                         "unit": "GB/s", "frac": (k_ach / kpeak) if k_ach else None, "traffic": traffic,
+            "roofline": {"bound": "hbm" if rw == 2 else "nvlink", "achieved": b2b_ach, "peak": kpeak,
+                         "unit": "GB/s", "frac": b2b_ach / kpeak, "traffic": traffic,
                          "kernel": "gr_copy (K2') leg B" + (" same-GPU" if rw == 2 else " NVLink push"),
                          "peak_source": peak_src if rw == 2 else "north star: 900 GB/s per direction",
-                         "launches": tl, "avg_launch_us": k_us,
-                         "alg_bytes_per_launch": rw * t_bytes / max(tl, 1),
-                         "timing": "CUDA events recorded around every gr_copy launch on its own stream "
-                                   "(GROUTER_PROFILE) during the timed region; each launch runs alone "
-                                   "(requests are PCIe-paced), so it pays its own ramp-up",
+                         "launches": b2b_l, "avg_launch_us": b2b_us, "alg_bytes_per_launch": rw * n,
+                         "timing": "leg B's own timed region: the gFn get_into's of 20 HBM-resident 38.5 MB "
+                                   "objects into 8 rotating bindings, 200 x 20 launches back to back, CUDA events "
+                                   "on the consumer stream the kernels run on / launches (no per-launch events: "
+                                   "they would sit between the launches)",
                          "traffic_note": "ncu --set full, per launch (profiles/); steady traffic without "
                                          "cache flushes in traffic_steady", "traffic_steady": traffic_steady,
-                         "peak_live": live_peaks},
+                         "peak_live": live_peaks,
+                         "in_step": {"avg_launch_us": k_us, "achieved": k_ach,
+                                     "frac": (k_ach / kpeak) if k_ach else None, "launches": tl,
+                                     "what": "the same kernel inside the workflow's timed region, CUDA events "
+                                             "recorded around every launch on its stream (GROUTER_PROFILE): "
+                                             "each launch runs alone (requests are PCIe-paced), so the "
+                                             "interval also holds the launch latency and the grid's ramp-up "
+                                             "that back-to-back launches overlap (tools/instep.py)"}},
             "roofline_step": {"bound": "pcie", "achieved": value / world * N_BYTES / 1e9,
                               "peak": link_peak, "unit": "GB/s",
                               "frac": value / world * N_BYTES / 1e9 / link_peak,
                               "what": "per-GPU payload GB/s of the workflow against this box's pinned "
                                       "single-link H2D (bare cudaMemcpyAsync of 256 MiB back to back): the "
                                       "link every request crosses once"},
-            "kernel_b2b": {"what": "leg B alone: gFn get_into of 20 HBM-resident objects back to back "
-                                   "(CUDA events on the consumer stream / launches)",
-                           "us_per_launch": b2b_us, "achieved": b2b_ach, "peak": kpeak,
-                           "frac": b2b_ach / kpeak, "launches": b2b_l},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "req/s", "h2d_bytes_per_step": R * N_BYTES,
                     "d2h_bytes_per_step": R * 8, "steps": e2e_steps, "outstanding": Q,

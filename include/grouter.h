@@ -58,10 +58,9 @@ extern "C" {
 #define GROUTER_PLAN_ONLY     0x4u /* no CUDA at all: planner/introspection only            */
 #define GROUTER_LOG           0x8u /* keep the dispatch log in real-time mode too           */
 #define GROUTER_COPY_TMA      0x10u/* SM copy kernel uses cp.async.bulk (TMA) staging       */
-#define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream;
-                                      the stream is held at a host-released gate until start
-                                      event, kernel and stop event are enqueued, so the interval
-                                      is the launch alone (measurement mode)                    */
+#define GROUTER_PROFILE       0x20u/* time every copy-kernel launch with CUDA events on its stream
+                                      (measurement mode: the events sit between launches and
+                                      cost the programmatic-dependent-launch overlap)           */
 #define GROUTER_D2H_MULTIPATH 0x80u/* gFn-host striping (L178, Fig. 5a; R45): a GPU
                                       object read into host memory is split over R(src) like a
                                       host->GPU plan; route r's copy engine moves its share      */

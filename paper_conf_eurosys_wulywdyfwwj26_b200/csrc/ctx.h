@@ -236,11 +236,6 @@ struct PhysDev {
   uint32_t n_scratch = 0, next_scratch = 0;
   std::vector<Fences> scratch_busy;
   std::vector<cudaEvent_t> timing_free;  // timing-enabled events (GROUTER_PROFILE)
-  // GROUTER_PROFILE gate: a host-mapped word the profiled stream waits on
-  // until start event, kernel and stop event are all enqueued, so the timed
-  // interval holds the launch alone (no host submission gap inside it)
-  volatile uint32_t *gate = nullptr;
-  uint32_t gate_seq = 0;
 };
 
 struct ProfRec {

@@ -439,7 +439,6 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       for (auto &pb : pubs)
         if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path]) p->pub[k].value = pb.x->value_after(pb.path);
     ProfRec pr{s.phys, nullptr, nullptr, bytes};
-    uint32_t gate_v = 0;
     if (prof) {
       for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
         if (!pd.timing_free.empty()) {
@@ -449,25 +448,8 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
           GR_CUDA(cudaEventCreate(e));
         }
       }
-      static const bool no_gate = getenv("GR_NO_GATE") != nullptr;  // diagnostics
-      if (!pd.gate && !no_gate) {
-        GR_CUDA(cudaHostAlloc((void **)&pd.gate, 64, cudaHostAllocMapped | cudaHostAllocPortable));
-        *pd.gate = 0;
-      }
-      if (!no_gate) {
-        gate_v = ++pd.gate_seq;  // released below, after the stop event is enqueued
-        GR_CU(drv().streamWaitValue32((CUstream)st, (CUdeviceptr)(uintptr_t)pd.gate, gate_v,
-                                      CU_STREAM_WAIT_VALUE_GEQ));
-      }
       GR_CUDA(cudaEventRecord(pr.start, st));
     }
-    struct GateRelease {  // the gate opens on every path out (an exception must not park the stream)
-      volatile uint32_t *g;
-      uint32_t v;
-      ~GateRelease() {
-        if (v) __atomic_store_n(g, v, __ATOMIC_RELEASE);
-      }
-    } gate_release{pd.gate, gate_v};
     HostProf &hp = hprof();
     uint64_t tl = hp.on ? now_ns() : 0;
     if (hp.on) hp.t[6] += tl - tparams;
@@ -488,7 +470,6 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       GR_CUDA(cudaEventRecord(pr.stop, st));
       c->prof.push_back(pr);
     }
-    (void)gate_release;
     c->stats.kernel_launches++;
     if (!local) c->stats.peer_launches++;
   }
@@ -1243,7 +1224,6 @@ void engine_shutdown(grouter_ctx *c) {
     DeviceGuard g(kv.first);
     if (kv.second->scratch) cudaFree(kv.second->scratch);
     for (cudaEvent_t e : kv.second->timing_free) cudaEventDestroy(e);
-    if (kv.second->gate) cudaFreeHost((void *)kv.second->gate);
     kv.second->scratch_busy.clear();
   }
   ipc_release_all(c);  // dedicated (exported) allocations; their fences hold pooled events
