@@ -368,6 +368,15 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   std::vector<grouter_chunk> plan;
   if (src_loc == GROUTER_REMOTE) c->planner.plan_single(n, dst_loc, plan);  // consumer GPU pulls
   else c->planner.plan(src_loc, dst_loc, n, plan, pool_src);
+  const int kind0 = server_kind_for(src_loc, dst_loc);
+  if (!caller && !pageable_src && (kind0 == SK_H2D || kind0 == SK_D2H)) {  // host caller, idle copy engine
+    XferRef fx = fast_ce(c, tenant, kind0, plan, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, n, deps);
+    if (fx) {
+      if (direct) *direct = false;
+      if (hprof().on) hprof().t[4] += now_ns() - tst;
+      return fx;
+    }
+  }
   XferRef x = new_xfer(c, tenant, plan);
   x->deps = std::move(deps);
   x->pageable_src = pageable_src;

@@ -329,6 +329,8 @@ void harvest_profile(grouter_ctx *c, bool wait);       // completed timed launch
 // is idle (or only busy with direct launches on that same stream).  Returns
 // false (nothing done) when the server path must be used.
 bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys);
+XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<grouter_chunk> &plan, uint64_t src,
+                uint64_t dst, uint64_t n, const Fences &deps);
 XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
                     int caller_phys);

@@ -572,9 +572,15 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
                                return std::find(evented.begin(), evented.end(), it.x) != evented.end();
                              }),
               seg.end());
+  // Only the round that carries a path's LAST chunk writes that path's word
+  // (consumers never see partial progress, R5; the copies of one path on one
+  // server are in stream order, so the final write covers the earlier rounds):
+  // a stream write costs ~1-2 us per round on a multi-round transfer.  Every
+  // fence on a word waits for its final value (done_fences).
   for (auto &p : issue(seg))
-    GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
-                                   p.x->value_after(p.path), 0));
+    if (p.x->issued[p.path] == p.x->total[p.path])
+      GR_CU(drv().streamWriteValue32((CUstream)s.stream, (CUdeviceptr)(uintptr_t)&p.x->words[p.path],
+                                     p.x->value_after(p.path), 0));
   seg.clear();
 }
 
@@ -619,7 +625,19 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   // chunk k+1, and the relay adds one chunk's forward to the tail instead of
   // a whole round's.  The forward kernels run only while a chunk is moving
   // (no SMs parked polling for PCIe arrivals).
+  // GR_SEGMENT_FWD=1 (measurement only, tools/relaytail.py): the round-1
+  // design -- one forward launch per segment after all its CE copies
+  static const bool segment_fwd = getenv("GR_SEGMENT_FWD") != nullptr;
+  std::vector<ChunkItem> seg_relay;
+  std::vector<uint64_t> seg_src;
+  std::vector<uint32_t> seg_slots;
   auto forward_chunk = [&](const ChunkItem &it, uint64_t slot, uint32_t k) {
+    if (segment_fwd) {
+      seg_relay.push_back(it);
+      seg_src.push_back(slot);
+      seg_slots.push_back(k);
+      return;
+    }
     EventRef ce = record(c, s.stream, s.phys);
     GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
     const std::vector<ChunkItem> one(1, it);
@@ -630,6 +648,16 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   auto end_segment = [&]() {
     flush_run();
     publish_ce(c, s, direct, evented);
+    if (!seg_relay.empty()) {
+      EventRef ce = record(c, s.stream, s.phys);
+      GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
+      launch_round(c, s, s.fwd_stream, s.fwd_scratch, seg_relay, seg_src.data());
+      last_fwd = record(c, s.fwd_stream, s.phys);
+      for (uint32_t k : seg_slots) s.slot_free[k] = last_fwd;
+      seg_relay.clear();
+      seg_src.clear();
+      seg_slots.clear();
+    }
   };
   for (size_t i = 0; i < items.size(); ++i) {
     const ChunkItem &it = items[i];
@@ -846,6 +874,55 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
     s.inflight.back().w = w;
   else
     s.inflight.push_back({w, caller, nb});
+  return x;
+}
+
+// Copy-engine transfer of an idle H2D / D2H server without the queues, for
+// a single-route plan of at most two batches (so <= 2 batches in flight
+// holds): one cudaMemcpyAsync on the server's stream and an
+// event, with the same scheduler accounting (Stride::account_solo), tenant
+// bytes, rate monitor and stats as a queued dispatch.  Real-time mode only
+// (no LOG / PROFILE); null when the queued path must be used.
+XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<grouter_chunk> &plan, uint64_t src,
+                uint64_t dst, uint64_t n, const Fences &deps) {
+  static const bool off = getenv("GR_NO_FAST") != nullptr;
+  if (off || c->replay || (c->cfg.flags & (GROUTER_LOG | GROUTER_PROFILE)) || plan.empty()) return nullptr;
+  const int route = plan[0].route_gpu;
+  for (auto &ch : plan)
+    if (ch.route_gpu != route || ch.path != 0) return nullptr;  // striped: the queued path relays
+  Server &s = server_of(c, kind, route);
+  if (n > 2 * batch_budget(c, s) || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
+  if (!s.inflight.empty()) {
+    retire(s);
+    if (!s.inflight.empty()) return nullptr;
+  }
+  for (auto &w : deps)
+    if (!is_submitted(w)) return nullptr;
+  auto x = std::make_shared<Xfer>();
+  x->id = ++c->xfer_seq;
+  x->tenant = tenant;
+  x->epoch = c->epoch;
+  x->npath = 1;
+  x->nchunks = x->submitted_chunks = (uint32_t)plan.size();
+  c->stats.xfer_count++;
+  DeviceGuard g(s.phys);
+  stream_wait(c, s.stream, s.phys, deps);
+  GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, n,
+                          kind == SK_H2D ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToHost, s.stream));
+  x->done_ev = record(c, s.stream, s.phys);
+  x->done_stream = s.stream;
+  s.sched.account_solo(tenant, n, plan[0].bytes, weight_of(c, tenant));
+  c->tenant_bytes[tenant][kind] += n;
+  {
+    auto &lg = c->tenant_log[tenant];
+    const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
+    lg.emplace_back(now, n);
+    while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
+  }
+  c->stats.link_bytes[kind][s.logical] += n;
+  c->stats.rounds++;
+  s.inflight.push_back({ev_wait(c, x->done_ev), nullptr,
+                        (uint32_t)((plan.size() + s.sched.batch - 1) / s.sched.batch)});
   return x;
 }
 
