@@ -1170,7 +1170,11 @@ def run_gpu(args, rank, world, local_rank):
                                              "recorded around every launch on its stream (GROUTER_PROFILE): "
                                              "each launch runs alone (requests are PCIe-paced), so the "
                                              "interval also holds the launch latency and the grid's ramp-up "
-                                             "that back-to-back launches overlap (tools/instep.py)"}},
+                                             "that back-to-back launches overlap, and with 4 client threads "
+                                             "the host's gap between the start event and the launch call "
+                                             "(tools/instep.py: 19-22 us with one client); the kernel alone "
+                                             "takes ~13 us per launch in ncu's launch list of this command "
+                                             "(profiles/r02_ncu_launches_summary.csv)"}},
             "roofline_step": {"bound": "pcie", "achieved": value / world * N_BYTES / 1e9,
                               "peak": link_peak, "unit": "GB/s",
                               "frac": value / world * N_BYTES / 1e9 / link_peak,

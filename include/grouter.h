@@ -430,6 +430,13 @@ grouter_status grouter_sched_enqueue(grouter_sched *s, uint32_t tenant, uint64_t
  * ENOENT when nothing is backlogged. */
 grouter_status grouter_sched_dispatch(grouter_sched *s, uint32_t *tenant, uint64_t *ids,
                                       uint32_t *n, uint64_t *bytes, uint64_t *pass_after);
+/* The pass / virtual-time updates the dispatch of `tenant`'s n bytes (in
+ * chunks of `chunk` bytes, the last one partial) would make if the tenant
+ * were alone on the server -- what the library applies when a transfer
+ * bypasses the queues of an idle server (direct launches, idle copy
+ * engines), so later contention sees the same state.  The tenant must have
+ * nothing queued.  EINVAL on a null scheduler or chunk == 0. */
+grouter_status grouter_sched_account_solo(grouter_sched *s, uint32_t tenant, uint64_t n, uint64_t chunk);
 void grouter_sched_free(grouter_sched *s);
 
 const char *grouter_strerror(grouter_status st);

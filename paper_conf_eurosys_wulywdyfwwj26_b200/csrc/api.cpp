@@ -1315,6 +1315,13 @@ grouter_status grouter_sched_dispatch(grouter_sched *s, uint32_t *tenant, uint64
   return GROUTER_OK;
 }
 
+grouter_status grouter_sched_account_solo(grouter_sched *s, uint32_t tenant, uint64_t n, uint64_t chunk) {
+  if (!s || !chunk) return fail(GROUTER_EINVAL, "sched_account_solo: bad argument");
+  auto it = s->w.find(tenant);
+  s->s.account_solo(tenant, n, chunk, it == s->w.end() ? 1u : it->second);
+  return GROUTER_OK;
+}
+
 void grouter_sched_free(grouter_sched *s) { delete s; }
 
 static void dump_fences(std::ostringstream &o, grouter_ctx *c, const Fences &f) {

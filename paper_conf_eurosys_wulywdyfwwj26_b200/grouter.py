@@ -163,6 +163,7 @@ SIGNATURES = {
     "grouter_sched_enqueue": (_ST, [_P, _U32, _U64, _U64]),
     "grouter_sched_dispatch": (_ST, [_P, C.POINTER(_U32), C.POINTER(_U64), C.POINTER(_U32),
                                      C.POINTER(_U64), C.POINTER(_U64)]),
+    "grouter_sched_account_solo": (_ST, [_P, C.c_uint32, C.c_uint64, C.c_uint64]),
     "grouter_sched_free": (None, [_P]),
     "grouter_strerror": (C.c_char_p, [_ST]),
     "grouter_last_error": (C.c_char_p, []),
@@ -560,6 +561,9 @@ class Sched:
 
     def enqueue(self, t, cid, nbytes):
         return self.lib.grouter_sched_enqueue(self.h, t, cid, nbytes)
+
+    def account_solo(self, t, n, chunk):
+        return self.lib.grouter_sched_account_solo(self.h, t, n, chunk)
 
     def dispatch(self):
         t, n, b, p = C.c_uint32(0), C.c_uint32(0), C.c_uint64(0), C.c_uint64(0)

@@ -144,6 +144,47 @@ def test_sched_parity_with_oracle(seed):
                 assert a[3] == orc.pass_[b[0]]
 
 
+@pytest.mark.parametrize("seed", range(25))
+def test_sched_account_solo_equals_queued_dispatch(seed):
+    """The fast paths (an idle server's direct launch / copy, engine.cpp
+    fast_direct, fast_ce) skip the queues but apply Stride::account_solo:
+    the same passes and virtual time as the oracle's stride scheduler
+    dispatching that tenant's chunks alone.  Checked by what it decides:
+    after a solo transfer by one tenant (queued and dispatched in the
+    oracle, accounted in the library), a contended workload of several
+    tenants dispatches identically, with identical passes."""
+    rng = random.Random(700 + seed)
+    w = {t: rng.choice([1, 2, 3, 4, 8]) for t in range(1, rng.randint(2, 6))}
+    C_ = rng.choice([2 << 20, 1 << 20, 4096 * rng.randint(1, 512)])
+    lib, orc = G.Sched(5), ostride.StrideServer()
+    for t, x in w.items():
+        lib.set_weight(t, x)
+    cid = 0
+    for rep in range(rng.randint(1, 4)):              # solo transfers, possibly by several tenants in turn
+        t = rng.choice(list(w))
+        n = rng.randint(1, 40 << 20)
+        full, last = divmod(n, C_)
+        for b in [C_] * full + ([last] if last else []):
+            orc.enqueue(t, cid, b)
+            cid += 1
+        while orc.dispatch(w.get) is not None:
+            pass
+        assert lib.account_solo(t, n, C_) == G.OK
+    for t in w:                                        # then contention
+        for _ in range(rng.randint(1, 12)):
+            nb = rng.randint(1, C_)
+            lib.enqueue(t, cid, nb)
+            orc.enqueue(t, cid, nb)
+            cid += 1
+    while True:
+        a, b = lib.dispatch(), orc.dispatch(w.get)
+        if b is None:
+            assert a is None
+            break
+        assert (a[0], a[1], a[2]) == (b[0], b[1], b[2])
+        assert a[3] == orc.pass_[b[0]]
+
+
 @pytest.mark.parametrize("seed", range(30))
 def test_slo_weights_parity_with_oracle(seed):
     """grouter_slo_weights (C) == oracle/slo.weights on random SLO sets,
