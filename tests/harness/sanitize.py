@@ -69,4 +69,33 @@ s.synchronize()
 for d in dsts:
     assert G.test_verify(d.data_ptr(), n, 11, 0, 0)[1] == 0
 ctx.close()
+# cfg1 at full size on two logical GPUs in real time: the striped put relays
+# through logical GPU1's staging ring with one forward launch per chunk
+# (K4'), then a D2D get; once more with every copy on the peer branch
+for flags in (0, G.FORCE_REMOTE):
+    ops = T.cfg1(2, iters=2)
+    r = LibRunner(calib, replay=False, keep_bytes=False, flags=flags)
+    out = r(ops)
+    r.close()
+    orc = orun.run(ops, calib)
+    for o, l in zip(orc["records"], out["records"]):
+        assert o["status"] == l["status"] and o.get("digest") == l.get("digest")
+    assert out["stats"].kernel_launches > 0
+# blocking small puts/gets on an idle copy engine (fast_ce) and small direct copies (fast_direct)
+ctx = G.Ctx(G.config_from_calib(c1, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED], pool_floor_bytes=64 * MiB))
+host = torch.empty(1 << 20, dtype=torch.uint8, pin_memory=True)
+host.copy_(torch.arange(1 << 20, dtype=torch.int64).to(torch.uint8))
+cf = G.fn(3, 1, G.HOST)
+for i in range(6):
+    n = 4096 << i
+    st, oid = ctx.put(cf, host.data_ptr(), n, 0, 0)
+    G.check(st, "put")
+    st, ptr, nn = ctx.get(cf, oid, 0)
+    G.check(st, "get")
+    import ctypes
+    import numpy as np
+    assert bytes((ctypes.c_uint8 * n).from_address(ptr)) == host.numpy()[:n].tobytes()
+    ctx.release(cf, oid, ptr, 0)
+    ctx.free(cf, oid)
+ctx.close()
 print("sanitize workload OK", os.environ.get("GR_COPY", "default"))

@@ -17,4 +17,6 @@ timeout 600 ncu --cache-control none --clock-control none --metrics dram__bytes_
   -k regex:gr_copy -s 200 -c 20 --csv --log-file $D/steady.csv $B > $D/ncu_steady.log 2>&1
 timeout 1500 python tests/harness/workflows.py $D/cfg5i.json cfg5i > $D/cfg5i.log 2>&1
 timeout 900 python tests/harness/workflows.py $D/workflows.json > $D/workflows.log 2>&1
+# NVLink evidence when the box has two or more GPUs (in-round gpurun has one)
+if [ "$(nvidia-smi -L | wc -l)" -ge 2 ]; then bash tools/ncu_nvlink.sh; fi
 tail -c 300 $D/bench.json
