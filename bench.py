@@ -611,7 +611,8 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
     out = {"probe_h2d_GBps": [round(b / 1e9, 2) for b in calib["h2d_Bps"]],
            "probe_nvl_GBps": round(calib["nvl_Bps"] / 1e9, 1)}
     # TA off (GROUTER_NO_TOPOLOGY, Fig. 16): GPUs behind one PCIe switch both stage (R48)
-    for name, flags in (("direct", G.NO_MULTIPATH), ("striped", 0), ("striped_no_topology", G.NO_TOPOLOGY)):
+    for name, flags in (("direct", G.NO_MULTIPATH), ("striped", 0), ("striped_no_topology", G.NO_TOPOLOGY),
+                        ("striped_ce_relay", G.CE_RELAY)):
         ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, flags=flags,
                                         pool_cap=[G.UNLIMITED] * world, pool_floor_bytes=64 << 20))
         st, routes = ctx.route_set(0)
@@ -642,6 +643,7 @@ def measure_multipath(world, G, nbytes=1 << 30, reps=3):
         out[name]["GBps_by_size"] = sweep
         ctx.close()
     out["speedup"] = round(out["striped"]["GBps"] / out["direct"]["GBps"], 2)
+    out["ce_relay_speedup"] = round(out["striped_ce_relay"]["GBps"] / out["direct"]["GBps"], 2)
     out["topology_gain"] = round(out["striped"]["GBps"] / out["striped_no_topology"]["GBps"], 2)
     # gFn-host (L178, Fig. 5a): a GPU0 object read into host memory by a cFn,
     # direct D2H vs striped over R(0) (GROUTER_D2H_MULTIPATH)

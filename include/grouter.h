@@ -82,6 +82,11 @@ extern "C" {
                                       engines (the gFn-host plan, L178), restores come back over
                                       R(d) with relays like a fetch (L178, L366 "parallel PCIe
                                       transfers ... mitigate the overhead"); R47      */
+#define GROUTER_CE_RELAY      0x2000u/* host->GPU striping without the staging hop: route GPU r's copy
+                                      engine reads its share from host memory over r's PCIe link
+                                      and writes the destination's pages directly (over NVLink on
+                                      a multi-GPU box) -- no staging slot, no forward launch.
+                                      Opt-in until measured on a multi-GPU box */
 #define GROUTER_FORCE_REMOTE  0x1000u/* TEST ONLY: every copy-kernel round is launched as if its
                                       sources and destinations were on another GPU (the NVLink
                                       branch: system-scope fences, no L2 prefetch, no TMA bulk

@@ -544,7 +544,7 @@ static std::vector<Xfer *> whole_in_round(grouter_ctx *c, const Server &s, const
   for (auto &it : items) {
     Xfer *x = it.x;
     if (x->word_fenced || x->submitted_chunks || !x->waiters.empty()) continue;
-    if (s.kind == SK_H2D && it.dst_logical != s.logical) {
+    if (s.kind == SK_H2D && it.dst_logical != s.logical && !(c->cfg.flags & GROUTER_CE_RELAY)) {
       n[x] = UINT32_MAX;  // a relayed chunk: the forward kernel publishes
       continue;
     }
@@ -588,6 +588,7 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
 // for r itself land in the lease; relayed chunks go through r's staging ring
 // and a forward round kernel on r pushes them to their destination.
 static size_t round_h2d(grouter_ctx *c, Server &s) {
+  const bool ce_relay = (c->cfg.flags & GROUTER_CE_RELAY) != 0;
   const uint64_t budget = batch_budget(c, s);
   const uint64_t tr0 = tl_put_t0 ? now_ns() : 0;
   const uint32_t nb = refill_one(c, s);
@@ -604,8 +605,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   auto flush_run = [&]() {
     if (run_len) {
       const uint64_t tm = tl_put_t0 ? now_ns() : 0;
-      GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyHostToDevice,
-                              s.stream));
+      GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyDefault, s.stream));
       if (tl_put_t0) {  // profiling: put call -> its first H2D copy submitted
         const uint64_t te = now_ns();
         hprof().t[14] += te - tl_put_t0;
@@ -668,7 +668,10 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
     uint64_t src = it.src;
     uint32_t bslot = 0;
     if (it.x->pageable_src) src = bounce(c, it.src, it.bytes, &bslot);
-    if (it.dst_logical == s.logical) {
+    // GROUTER_CE_RELAY: the route GPU's copy engine reads host memory over its
+    // own PCIe link and writes the destination's pages directly (over NVLink
+    // on a multi-GPU box): no staging slot, no forward launch
+    if (it.dst_logical == s.logical || ce_relay) {
       if (run_len && !it.x->pageable_src && run_src + run_len == src && run_dst + run_len == it.dst) {
         run_len += it.bytes;
       } else {

@@ -292,6 +292,46 @@ def test_config_traces_forced_remote(replay):
         assert st.peer_launches == st.kernel_launches > 0
 
 
+@pytest.mark.parametrize("replay", [True, False])
+def test_ce_relay_parity(replay):
+    """GROUTER_CE_RELAY: the route GPUs' copy engines write the destination's
+    pages directly (no staging slot, no forward launch).  Random traces and
+    cfg1/cfg5 on virtual topologies equal the oracle (placements, victims,
+    bytes, dispatch logs: the relay changes the hop, not the plan), and a
+    striped put launches no kernel at all."""
+    for k, seed in ((2, 1), (3, 2), (4, 3)):
+        rng = random.Random(4000 + seed)
+        calib = C.virtual(k)
+        ops = T.random_trace(rng, k, n_ops=100, max_n=5 * MiB, run_seed=seed)
+        caps = [rng.choice([8, 16, 64]) * MiB for _ in range(k)]
+        orc, lib_out = _both(ops, calib, replay=replay, host_store_bytes=48 * MiB, pool_cap=caps,
+                             flags=G.CE_RELAY)
+        compare(orc, lib_out, check_dispatch=replay)
+    calib = C.virtual(4)
+    for ops in (T.cfg1(4, iters=3, scale=4), T.cfg5(4, requests=2, limit_frac=0.1, scale=64, layers=4)):
+        orc, lib_out = _both(ops, calib, replay=replay, flags=G.CE_RELAY)
+        assert compare(orc, lib_out, check_dispatch=replay) > 0
+    ctx = G.Ctx(G.config_from_calib(C.virtual(2), host_store_bytes=256 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    flags=G.CE_RELAY))
+    try:
+        n = 38_535_168
+        st, plan = ctx.plan(G.HOST, 0, n)
+        assert {c[3] for c in plan} == {0, 1}                 # striped over both routes
+        host = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        tmp = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(tmp.data_ptr(), n, 55, 0, 0))
+        host.copy_(tmp)
+        st, oid = ctx.put(G.fn(1, 1, G.HOST), host.data_ptr(), n, 0, 0)
+        G.check(st, "put")
+        assert ctx.stats().kernel_launches == 0               # no forward hop
+        st, nn = ctx.get_into(G.fn(1, 2, 0), oid, tmp.data_ptr(), n, 0)
+        G.check(st, "get_into")
+        assert G.test_verify(tmp.data_ptr(), n, 55, 0, 0)[1] == 0
+        ctx.free(G.fn(1, 1, G.HOST), oid)
+    finally:
+        ctx.close()
+
+
 def test_fig11b_restore():
     """PAPER.md L260-L262 worked example on the device: a2's output is
     migrated, then reloaded once a1's output has been processed."""
