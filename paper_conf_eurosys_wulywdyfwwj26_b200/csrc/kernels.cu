@@ -368,14 +368,16 @@ __device__ __forceinline__ void st256(V8 *p, const V8 &v) {
                : "memory");
 }
 
-// wv8: warp-strided copy with 256-bit accesses over 8 KiB units; warp w of W
-// takes units w, w+W, ...; each lane keeps 8 x 32 B loads in flight per
-// unit.  32 B co-aligned full units take the 256-bit path, 16 B co-aligned
-// ones a 16 B path with 8 loads in flight per lane, anything else bytes
-// (misaligned rounds go to ldst8 instead, see launch_copy).
-template <bool COUNT, class KP>
+// wv8: warp-strided copy with 256-bit accesses over 8 KiB units (LG = 13);
+// warp w of W takes units w, w+W, ...; each lane keeps 8 x 32 B loads in
+// flight per unit.  32 B co-aligned full units take the 256-bit path, 16 B
+// co-aligned ones a 16 B path with 8 loads in flight per lane, anything else
+// bytes (misaligned rounds go to ldst8 instead, see launch_copy).  Small
+// rounds (<= 4 MiB) use 1 KiB units (LG = 10, one 32 B load per lane): the
+// copy spreads over 8x more warps and SMs, so a latency-bound small copy
+// waits for one DRAM round trip per lane instead of eight in a row.
+template <bool COUNT, int LG, class KP>
 __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ KP p) {
-  constexpr int LG = 13;
   constexpr uint32_t kUnit = 1u << LG;
   constexpr int kPer = (int)(kUnit / (32 * 32));  // 32 B loads per lane per unit
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
@@ -561,12 +563,11 @@ static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   else launch_pdl(gr_copy_ldst<false, 8, 1, KP>, grid, kThreads, 0, s, p);
 }
 
-template <class KP>
+template <int LG, class KP>
 static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
-  constexpr int LG = 13;
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, KP>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, LG, KP>, kThreads, 0);
     if (occ <= 0) occ = 1;
   }
   const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
@@ -581,15 +582,26 @@ static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   const uint64_t cap = (uint64_t)sm_count * per_sm;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
-  if (p.counts) launch_pdl(gr_copy_wv<true, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_wv<false, KP>, grid, kThreads, 0, s, p);
+  if (p.counts) launch_pdl(gr_copy_wv<true, LG, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_wv<false, LG, KP>, grid, kThreads, 0, s, p);
+}
+
+static bool getenv_wv_big() {  // GR_WV_BIG=1: 8 KiB units at every size (measurement only)
+  static const bool b = getenv("GR_WV_BIG") != nullptr;
+  return b;
 }
 
 template <class KP>
 static void launch_engine(KP &p, int v, int sm_count, int ctas_per_sm, cudaStream_t s) {
   switch (v) {
     case kEngTmas4: launch_tmas(p, sm_count, s); break;
-    case kEngWv8: launch_wv(p, sm_count, ctas_per_sm, s); break;
+    case kEngWv8: {
+      uint64_t total = 0;
+      for (uint32_t i = 0; i < p.n_chunks; ++i) total += p.chunk[i].bytes;
+      if (total <= (4ull << 20) && !getenv_wv_big()) launch_wv<10>(p, sm_count, ctas_per_sm, s);
+      else launch_wv<13>(p, sm_count, ctas_per_sm, s);
+      break;
+    }
     default: launch_ldst(p, sm_count, ctas_per_sm, s); break;
   }
 }

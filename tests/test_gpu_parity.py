@@ -62,10 +62,12 @@ def test_verify_kernel_detects_corruption():
 
 
 # ------------------------------------------------------------------ copy kernel, exactly once
+@pytest.mark.parametrize("big", [True, False])
 @pytest.mark.parametrize("tma", [False, True])
 @pytest.mark.parametrize("src_off,dst_off", [(0, 0), (16, 32), (3, 3), (1, 0), (0, 5), (7, 13), (15, 1)])
-def test_copy_kernel_exactly_once(tma, src_off, dst_off):
-    _copy_exactly_once(tma, src_off, dst_off)
+def test_copy_kernel_exactly_once(tma, src_off, dst_off, big):
+    """big: 5 MiB + r (wv8 with 8 KiB units); small: 1 MiB + r (<= 4 MiB: 1 KiB units)."""
+    _copy_exactly_once(tma, src_off, dst_off, 5 if big else 1)
 
 
 VARIANTS = ["ldst8", "wv8", "tmas4"]
@@ -84,7 +86,7 @@ def test_copy_kernel_variants(variant):
     env = dict(os.environ, GR_COPY=name)
     env.update(kv.split("=", 1) for kv in extra)
     code = ("import sys; sys.path.insert(0, '.'); from tests.test_gpu_parity import _copy_exactly_once as f; "
-            "[f(t, a, b) for t in (False, True) for a, b in ((0, 0), (3, 3), (1, 0), (7, 13), (32, 64))]")
+            "[f(t, a, b, m) for m in (5, 1) for t in (False, True) for a, b in ((0, 0), (3, 3), (1, 0), (7, 13), (32, 64))]")
     r = subprocess.run([sys.executable, "-c", code], env=env,
                        capture_output=True, text=True, timeout=240)
     assert r.returncode == 0, r.stderr[-2000:]
@@ -124,12 +126,12 @@ def _copy_aligned(n, seed):
     assert (d[:128] == 0xA5).all() and (d[128 + n:] == 0xA5).all()
 
 
-def _copy_exactly_once(tma, src_off, dst_off):
+def _copy_exactly_once(tma, src_off, dst_off, mib=5):
     """Invariant I1 on the production kernel: every destination byte of a
     chunk list tiling [0, n) is written exactly once; bytes are identical;
     guard bands stay untouched."""
     rng = random.Random(src_off * 31 + dst_off + tma)
-    n = 5 * MiB + rng.randint(0, 4095)
+    n = mib * MiB + rng.randint(0, 4095)
     cuts = sorted(rng.sample(range(1, n), 6))
     bounds = [0] + cuts + [n]
     chunks = [(a, b - a, 0, 0) for a, b in zip(bounds, bounds[1:])]
