@@ -479,7 +479,10 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
                 xs.append((time.perf_counter() - t) * 1e6)
             return xs
 
-        for n in sizes:
+        import gc
+        gc_was = gc.isenabled()
+        gc.disable()          # no collector pauses inside single-call samples
+        for n in [sizes[0]] + list(sizes):   # the first size twice: its first pass is a warm-up
             reps = _samples(n)
             row = {"bytes": n}
             st, oid = ctx.put(cfn, hp, n, 0, 0)
@@ -513,11 +516,15 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
             s.synchronize()
             st, bad, _ = G.test_verify(dst_at(4), n, 31337, 0, 0)
             assert st == 0 and bad == 0, f"sweep get_into {n}: {bad} bytes differ"
-            lib1 = dev_single(gi, reps)
-            b2b = dev_b2b(gi, max(10, min(reps, 200)))
             for _ in range(3):
                 mc()
-            base1 = dev_single(mc, reps)
+            # single calls, library and baseline interleaved sample by sample (drift
+            # and host noise hit both alike)
+            lib1, base1 = [], []
+            for _ in range(reps):
+                lib1 += dev_single(gi, 1)
+                base1 += dev_single(mc, 1)
+            b2b = dev_b2b(gi, max(10, min(reps, 200)))
             bb2b = dev_b2b(mc, max(10, min(reps, 200)))
             row["get_into"] = dict(_stats(lib1, n, 2), b2b_us=round(b2b, 2), b2b_GBps=round(2 * n / b2b / 1e3, 1),
                                    b2b_frac_hbm=round(2 * n / b2b / 1e3 / hbm_peak, 3),
@@ -540,8 +547,10 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
             put_timed(3)
             for _ in range(3):
                 h2d()
-            lp = put_timed(reps)
-            bp = host_single(h2d, reps)
+            lp, bp = [], []
+            for _ in range(reps):
+                lp += put_timed(1)
+                bp += host_single(h2d, 1)
             row["put_h2d"] = dict(_stats(lp, n), frac_link=round(n / pct(lp, 50) / 1e3 / h2d_peak, 3),
                                   memcpy=_stats(bp, n))
             # cFn get (D2H into a host lease) vs bare D2H; the lease's release
@@ -562,8 +571,10 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
             get_timed(3)
             for _ in range(3):
                 d2h()
-            lg = get_timed(reps)
-            bg = host_single(d2h, reps)
+            lg, bg = [], []
+            for _ in range(reps):
+                lg += get_timed(1)
+                bg += host_single(d2h, 1)
             row["get_d2h"] = dict(_stats(lg, n), memcpy=_stats(bg, n))
 
             def zc_timed(reps):   # gFn zero-copy get; the release is outside the timed call
@@ -595,6 +606,9 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
                 row["oracle_get_into"] = {"p50_us": round(pct(xs, 50), 2), "samples": len(xs)}
             row["samples"] = reps
             out.append(row)
+        out = out[1:]                         # drop the warm-up pass
+        if gc_was:
+            gc.enable()
     finally:
         ctx.close()
     return out

@@ -90,8 +90,11 @@ extern "C" {
 #define GROUTER_FORCE_REMOTE  0x1000u/* TEST ONLY: every copy-kernel round is launched as if its
                                       sources and destinations were on another GPU (the NVLink
                                       branch: system-scope fences, no L2 prefetch, no TMA bulk
-                                      engine, completion published in-kernel), so one-GPU test
-                                      boxes execute the code a physical peer transfer runs    */
+                                      engine, completion published in-kernel), and a copy between
+                                      two logical GPUs never runs as a direct launch on the
+                                      consumer's stream (the source's copy server pushes, the
+                                      consumer waits on completion words), so one-GPU test boxes
+                                      execute the code a physical peer transfer runs          */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;

@@ -355,7 +355,12 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
     pump(c, false);
     return x2;
   }
-  if (caller && direct && n && server_kind_for(src_loc, dst_loc) == SK_COPY) {
+  // GROUTER_FORCE_REMOTE: a copy between two logical GPUs takes the path a
+  // physical pair takes (the consumer's stream is on another device there, so
+  // never a direct launch): the source's copy server pushes, the consumer
+  // stream waits on the completion words
+  const bool may_direct = !(c->cfg.flags & GROUTER_FORCE_REMOTE) || src_loc == dst_loc;
+  if (caller && direct && n && may_direct && server_kind_for(src_loc, dst_loc) == SK_COPY) {
     const int server = src_loc == GROUTER_REMOTE ? dst_loc : src_loc;
     XferRef fx = fast_direct(c, tenant, server, dst_loc, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, n,
                              pool_src && src_loc >= 0, deps, caller, c->dev[caller_logical].phys);
@@ -385,7 +390,7 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   enqueue_plan(c, x, plan, kind, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, dst_loc);
   if (hprof().on) hprof().t[4] += now_ns() - tst;
   if (direct) *direct = false;
-  if (caller && kind == SK_COPY && direct &&
+  if (caller && kind == SK_COPY && direct && may_direct &&
       try_direct(c, x, src_loc == GROUTER_REMOTE ? dst_loc : src_loc, caller, c->dev[caller_logical].phys)) {
     *direct = true;
     return x;
