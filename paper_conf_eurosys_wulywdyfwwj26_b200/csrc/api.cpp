@@ -560,6 +560,7 @@ grouter_status grouter_finalize(grouter_ctx *c) {
 // ------------------------------------------------------------------ put / alloc / seal
 grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src, uint64_t n,
                            int32_t hint, uint32_t consumers, void *stream, grouter_oid *out) {
+  gr::NvtxRange nvtx_("grouter_put", n);
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->seq++;
@@ -641,6 +642,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
 
 grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, int32_t hint,
                              uint32_t consumers, void **buf, grouter_oid *out) {
+  gr::NvtxRange nvtx_("grouter_alloc", n);
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->seq++;
@@ -675,6 +677,7 @@ grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, i
 }
 
 grouter_status grouter_seal(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *stream) {
+  gr::NvtxRange nvtx_("grouter_seal");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->seq++;
@@ -712,6 +715,7 @@ static grouter_status get_common(grouter_ctx *c, const grouter_fn *fn, grouter_o
 
 grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *stream,
                            const void **ptr, uint64_t *n_out) {
+  gr::NvtxRange nvtx_("grouter_get");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->seq++;
@@ -781,6 +785,7 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
 
 grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid, void *dst,
                                 uint64_t dst_cap, void *stream, uint64_t *n_out) {
+  gr::NvtxRange nvtx_("grouter_get_into");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   HostProf &hp = hprof();
   uint64_t t0 = hp.on ? now_ns() : 0, t1 = 0, t2 = 0, t3 = 0;
@@ -843,6 +848,7 @@ grouter_status grouter_get_into(grouter_ctx *c, const grouter_fn *fn, grouter_oi
 // ------------------------------------------------------------------ release / free
 grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid,
                                const void *ptr, void *stream) {
+  gr::NvtxRange nvtx_("grouter_release");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
@@ -883,6 +889,7 @@ grouter_status grouter_release(grouter_ctx *c, const grouter_fn *fn, grouter_oid
 }
 
 grouter_status grouter_free(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid) {
+  gr::NvtxRange nvtx_("grouter_free");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
@@ -902,6 +909,7 @@ grouter_status grouter_free(grouter_ctx *c, const grouter_fn *fn, grouter_oid oi
 // ------------------------------------------------------------------ cross-process handoff
 grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid,
                                   grouter_ipc_desc *desc) {
+  gr::NvtxRange nvtx_("grouter_export_ipc");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
@@ -949,6 +957,7 @@ grouter_status grouter_export_ipc(grouter_ctx *c, const grouter_fn *fn, grouter_
 
 grouter_status grouter_import_ipc(grouter_ctx *c, const grouter_fn *fn, const grouter_ipc_desc *d,
                                   uint32_t consumers, grouter_oid *out) {
+  gr::NvtxRange nvtx_("grouter_import_ipc");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();
@@ -1086,6 +1095,7 @@ grouter_status grouter_set_next_use(grouter_ctx *c, grouter_oid oid, uint64_t po
 }
 
 grouter_status grouter_set_pool_limit(grouter_ctx *c, int32_t d, uint64_t bytes) {
+  gr::NvtxRange nvtx_("grouter_set_pool_limit");
   if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
   Guard g(c);
   c->victims.clear();

@@ -10,6 +10,7 @@
 
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <cstdint>
 #include <cstring>
@@ -72,6 +73,27 @@ struct Driver {
   CUresult (*launchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **);
 };
 const Driver &drv();
+
+// NVTX ranges (SURVEY §5 tracing): one per data-path call and one per
+// dispatch round / direct launch, in the "grouter" domain, with the bytes as
+// payload.  nvtx3 is header-only: without an attached tool (nsys, ncu range
+// replay) a push/pop costs a few ns.
+nvtxDomainHandle_t nvtx_domain();
+struct NvtxRange {
+  explicit NvtxRange(const char *name, uint64_t bytes = 0) {
+    nvtxEventAttributes_t a = {};
+    a.version = NVTX_VERSION;
+    a.size = NVTX_EVENT_ATTRIB_STRUCT_SIZE;
+    a.messageType = NVTX_MESSAGE_TYPE_ASCII;
+    a.message.ascii = name;
+    a.payloadType = NVTX_PAYLOAD_TYPE_UNSIGNED_INT64;
+    a.payload.ullValue = bytes;
+    nvtxDomainRangePushEx(nvtx_domain(), &a);
+  }
+  ~NvtxRange() { nvtxDomainRangePop(nvtx_domain()); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 // Saves/restores the caller's current device around library work.
 struct DeviceGuard {

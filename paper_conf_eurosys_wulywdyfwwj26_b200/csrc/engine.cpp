@@ -495,6 +495,7 @@ void harvest_profile(grouter_ctx *c, bool wait) {
 // SM-copy server: one kernel launch per round segment (D2D push over
 // NVLink, or a same-GPU HBM copy).
 static size_t round_copy(grouter_ctx *c, Server &s) {
+  NvtxRange nvtx_("round copy");
   const uint32_t nb = refill_one(c, s);
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
@@ -588,6 +589,7 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
 // for r itself land in the lease; relayed chunks go through r's staging ring
 // and a forward round kernel on r pushes them to their destination.
 static size_t round_h2d(grouter_ctx *c, Server &s) {
+  NvtxRange nvtx_("round h2d");
   const bool ce_relay = (c->cfg.flags & GROUTER_CE_RELAY) != 0;
   const uint64_t budget = batch_budget(c, s);
   const uint64_t tr0 = tl_put_t0 ? now_ns() : 0;
@@ -711,6 +713,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
 // D2H server: CE copies device -> host (host store, host leases, caller
 // host buffers, and urgent spills).
 static size_t round_d2h(grouter_ctx *c, Server &s) {
+  NvtxRange nvtx_("round d2h");
   const uint32_t nb = refill_one(c, s);
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
@@ -813,6 +816,7 @@ void flush_all(grouter_ctx *c) {
 XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
                     int caller_phys) {
+  NvtxRange nvtx_("fast direct copy", n);
   static const bool off = getenv("GR_NO_FAST") != nullptr || getenv("GR_COPY") != nullptr;
   const uint32_t never = GROUTER_LOG | GROUTER_PROFILE | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
   if (off || c->replay || !caller || (c->cfg.flags & never) || !n || ((src | dst) & 15)) return nullptr;
@@ -888,6 +892,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
 // (no LOG / PROFILE); null when the queued path must be used.
 XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<grouter_chunk> &plan, uint64_t src,
                 uint64_t dst, uint64_t n, const Fences &deps) {
+  NvtxRange nvtx_(kind == SK_H2D ? "fast ce h2d" : "fast ce d2h", n);
   static const bool off = getenv("GR_NO_FAST") != nullptr;
   if (off || c->replay || (c->cfg.flags & (GROUTER_LOG | GROUTER_PROFILE)) || plan.empty()) return nullptr;
   const int route = plan[0].route_gpu;
@@ -930,6 +935,7 @@ XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<gro
 }
 
 bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream_t caller, int caller_phys) {
+  NvtxRange nvtx_("direct launch");
   if (c->replay || !caller) return false;
   Server &s = c->dev[server_logical].copy;
   if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty()) return false;
@@ -996,6 +1002,7 @@ bool try_direct(grouter_ctx *c, const XferRef &x, int server_logical, cudaStream
 // GPU's copy engine reading its share straight from the source pool pages
 // (mapped for every GPU) -- the gFn-host plan of L178 / R45.
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
+  NvtxRange nvtx_("spill", o.n);
   std::vector<grouter_chunk> plan;
   if (c->cfg.flags & GROUTER_STRIPED_MIGRATION) c->planner.plan_h2d(o.loc, o.n, plan);
   else c->planner.plan_single(o.n, o.loc, plan);
@@ -1021,6 +1028,7 @@ void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst) {
 // urgent, unscheduled transfer, single-path on d's own H2D engine (R42), or
 // striped over R(d) with relays under GROUTER_STRIPED_MIGRATION (R47).
 void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst) {
+  NvtxRange nvtx_("restore", o.n);
   std::vector<grouter_chunk> plan;
   if (c->cfg.flags & GROUTER_STRIPED_MIGRATION) c->planner.plan_h2d(d, o.n, plan);
   else c->planner.plan_single(o.n, d, plan);

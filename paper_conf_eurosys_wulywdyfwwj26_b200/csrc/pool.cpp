@@ -64,6 +64,11 @@ uint64_t now_ns() {
       .count();
 }
 
+nvtxDomainHandle_t nvtx_domain() {
+  static nvtxDomainHandle_t d = nvtxDomainCreateA("grouter");
+  return d;
+}
+
 // ------------------------------------------------------------------ errors
 static thread_local std::string tl_error;
 void set_error(const std::string &msg) { tl_error = msg; }
