@@ -816,7 +816,6 @@ void flush_all(grouter_ctx *c) {
 XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
                     int caller_phys) {
-  NvtxRange nvtx_("fast direct copy", n);
   static const bool off = getenv("GR_NO_FAST") != nullptr || getenv("GR_COPY") != nullptr;
   const uint32_t never = GROUTER_LOG | GROUTER_PROFILE | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
   if (off || c->replay || !caller || (c->cfg.flags & never) || !n || ((src | dst) & 15)) return nullptr;
@@ -831,6 +830,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
     }
   for (auto &w : deps)
     if (!is_submitted(w)) return nullptr;
+  NvtxRange nvtx_("fast direct copy", n);
   const uint64_t C = c->cfg.chunk_bytes;
   auto x = std::make_shared<Xfer>();
   x->id = ++c->xfer_seq;
@@ -892,7 +892,6 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
 // (no LOG / PROFILE); null when the queued path must be used.
 XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<grouter_chunk> &plan, uint64_t src,
                 uint64_t dst, uint64_t n, const Fences &deps) {
-  NvtxRange nvtx_(kind == SK_H2D ? "fast ce h2d" : "fast ce d2h", n);
   static const bool off = getenv("GR_NO_FAST") != nullptr;
   if (off || c->replay || (c->cfg.flags & (GROUTER_LOG | GROUTER_PROFILE)) || plan.empty()) return nullptr;
   const int route = plan[0].route_gpu;
@@ -906,6 +905,7 @@ XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<gro
   }
   for (auto &w : deps)
     if (!is_submitted(w)) return nullptr;
+  NvtxRange nvtx_(kind == SK_H2D ? "fast ce h2d" : "fast ce d2h", n);
   auto x = std::make_shared<Xfer>();
   x->id = ++c->xfer_seq;
   x->tenant = tenant;
