@@ -63,6 +63,11 @@ grouter_status grouter_test_race(int32_t iters, int64_t *out);
  * the full length needed in *len (may be NULL). */
 grouter_status grouter_test_dump(grouter_ctx *ctx, char *buf, uint64_t cap, uint64_t *len);
 
+/* Fault injection (tests only): what = 1 -- the next `count` dispatch rounds
+ * fail as a CUDA error would (the context turns sticky-ECUDA; callers blocked
+ * waiting for a submission wake up and fail instead of hanging). */
+grouter_status grouter_test_inject(grouter_ctx *ctx, int32_t what, int32_t count);
+
 /* Fixes the clock the pool-sizing samples and targets use (fixed != 0) to
  * t_ns, or returns to the monotonic clock (fixed == 0).  For deterministic
  * parity traces (R44). */

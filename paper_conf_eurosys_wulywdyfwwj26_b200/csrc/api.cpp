@@ -254,7 +254,7 @@ void block_on(grouter_ctx *c, Guard &g, const Fences &f) {
   g.lk.unlock();
   if (hprof().on) hprof().t[13] += now_ns() - t0;  // pump + daemon notify
   const uint64_t t1 = hprof().on ? now_ns() : 0;
-  host_wait(f);
+  host_wait(f, 120.0, &c->sticky_error);
   if (hprof().on) hprof().t[15] += now_ns() - t1;
 }
 
@@ -1240,6 +1240,13 @@ grouter_status grouter_pool_target(grouter_ctx *c, int32_t d, uint64_t *target) 
   Guard g(c);
   if (d < 0 || d >= (int)c->dev.size()) return fail(GROUTER_EINVAL, "pool_target: bad device");
   *target = pool_target(c, d);
+  return GROUTER_OK;
+}
+
+grouter_status grouter_test_inject(grouter_ctx *c, int32_t what, int32_t count) {
+  if (!c || what != 1 || count < 0) return fail(GROUTER_EINVAL, "test_inject: bad argument");
+  Guard g(c);
+  c->inject_round_failures = count;
   return GROUTER_OK;
 }
 

@@ -300,6 +300,7 @@ struct grouter_ctx {
   std::condition_variable submit_cv;                   // a transfer became fully submitted
   bool stop = false;
   std::atomic<bool> sticky_error{false};
+  int inject_round_failures = 0;                       // grouter_test_inject (tests only)
   // cross-process export (ipc.cpp)
   uint32_t ctx_id = 0;
   int ipc_listen = -1;
@@ -342,7 +343,9 @@ void done_fences(const XferRef &x, Fences &f);
 bool is_submitted(const Waitable &w);
 EventRef record(grouter_ctx *c, cudaStream_t s, int phys);       // library streams only
 Waitable signal(grouter_ctx *c, cudaStream_t s, int phys);       // caller streams
-void host_wait(const Fences &f, double timeout_s = 120.0);
+// abort (optional): a sticky-error flag; a wait on words that will never be
+// written (the producing round failed) ends with ECUDA instead of the timeout
+void host_wait(const Fences &f, double timeout_s = 120.0, const std::atomic<bool> *abort = nullptr);
 bool grounded(const grouter_ctx *c, const Fences &f);
 void spill_copy(grouter_ctx *c, Obj &o, uint8_t *host_dst);  // D2H of a victim (unscheduled)
 void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst);  // H2D back home (unscheduled)

@@ -115,7 +115,7 @@ EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
   return e;
 }
 
-void host_wait(const Fences &f, double timeout_s) {
+void host_wait(const Fences &f, double timeout_s, const std::atomic<bool> *abort) {
   auto t0 = std::chrono::steady_clock::now();
   for (auto &w : f) {
     if (w.ev && !w.word) {
@@ -130,6 +130,8 @@ void host_wait(const Fences &f, double timeout_s) {
     while (!w.done()) {
       if (++spins > 64) std::this_thread::yield();
       if ((spins & 1023) == 0) {
+        if (abort && abort->load(std::memory_order_relaxed))
+          throw Error(GROUTER_ECUDA, "sticky CUDA error while waiting for a transfer");
         double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
         if (dt > timeout_s) throw Error(GROUTER_ECUDA, "timeout waiting for a transfer");
       }
@@ -772,6 +774,10 @@ static size_t pump_server(grouter_ctx *c, Server &s, bool force) {
   if (!force && s.inflight.size() >= 2) retire(s);
   size_t total = 0;
   while (has_work(s) && (force || s.inflight.size() < 2 || (retire(s), s.inflight.size() < 2))) {
+    if (c->inject_round_failures > 0) {  // grouter_test_inject: fault injection (tests only)
+      --c->inject_round_failures;
+      throw Error(GROUTER_ECUDA, "injected dispatch-round failure (grouter_test_inject)");
+    }
     size_t n = s.kind == SK_COPY ? round_copy(c, s) : s.kind == SK_H2D ? round_h2d(c, s) : round_d2h(c, s);
     if (!n) break;  // blocked on another server's submission
     total += n;

@@ -176,6 +176,7 @@ SIGNATURES = {
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
     "grouter_test_memcpy": (_ST, [_P, _P, C.c_uint64, _P, C.c_int32]),
     "grouter_test_race": (_ST, [C.c_int32, C.POINTER(C.c_int64)]),
+    "grouter_test_inject": (_ST, [_CTX, C.c_int32, C.c_int32]),
 }
 
 _lib = None
@@ -377,6 +378,10 @@ class Ctx:
         v = C.c_uint64(0)
         check(self.lib.grouter_pool_target(self.h, dev, C.byref(v)), "pool_target")
         return v.value
+
+    def inject_round_failures(self, count):
+        """Fault injection (tests only): the next `count` dispatch rounds fail."""
+        return self.lib.grouter_test_inject(self.h, 1, count)
 
     def set_clock(self, t_ns=None):
         """Fix the pool-sizing clock to t_ns (None: back to the monotonic clock)."""

@@ -829,6 +829,49 @@ def test_two_batches_in_flight_under_contention():
         ctx.close()
 
 
+def test_blocked_callers_fail_on_sticky_error():
+    """A dispatch round that fails (here injected: grouter_test_inject) turns
+    the context sticky-ECUDA, and every caller waiting for work that will now
+    never be submitted returns ECUDA at once instead of hanging: a device
+    caller blocked in order_after (its H2D queued behind a saturating put)
+    and the host caller blocked in that put.  The context still closes."""
+    import threading
+    import time
+    calib = dict(C.b200_hgx(1), device_map=[0])
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=512 * MiB, pool_cap=[G.UNLIMITED]))
+    closed = False
+    try:
+        big, small = 256 * MiB, 8 * MiB
+        host = torch.empty(big, dtype=torch.uint8, pin_memory=True)
+        st, o_host = ctx.put(G.fn(1, 1, G.HOST), host.data_ptr(), small, G.NOHINT, 0)   # in the host store
+        G.check(st, "put")
+        res = {}
+
+        def saturate():
+            t = time.perf_counter()
+            res["put"] = ctx.put(G.fn(2, 1, G.HOST), host.data_ptr(), big, 0, 0)[0]
+            res["put_s"] = time.perf_counter() - t
+        th = threading.Thread(target=saturate)
+        th.start()
+        time.sleep(0.02)                                    # the big put owns the H2D engine
+        G.check(ctx.inject_round_failures(1), "inject")
+        dst = torch.empty(small, dtype=torch.uint8, device="cuda")
+        s = torch.cuda.Stream()
+        t = time.perf_counter()
+        st, _ = ctx.get_into(G.fn(1, 2, 0), o_host, dst.data_ptr(), small, s.cuda_stream)
+        dt = time.perf_counter() - t
+        th.join(timeout=30)
+        assert not th.is_alive(), "the blocked put hung"
+        assert st == G.ECUDA and dt < 10, (G.STATUS[st], dt)
+        assert res["put"] in (G.OK, G.ECUDA) and res["put_s"] < 30, res
+        assert ctx.sync() == G.ECUDA                         # sticky
+        ctx.close()
+        closed = True
+    finally:
+        if not closed:
+            ctx.close()
+
+
 def test_probe_calibration():
     """grouter_probe (a5, L178/L131/L271): on one B200 the solo pinned H2D rate
     is a PCIe Gen5 x16 figure, per-copy and first-chunk costs are positive,
