@@ -36,6 +36,8 @@ Also in the line:
                GB/s of same-GPU get_into, cFn put (H2D), cFn get (D2H) and
                zero-copy get, each beside a bare cudaMemcpyAsync on the same
                buffers through the same binding, plus the oracle's get_into
+  cfg2         BASELINE configs[1] (traffic monitoring) at one GPU: req/s of the
+               frame put + zero-copy fan-out, wall clock
   cpu_baseline the oracle (oracle/, numpy memcpy on simulated buffers) on the
                same cfg1 request, single-threaded as it stands, plus the
                striped put variant (one thread per route of the 8-GPU HGX
@@ -884,6 +886,90 @@ def nccl_ring_baseline(world, rank, dev, n, per_step, steps):
 
 # ------------------------------------------------------------------ GPU arm
 
+# ------------------------------------------------------------------ cfg2 (BASELINE configs[1]) at one GPU
+def measure_cfg2(G, dev, seconds=2.0, outstanding=4):
+    """Traffic-monitoring workflow (BASELINE configs[1]),
+    data plane only, closed loop with `outstanding` clients: a decode cFn puts a
+    39,321,600 B frame (8x3x640x640 fp32) with hint GPU0 (PCIe H2D); the YOLO
+    gFn gets it (zero copy, co-located), allocs + seals person and vehicle crop
+    batches (K x 602,112 B, K ~ Poisson(4) clipped to [0, 32]); the two
+    recognition gFns get them (zero copy at one GPU) and everyone releases.
+    Wall-clock req/s and per-request latency."""
+    import math
+    import random
+    import torch
+    from synth.calib import b200_hgx
+    FRAME, CROP = 39_321_600, 602_112
+    calib = b200_hgx(1)
+    calib["device_map"] = [dev]
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED]))
+    frames = [torch.empty(FRAME, dtype=torch.uint8, pin_memory=True) for _ in range(outstanding)]
+    streams = [torch.cuda.Stream(device=dev) for _ in range(outstanding)]
+    lat, done, stop = [], [0] * outstanding, threading.Event()
+    go = threading.Barrier(outstanding + 1)
+
+    def poisson(rng, lam=4.0):
+        L, k, p = math.exp(-lam), 0, 1.0
+        while True:
+            p *= rng.random()
+            if p <= L:
+                return min(k, 32)
+            k += 1
+
+    def worker(t):
+        torch.cuda.set_device(dev)
+        rng = random.Random(2000 + t)
+        s = streams[t].cuda_stream
+        go.wait()
+        i = 0
+        while not stop.is_set():
+            wf = 10 + t * 100000 + i
+            dec, yolo, rp, rv = G.fn(wf, 1, G.HOST), G.fn(wf, 2, 0), G.fn(wf, 3, 0), G.fn(wf, 4, 0)
+            t0 = time.perf_counter()
+            st, o = ctx.put(dec, frames[t].data_ptr(), FRAME, 0, 1)
+            G.check(st, "put")
+            st, fp, _ = ctx.get(yolo, o, s)
+            G.check(st, "get")
+            crops = []
+            for k in (poisson(rng), poisson(rng)):
+                st, buf, a = ctx.alloc(yolo, k * CROP, G.NOHINT, 1)
+                G.check(st, "alloc")
+                G.check(ctx.seal(yolo, a, s), "seal")
+                crops.append(a)
+            leases = []
+            for f, a in ((rp, crops[0]), (rv, crops[1])):
+                st, ptr, _ = ctx.get(f, a, s)
+                G.check(st, "get crops")
+                leases.append((f, a, ptr))
+            G.check(ctx.release(yolo, o, fp, s), "release")
+            for f, a, ptr in leases:
+                if ptr:
+                    G.check(ctx.release(f, a, ptr, s), "release crops")
+            streams[t].synchronize()
+            lat.append((time.perf_counter() - t0) * 1e6)
+            done[t] += 1
+            i += 1
+    ths = [threading.Thread(target=worker, args=(t,)) for t in range(outstanding)]
+    for th in ths:
+        th.start()
+    go.wait()
+    t0 = time.perf_counter()
+    time.sleep(seconds)
+    stop.set()
+    for th in ths:
+        th.join()
+    dt = time.perf_counter() - t0
+    ctx.sync()
+    used = ctx.stats().used[0]
+    ctx.close()
+    n = sum(done)
+    return {"what": "cfg2 traffic monitoring (BASELINE configs[1]) at one GPU, data plane: frame put + zero-copy "
+                    "YOLO get + crop alloc/seal + two zero-copy recognition gets, 4 clients, wall clock",
+            "req_per_s": round(n / dt, 1), "frame_GBps": round(n * FRAME / dt / 1e9, 2),
+            "latency_us": {"p50": round(pct(lat, 50), 1), "p99": round(pct(lat, 99), 1)}, "requests": n,
+            "pool_used_after": used}
+
+
 # ------------------------------------------------------------------ GPU arm
 def h2d_link_peak(G, dev, nbytes=256 << 20, reps=4):
     """Pinned single-link H2D GB/s on this box (bare cudaMemcpyAsync back to
@@ -1145,6 +1231,13 @@ def run_gpu(args, rank, world, local_rank):
         except Exception as e:   # reported, never fatal for the line
             sweep = [{"error": f"{type(e).__name__}: {e}"[:300]}]
 
+    cfg2 = None
+    if rank == 0 and world == 1 and not args.no_sweep:
+        try:
+            cfg2 = measure_cfg2(G, dev)
+        except Exception as e:   # reported, never fatal for the line
+            cfg2 = {"error": f"{type(e).__name__}: {e}"[:300]}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline_obj(args.cpu_seconds)
@@ -1205,6 +1298,8 @@ def run_gpu(args, rank, world, local_rank):
             "gpu_launches": launches,
             "clocks": clocks,
         }
+        if cfg2 is not None:
+            line["cfg2"] = cfg2
         if sweep is not None:
             line["sweep"] = sweep
         if nccl is not None:
