@@ -904,7 +904,8 @@ XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<gro
   for (auto &ch : plan)
     if (ch.route_gpu != route || ch.path != 0) return nullptr;  // striped: the queued path relays
   Server &s = server_of(c, kind, route);
-  if (n > 2 * batch_budget(c, s) || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
+  if (plan.size() > 2ull * s.sched.batch || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty())
+    return nullptr;  // more than two batches: the queued path keeps them preemptible (O8)
   if (!s.inflight.empty()) {
     retire(s);
     if (!s.inflight.empty()) return nullptr;
