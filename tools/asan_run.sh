@@ -7,7 +7,8 @@ set -x
 D=gpurun_out/asan
 mkdir -p $D
 python paper_conf_eurosys_wulywdyfwwj26_b200/_build.py --asan
-export LD_PRELOAD=$(gcc -print-file-name=libasan.so) GROUTER_LIB=asan
+# libstdc++ preloaded too: the runtime must see it at start (the library throws C++ exceptions)
+export LD_PRELOAD="$(gcc -print-file-name=libasan.so) $(gcc -print-file-name=libstdc++.so)" GROUTER_LIB=asan
 export ASAN_OPTIONS="protect_shadow_gap=0:detect_leaks=0:halt_on_error=0:log_path=$D/asan"
 GR_STRESS_OPS=200 timeout 1200 python -m pytest tests/test_gpu_concurrency.py -m gpu -q -p no:cacheprovider > $D/stress_pytest.txt 2>&1
 echo stress_rc=$?
