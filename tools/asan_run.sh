@@ -1,7 +1,9 @@
 #!/bin/bash
 # AddressSanitizer build of the host library under the concurrency
 # stress and the real-time soak; CUDA needs protect_shadow_gap=0, leak
-# checking is off (the CUDA runtime keeps allocations until exit).  Reports land
+# checking is off (the CUDA runtime keeps allocations until exit).  The two-process
+# IPC test is left out: its child process inherits the preload and cannot create
+# a CUDA context under it ("device busy or unavailable").  Reports land
 # in gpurun_out/asan/.
 set -x
 D=gpurun_out/asan
@@ -13,7 +15,7 @@ export ASAN_OPTIONS="protect_shadow_gap=0:detect_leaks=0:halt_on_error=0:log_pat
 GR_STRESS_OPS=200 timeout 1200 python -m pytest tests/test_gpu_concurrency.py -m gpu -q -p no:cacheprovider > $D/stress_pytest.txt 2>&1
 echo stress_rc=$?
 GR_SOAK_SEEDS=6 timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_ipc.py -m gpu -q -p no:cacheprovider \
-  -k "random_traces_realtime or two_batches or forced_remote or ce_relay or sticky or two_processes or two_contexts" > $D/soak_pytest.txt 2>&1
+  -k "random_traces_realtime or two_batches or forced_remote or ce_relay or sticky or two_contexts" > $D/soak_pytest.txt 2>&1
 echo soak_rc=$?
 tail -n 3 $D/stress_pytest.txt $D/soak_pytest.txt
 ls $D
