@@ -57,6 +57,9 @@ grouter_status grouter_test_memcpy(void *dst, const void *src, uint64_t n, void 
  * a ThreadSanitizer build must report exactly this data race.  Returns the
  * final count in *out (any value; the race is the point). */
 grouter_status grouter_test_race(int32_t iters, int64_t *out);
+/* Positive control for AddressSanitizer builds: a deliberate one-past-the-end
+ * heap read (the sanitizer must report it; a product build just returns). */
+grouter_status grouter_test_oob(int32_t *out);
 
 /* Text dump of the context's internal state (servers, objects, leases,
  * pending completion words) for debugging; truncated to cap bytes.  Returns

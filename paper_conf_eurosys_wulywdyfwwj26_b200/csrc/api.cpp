@@ -435,6 +435,16 @@ static void race_body(int32_t iters) {
     g_race_counter = v + 1;
   }
 }
+// Positive control for AddressSanitizer builds: reads one element past the
+// end of a heap array (an ASan build reports a heap-buffer-overflow here).
+grouter_status grouter_test_oob(int32_t *out) {
+  if (!out) return GROUTER_EINVAL;
+  std::vector<int32_t> v(4, 7);
+  volatile int32_t *p = v.data();
+  *out = p[4];
+  return GROUTER_OK;
+}
+
 grouter_status grouter_test_race(int32_t iters, int64_t *out) {
   if (!out || iters < 0) return GROUTER_EINVAL;
   g_race_counter = 0;

@@ -176,6 +176,7 @@ SIGNATURES = {
     "grouter_test_copy": (_ST, [_P, _P, C.POINTER(grouter_chunk), _U32, _P, C.c_int, _P]),
     "grouter_test_memcpy": (_ST, [_P, _P, C.c_uint64, _P, C.c_int32]),
     "grouter_test_race": (_ST, [C.c_int32, C.POINTER(C.c_int64)]),
+    "grouter_test_oob": (_ST, [C.POINTER(C.c_int32)]),
     "grouter_test_inject": (_ST, [_CTX, C.c_int32, C.c_int32]),
 }
 
