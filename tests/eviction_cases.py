@@ -81,4 +81,28 @@ def case_d():
     return b.ops, {"pool_cap": [2 * MiB], "host_store_bytes": 4 * MiB}
 
 
-CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d}
+def case_e():
+    """Status rules of the boundary (SURVEY §8(b) conventions, R19, R35)."""
+    b = T.Builder(25)
+    g, other = T.fn(1, 1, 0), T.fn(2, 1, 0)
+    o1 = b.alloc(g, MiB)                                    # 0 OPEN
+    b.free(g, o1)                                           # 1 EBUSY
+    b.get(g, o1)                                            # 2 ENOENT (unsealed)
+    b.seal(other, o1)                                       # 3 EPERM
+    b.seal(g, o1)                                           # 4
+    b.seal(g, o1)                                           # 5 ESTATE
+    b.get_into(g, o1, cap=MiB - 1)                          # 6 EINVAL
+    z = b.get(g, o1)                                        # 7 zero copy
+    b.release(other, z)                                     # 8 EPERM
+    b.free(other, o1)                                       # 9 EPERM
+    b.weight(1, 0)                                          # 10 EINVAL
+    b.next_use(1, 5)                                        # 11 ENOENT (op 1 created nothing)
+    b.pool_limit(3, 0)                                      # 12 EINVAL (one GPU)
+    b.release(g, z)                                         # 13
+    b.free(g, o1)                                           # 14
+    b.get(g, o1)                                            # 15 ENOENT (freed)
+    b.flush()                                               # 16
+    return b.ops, {"host_store_bytes": 64 * MiB}
+
+
+CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d, "E": case_e}

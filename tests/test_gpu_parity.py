@@ -196,7 +196,7 @@ def test_golden_trace_on_virtual_pair():
 
 
 @pytest.mark.parametrize("replay", [True, False])
-@pytest.mark.parametrize("case", ["A", "B", "C", "D"])
+@pytest.mark.parametrize("case", ["A", "B", "C", "D", "E"])
 def test_eviction_branch_golden_cases(case, replay):
     """The hand-derived eviction-branch cases (tests/golden/eviction_branches.md:
     R15 mixed hints, R33/R16 all-or-nothing reserve, R34 limit below the

@@ -35,6 +35,12 @@ MUTATIONS = [
     ("R32 host admission >=", "        if self.host_used + c > self.H:", "        if self.host_used + c >= self.H:"),
     ("R32 host leases not charged", "            ok = self._host_reserve(c) if d == HOST else self._reserve(d, c)",
      "            ok = True if d == HOST else self._reserve(d, c)"),
+    ("seal twice accepted", "            return ESTATE, {}", "            pass"),
+    ("free of an OPEN object -> ENOENT", "            return EBUSY, {}", "            return ENOENT, {}"),
+    ("get_into accepts dst_cap = n - 1", "        if cap < o.n or (dst is None and o.n > 0):",
+     "        if cap < o.n - 1 or (dst is None and o.n > 0):"),
+    ("weight 0 accepted", "        if w < 1:", "        if w < 0:"),
+    ("R35 release of a pin skips the workflow check", '            if o.wf != fn["wf"]:', "            if False:"),
 ]
 
 
