@@ -105,4 +105,18 @@ def case_e():
     return b.ops, {"host_store_bytes": 64 * MiB}
 
 
-CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d, "E": case_e}
+def case_f():
+    """Placement rules (R23, R38; PAPER.md L165 locality): two GPUs."""
+    b = T.Builder(26)
+    g0, c, g1 = T.fn(1, 1, 0), T.fn(1, 2, T.HOST), T.fn(1, 3, 1)
+    o1 = b.put(g0, MiB, hint=1)                             # 0 gFn put: local, hint ignored
+    b.put(c, MiB, hint=1)                                   # 1 cFn put with a hint: staged to GPU1
+    b.put(c, MiB)                                           # 2 cFn put without a hint: host store
+    b.alloc(c, MiB, hint=1)                                 # 3 cFn alloc: caller's location (host)
+    b.alloc(g0, MiB, hint=1)                                # 4 gFn alloc: its own GPU
+    b.get(g1, o1)                                           # 5 another GPU: copy lease on GPU1
+    b.flush()                                               # 6
+    return b.ops, {"host_store_bytes": 64 * MiB, "n_gpus": 2}
+
+
+CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d, "E": case_e, "F": case_f}

@@ -196,7 +196,7 @@ def test_golden_trace_on_virtual_pair():
 
 
 @pytest.mark.parametrize("replay", [True, False])
-@pytest.mark.parametrize("case", ["A", "B", "C", "D", "E"])
+@pytest.mark.parametrize("case", ["A", "B", "C", "D", "E", "F"])
 def test_eviction_branch_golden_cases(case, replay):
     """The hand-derived eviction-branch cases (tests/golden/eviction_branches.md:
     R15 mixed hints, R33/R16 all-or-nothing reserve, R34 limit below the
@@ -207,8 +207,10 @@ def test_eviction_branch_golden_cases(case, replay):
     from tests.eviction_cases import CASES
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "eviction_branches.json")))
     ops, kw = CASES[case]()
-    calib = C.b200_hgx(1)
-    calib["device_map"] = [0]
+    kw = dict(kw)
+    k = kw.pop("n_gpus", 1)
+    calib = C.b200_hgx(k, shared_pairs=False)
+    calib["device_map"] = [0] * k
     orc, lib_out = _both(ops, calib, replay=replay, **kw)
     compare(orc, lib_out, check_dispatch=replay)
     for r in lib_out["records"]:

@@ -22,7 +22,8 @@ MiB = GOLD["MiB"]
 
 def _check(case):
     ops, kw = CASES[case]()
-    out = runner.run(ops, C.b200_hgx(1), **kw)
+    kw = dict(kw)
+    out = runner.run(ops, C.b200_hgx(kw.pop("n_gpus", 1), shared_pairs=False), **kw)
     recs, exp = out["records"], GOLD[case]["expect"]
     for r in recs:
         e = exp.get(str(r["i"]), {})

@@ -41,6 +41,10 @@ MUTATIONS = [
      "        if cap < o.n - 1 or (dst is None and o.n > 0):"),
     ("weight 0 accepted", "        if w < 1:", "        if w < 0:"),
     ("R35 release of a pin skips the workflow check", '            if o.wf != fn["wf"]:', "            if False:"),
+    ("R23 gFn put follows its hint", "            home = dev", "            home = hint if hint >= 0 else dev"),
+    ("R23 cFn hint ignored", "        elif hint >= 0:", "        elif False:"),
+    ("R38 alloc follows the hint", "        home = dev\n        if home != HOST:",
+     "        home = hint if hint >= 0 else dev\n        if home != HOST:"),
 ]
 
 
