@@ -51,9 +51,6 @@ if __name__ == "__main__":
     if len(sys.argv) > 1 and sys.argv[1] == "--child":
         child(sys.argv[2])
     else:
-        for v in (sys.argv[1:] or ["torch", "ldst8", "wv8", "tmas4"]):
-            name, _, ctas = v.partition("@")
+        for name in (sys.argv[1:] or ["torch", "ldst8", "wv8", "tmas4"]):
             env = dict(os.environ, GR_COPY=name)
-            if ctas:
-                env["GR_CTAS"] = ctas
             subprocess.run([sys.executable, __file__, "--child", name], env=env, timeout=300)

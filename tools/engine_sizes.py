@@ -69,8 +69,7 @@ def child():
         del dsts
         torch.cuda.empty_cache()
     ctx.close()
-    print(json.dumps({"engine": ("ce" if os.environ.get("GR_SIZES_CE") == "1" else os.environ.get("GR_COPY", "default"))
-                      + (f" ctas={os.environ['GR_TMAS_CTAS']}" if "GR_TMAS_CTAS" in os.environ else ""), "pf": os.environ.get("GR_PF", "1"),
+    print(json.dumps({"engine": "ce" if os.environ.get("GR_SIZES_CE") == "1" else os.environ.get("GR_COPY", "default"),
                       "res": out}), flush=True)
 
 
