@@ -264,6 +264,16 @@ static void log_batch(grouter_ctx *c, Server &s, uint32_t tenant,
   if (c->dlog.size() > (1u << 20)) c->dlog.pop_front();
 }
 
+// Per-tenant accounting of dispatched bytes (grouter_tenant_stats) and the
+// rate monitor's records (L197: 10 s of dispatch records per tenant).
+static void note_dispatch(grouter_ctx *c, uint32_t tenant, int kind, uint64_t bytes) {
+  c->tenant_bytes[tenant][kind] += bytes;
+  auto &lg = c->tenant_log[tenant];
+  const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
+  lg.emplace_back(now, bytes);
+  while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
+}
+
 // Moves whole batches (stride order, logged) from the scheduler into the
 // carry queue until the round budget is covered; returns how many.
 static uint32_t refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t max_bytes,
@@ -279,13 +289,7 @@ static uint32_t refill(grouter_ctx *c, Server &s, uint32_t max_batches, uint64_t
     uint32_t t = s.sched.dispatch([&](uint32_t tn) { return weight_of(c, tn); }, b, &bb);
     if (t == UINT32_MAX) break;
     log_batch(c, s, t, b, bb);
-    c->tenant_bytes[t][s.kind] += bb;
-    {  // rate monitor (L197): keep 10 s of dispatch records per tenant
-      auto &lg = c->tenant_log[t];
-      const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
-      lg.emplace_back(now, bb);
-      while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
-    }
+    note_dispatch(c, t, s.kind, bb);
     for (auto &it : b) s.carry.push_back(it);
     bytes += bb;
     ++nb;
@@ -867,13 +871,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   x->done_stream = caller;
   // the bookkeeping a queued dispatch would have done
   s.sched.account_solo(tenant, n, C, weight_of(c, tenant));
-  c->tenant_bytes[tenant][SK_COPY] += n;
-  {
-    auto &lg = c->tenant_log[tenant];
-    const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
-    lg.emplace_back(now, n);
-    while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
-  }
+  note_dispatch(c, tenant, SK_COPY, n);
   c->stats.link_bytes[0][s.logical] += n;
   c->stats.rounds++;
   c->stats.kernel_launches++;
@@ -927,13 +925,7 @@ XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<gro
   x->done_ev = record(c, s.stream, s.phys);
   x->done_stream = s.stream;
   s.sched.account_solo(tenant, n, plan[0].bytes, weight_of(c, tenant));
-  c->tenant_bytes[tenant][kind] += n;
-  {
-    auto &lg = c->tenant_log[tenant];
-    const uint64_t now = c->clock_fixed ? c->clock_ns : now_ns();
-    lg.emplace_back(now, n);
-    while (!lg.empty() && (lg.size() > 65536 || lg.front().first + 10000000000ull < now)) lg.pop_front();
-  }
+  note_dispatch(c, tenant, kind, n);
   c->stats.link_bytes[kind][s.logical] += n;
   c->stats.rounds++;
   s.inflight.push_back({ev_wait(c, x->done_ev), nullptr,
