@@ -210,6 +210,52 @@ def test_two_processes():
         p.wait(timeout=60)
 
 
+def test_export_free_trim_reexport():
+    """ADVICE r01 (stale descriptors): export A, import it, free A, let the
+    pool trim, put and export B, import B.  B's import reads B's bytes, A's
+    old descriptor is refused, and the mapping of A taken before the free
+    still reads A's bytes (its pages were A's own allocation, never
+    recycled by the pool)."""
+    import time
+    a, b = _ctx(), _ctx()
+    try:
+        n = 6 * (1 << 20) + 11
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        f, g = G.fn(4, 1, 0), G.fn(4, 2, 0)
+        G.check(G.test_fill(src.data_ptr(), n, 61, 0, 0))
+        torch.cuda.synchronize()
+        st, oa = a.put(f, src.data_ptr(), n, G.NOHINT, 0, 0)
+        st, da = a.export_ipc(f, oa)
+        assert st == G.OK
+        st, ra = b.import_ipc(g, da)
+        assert st == G.OK
+        st, pa, _ = b.get(g, ra, 0)
+        assert st == G.OK
+        assert a.release(f, oa, G.Ctx.desc_exporter_ptr(da), 0) == G.OK and a.free(f, oa) == G.OK
+        a.sync()
+        time.sleep(1.3)                                    # the daemon trims excess pool segments after 1 s
+        G.check(G.test_fill(src.data_ptr(), n, 62, 0, 0))
+        torch.cuda.synchronize()
+        st, ob = a.put(f, src.data_ptr(), n, G.NOHINT, 0, 0)
+        st, db = a.export_ipc(f, ob)
+        assert st == G.OK
+        assert b.import_ipc(g, da)[0] == G.ENOENT           # A's export ended with A
+        st, rb = b.import_ipc(g, db)
+        assert st == G.OK
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+        st, nn = b.get_into(g, rb, dst.data_ptr(), n, 0)
+        assert st == G.OK
+        assert G.test_verify(dst.data_ptr(), n, 62, 0, 0)[1] == 0      # B's bytes
+        assert np.array_equal(read_device(pa, n, 0), payload(61, n))   # A's pages, still A's bytes
+        assert b.release(g, ra, pa, 0) == G.OK
+        for roid in (ra, rb):
+            assert b.free(g, roid) == G.OK
+        assert a.release(f, ob, G.Ctx.desc_exporter_ptr(db), 0) == G.OK and a.free(f, ob) == G.OK
+    finally:
+        b.close()
+        a.close()
+
+
 def test_export_requires_no_zero_copy_leases():
     """The first export moves the object into its own allocation; an object a
     zero-copy lease still aliases cannot move (EBUSY), once the lease is
