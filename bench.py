@@ -1105,6 +1105,8 @@ def run_gpu(args, rank, world, local_rank):
     tl = st1.timed_launches - st0.timed_launches
     t_ns = st1.timed_ns - st0.timed_ns
     t_bytes = st1.timed_bytes - st0.timed_bytes
+    tk = st1.timed_kernel_launches - st0.timed_kernel_launches      # %globaltimer stamps
+    tk_ns = st1.timed_kernel_ns - st0.timed_kernel_ns
 
     # ---------------------------------------------------------- e2e (host-timed, + 8 B result read)
     e2e_steps = max(1, min(args.steps, args.e2e_steps))
@@ -1275,15 +1277,23 @@ def run_gpu(args, rank, world, local_rank):
                          "peak_live": live_peaks,
                          "in_step": {"avg_launch_us": k_us, "achieved": k_ach,
                                      "frac": (k_ach / kpeak) if k_ach else None, "launches": tl,
+                                     "kernel_us": tk_ns / tk / 1e3 if tk else None,
+                                     "kernel_achieved": (rw * t_bytes / max(tl, 1)) / (tk_ns / tk) if tk else None,
+                                     "kernel_frac": ((rw * t_bytes / max(tl, 1)) / (tk_ns / tk) / kpeak) if tk
+                                     else None,
+                                     "kernel_what": "the same launches timed by the kernel itself: latest CTA end "
+                                                    "minus earliest CTA start (%globaltimer), host submission "
+                                                    "and launch latency excluded",
                                      "what": "the same kernel inside the workflow's timed region, CUDA events "
                                              "recorded around every launch on its stream (GROUTER_PROFILE): "
                                              "each launch runs alone (requests are PCIe-paced), so the "
                                              "interval also holds the launch latency and the grid's ramp-up "
                                              "that back-to-back launches overlap, and with 4 client threads "
                                              "the host's gap between the start event and the launch call "
-                                             "(tools/instep.py: 19-22 us with one client); the kernel alone "
-                                             "takes ~13 us per launch in ncu's launch list of this command "
-                                             "(profiles/r02_ncu_launches_summary.csv)"}},
+                                             "(tools/instep.py: 19-22 us with one client); kernel_us is the "
+                                             "kernel's own span in the same launches -- shorter than back to "
+                                             "back because the tensor the copy engine has just written is "
+                                             "partly still in L2"}},
             "roofline_step": {"bound": "pcie", "achieved": value / world * N_BYTES / 1e9,
                               "peak": link_peak, "unit": "GB/s",
                               "frac": value / world * N_BYTES / 1e9 / link_peak,

@@ -177,6 +177,10 @@ typedef struct {
   uint64_t peer_launches;                /* copy-kernel launches on the peer (NVLink) branch:
                                             a destination or source outside the launching GPU,
                                             or GROUTER_FORCE_REMOTE                         */
+  uint64_t timed_kernel_launches;        /* GROUTER_PROFILE: launches with kernel stamps     */
+  uint64_t timed_kernel_ns;              /* their summed kernel time: latest CTA end minus
+                                            earliest CTA start, %globaltimer (the kernel's
+                                            own duration, host submission excluded)         */
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE

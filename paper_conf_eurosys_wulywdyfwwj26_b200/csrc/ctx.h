@@ -236,12 +236,18 @@ struct PhysDev {
   uint32_t n_scratch = 0, next_scratch = 0;
   std::vector<Fences> scratch_busy;
   std::vector<cudaEvent_t> timing_free;  // timing-enabled events (GROUTER_PROFILE)
+  // GROUTER_PROFILE kernel stamps (%globaltimer start/end per launch, device
+  // memory, a ring of slots; a slot is reused once its launch was harvested)
+  unsigned long long *stamps = nullptr;
+  std::vector<char> stamp_busy;
+  uint32_t next_stamp = 0;
 };
 
 struct ProfRec {
   int phys;
   cudaEvent_t start, stop;
   uint64_t bytes;
+  int stamp = -1;  // slot of PhysDev::stamps, -1 if none was free
 };
 
 }  // namespace gr

@@ -445,6 +445,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       for (auto &pb : pubs)
         if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path]) p->pub[k].value = pb.x->value_after(pb.path);
     ProfRec pr{s.phys, nullptr, nullptr, bytes};
+    p->stamp = nullptr;
     if (prof) {
       for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
         if (!pd.timing_free.empty()) {
@@ -453,6 +454,22 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
         } else {
           GR_CUDA(cudaEventCreate(e));
         }
+      }
+      static const uint32_t kStampSlots = 4096;
+      if (!pd.stamps) {  // [start, end] per slot: UINT64_MAX / 0 until a kernel stamps it
+        std::vector<unsigned long long> init(2 * kStampSlots);
+        for (uint32_t k = 0; k < kStampSlots; ++k) init[2 * k] = ~0ull, init[2 * k + 1] = 0;
+        GR_CUDA(cudaMalloc(&pd.stamps, init.size() * sizeof(unsigned long long)));
+        GR_CUDA(cudaMemcpy(pd.stamps, init.data(), init.size() * sizeof(unsigned long long),
+                           cudaMemcpyHostToDevice));
+        pd.stamp_busy.assign(kStampSlots, 0);
+      }
+      const uint32_t k = pd.next_stamp;
+      if (!pd.stamp_busy[k]) {  // else: no stamp for this launch (slots not harvested yet)
+        pd.next_stamp = (k + 1) % kStampSlots;
+        pd.stamp_busy[k] = 1;
+        pr.stamp = (int)k;
+        p->stamp = pd.stamps + 2 * k;
       }
       GR_CUDA(cudaEventRecord(pr.start, st));
     }
@@ -491,6 +508,18 @@ void harvest_profile(grouter_ctx *c, bool wait) {
     c->stats.timed_launches++;
     c->stats.timed_ns += (uint64_t)((double)ms * 1e6);
     c->stats.timed_bytes += r.bytes;
+    if (r.stamp >= 0) {  // the kernel's own start/end (completed: the stop event fired)
+      PhysDev &pd = *c->phys.at(r.phys);
+      unsigned long long t[2], init[2] = {~0ull, 0ull};
+      DeviceGuard g(r.phys);
+      GR_CUDA(cudaMemcpy(t, pd.stamps + 2 * r.stamp, sizeof(t), cudaMemcpyDeviceToHost));
+      GR_CUDA(cudaMemcpy(pd.stamps + 2 * r.stamp, init, sizeof(init), cudaMemcpyHostToDevice));
+      pd.stamp_busy[r.stamp] = 0;
+      if (t[1] > t[0] && t[0] != ~0ull) {
+        c->stats.timed_kernel_launches++;
+        c->stats.timed_kernel_ns += t[1] - t[0];
+      }
+    }
     auto &fl = c->phys.at(r.phys)->timing_free;
     fl.push_back(r.start);
     fl.push_back(r.stop);
@@ -861,6 +890,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   p->scratch = nullptr;
   p->counts = nullptr;
   p->count_base = 0;
+  p->stamp = nullptr;
   p->chunk[0] = {src, dst, n};
   bool host_pub = false;
   PhysDev &pd = *c->phys.at(s.phys);
@@ -1311,6 +1341,7 @@ void engine_shutdown(grouter_ctx *c) {
     DeviceGuard g(kv.first);
     if (kv.second->scratch) cudaFree(kv.second->scratch);
     for (cudaEvent_t e : kv.second->timing_free) cudaEventDestroy(e);
+    if (kv.second->stamps) cudaFree(kv.second->stamps);
     kv.second->scratch_busy.clear();
   }
   ipc_release_all(c);  // dedicated (exported) allocations; their fences hold pooled events

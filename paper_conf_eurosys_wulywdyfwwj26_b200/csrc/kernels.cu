@@ -67,6 +67,25 @@ __device__ __forceinline__ void st_release_sys(uint64_t addr, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(addr), "r"(v) : "memory");
 }
 
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// GROUTER_PROFILE stamps: every CTA after its PDL wait, and once all its
+// threads are done (p.stamp is grid-uniform, so the barrier is too)
+template <class KP>
+__device__ __forceinline__ void stamp_begin(const KP &p) {
+  if (p.stamp && threadIdx.x == 0) atomicMin(&p.stamp[0], gtimer());
+}
+template <class KP>
+__device__ __forceinline__ void stamp_end(const KP &p) {
+  if (p.stamp) {
+    __syncthreads();
+    if (threadIdx.x == 0) atomicMax(&p.stamp[1], gtimer());
+  }
+}
+
 template <bool COUNT, class KP>
 __device__ __forceinline__ void count_bytes(const KP &p, uint64_t dst_addr, uint32_t nbytes) {
   if (COUNT) atomicAdd(&p.counts[(dst_addr - p.count_base) >> 4], nbytes);
@@ -244,6 +263,7 @@ __device__ __forceinline__ void finish_round(const KP &p) {
 template <bool COUNT, int U, int MINB, class KP>
 __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_constant__ KP p) {
   pdl_wait();
+  stamp_begin(p);
   __shared__ uint32_t s_tile;
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   for (;;) {
@@ -260,6 +280,7 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
                      reinterpret_cast<const uint8_t *>(ch.src + off), len);
   }
   pdl_trigger();
+  stamp_end(p);
   finish_round(p);
 }
 
@@ -289,6 +310,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constan
       }
   }
   pdl_wait();
+  stamp_begin(p);
   if (threadIdx.x == 0) {
     uint64_t dst_of[STAGES];
     uint32_t bytes_of[STAGES];
@@ -324,6 +346,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constan
   }
   __syncthreads();
   pdl_trigger();
+  stamp_end(p);
   finish_round(p);
 }
 
@@ -385,6 +408,7 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
   const uint32_t W = gridDim.x * (kThreads / 32);
   prefetch_units<LG>(p, blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5), W, total, lane);
   pdl_wait();
+  stamp_begin(p);
   for (uint32_t id = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5); id < total; id += W) {
     const int c = find_chunk(p, id);
     const KChunk &ch = p.chunk[c];
@@ -439,6 +463,7 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
     }
   }
   pdl_trigger();
+  stamp_end(p);
   finish_round(p);
 }
 
@@ -690,6 +715,7 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
     q.scratch = p.scratch;
     q.counts = p.counts;
     q.count_base = p.count_base;
+    q.stamp = p.stamp;
     for (uint32_t i = 0; i < p.n_chunks; ++i) q.chunk[i] = p.chunk[i];
     for (uint32_t i = 0; i < p.n_pub; ++i) q.pub[i] = p.pub[i];
     if (g_launch_prof_on) lp1 = lp_now();

@@ -47,6 +47,10 @@ struct KParams {
   uint32_t *scratch = nullptr;   // [0] tile ticket, [1] finished CTAs; zero between launches
   uint32_t *counts = nullptr;    // test only: bytes written per 16 B granule
   uint64_t count_base = 0;
+  // GROUTER_PROFILE: [0] = earliest CTA start, [1] = latest CTA end, in
+  // %globaltimer ns (device memory; the kernel's own duration, independent of
+  // the host's submission timing); null otherwise
+  unsigned long long *stamp = nullptr;
   uint64_t tile_prefix[C + 1] = {};
   KChunk chunk[C];
   KPublish pub[P];

@@ -82,6 +82,7 @@ class grouter_stats_t(C.Structure):
         ("timed_bytes", C.c_uint64), ("restore_count", C.c_uint64), ("restore_bytes", C.c_uint64),
         ("pool_target", C.c_uint64 * MAX_GPUS), ("tracked_functions", C.c_uint64),
         ("tracked_tenants", C.c_uint64), ("peer_launches", C.c_uint64),
+        ("timed_kernel_launches", C.c_uint64), ("timed_kernel_ns", C.c_uint64),
     ]
 
 
