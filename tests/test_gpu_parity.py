@@ -874,6 +874,33 @@ def test_blocked_callers_fail_on_sticky_error():
             ctx.close()
 
 
+def test_profile_stamps():
+    """GROUTER_PROFILE: every timed launch also carries the kernel's own span
+    (%globaltimer, earliest CTA start to latest CTA end), positive and no
+    longer than the CUDA-event interval around the launch; bytes unchanged."""
+    calib = dict(C.b200_hgx(1), device_map=[0])
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED], flags=G.PROFILE))
+    try:
+        n = 38_535_168
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 71, 0, 0))
+        torch.cuda.synchronize()
+        st, oid = ctx.put(G.fn(1, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+        s = torch.cuda.Stream()
+        for _ in range(8):
+            G.check(ctx.get_into(G.fn(1, 2, 0), oid, dst.data_ptr(), n, s.cuda_stream)[0], "get_into")
+        s.synchronize()
+        G.check(ctx.sync(), "sync")
+        st_ = ctx.stats()
+        assert st_.timed_launches >= 8 and st_.timed_kernel_launches == st_.timed_launches
+        assert 0 < st_.timed_kernel_ns <= st_.timed_ns
+        assert G.test_verify(dst.data_ptr(), n, 71, 0, 0)[1] == 0
+    finally:
+        ctx.close()
+
+
 def test_probe_calibration():
     """grouter_probe (a5, L178/L131/L271): on one B200 the solo pinned H2D rate
     is a PCIe Gen5 x16 figure, per-copy and first-chunk costs are positive,
