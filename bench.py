@@ -887,7 +887,7 @@ def nccl_ring_baseline(world, rank, dev, n, per_step, steps):
 # ------------------------------------------------------------------ GPU arm
 
 # ------------------------------------------------------------------ cfg2 (BASELINE configs[1]) at one GPU
-def measure_cfg2(G, dev, seconds=2.0, outstanding=4):
+def measure_cfg2(G, dev, seconds=2.0, outstanding=4, oracle=True):
     """Traffic-monitoring workflow (BASELINE configs[1]),
     data plane only, closed loop with `outstanding` clients: a decode cFn puts a
     39,321,600 B frame (8x3x640x640 fp32) with hint GPU0 (PCIe H2D); the YOLO
@@ -963,11 +963,19 @@ def measure_cfg2(G, dev, seconds=2.0, outstanding=4):
     used = ctx.stats().used[0]
     ctx.close()
     n = sum(done)
-    return {"what": "cfg2 traffic monitoring (BASELINE configs[1]) at one GPU, data plane: frame put + zero-copy "
-                    "YOLO get + crop alloc/seal + two zero-copy recognition gets, 4 clients, wall clock",
-            "req_per_s": round(n / dt, 1), "frame_GBps": round(n * FRAME / dt / 1e9, 2),
-            "latency_us": {"p50": round(pct(lat, 50), 1), "p99": round(pct(lat, 99), 1)}, "requests": n,
-            "pool_used_after": used}
+    out = {"what": "cfg2 traffic monitoring (BASELINE configs[1]) at one GPU, data plane: frame put + zero-copy "
+                   "YOLO get + crop alloc/seal + two zero-copy recognition gets, 4 clients, wall clock",
+           "req_per_s": round(n / dt, 1), "frame_GBps": round(n * FRAME / dt / 1e9, 2),
+           "latency_us": {"p50": round(pct(lat, 50), 1), "p99": round(pct(lat, 99), 1)}, "requests": n,
+           "pool_used_after": used}
+    if oracle:   # the oracle on the same request structure (synth.traces.cfg2), one thread
+        from oracle import runner as orun
+        from synth import traces as TT
+        ops = TT.cfg2(1, requests=8)
+        t1 = time.perf_counter()
+        orun.run(ops, b200_hgx(1))
+        out["oracle_req_per_s"] = round(8 / (time.perf_counter() - t1), 1)
+    return out
 
 
 # ------------------------------------------------------------------ GPU arm
@@ -1236,7 +1244,7 @@ def run_gpu(args, rank, world, local_rank):
     cfg2 = None
     if rank == 0 and world == 1 and not args.no_sweep:
         try:
-            cfg2 = measure_cfg2(G, dev)
+            cfg2 = measure_cfg2(G, dev, oracle=not args.no_cpu_baseline)
         except Exception as e:   # reported, never fatal for the line
             cfg2 = {"error": f"{type(e).__name__}: {e}"[:300]}
 

@@ -74,13 +74,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 // GROUTER_PROFILE stamps: every CTA after its PDL wait, and once all its
 // threads are done (p.stamp is grid-uniform, so the barrier is too)
-template <class KP>
+// (separate kernel instantiations: launches without stamps carry no trace of them)
+template <bool STAMP, class KP>
 __device__ __forceinline__ void stamp_begin(const KP &p) {
-  if (p.stamp && threadIdx.x == 0) atomicMin(&p.stamp[0], gtimer());
+  if (STAMP && threadIdx.x == 0) atomicMin(&p.stamp[0], gtimer());
 }
-template <class KP>
+template <bool STAMP, class KP>
 __device__ __forceinline__ void stamp_end(const KP &p) {
-  if (p.stamp) {
+  if (STAMP) {
     __syncthreads();
     if (threadIdx.x == 0) atomicMax(&p.stamp[1], gtimer());
   }
@@ -260,10 +261,10 @@ __device__ __forceinline__ void finish_round(const KP &p) {
   }
 }
 
-template <bool COUNT, int U, int MINB, class KP>
+template <bool COUNT, int U, int MINB, bool STAMP, class KP>
 __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_constant__ KP p) {
   pdl_wait();
-  stamp_begin(p);
+  stamp_begin<STAMP>(p);
   __shared__ uint32_t s_tile;
   const uint32_t total = (uint32_t)p.tile_prefix[p.n_chunks];
   for (;;) {
@@ -280,7 +281,7 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
                      reinterpret_cast<const uint8_t *>(ch.src + off), len);
   }
   pdl_trigger();
-  stamp_end(p);
+  stamp_end<STAMP>(p);
   finish_round(p);
 }
 
@@ -293,7 +294,7 @@ __global__ void __launch_bounds__(kThreads, MINB) gr_copy_ldst(const __grid_cons
 // STAGES units of SOURCE into L2 (local sources only, like wv), so the DRAM
 // read ramp of launch i+1 overlaps the tail of launch i.  16 B-aligned
 // rounds only (bulk copies need 16 B addresses and sizes).
-template <int STAGES, class KP>
+template <int STAGES, bool STAMP, class KP>
 __global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constant__ KP p) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bars[STAGES];
@@ -310,7 +311,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constan
       }
   }
   pdl_wait();
-  stamp_begin(p);
+  stamp_begin<STAMP>(p);
   if (threadIdx.x == 0) {
     uint64_t dst_of[STAGES];
     uint32_t bytes_of[STAGES];
@@ -346,7 +347,7 @@ __global__ void __launch_bounds__(kTmaThreads) gr_copy_tmas(const __grid_constan
   }
   __syncthreads();
   pdl_trigger();
-  stamp_end(p);
+  stamp_end<STAMP>(p);
   finish_round(p);
 }
 
@@ -399,7 +400,7 @@ __device__ __forceinline__ void st256(V8 *p, const V8 &v) {
 // rounds (<= 4 MiB) use 1 KiB units (LG = 10, one 32 B load per lane): the
 // copy spreads over 8x more warps and SMs, so a latency-bound small copy
 // waits for one DRAM round trip per lane instead of eight in a row.
-template <bool COUNT, int LG, class KP>
+template <bool COUNT, int LG, bool STAMP, class KP>
 __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ KP p) {
   constexpr uint32_t kUnit = 1u << LG;
   constexpr int kPer = (int)(kUnit / (32 * 32));  // 32 B loads per lane per unit
@@ -408,7 +409,7 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
   const uint32_t W = gridDim.x * (kThreads / 32);
   prefetch_units<LG>(p, blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5), W, total, lane);
   pdl_wait();
-  stamp_begin(p);
+  stamp_begin<STAMP>(p);
   for (uint32_t id = blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5); id < total; id += W) {
     const int c = find_chunk(p, id);
     const KChunk &ch = p.chunk[c];
@@ -463,7 +464,7 @@ __global__ void __launch_bounds__(kThreads) gr_copy_wv(const __grid_constant__ K
     }
   }
   pdl_trigger();
-  stamp_end(p);
+  stamp_end<STAMP>(p);
   finish_round(p);
 }
 
@@ -554,7 +555,8 @@ static void launch_tmas(KP &p, int sm_count, cudaStream_t s) {
   static bool attr_set = false;
   const int smem = STAGES * kTmaStage;
   if (!attr_set) {
-    cudaFuncSetAttribute(gr_copy_tmas<STAGES, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gr_copy_tmas<STAGES, false, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gr_copy_tmas<STAGES, true, KP>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr_set = true;
   }
   p.tile_log2 = 14;  // units of kTmaStage bytes
@@ -567,7 +569,8 @@ static void launch_tmas(KP &p, int sm_count, cudaStream_t s) {
   uint64_t grid = (uint64_t)sm_count;
   if (grid > t) grid = t;
   if (grid == 0) grid = 1;
-  launch_pdl(gr_copy_tmas<STAGES, KP>, grid, kTmaThreads, smem, s, p);
+  if (p.stamp) launch_pdl(gr_copy_tmas<STAGES, true, KP>, grid, kTmaThreads, smem, s, p);
+  else launch_pdl(gr_copy_tmas<STAGES, false, KP>, grid, kTmaThreads, smem, s, p);
 }
 
 // ldst8: 256-thread CTAs claim 32-256 KiB tiles from a ticket, 8 x 16 B in
@@ -576,7 +579,7 @@ template <class KP>
 static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ldst<false, 8, 1, KP>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_ldst<false, 8, 1, false, KP>, kThreads, 0);
     if (occ <= 0) occ = 1;
   }
   const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
@@ -584,15 +587,16 @@ static void launch_ldst(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   choose_tiles(p, cap, 15, 18);
   uint64_t tiles = p.tile_prefix[p.n_chunks];
   uint64_t grid = cap > tiles ? tiles : cap;
-  if (p.counts) launch_pdl(gr_copy_ldst<true, 8, 1, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_ldst<false, 8, 1, KP>, grid, kThreads, 0, s, p);
+  if (p.counts) launch_pdl(gr_copy_ldst<true, 8, 1, false, KP>, grid, kThreads, 0, s, p);
+  else if (p.stamp) launch_pdl(gr_copy_ldst<false, 8, 1, true, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_ldst<false, 8, 1, false, KP>, grid, kThreads, 0, s, p);
 }
 
 template <int LG, class KP>
 static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   static int occ = 0;
   if (!occ) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, LG, KP>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, gr_copy_wv<false, LG, false, KP>, kThreads, 0);
     if (occ <= 0) occ = 1;
   }
   const int per_sm = ctas_per_sm < occ ? ctas_per_sm : occ;
@@ -607,8 +611,9 @@ static void launch_wv(KP &p, int sm_count, int ctas_per_sm, cudaStream_t s) {
   const uint64_t cap = (uint64_t)sm_count * per_sm;
   if (grid > cap) grid = cap;
   if (grid == 0) grid = 1;
-  if (p.counts) launch_pdl(gr_copy_wv<true, LG, KP>, grid, kThreads, 0, s, p);
-  else launch_pdl(gr_copy_wv<false, LG, KP>, grid, kThreads, 0, s, p);
+  if (p.counts) launch_pdl(gr_copy_wv<true, LG, false, KP>, grid, kThreads, 0, s, p);
+  else if (p.stamp) launch_pdl(gr_copy_wv<false, LG, true, KP>, grid, kThreads, 0, s, p);
+  else launch_pdl(gr_copy_wv<false, LG, false, KP>, grid, kThreads, 0, s, p);
 }
 
 static bool getenv_wv_big() {  // GR_WV_BIG=1: 8 KiB units at every size (measurement only)
