@@ -52,3 +52,15 @@ def test_single_rank_is_identity():
     import bench
     assert bench.exchange("x", 1) == ["x"]
     assert bench.max_over_ranks(3.5, 1) == 3.5
+
+
+def test_bench_helpers():
+    """bench.py's nearest-rank percentile (R26) and host description."""
+    import bench
+    xs = list(range(1, 101))
+    assert bench.pct(xs, 50) == 50 and bench.pct(xs, 99) == 99 and bench.pct(xs, 100) == 100
+    assert bench.pct([7], 99) == 7 and bench.pct([], 50) is None
+    assert bench.pct([3, 1, 2], 50) == 2            # sorts its input
+    cores, model = bench.host_info()
+    assert cores >= 1 and (model is None or isinstance(model, str))
+    assert bench.peer_of(3, 4) == 0 and bench.peer_of(0, 2) == 1
