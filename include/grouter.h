@@ -147,10 +147,14 @@ typedef struct {
   uint32_t batch_chunks;       /* default 5 (L229)                            */
   uint64_t granule;            /* split granule g, default 4096               */
   uint64_t pool_floor_bytes;   /* trim floor, default 300 MiB (L256, R13)     */
-  uint32_t pool_cap_permille;  /* auto cap = permille of free, default 500 (L262) */
-  uint64_t pool_cap_bytes[GROUTER_MAX_GPUS]; /* explicit cap; 0 = auto         */
+  uint32_t pool_cap_permille;  /* auto cap = permille of available, default 500 (L262) */
+  uint64_t pool_cap_bytes[GROUTER_MAX_GPUS]; /* explicit cap; 0 = auto (O10) */
   uint64_t host_store_bytes;   /* pinned host store H, default 1 GiB          */
-  uint64_t round_bytes;        /* unused since rounds carry one batch (O8)     */
+  uint64_t auto_cap_period_us; /* auto-mode GPUs: the background thread re-reads
+                                  free memory and re-applies the cap this often
+                                  (grouter_refresh_cap); default 20000; 0 = only
+                                  on explicit grouter_refresh_cap calls; never
+                                  in GROUTER_REPLAY mode                      */
   uint32_t copy_ctas_per_sm;   /* SM copy kernel CTAs per SM cap, default 4   */
   uint32_t flags;              /* GROUTER_* flags                              */
 } grouter_config;
@@ -181,6 +185,13 @@ typedef struct {
   uint64_t timed_kernel_ns;              /* their summed kernel time: latest CTA end minus
                                             earliest CTA start, %globaltimer (the kernel's
                                             own duration, host submission excluded)         */
+  /* auto cap (O10, R54): the input of the last grouter_refresh_cap of each GPU
+   * (explicit or by the background thread): available = free + the pool's own
+   * mapped bytes; cap[] is then the O10 function of it */
+  uint64_t auto_avail[GROUTER_MAX_GPUS];
+  uint64_t auto_refreshes;               /* refreshes applied (all GPUs)                     */
+  uint32_t auto_mode;                    /* bit d set: GPU d's cap follows free memory       */
+  uint32_t pad_;
 } grouter_stats_t;
 
 /* One dispatched batch (L229: <= batch_chunks chunks of ONE tenant on ONE
@@ -328,8 +339,29 @@ grouter_status grouter_slo_weights(uint32_t n, const uint32_t *ids, const uint64
  * workflow check (L394 authenticates the data-path calls). */
 grouter_status grouter_set_next_use(grouter_ctx *ctx, grouter_oid oid, uint64_t queue_pos);
 /* Pool cap of a GPU (GROUTER_UNLIMITED = no cap); evicts at once until used <= cap
- * (L262).  ENOMEM if unevictable data keeps the pool above the cap. */
+ * (L262).  ENOMEM if unevictable data keeps the pool above the cap.  An
+ * explicit limit takes the GPU out of auto mode (grouter_refresh_cap puts it
+ * back). */
 grouter_status grouter_set_pool_limit(grouter_ctx *ctx, int32_t device, uint64_t bytes);
+/* Auto cap (O10; "GROUTER triggers data migration and
+ * restoration automatically based on available GPU memory, maintaining storage
+ * usage within a fixed threshold (50% of free memory in our experiments)";
+ * readings R12, R54).  Puts GPU `device` in auto mode and applies
+ *   cap = floor(avail * pool_cap_permille / 1000 / 2 MiB) * 2 MiB
+ * exactly as grouter_set_pool_limit(device, cap) would: victims migrate to the
+ * host in queue-aware order until used <= cap, and with GROUTER_RESTORE host
+ * objects come back while they fit.  avail_bytes = memory available to the
+ * store; GROUTER_AUTO_AVAIL = measure it now: cudaMemGetInfo's free bytes of
+ * the GPU's device plus the bytes its pool has mapped (the pool's own memory
+ * is the store's, so its growth does not shrink its cap; logical GPUs sharing
+ * one device each see that device's free bytes).  Any other value is taken as
+ * the measurement (a platform that accounts function memory itself, tests).
+ * The background thread repeats the measured form every auto_cap_period_us
+ * for every auto-mode GPU; its victims count in stats but are not listed by
+ * grouter_victims.  *cap_out (nullable) = the cap applied.  EINVAL: bad
+ * device; ENOMEM as grouter_set_pool_limit (the cap stays). */
+#define GROUTER_AUTO_AVAIL UINT64_MAX
+grouter_status grouter_refresh_cap(grouter_ctx *ctx, int32_t device, uint64_t avail_bytes, uint64_t *cap_out);
 /* Replay mode: dispatch every queued chunk (stride order); no-op otherwise. */
 grouter_status grouter_flush(grouter_ctx *ctx);
 /* Blocks until all library work issued so far has completed. */

@@ -21,5 +21,6 @@ Parity status per function:
                                     hand-computed golden log)
   model.Oracle                      pinned (identity, I1-I7 invariants, Fig. 11b worked
                                     example L258, hand-derived golden traces)
-  model cap auto-mode (O10)         parity unpinned (depends on live free memory)
+  model.auto_cap / refresh_cap (O10) pinned (closed forms by hand, hand-derived golden
+                                    case G; the measured availability is an input)
 """

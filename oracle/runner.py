@@ -108,6 +108,10 @@ def run(ops: list, calib: dict, host_store_bytes: int = 1 << 40, pool_cap=None,
             st, out = orc.set_next_use(oid, op["pos"])
         elif k == "pool_limit":
             st, out = orc.set_pool_limit(op["dev"], op["bytes"])
+        elif k == "refresh_cap":
+            st, out = orc.refresh_cap(op["dev"], op["avail"])
+            if "cap" in out:
+                rec["cap"] = out["cap"]
         elif k == "flush":
             st, out = orc.flush()
             rec["dispatched"] = out["dispatched"]

@@ -410,6 +410,43 @@ bool check_ready(grouter_ctx *c) {
 
 }  // namespace
 
+// O10 auto cap and the cap rule shared by set_pool_limit / refresh_cap (L262)
+bool gr::apply_cap(grouter_ctx *c, int d, uint64_t bytes) {
+  LogicalDev &D = c->dev[d];
+  D.cap = bytes;
+  if (bytes != GROUTER_UNLIMITED && D.used > bytes)
+    for (Obj *o : candidates(c, d)) {  // migrate until under the new cap (L262)
+      if (D.used <= D.cap) break;
+      if (c->host_used + charge(o->n) > c->host_cap) break;
+      spill(c, *o);
+    }
+  const bool ok = bytes == GROUTER_UNLIMITED || D.used <= D.cap;
+  if (ok) restore(c, d);
+  return ok;
+}
+
+uint64_t gr::auto_cap_bytes(uint32_t permille, uint64_t avail) {
+  return (uint64_t)((unsigned __int128)avail * permille / 1000) / kPage * kPage;
+}
+
+uint64_t gr::refresh_cap(grouter_ctx *c, int d, uint64_t avail, bool *ok) {
+  LogicalDev &D = c->dev[d];
+  if (avail == GROUTER_AUTO_AVAIL) {  // free + the store's own device memory
+    DeviceGuard g(D.phys);
+    size_t fr = 0, tot = 0;
+    GR_CUDA(cudaMemGetInfo(&fr, &tot));
+    avail = (uint64_t)fr + D.pool.mapped;
+    for (auto &kv : c->dedicated)
+      if (kv.second.logical == d) avail += kv.second.size;
+  }
+  const uint64_t cap = auto_cap_bytes(c->cfg.pool_cap_permille, avail);
+  D.auto_cap = true;
+  c->stats.auto_avail[d] = avail;
+  c->stats.auto_refreshes++;
+  *ok = apply_cap(c, d, cap);
+  return cap;
+}
+
 extern "C" {
 
 const char *grouter_strerror(grouter_status st) {
@@ -474,7 +511,7 @@ void grouter_config_default(grouter_config *cfg) {
   cfg->pool_floor_bytes = 300ull << 20;
   cfg->pool_cap_permille = 500;
   cfg->host_store_bytes = 1ull << 30;
-  cfg->round_bytes = 64ull << 20;
+  cfg->auto_cap_period_us = 20000;
   cfg->copy_ctas_per_sm = 4;
 }
 
@@ -492,7 +529,6 @@ grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
   }
   if (cfg.n_gpus == 0 || cfg.n_gpus > GROUTER_MAX_GPUS) return fail(GROUTER_EINVAL, "bad n_gpus");
   if (cfg.copy_ctas_per_sm == 0) cfg.copy_ctas_per_sm = 4;
-  if (cfg.round_bytes == 0) cfg.round_bytes = 64ull << 20;
   auto *c = new grouter_ctx();
   c->cfg = cfg;
   c->replay = (cfg.flags & GROUTER_REPLAY) != 0;
@@ -1112,17 +1148,23 @@ grouter_status grouter_set_pool_limit(grouter_ctx *c, int32_t d, uint64_t bytes)
   c->restored.clear();
   API_TRY
   if (!valid_gpu(c, d)) return fail(GROUTER_EINVAL, "set_pool_limit: bad device");
-  LogicalDev &D = c->dev[d];
-  D.cap = bytes;
-  if (bytes != GROUTER_UNLIMITED)
-    for (Obj *o : candidates(c, d)) {  // migrate until under the new cap (L262)
-      if (D.used <= D.cap) break;
-      if (c->host_used + charge(o->n) > c->host_cap) break;
-      spill(c, *o);
-    }
-  if (bytes == GROUTER_UNLIMITED || D.used <= D.cap) restore(c, d);
-  return (bytes == GROUTER_UNLIMITED || D.used <= D.cap) ? GROUTER_OK
-                                                         : fail(GROUTER_ENOMEM, "pool above cap");
+  c->dev[d].auto_cap = false;
+  return apply_cap(c, d, bytes) ? GROUTER_OK : fail(GROUTER_ENOMEM, "pool above cap");
+  API_CATCH(c)
+}
+
+grouter_status grouter_refresh_cap(grouter_ctx *c, int32_t d, uint64_t avail, uint64_t *cap_out) {
+  gr::NvtxRange nvtx_("grouter_refresh_cap");
+  if (!c || c->plan_only) return fail(GROUTER_EINVAL, "no data-path context");
+  Guard g(c);
+  c->victims.clear();
+  c->restored.clear();
+  API_TRY
+  if (!valid_gpu(c, d)) return fail(GROUTER_EINVAL, "refresh_cap: bad device");
+  bool ok = false;
+  const uint64_t cap = refresh_cap(c, d, avail, &ok);
+  if (cap_out) *cap_out = cap;
+  return ok ? GROUTER_OK : fail(GROUTER_ENOMEM, "pool above cap");
   API_CATCH(c)
 }
 
@@ -1237,6 +1279,7 @@ grouter_status grouter_stats(grouter_ctx *c, grouter_stats_t *out) {
     out->cap[i] = c->dev[i].cap;
     out->mapped[i] = c->dev[i].pool.mapped;
     out->pool_target[i] = pool_target(c, (int)i);
+    if (c->dev[i].auto_cap) out->auto_mode |= 1u << i;
   }
   out->host_used = c->host_used;
   out->host_cap = c->host_cap;

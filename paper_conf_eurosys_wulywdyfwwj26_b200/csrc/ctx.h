@@ -221,6 +221,7 @@ struct LogicalDev {
   int phys = -1;
   DevicePool pool;
   uint64_t used = 0, cap = GROUTER_UNLIMITED;
+  bool auto_cap = false;  // cap follows available memory (O10, grouter_refresh_cap)
   Server copy, h2d, d2h;
 };
 
@@ -363,6 +364,14 @@ void ipc_unmap(RemoteMap &m);
 void ipc_dedicate(grouter_ctx *c, Obj &o);                       // move into an own allocation
 uint64_t ipc_export_record(grouter_ctx *c, uint64_t va, uint64_t nonce[2]);
 bool ded_free(grouter_ctx *c, uint8_t *p, Fences &&f);          // false: not dedicated
+// cap_d := bytes; migrate victims until used <= cap, then restore what fits
+// (L262); false when unevictable data keeps the pool above the cap
+bool apply_cap(grouter_ctx *c, int d, uint64_t bytes);
+// O10 (R12, R54): cap = floor(avail * permille / 1000 / page) * page
+uint64_t auto_cap_bytes(uint32_t permille, uint64_t avail);
+// auto mode on d: measure (avail == GROUTER_AUTO_AVAIL) or take avail, apply
+// the O10 cap; *ok = apply_cap's result; returns the cap
+uint64_t refresh_cap(grouter_ctx *c, int d, uint64_t avail, bool *ok);
 void ded_sweep(grouter_ctx *c, std::unique_lock<std::mutex> *lk, bool wait);
 void ipc_release_all(grouter_ctx *c);
 // pool.cpp

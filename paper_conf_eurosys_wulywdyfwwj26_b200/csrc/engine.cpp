@@ -1099,6 +1099,7 @@ static constexpr uint64_t kTrimDelayNs = 1000000000ull;  // 1 s of sustained exc
 static void daemon_main(grouter_ctx *c) {
   std::unique_lock<std::mutex> lk(c->mu);
   auto last_trim = std::chrono::steady_clock::now();
+  auto last_cap = last_trim;
   while (!c->stop) {
     bool backlog = false, busy = false;
     try {
@@ -1113,6 +1114,20 @@ static void daemon_main(grouter_ctx *c) {
         }
       }
       auto now = std::chrono::steady_clock::now();
+      // auto cap (O10, L262): re-read available memory and migrate / restore
+      // to stay within permille of it
+      if (!c->replay && c->cfg.auto_cap_period_us &&
+          now - last_cap >= std::chrono::microseconds(c->cfg.auto_cap_period_us)) {
+        last_cap = now;
+        for (size_t i = 0; i < c->dev.size(); ++i)
+          if (c->dev[i].auto_cap) {
+            bool ok = false;
+            const size_t nv = c->victims.size(), nr = c->restored.size();
+            refresh_cap(c, (int)i, GROUTER_AUTO_AVAIL, &ok);
+            c->victims.resize(nv);  // grouter_victims lists the API calls' own victims
+            c->restored.resize(nr);
+          }
+      }
       if (now - last_trim > std::chrono::milliseconds(50)) {  // I/O thread: reclaim (L269)
         last_trim = now;
         static const bool diag = getenv("GR_DIAG") != nullptr;
@@ -1265,8 +1280,13 @@ void engine_init(grouter_ctx *c) {
     DeviceGuard g(d.phys);
     size_t fr = 0, tot = 0;
     GR_CUDA(cudaMemGetInfo(&fr, &tot));
-    if (c->cfg.pool_cap_bytes[i]) d.cap = c->cfg.pool_cap_bytes[i];
-    else d.cap = (uint64_t)((unsigned __int128)fr * c->cfg.pool_cap_permille / 1000) / kPage * kPage;
+    if (c->cfg.pool_cap_bytes[i]) {
+      d.cap = c->cfg.pool_cap_bytes[i];
+    } else {  // auto mode (O10): nothing mapped yet, so available = free
+      d.auto_cap = true;
+      d.cap = auto_cap_bytes(c->cfg.pool_cap_permille, fr);
+      c->stats.auto_avail[i] = fr;
+    }
     uint64_t prewarm = std::min<uint64_t>(c->cfg.pool_floor_bytes, d.cap == GROUTER_UNLIMITED ? c->cfg.pool_floor_bytes : d.cap);
     if (c->cfg.flags & GROUTER_NO_POOL) prewarm = 0;  // ablation: nothing pooled
     d.pool.init(i, d.phys, (uint64_t)tot * 2 / kPage * kPage, phys_list, prewarm / kPage * kPage);

@@ -24,6 +24,7 @@ HOST = -1
 NOHINT = -2
 REMOTE = -3
 UNLIMITED = (1 << 64) - 1
+AUTO_AVAIL = (1 << 64) - 1   # grouter_refresh_cap: measure free memory now
 
 REPLAY, NO_MULTIPATH, PLAN_ONLY, LOG, COPY_TMA, PROFILE, RESTORE, D2H_MULTIPATH = \
     0x1, 0x2, 0x4, 0x8, 0x10, 0x20, 0x40, 0x80
@@ -66,7 +67,7 @@ class grouter_config(C.Structure):
         ("pool_cap_permille", C.c_uint32),
         ("pool_cap_bytes", C.c_uint64 * MAX_GPUS),
         ("host_store_bytes", C.c_uint64),
-        ("round_bytes", C.c_uint64),
+        ("auto_cap_period_us", C.c_uint64),
         ("copy_ctas_per_sm", C.c_uint32),
         ("flags", C.c_uint32),
     ]
@@ -83,6 +84,8 @@ class grouter_stats_t(C.Structure):
         ("pool_target", C.c_uint64 * MAX_GPUS), ("tracked_functions", C.c_uint64),
         ("tracked_tenants", C.c_uint64), ("peer_launches", C.c_uint64),
         ("timed_kernel_launches", C.c_uint64), ("timed_kernel_ns", C.c_uint64),
+        ("auto_avail", C.c_uint64 * MAX_GPUS), ("auto_refreshes", C.c_uint64),
+        ("auto_mode", C.c_uint32), ("pad_", C.c_uint32),
     ]
 
 
@@ -133,6 +136,7 @@ SIGNATURES = {
     "grouter_set_tenant_weight": (_ST, [_CTX, _U32, _U32]),
     "grouter_set_next_use": (_ST, [_CTX, _U64, _U64]),
     "grouter_set_pool_limit": (_ST, [_CTX, _I32, _U64]),
+    "grouter_refresh_cap": (_ST, [_CTX, _I32, _U64, C.POINTER(C.c_uint64)]),
     "grouter_flush": (_ST, [_CTX]),
     "grouter_sync": (_ST, [_CTX]),
     "grouter_plan": (_ST, [_CTX, _I32, _I32, _U64, C.POINTER(grouter_chunk), _U64, C.POINTER(_U64)]),
@@ -397,6 +401,12 @@ class Ctx:
 
     def set_pool_limit(self, dev, nbytes):
         return self.lib.grouter_set_pool_limit(self.h, dev, nbytes)
+
+    def refresh_cap(self, dev, avail=AUTO_AVAIL):
+        """O10 auto cap: (status, cap applied)."""
+        cap = C.c_uint64(0)
+        st = self.lib.grouter_refresh_cap(self.h, dev, avail, C.byref(cap))
+        return st, cap.value
 
     def flush(self):
         return self.lib.grouter_flush(self.h)

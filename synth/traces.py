@@ -19,6 +19,7 @@ ops:
   weight    wf w
   next_use  ref pos
   pool_limit dev bytes
+  refresh_cap dev avail      (O10 auto cap with `avail` bytes available to the store)
   flush
 """
 from __future__ import annotations
@@ -96,6 +97,9 @@ class Builder:
 
     def pool_limit(self, dev, nbytes):
         return self._add({"op": "pool_limit", "dev": dev, "bytes": nbytes})
+
+    def refresh_cap(self, dev, avail):
+        return self._add({"op": "refresh_cap", "dev": dev, "avail": avail})
 
     def flush(self):
         return self._add({"op": "flush"})
@@ -342,8 +346,10 @@ def random_trace(rng: random.Random, n_gpus: int, n_ops: int = 200, max_n: int =
         elif r < 0.90 and live:
             i, _ = rng.choice(live)
             b.next_use(i, rng.randint(0, 20))
-        elif r < 0.93 and limits:
+        elif r < 0.915 and limits:
             b.pool_limit(rng.randrange(n_gpus), rng.randint(0, 16) * 2 * MiB)
+        elif r < 0.93 and limits:   # O10 auto cap at an arbitrary (unaligned) availability
+            b.refresh_cap(rng.randrange(n_gpus), rng.randint(0, 64 * MiB))
         elif r < 0.95 and opened:
             i, f = rng.choice(opened)
             b.get(f, i)  # unsealed -> ENOENT

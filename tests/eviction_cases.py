@@ -119,4 +119,25 @@ def case_f():
     return b.ops, {"host_store_bytes": 64 * MiB, "n_gpus": 2}
 
 
-CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d, "E": case_e, "F": case_f}
+def case_g():
+    """O10 auto cap (L262 "triggers data migration and restoration
+    automatically based on available GPU memory ... 50% of free memory";
+    R12, R54) with proactive restore (R42)."""
+    b = T.Builder(27)
+    f, g = T.fn(1, 1, 0), T.fn(1, 2, 0)
+    A = b.put(f, 3 * MiB)                                   # 0
+    B = b.put(f, MiB)                                       # 1
+    b.put(f, MiB)                                           # 2 C, no hint
+    b.next_use(A, 2)                                        # 3
+    b.next_use(B, 5)                                        # 4
+    b.refresh_cap(0, 9 * MiB + 123)                         # 5 cap 4 MiB
+    b.refresh_cap(0, 12 * MiB)                              # 6 cap 6 MiB
+    b.refresh_cap(0, 3 * MiB)                               # 7 cap 0
+    b.refresh_cap(5, MiB)                                   # 8 EINVAL (one GPU)
+    b.get_into(g, B)                                        # 9 from the host store
+    b.refresh_cap(0, 100 * MiB + 1)                         # 10 cap 50 MiB
+    b.flush()                                               # 11
+    return b.ops, {"host_store_bytes": 64 * MiB, "restore": True}
+
+
+CASES = {"A": case_a, "B": case_b, "C": case_c, "D": case_d, "E": case_e, "F": case_f, "G": case_g}

@@ -61,8 +61,10 @@ class LibRunner:
         self.n = n
         self.phys = calib.get("device_map", list(range(n)))
         caps = pool_cap if pool_cap is not None else [G.UNLIMITED] * n
+        # auto_cap_period_us=0: a trace's refresh_cap ops are the only cap
+        # refreshes (the background thread would re-measure free memory)
         kw = dict(host_store_bytes=host_store_bytes, pool_cap=caps, pool_floor_bytes=pool_floor,
-                  flags=(G.REPLAY if replay else 0) | flags)
+                  flags=(G.REPLAY if replay else 0) | flags, auto_cap_period_us=0)
         if chunk_bytes:
             kw["chunk_bytes"] = chunk_bytes
         self.ctx = G.Ctx(G.config_from_calib(calib, **kw))
@@ -224,6 +226,10 @@ class LibRunner:
                 st = ctx.set_next_use(oid, op["pos"])
             elif k == "pool_limit":
                 st = ctx.set_pool_limit(op["dev"], op["bytes"])
+            elif k == "refresh_cap":
+                st, cap = ctx.refresh_cap(op["dev"], op["avail"])
+                if st in (G.OK, G.ENOMEM):
+                    rec["cap"] = cap
             elif k == "flush":
                 st = ctx.flush()
                 self._flush_and_verify()
@@ -281,6 +287,7 @@ def compare(orc_out, lib_out, check_dispatch=True):
             assert l["pool_target"] == o["pool_target"], (ctx, o["pool_target"], l["pool_target"])
         assert l["used"] == o["used"], (ctx, o["used"], l["used"])
         assert l["host_used"] == o["host_used"], ctx
+        assert l.get("cap") == o.get("cap"), (ctx, o.get("cap"), l.get("cap"))
         if o["status"] == "OK" and o["op"] in ("get", "get_into"):
             assert l["n"] == o["n"], ctx
             if "bytes" in o and "bytes" in l:

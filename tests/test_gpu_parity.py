@@ -196,12 +196,13 @@ def test_golden_trace_on_virtual_pair():
 
 
 @pytest.mark.parametrize("replay", [True, False])
-@pytest.mark.parametrize("case", ["A", "B", "C", "D", "E", "F"])
+@pytest.mark.parametrize("case", ["A", "B", "C", "D", "E", "F", "G"])
 def test_eviction_branch_golden_cases(case, replay):
     """The hand-derived eviction-branch cases (tests/golden/eviction_branches.md:
     R15 mixed hints, R33/R16 all-or-nothing reserve, R34 limit below the
-    unevictable floor, R32 full host store): the library equals the oracle
-    op by op, and both equal the hand-derived values."""
+    unevictable floor, R32 full host store, boundary statuses, placement,
+    O10 auto cap with restore): the library equals the oracle op by op, and
+    both equal the hand-derived values."""
     import json
     import os
     from tests.eviction_cases import CASES
@@ -217,6 +218,10 @@ def test_eviction_branch_golden_cases(case, replay):
         e = g[case]["expect"].get(str(r["i"]), {})
         assert r["status"] == e.get("status", "OK"), (case, r["i"])
         assert r["victims"] == e.get("victims", []), (case, r["i"])
+        if "cap" in e:
+            assert r["cap"] == e["cap"] * MiB, (case, r["i"])
+        if "restored" in e:
+            assert r["restored"] == e["restored"], (case, r["i"])
 
 
 @pytest.mark.parametrize("k", [1, 2, 4])

@@ -39,6 +39,10 @@ def _check(case):
             assert r["host_used"] == e["host_used"] * MiB, (case, r["i"], r["host_used"])
         if "plan" in e:
             assert r["plan"] == e["plan"], (case, r["i"])
+        if "restored" in e:
+            assert r["restored"] == e["restored"], (case, r["i"], r["restored"])
+        if "cap" in e:
+            assert r["cap"] == e["cap"] * MiB, (case, r["i"], r["cap"])
     orc = out["oracle"]
     for oid, loc in GOLD[case]["final_where"].items():
         assert orc.where(int(oid)) == loc, (case, oid, orc.where(int(oid)))
@@ -55,3 +59,38 @@ def test_case_c_cap_stays_after_enomem():
     had no cap before op 4)."""
     out = _check("C")
     assert out["oracle"].cap == [2 * MiB]
+
+
+def test_auto_cap_closed_forms():
+    """O10 (L262 "50% of free memory", R12, R54) by hand: half of the
+    availability, rounded down to whole 2 MiB pages."""
+    from oracle.model import auto_cap
+    assert auto_cap(10 << 30) == 5 << 30
+    assert auto_cap(1000 * MiB + 3) == 500 * MiB          # 500 MiB + 1 B -> 250 pages
+    assert auto_cap(4 * MiB - 1) == 0                     # 2 MiB - 0.5 B: no whole page
+    assert auto_cap(4 * MiB) == 2 * MiB
+    assert auto_cap(0) == 0
+    assert auto_cap(183_359 * MiB) == 91_678 * MiB        # a whole B200 (nvidia-smi total)
+    assert auto_cap(7 * MiB, permille=1000) == 6 * MiB
+    assert auto_cap(100 * MiB, permille=20) == 2 * MiB
+
+
+def test_refresh_cap_is_set_pool_limit_of_auto_cap():
+    """refresh_cap(d, avail) == set_pool_limit(d, auto_cap(avail)) op by op on
+    random traces (victims, restores, pools); the only extra is the cap."""
+    import random
+    from oracle.model import auto_cap
+    from synth import traces as T
+    n_refresh = 0
+    for seed in range(6):
+        ops = T.random_trace(random.Random(seed + 300), n_gpus=2, n_ops=160)
+        n_refresh += sum(op["op"] == "refresh_cap" for op in ops)
+        alt = [dict(op, op="pool_limit", bytes=auto_cap(op["avail"])) if op["op"] == "refresh_cap" else op
+               for op in ops]
+        cal = C.b200_hgx(2, shared_pairs=False)
+        a = runner.run(ops, cal, host_store_bytes=64 * MiB, restore=bool(seed % 2))
+        b = runner.run(alt, cal, host_store_bytes=64 * MiB, restore=bool(seed % 2))
+        for ra, rb in zip(a["records"], b["records"]):
+            for key in ("status", "victims", "restored", "used", "host_used", "oid", "where"):
+                assert ra.get(key) == rb.get(key), (seed, ra["i"], key)
+    assert n_refresh >= 6

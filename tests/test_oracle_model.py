@@ -289,14 +289,20 @@ def test_restore_preserves_bytes_and_caps(seed):
     r = runner.run(ops, c, host_store_bytes=1 << 30, pool_cap=caps, restore=True)
     moved = 0
     caps = list(caps)
+    prev = [0] * n
     for op, x, y in zip(ops, a, r["records"]):
-        if op["op"] == "pool_limit":
+        if op["op"] == "pool_limit" and 0 <= op["dev"] < n:
             caps[op["dev"]] = op["bytes"]
+        if op["op"] == "refresh_cap" and 0 <= op["dev"] < n:
+            caps[op["dev"]] = y["cap"]
         moved += len(y["restored"])
         if x["op"] in ("get", "get_into") and x["status"] == y["status"] == "OK":
             assert x.get("digest") == y.get("digest"), x["i"]
         if y["restored"] and y["op"] in ("release", "free", "get", "get_into"):
-            assert all(u <= cp for u, cp in zip(y["used"], caps))
+            # a GPU that grew (restore target) is within its cap (another may
+            # sit above an unreachable cap with unevictable data, R34)
+            assert all(u <= cp for u, cp, p in zip(y["used"], caps, prev) if u > p)
+        prev = y["used"]
     assert moved > 0 or seed % 3 == 0     # most traces exercise restore
 
 

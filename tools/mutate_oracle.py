@@ -43,6 +43,12 @@ MUTATIONS = [
     ("R35 release of a pin skips the workflow check", '            if o.wf != fn["wf"]:', "            if False:"),
     ("R23 gFn put follows its hint", "            home = dev", "            home = hint if hint >= 0 else dev"),
     ("R23 cFn hint ignored", "        elif hint >= 0:", "        elif False:"),
+    ("O10 threshold rounded up", "    return avail * permille // 1000 // PAGE * PAGE",
+     "    return -(-(avail * permille // 1000) // PAGE) * PAGE"),
+    ("O10 whole availability, not half", "    return avail * permille // 1000 // PAGE * PAGE",
+     "    return avail // PAGE * PAGE"),
+    ("O10 no rounding to pages", "    return avail * permille // 1000 // PAGE * PAGE",
+     "    return avail * permille // 1000"),
     ("R38 alloc follows the hint", "        home = dev\n        if home != HOST:",
      "        home = hint if hint >= 0 else dev\n        if home != HOST:"),
 ]
