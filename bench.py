@@ -1283,6 +1283,10 @@ def run_gpu(args, rank, world, local_rank):
                          "traffic_note": "ncu --set full, per launch (profiles/); steady traffic without "
                                          "cache flushes in traffic_steady", "traffic_steady": traffic_steady,
                          "peak_live": live_peaks,
+                         "frac_note": "peak = a measured torch copy_ (read + write bytes), not a hardware limit: "
+                                      "the kernel's steady DRAM traffic equals its algorithmic bytes "
+                                      "(traffic_steady: ncu, back to back), so a frac a little above 1 is a "
+                                      "faster copy than torch's, not skipped bytes",
                          "in_step": {"avg_launch_us": k_us, "achieved": k_ach,
                                      "frac": (k_ach / kpeak) if k_ach else None, "launches": tl,
                                      "kernel_us": tk_ns / tk / 1e3 if tk else None,

@@ -416,7 +416,8 @@ grouter_status grouter_victims(grouter_ctx *ctx, grouter_oid *out, uint64_t cap,
 /* Takes (and clears) the objects proactively restored to a GPU pool since the
  * last call, in order (GROUTER_RESTORE, R42).
  * Like grouter_victims the list is also reset at the start of every data-path
- * call, so it reports the restores of the latest call. */
+ * call, so it reports the restores of the latest call (the background auto-cap
+ * refresh's migrations and restores are counted in grouter_stats only). */
 grouter_status grouter_restored(grouter_ctx *ctx, grouter_oid *out, uint64_t cap, uint64_t *n_out);
 /* Takes (and clears) up to cap dispatch records, oldest first. */
 grouter_status grouter_dispatch_log(grouter_ctx *ctx, grouter_dispatch *out, uint64_t cap,

@@ -22,6 +22,7 @@
 // pages stay alive exactly as long as an importer maps them (VMM reference
 // counting) -- no page an importer still maps is ever reused for other data.
 #include <sys/socket.h>
+#include <sys/time.h>
 #include <sys/un.h>
 #include <unistd.h>
 
@@ -55,6 +56,15 @@ struct Rsp {
   uint32_t ok, pad;
   uint64_t size;
 };
+
+// A peer that connects and then stalls must not hold the serving thread (or
+// grouter_finalize, which joins it) -- nor an importer wait forever on a
+// stalled exporter: every accepted / connecting socket gets I/O timeouts.
+static void set_timeouts(int fd, int ms) {
+  timeval tv{ms / 1000, (ms % 1000) * 1000};
+  (void)::setsockopt(fd, SOL_SOCKET, SO_RCVTIMEO, &tv, sizeof(tv));
+  (void)::setsockopt(fd, SOL_SOCKET, SO_SNDTIMEO, &tv, sizeof(tv));
+}
 
 static bool read_full(int fd, void *p, size_t n) {
   uint8_t *b = (uint8_t *)p;
@@ -193,6 +203,7 @@ static void serve(grouter_ctx *c) {
       if (errno == EINTR) continue;
       return;  // listening socket closed: shutting down
     }
+    set_timeouts(cfd, 1000);
     Req rq;
     Rsp rsp{0, 0, 0};
     int fd = -1;
@@ -282,6 +293,7 @@ std::shared_ptr<RemoteMap> ipc_map(grouter_ctx *c, const grouter_ipc_desc &d, in
   sockaddr_un a;
   socklen_t len;
   sock_name(a, len, d.pid, d.ctx_id);
+  set_timeouts(s, 10000);
   if (::connect(s, (sockaddr *)&a, len) != 0) {
     ::close(s);
     throw Error(GROUTER_EINVAL, "ipc: exporter not reachable (process gone or other namespace)");

@@ -286,3 +286,51 @@ def test_export_requires_no_zero_copy_leases():
         assert a.stats().used[0] == 0
     finally:
         a.close()
+
+
+def test_stalled_peer_does_not_block_imports_or_close():
+    """A same-uid peer that connects to the exporter's socket and never sends
+    its request holds the serving thread for at most its 1 s I/O timeout:
+    a real import behind it still succeeds, and close() does not hang."""
+    import socket
+    import time
+    a, b = _ctx(), _ctx()
+    stalled = []
+    try:
+        n = 1 << 20
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 77, 0, 0))
+        torch.cuda.synchronize()
+        producer, consumer = G.fn(8, 1, 0), G.fn(8, 2, 0)
+        st, oid = a.put(producer, src.data_ptr(), n, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        st, desc = a.export_ipc(producer, oid)
+        G.check(st, "export")
+        d = G.grouter_ipc_desc.from_buffer_copy(desc)
+        for _ in range(3):   # connect, send nothing
+            s = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+            s.connect(b"\0" + f"grouter.{d.pid}.{d.ctx_id}".encode())
+            stalled.append(s)
+        t0 = time.time()
+        st, rid = b.import_ipc(consumer, desc)
+        assert st == G.OK, G.last_error()
+        assert time.time() - t0 < 8.0
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(b.get_into(consumer, rid, dst.data_ptr(), n, 0)[0], "get_into")
+        torch.cuda.synchronize()
+        st2, bad, _ = G.test_verify(dst.data_ptr(), n, 77, 0, 0)
+        assert st2 == G.OK and bad == 0
+        assert b.free(consumer, rid) == G.OK
+        assert a.release(producer, oid, G.Ctx.desc_exporter_ptr(desc), 0) == G.OK
+        assert a.free(producer, oid) == G.OK
+    finally:
+        if stalled:   # one more stalled peer at close
+            s = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+            s.connect(stalled[0].getpeername())
+            stalled.append(s)
+        t0 = time.time()
+        b.close()
+        a.close()
+        assert time.time() - t0 < 8.0
+        for s in stalled:
+            s.close()
