@@ -536,9 +536,13 @@ def measure_sweep(G, dev, hbm_peak, h2d_peak, sizes=SWEEP_SIZES, oracle=True):
             def put_timed(reps):
                 xs = []
                 for _ in range(reps):
+                    m0 = ctx.stats().mapped[0] if SWEEP_DEBUG else 0
                     t = time.perf_counter()
                     st, o2 = ctx.put(cfn, hp, n, 0, 0)
                     xs.append((time.perf_counter() - t) * 1e6)
+                    if SWEEP_DEBUG:
+                        print(f"[sweep] put {n} {xs[-1]:.0f} us mapped {m0 >> 20} -> "
+                              f"{ctx.stats().mapped[0] >> 20} MiB", file=sys.stderr, flush=True)
                     if st:
                         G.check(st, "put")
                     ctx.free(cfn, o2)
@@ -979,6 +983,9 @@ def measure_cfg2(G, dev, seconds=2.0, outstanding=4, oracle=True):
 
 
 # ------------------------------------------------------------------ GPU arm
+SWEEP_DEBUG = os.environ.get("GR_SWEEP_DEBUG") == "1"
+
+
 def h2d_link_peak(G, dev, nbytes=256 << 20, reps=4):
     """Pinned single-link H2D GB/s on this box (bare cudaMemcpyAsync back to
     back, CUDA events): the PCIe roofline of the workflow."""

@@ -59,7 +59,17 @@ struct DevicePool {
   PageHeap heap;
   std::vector<int> access;  // physical devices that may access the pages
   void init(int logical, int phys, uint64_t va, const std::vector<int> &access, uint64_t prewarm);
-  void grow(uint64_t need);
+  void grow(uint64_t need);  // on demand, lock held
+  // pre-warm in three steps so the driver calls (cuMemCreate / cuMemSetAccess
+  // took up to ~60 ms while copies streamed, tools/vmmlat.cu) run without the
+  // context lock and off the dispatch thread: reserve() takes a VA range
+  // (lock held), map_seg() creates and maps it (lock NOT held), publish()
+  // hands it to the heap (lock held); unreserve() after a failed map_seg
+  bool reserve(uint64_t size, uint64_t &off);
+  static Seg map_seg(CUdeviceptr base, uint64_t off, uint64_t size, int phys, const std::vector<int> &access,
+                     bool fallback_ok, uint64_t need);
+  void publish(const Seg &s);
+  void unreserve(uint64_t off, uint64_t size);
   // trim in two steps so the (slow, up to ~0.8 s measured) cuMemUnmap runs
   // without the context lock: detach() takes trailing free segments out of
   // the heap (lock held), unmap() releases them (lock NOT held), settle()
@@ -303,6 +313,8 @@ struct grouter_ctx {
   grouter_stats_t stats{};
   // background I/O + dispatch thread (L269, L271)
   std::thread daemon;
+  std::thread pool_thread;               // pool pre-warm / trim, auto cap, housekeeping
+  std::condition_variable pool_cv;
   std::condition_variable cv;
   std::condition_variable submit_cv;                   // a transfer became fully submitted
   bool stop = false;

@@ -1096,10 +1096,11 @@ void restore_copy(grouter_ctx *c, Obj &o, int d, uint8_t *dev_dst) {
 // ------------------------------------------------------------------ lifecycle
 static constexpr uint64_t kTrimDelayNs = 1000000000ull;  // 1 s of sustained excess before a trim
 
+// Dispatch thread (L269-L271 I/O daemon): pumps the servers' queues and
+// retires completed rounds.  Nothing here may block in a slow driver call:
+// while a blocking host put waits, this thread alone issues its next batches.
 static void daemon_main(grouter_ctx *c) {
   std::unique_lock<std::mutex> lk(c->mu);
-  auto last_trim = std::chrono::steady_clock::now();
-  auto last_cap = last_trim;
   while (!c->stop) {
     bool backlog = false, busy = false;
     try {
@@ -1113,6 +1114,89 @@ static void daemon_main(grouter_ctx *c) {
           retire(d.d2h);
         }
       }
+    } catch (const Error &e) {
+      set_error(e.what());
+      c->sticky_error = true;
+      c->submit_cv.notify_all();  // callers blocked in order_after fail with ECUDA
+    }
+    if (backlog && !c->replay) {
+      lk.unlock();
+      std::this_thread::sleep_for(std::chrono::microseconds(20));
+      lk.lock();
+    } else {
+      c->cv.wait_for(lk, busy ? std::chrono::milliseconds(1) : std::chrono::milliseconds(20));
+    }
+  }
+}
+
+// One pool tick of logical GPU i (L250-L256 histogram-driven size, R44; L269
+// reclaim): pre-warm one segment toward the target, trim back to
+// max(used, target) once the excess has lasted kTrimDelay and the GPU's
+// servers are idle.  The slow driver calls (create / map / set access;
+// unmap) run WITHOUT the context lock.
+static void pool_tick(grouter_ctx *c, size_t i, std::unique_lock<std::mutex> &lk) {
+  static const bool diag = getenv("GR_DIAG") != nullptr;
+  LogicalDev &d = c->dev[i];
+  DeviceGuard g(d.phys);
+  d.pool.heap.reclaim();
+  const uint64_t tgt = pool_target(c, (int)i);
+  const uint64_t t0 = diag ? now_ns() : 0, m0 = d.pool.mapped;
+  if (d.pool.mapped < tgt && !(c->cfg.flags & GROUTER_NO_POOL)) {
+    const uint64_t need = charge(std::min<uint64_t>(tgt - d.pool.mapped, 64ull << 20));
+    const uint64_t seg = std::max<uint64_t>(need, 64ull << 20);
+    uint64_t off = 0;
+    if (d.pool.reserve(seg, off)) {
+      const CUdeviceptr base = d.pool.base;
+      const int phys = d.pool.phys;
+      const std::vector<int> access = d.pool.access;
+      lk.unlock();
+      bool ok = true;
+      DevicePool::Seg sg{};
+      try {
+        sg = DevicePool::map_seg(base, off, seg, phys, access, false, need);
+      } catch (const Error &) {
+        ok = false;  // HBM short: pre-warming is best effort
+      }
+      lk.lock();
+      if (ok) d.pool.publish(sg);
+      else d.pool.unreserve(off, seg);
+    }
+  }
+  const uint64_t t1 = diag ? now_ns() : 0, m1 = d.pool.mapped;
+  const uint64_t keep = std::max<uint64_t>(d.used, tgt) + (64ull << 20);
+  const uint64_t tnow = now_ns();
+  if (d.pool.mapped <= keep) d.pool.excess_since = 0;
+  else if (!d.pool.excess_since) d.pool.excess_since = tnow;
+  const bool idle = d.copy.inflight.empty() && d.h2d.inflight.empty() && d.d2h.inflight.empty() &&
+                    !has_work(d.copy) && !has_work(d.h2d) && !has_work(d.d2h);
+  if (d.pool.excess_since && tnow - d.pool.excess_since >= kTrimDelayNs && idle) {
+    std::vector<DevicePool::Seg> v = d.pool.detach(keep);
+    if (!v.empty()) {
+      const CUdeviceptr base = d.pool.base;
+      lk.unlock();
+      DevicePool::unmap(base, v);
+      lk.lock();
+      d.pool.settle(v);
+    }
+    d.pool.excess_since = 0;
+  }
+  if (diag && now_ns() - t0 > 5000000)
+    fprintf(stderr, "[grouter diag] pool tick dev %zu: grow %.1f ms (%llu -> %llu MiB), trim %.1f ms "
+                    "(-> %llu MiB), used %llu MiB, target %llu MiB\n",
+            i, (t1 - t0) / 1e6, (unsigned long long)(m0 >> 20), (unsigned long long)(m1 >> 20),
+            (now_ns() - t1) / 1e6, (unsigned long long)(d.pool.mapped >> 20),
+            (unsigned long long)(d.used >> 20), (unsigned long long)(tgt >> 20));
+}
+
+// Housekeeping thread: the auto cap (O10), pool pre-warm / trim, quarantine
+// reclaim, bounded bookkeeping -- off the dispatch thread, so a slow driver
+// call here never holds back a batch.
+static void pool_main(grouter_ctx *c) {
+  std::unique_lock<std::mutex> lk(c->mu);
+  auto last_trim = std::chrono::steady_clock::now();
+  auto last_cap = last_trim;
+  while (!c->stop) {
+    try {
       auto now = std::chrono::steady_clock::now();
       // auto cap (O10, L262): re-read available memory and migrate / restore
       // to stay within permille of it
@@ -1130,13 +1214,10 @@ static void daemon_main(grouter_ctx *c) {
       }
       if (now - last_trim > std::chrono::milliseconds(50)) {  // I/O thread: reclaim (L269)
         last_trim = now;
-        static const bool diag = getenv("GR_DIAG") != nullptr;
-        for (size_t i = 0; i < c->dev.size(); ++i) {
-          LogicalDev &d = c->dev[i];
-          DeviceGuard g(d.phys);
-          d.pool.heap.reclaim();
+        for (size_t i = 0; i < c->dev.size() && !c->stop; ++i) {
           if (i == 0 && !c->nopool_pending.empty()) nopool_sweep(c, false);
-          for (Server *sv : {&d.copy, &d.h2d, &d.d2h}) sv->sched.prune();  // idle tenants (no-op for dispatch)
+          for (Server *sv : {&c->dev[i].copy, &c->dev[i].h2d, &c->dev[i].d2h})
+            sv->sched.prune();  // idle tenants (no-op for dispatch)
           if (i == 0) {  // rate-monitor records older than its 10 s horizon; bounded per-tenant counters
             const uint64_t tn = c->clock_fixed ? c->clock_ns : now_ns();
             for (auto it = c->tenant_log.begin(); it != c->tenant_log.end();)
@@ -1158,45 +1239,7 @@ static void daemon_main(grouter_ctx *c) {
                 if (!c->tenant_log.count(it->first)) it = c->tenant_bytes.erase(it);
                 else ++it;
           }
-          // histogram-driven size (L250-L256, R44): pre-warm one segment per
-          // tick toward the target, trim back to max(used, target)
-          const uint64_t tgt = pool_target(c, (int)i);
-          const uint64_t t0 = diag ? now_ns() : 0, m0 = d.pool.mapped;
-          if (d.pool.mapped < tgt && !(c->cfg.flags & GROUTER_NO_POOL)) {
-            try {
-              d.pool.grow(std::min<uint64_t>(tgt - d.pool.mapped, 64ull << 20));
-            } catch (const Error &) {
-              // HBM short: pre-warming is best effort
-            }
-          }
-          const uint64_t t1 = diag ? now_ns() : 0, m1 = d.pool.mapped;
-          // trim only once the excess has lasted kTrimDelay and this GPU's
-          // servers are idle, and unmap WITHOUT the context lock: cuMemUnmap
-          // of a few hundred MiB took up to ~0.8 s under load (it drains the
-          // GPU), which stalled every API call behind the lock
-          const uint64_t keep = std::max<uint64_t>(d.used, tgt) + (64ull << 20);
-          const uint64_t tnow = now_ns();
-          if (d.pool.mapped <= keep) d.pool.excess_since = 0;
-          else if (!d.pool.excess_since) d.pool.excess_since = tnow;
-          const bool idle = d.copy.inflight.empty() && d.h2d.inflight.empty() && d.d2h.inflight.empty() &&
-                            !has_work(d.copy) && !has_work(d.h2d) && !has_work(d.d2h);
-          if (d.pool.excess_since && tnow - d.pool.excess_since >= kTrimDelayNs && idle) {
-            std::vector<DevicePool::Seg> v = d.pool.detach(keep);
-            if (!v.empty()) {
-              const CUdeviceptr base = d.pool.base;
-              lk.unlock();
-              DevicePool::unmap(base, v);
-              lk.lock();
-              d.pool.settle(v);
-            }
-            d.pool.excess_since = 0;
-          }
-          if (diag && now_ns() - t0 > 5000000)
-            fprintf(stderr, "[grouter diag] pool tick dev %zu: grow %.1f ms (%llu -> %llu MiB), trim %.1f ms "
-                            "(-> %llu MiB), used %llu MiB, target %llu MiB\n",
-                    i, (t1 - t0) / 1e6, (unsigned long long)(m0 >> 20), (unsigned long long)(m1 >> 20),
-                    (now_ns() - t1) / 1e6, (unsigned long long)(d.pool.mapped >> 20),
-                    (unsigned long long)(d.used >> 20), (unsigned long long)(tgt >> 20));
+          pool_tick(c, i, lk);
         }
         c->host.heap.reclaim();
         if (!c->ded_retire.empty()) ded_sweep(c, &lk, false);  // exported objects' own allocations
@@ -1206,13 +1249,7 @@ static void daemon_main(grouter_ctx *c) {
       c->sticky_error = true;
       c->submit_cv.notify_all();  // callers blocked in order_after fail with ECUDA
     }
-    if (backlog && !c->replay) {
-      lk.unlock();
-      std::this_thread::sleep_for(std::chrono::microseconds(20));
-      lk.lock();
-    } else {
-      c->cv.wait_for(lk, busy ? std::chrono::milliseconds(1) : std::chrono::milliseconds(20));
-    }
+    c->pool_cv.wait_for(lk, std::chrono::milliseconds(10));
   }
 }
 
@@ -1322,6 +1359,7 @@ void engine_init(grouter_ctx *c) {
     GR_CUDA(cudaDeviceSynchronize());
   }
   c->daemon = std::thread(daemon_main, c);
+  c->pool_thread = std::thread(pool_main, c);
 }
 
 void engine_shutdown(grouter_ctx *c) {
@@ -1330,8 +1368,10 @@ void engine_shutdown(grouter_ctx *c) {
     c->stop = true;
   }
   c->cv.notify_all();
+  c->pool_cv.notify_all();
   c->submit_cv.notify_all();
   if (c->daemon.joinable()) c->daemon.join();
+  if (c->pool_thread.joinable()) c->pool_thread.join();
   // drain the library's own streams (never the device: a caller stream may be
   // parked on a completion word that will not arrive after an error)
   auto t0 = std::chrono::steady_clock::now();

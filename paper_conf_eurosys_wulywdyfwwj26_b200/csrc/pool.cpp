@@ -257,24 +257,24 @@ void DevicePool::init(int lg, int ph, uint64_t va, const std::vector<int> &acc, 
   if (prewarm) grow(prewarm);
 }
 
-void DevicePool::grow(uint64_t need) {
-  need = charge(need);
-  uint64_t seg = std::max<uint64_t>(need, 64ull << 20);
-  if (va_top + seg > va_size) seg = need;
-  if (va_top + seg > va_size) throw Error(GROUTER_ENOMEM, "pool VA range exhausted");
+DevicePool::Seg DevicePool::map_seg(CUdeviceptr base, uint64_t off, uint64_t size, int phys,
+                                    const std::vector<int> &access, bool fallback_ok, uint64_t need) {
   CUmemAllocationProp prop = {};
   prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
   prop.location.id = phys;
   prop.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;  // IPC-exportable (L167)
   CUmemGenericAllocationHandle h;
-  CUresult r = drv().memCreate(&h, seg, &prop, 0);
-  if (r != CUDA_SUCCESS && seg > need) {
-    seg = need;
-    r = drv().memCreate(&h, seg, &prop, 0);
+  CUresult r = drv().memCreate(&h, size, &prop, 0);
+  if (r != CUDA_SUCCESS && fallback_ok && size > need) {
+    size = need;
+    r = drv().memCreate(&h, size, &prop, 0);
   }
   if (r != CUDA_SUCCESS) throw Error(GROUTER_ENOMEM, "cuMemCreate failed (HBM exhausted)");
-  GR_CU(drv().memMap(base + va_top, seg, 0, h, 0));
+  if (drv().memMap(base + off, size, 0, h, 0) != CUDA_SUCCESS) {
+    drv().memRelease(h);
+    throw Error(GROUTER_ECUDA, "cuMemMap failed");
+  }
   std::vector<CUmemAccessDesc> ad;
   for (int p : access) {
     CUmemAccessDesc a = {};
@@ -283,11 +283,44 @@ void DevicePool::grow(uint64_t need) {
     a.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
     ad.push_back(a);
   }
-  GR_CU(drv().memSetAccess(base + va_top, seg, ad.data(), ad.size()));
-  segs.push_back({va_top, seg, h});
-  heap.give(va_top, seg);
-  va_top += seg;
-  mapped += seg;
+  if (drv().memSetAccess(base + off, size, ad.data(), ad.size()) != CUDA_SUCCESS) {
+    drv().memUnmap(base + off, size);
+    drv().memRelease(h);
+    throw Error(GROUTER_ECUDA, "cuMemSetAccess failed");
+  }
+  return {off, size, h};
+}
+
+void DevicePool::publish(const Seg &s) {
+  // segments stay in VA order (an on-demand grow may have mapped above a
+  // pre-warm reservation meanwhile)
+  auto it = std::upper_bound(segs.begin(), segs.end(), s.off,
+                             [](uint64_t off, const Seg &x) { return off < x.off; });
+  segs.insert(it, s);
+  heap.give(s.off, s.size);
+  mapped += s.size;
+}
+
+void DevicePool::grow(uint64_t need) {
+  need = charge(need);
+  uint64_t seg = std::max<uint64_t>(need, 64ull << 20);
+  if (va_top + seg > va_size) seg = need;
+  if (va_top + seg > va_size) throw Error(GROUTER_ENOMEM, "pool VA range exhausted");
+  const uint64_t off = va_top;
+  Seg s = map_seg(base, off, seg, phys, access, true, need);
+  va_top = off + s.size;
+  publish(s);
+}
+
+bool DevicePool::reserve(uint64_t size, uint64_t &off) {
+  if (va_top + size > va_size) return false;
+  off = va_top;
+  va_top += size;
+  return true;
+}
+
+void DevicePool::unreserve(uint64_t off, uint64_t size) {
+  if (va_top == off + size) va_top = off;  // else a hole (never handed out)
 }
 
 // Detaches trailing segments that are entirely free while the mapping stays
