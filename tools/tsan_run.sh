@@ -23,8 +23,8 @@ TSAN_OPTIONS="report_signal_unsafe=0 halt_on_error=0 log_path=$D/stress" GR_STRE
   timeout 1200 python -m pytest tests/test_gpu_concurrency.py -m gpu -q -p no:cacheprovider > $D/stress_pytest.txt 2>&1
 echo stress_rc=$?
 TSAN_OPTIONS="report_signal_unsafe=0 halt_on_error=0 log_path=$D/soak" GR_SOAK_SEEDS=8 \
-  timeout 1200 python -m pytest tests/test_gpu_parity.py -m gpu -q -p no:cacheprovider \
-  -k "random_traces_realtime or two_batches or forced_remote" > $D/soak_pytest.txt 2>&1
+  timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_autocap.py -m gpu -q -p no:cacheprovider \
+  -k "random_traces_realtime or two_batches or forced_remote or background_refresh" > $D/soak_pytest.txt 2>&1
 echo soak_rc=$?
-tail -3 $D/stress_pytest.txt $D/soak_pytest.txt
+for f in $D/stress_pytest.txt $D/soak_pytest.txt; do tail -n 3 $f; done
 for f in $D/control* $D/stress* $D/soak*; do echo "$f: $(grep -c 'WARNING: ThreadSanitizer' $f 2>/dev/null)"; done
