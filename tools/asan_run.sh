@@ -24,8 +24,8 @@ print("control returned (ASan inactive?)")
 PY
 GR_STRESS_OPS=200 timeout 1200 python -m pytest tests/test_gpu_concurrency.py -m gpu -q -p no:cacheprovider > $D/stress_pytest.txt 2>&1
 echo stress_rc=$?
-GR_SOAK_SEEDS=6 timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_ipc.py -m gpu -q -p no:cacheprovider \
-  -k "random_traces_realtime or two_batches or forced_remote or ce_relay or sticky or two_contexts" > $D/soak_pytest.txt 2>&1
+GR_SOAK_SEEDS=6 timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_ipc.py tests/test_gpu_autocap.py -m gpu -q -p no:cacheprovider \
+  -k "random_traces_realtime or two_batches or forced_remote or ce_relay or sticky or two_contexts or stalled or background_refresh" > $D/soak_pytest.txt 2>&1
 echo soak_rc=$?
 tail -n 3 $D/stress_pytest.txt $D/soak_pytest.txt
 ls $D
