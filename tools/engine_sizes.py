@@ -79,13 +79,10 @@ if __name__ == "__main__":
     else:
         for e in sys.argv[1:] or ["default", "wv8", "tmas4"]:
             env = dict(os.environ)
-            e, *extra = e.split(":")        # ENGINE[@PF][:ENV=VAL ...]
+            name, *extra = e.split(":")     # ENGINE[:ENV=VAL ...]
             env.update(kv.split("=", 1) for kv in extra)
-            name, _, pf = e.partition("@")
             if name == "ce":
                 env["GR_SIZES_CE"] = "1"
             elif name != "default":
                 env["GR_COPY"] = name
-            if pf:
-                env["GR_PF"] = pf
             subprocess.run([sys.executable, __file__, "--child"], env=env, timeout=600)
