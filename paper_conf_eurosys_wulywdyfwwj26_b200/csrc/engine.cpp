@@ -395,6 +395,42 @@ static void after_submit(grouter_ctx *c, const std::vector<ChunkItem> &items) {
 // records an event instead (a stream write after a kernel costs ~3.5 us of
 // GPU time per launch and breaks programmatic dependent launch; an event
 // record costs neither).
+// GROUTER_PROFILE around one copy-kernel launch on stream st: timing events
+// (pooled) and a %globaltimer stamp slot the kernel writes its first CTA start
+// and last CTA end into (*stamp = null when every slot awaits harvesting).
+static void prof_begin(PhysDev &pd, cudaStream_t st, ProfRec &pr, unsigned long long *&stamp) {
+  for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
+    if (!pd.timing_free.empty()) {
+      *e = pd.timing_free.back();
+      pd.timing_free.pop_back();
+    } else {
+      GR_CUDA(cudaEventCreate(e));
+    }
+  }
+  static const uint32_t kStampSlots = 4096;
+  if (!pd.stamps) {  // [start, end] per slot: UINT64_MAX / 0 until a kernel stamps it
+    std::vector<unsigned long long> init(2 * kStampSlots);
+    for (uint32_t k = 0; k < kStampSlots; ++k) init[2 * k] = ~0ull, init[2 * k + 1] = 0;
+    GR_CUDA(cudaMalloc(&pd.stamps, init.size() * sizeof(unsigned long long)));
+    GR_CUDA(cudaMemcpy(pd.stamps, init.data(), init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice));
+    pd.stamp_busy.assign(kStampSlots, 0);
+  }
+  stamp = nullptr;
+  const uint32_t k = pd.next_stamp;
+  if (!pd.stamp_busy[k]) {  // else: no stamp for this launch (slots not harvested yet)
+    pd.next_stamp = (k + 1) % kStampSlots;
+    pd.stamp_busy[k] = 1;
+    pr.stamp = (int)k;
+    stamp = pd.stamps + 2 * k;
+  }
+  GR_CUDA(cudaEventRecord(pr.start, st));
+}
+
+static void prof_end(grouter_ctx *c, cudaStream_t st, ProfRec &pr) {
+  GR_CUDA(cudaEventRecord(pr.stop, st));
+  c->prof.push_back(pr);
+}
+
 static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *scratch,
                          const std::vector<ChunkItem> &items, const uint64_t *src_override,
                          bool *deferred_pub = nullptr) {
@@ -446,33 +482,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
         if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path]) p->pub[k].value = pb.x->value_after(pb.path);
     ProfRec pr{s.phys, nullptr, nullptr, bytes};
     p->stamp = nullptr;
-    if (prof) {
-      for (cudaEvent_t *e : {&pr.start, &pr.stop}) {
-        if (!pd.timing_free.empty()) {
-          *e = pd.timing_free.back();
-          pd.timing_free.pop_back();
-        } else {
-          GR_CUDA(cudaEventCreate(e));
-        }
-      }
-      static const uint32_t kStampSlots = 4096;
-      if (!pd.stamps) {  // [start, end] per slot: UINT64_MAX / 0 until a kernel stamps it
-        std::vector<unsigned long long> init(2 * kStampSlots);
-        for (uint32_t k = 0; k < kStampSlots; ++k) init[2 * k] = ~0ull, init[2 * k + 1] = 0;
-        GR_CUDA(cudaMalloc(&pd.stamps, init.size() * sizeof(unsigned long long)));
-        GR_CUDA(cudaMemcpy(pd.stamps, init.data(), init.size() * sizeof(unsigned long long),
-                           cudaMemcpyHostToDevice));
-        pd.stamp_busy.assign(kStampSlots, 0);
-      }
-      const uint32_t k = pd.next_stamp;
-      if (!pd.stamp_busy[k]) {  // else: no stamp for this launch (slots not harvested yet)
-        pd.next_stamp = (k + 1) % kStampSlots;
-        pd.stamp_busy[k] = 1;
-        pr.stamp = (int)k;
-        p->stamp = pd.stamps + 2 * k;
-      }
-      GR_CUDA(cudaEventRecord(pr.start, st));
-    }
+    if (prof) prof_begin(pd, st, pr, p->stamp);
     HostProf &hp = hprof();
     uint64_t tl = hp.on ? now_ns() : 0;
     if (hp.on) hp.t[6] += tl - tparams;
@@ -489,10 +499,7 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
     if (e != 0)
       throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
     if (host_pub) *deferred_pub = true;
-    if (prof) {
-      GR_CUDA(cudaEventRecord(pr.stop, st));
-      c->prof.push_back(pr);
-    }
+    if (prof) prof_end(c, st, pr);
     c->stats.kernel_launches++;
     if (!local) c->stats.peer_launches++;
   }
@@ -856,7 +863,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
                     int caller_phys) {
   static const bool off = getenv("GR_NO_FAST") != nullptr || getenv("GR_COPY") != nullptr;
-  const uint32_t never = GROUTER_LOG | GROUTER_PROFILE | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
+  const uint32_t never = GROUTER_LOG | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
   if (off || c->replay || !caller || (c->cfg.flags & never) || !n || ((src | dst) & 15)) return nullptr;
   Server &s = c->dev[server_logical].copy;
   if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
@@ -905,8 +912,12 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
     GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, n, cudaMemcpyDeviceToDevice, caller));
     host_pub = true;
   } else {
+    const bool prof = (c->cfg.flags & GROUTER_PROFILE) != 0;  // the same events and stamps as launch_round
+    ProfRec pr{s.phys, nullptr, nullptr, n};
+    if (prof) prof_begin(pd, caller, pr, p->stamp);
     int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm, false, caller, &host_pub);
     if (e != 0) throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
+    if (prof) prof_end(c, caller, pr);
   }
   if (!host_pub) throw Error(GROUTER_ECUDA, "internal: fast direct launch needs a static engine");
   x->done_ev = record(c, caller, s.phys);
@@ -936,12 +947,12 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
 // a single-route plan of at most two batches (so <= 2 batches in flight
 // holds): one cudaMemcpyAsync on the server's stream and an
 // event, with the same scheduler accounting (Stride::account_solo), tenant
-// bytes, rate monitor and stats as a queued dispatch.  Real-time mode only
-// (no LOG / PROFILE); null when the queued path must be used.
+// bytes, rate monitor and stats as a queued dispatch.  Real-time mode only,
+// no LOG (the dispatch log lists batches); null when the queued path must be used.
 XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<grouter_chunk> &plan, uint64_t src,
                 uint64_t dst, uint64_t n, const Fences &deps) {
   static const bool off = getenv("GR_NO_FAST") != nullptr;
-  if (off || c->replay || (c->cfg.flags & (GROUTER_LOG | GROUTER_PROFILE)) || plan.empty()) return nullptr;
+  if (off || c->replay || (c->cfg.flags & GROUTER_LOG) || plan.empty()) return nullptr;
   const int route = plan[0].route_gpu;
   for (auto &ch : plan)
     if (ch.route_gpu != route || ch.path != 0) return nullptr;  // striped: the queued path relays
