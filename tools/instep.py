@@ -40,7 +40,12 @@ def kstats(fn):
     torch.cuda.synchronize()
     s1 = ctx.stats()
     k = s1.timed_launches - s0.timed_launches
+    kk = s1.timed_kernel_launches - s0.timed_kernel_launches
+    KUS[0] = (s1.timed_kernel_ns - s0.timed_kernel_ns) / max(kk, 1) / 1e3
     return k, (s1.timed_ns - s0.timed_ns) / max(k, 1) / 1e3
+
+
+KUS = [0.0]
 
 
 def loop(q, total, drain):
@@ -59,11 +64,17 @@ def loop(q, total, drain):
         t.join()
 
 
-for name, q, drain in (("alone", 1, True), ("serial", 1, False), ("q4", 4, False), ("alone", 1, True)):
+MODES = (("alone", 1, True), ("serial", 1, False), ("q4", 4, False), ("alone", 1, True))
+if len(sys.argv) > 1:   # one mode only, then exit (GROUTER_HOST_PROFILE percentiles of that mode)
+    MODES = [m for m in MODES if m[0] == sys.argv[1]][:1]
+for name, q, drain in MODES:
     loop(q, 20, drain)
     k, us = kstats(lambda: loop(q, 200, drain))
-    print(f"{name:8s} launches {k}  avg {us:.2f} us", flush=True)
+    print(f"{name:8s} launches {k}  avg {us:.2f} us  (kernel stamps {KUS[0]:.2f} us)", flush=True)
 
+if len(sys.argv) > 1:
+    ctx.close()
+    sys.exit(0)
 res = []
 for i in range(8):
     st, oid = ctx.put(cfn, hs[i].data_ptr(), n, 0, 0)
@@ -78,7 +89,8 @@ def b2b():
 
 
 k, us = kstats(b2b)
-print(f"b2b      launches {k}  avg {us:.2f} us (PROFILE events between launches)", flush=True)
+print(f"b2b      launches {k}  avg {us:.2f} us (PROFILE events between launches; kernel stamps {KUS[0]:.2f} us)",
+      flush=True)
 
 
 def gap(delay_us):
@@ -94,5 +106,5 @@ def gap(delay_us):
 
 for d in (0, 50, 200, 700, 2000):
     k, us = kstats(gap(d))
-    print(f"idle gap {d:5d} us before each launch: avg {us:.2f} us", flush=True)
+    print(f"idle gap {d:5d} us before each launch: avg {us:.2f} us  (kernel stamps {KUS[0]:.2f} us)", flush=True)
 ctx.close()
