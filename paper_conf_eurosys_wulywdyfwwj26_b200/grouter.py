@@ -14,6 +14,7 @@ from __future__ import annotations
 
 import ctypes as C
 import os
+import threading
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libgrouter.so")
@@ -119,20 +120,22 @@ _U64, _U32, _I32 = C.c_uint64, C.c_uint32, C.c_int32
 _ST = C.c_int
 _CTX = C.c_void_p
 
-# name -> (restype, argtypes); every symbol declared in include/*.h
+# name -> (restype, argtypes); every symbol declared in include/*.h.  The
+# data-path calls take their grouter_fn* and out-pointers as plain addresses
+# (c_void_p): a typed POINTER argument costs ~0.2 us of ctypes conversion per
+# argument per call, which single small transfers (a few us) would feel.
 SIGNATURES = {
     "grouter_config_default": (None, [C.POINTER(grouter_config)]),
     "grouter_probe": (_ST, [C.POINTER(grouter_config), _U64]),
     "grouter_init": (_ST, [C.POINTER(grouter_config), C.POINTER(_CTX)]),
     "grouter_finalize": (_ST, [_CTX]),
-    "grouter_put": (_ST, [_CTX, C.POINTER(grouter_fn), _P, _U64, _I32, _U32, _P, C.POINTER(_U64)]),
-    "grouter_alloc": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _I32, _U32, C.POINTER(_P),
-                            C.POINTER(_U64)]),
-    "grouter_seal": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P]),
-    "grouter_get": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, C.POINTER(_P), C.POINTER(_U64)]),
-    "grouter_get_into": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, _U64, _P, C.POINTER(_U64)]),
-    "grouter_release": (_ST, [_CTX, C.POINTER(grouter_fn), _U64, _P, _P]),
-    "grouter_free": (_ST, [_CTX, C.POINTER(grouter_fn), _U64]),
+    "grouter_put": (_ST, [_CTX, _P, _P, _U64, _I32, _U32, _P, _P]),
+    "grouter_alloc": (_ST, [_CTX, _P, _U64, _I32, _U32, _P, _P]),
+    "grouter_seal": (_ST, [_CTX, _P, _U64, _P]),
+    "grouter_get": (_ST, [_CTX, _P, _U64, _P, _P, _P]),
+    "grouter_get_into": (_ST, [_CTX, _P, _U64, _P, _U64, _P, _P]),
+    "grouter_release": (_ST, [_CTX, _P, _U64, _P, _P]),
+    "grouter_free": (_ST, [_CTX, _P, _U64]),
     "grouter_set_tenant_weight": (_ST, [_CTX, _U32, _U32]),
     "grouter_set_next_use": (_ST, [_CTX, _U64, _U64]),
     "grouter_set_pool_limit": (_ST, [_CTX, _I32, _U64]),
@@ -302,6 +305,32 @@ def fn(wf: int, fid: int, dev: int) -> grouter_fn:
     return grouter_fn(wf, fid, dev)
 
 
+def _fa(f: grouter_fn) -> int:
+    """Address of a grouter_fn (cached on the object: it never moves)."""
+    try:
+        return f._a
+    except AttributeError:
+        if not isinstance(f, grouter_fn):
+            raise TypeError("expected a grouter_fn") from None
+        f._a = C.addressof(f)
+        return f._a
+
+
+_tls = threading.local()
+
+
+def _out():
+    """This thread's out-parameter slots (4 x u64) and their address; the
+    library writes them only on success, so they are zeroed per call."""
+    try:
+        b, a = _tls.b, _tls.a
+    except AttributeError:
+        b = _tls.b = (C.c_uint64 * 4)()
+        a = _tls.a = C.addressof(b)
+    b[0] = b[1] = 0
+    return b, a
+
+
 class Ctx:
     """Owns a grouter_ctx; methods mirror the C calls and return statuses."""
 
@@ -328,37 +357,35 @@ class Ctx:
         except Exception:
             pass
 
-    # data path
+    # data path (per-thread out-parameter slots: one context serves several client threads)
     def put(self, f, src: int, n: int, hint=NOHINT, consumers=0, stream=0):
-        oid = C.c_uint64(0)
-        st = self.lib.grouter_put(self.h, C.byref(f), src or None, n, hint, consumers, stream or None,
-                                  C.byref(oid))
-        return st, oid.value
+        b, a = _out()
+        st = self.lib.grouter_put(self.h, _fa(f), src, n, hint, consumers, stream, a)
+        return st, b[0]
 
     def alloc(self, f, n: int, hint=NOHINT, consumers=0):
-        buf, oid = C.c_void_p(), C.c_uint64(0)
-        st = self.lib.grouter_alloc(self.h, C.byref(f), n, hint, consumers, C.byref(buf), C.byref(oid))
-        return st, (buf.value or 0), oid.value
+        b, a = _out()
+        st = self.lib.grouter_alloc(self.h, _fa(f), n, hint, consumers, a, a + 8)
+        return st, b[0], b[1]
 
     def seal(self, f, oid: int, stream=0):
-        return self.lib.grouter_seal(self.h, C.byref(f), oid, stream or None)
+        return self.lib.grouter_seal(self.h, _fa(f), oid, stream)
 
     def get(self, f, oid: int, stream=0):
-        p, n = C.c_void_p(), C.c_uint64(0)
-        st = self.lib.grouter_get(self.h, C.byref(f), oid, stream or None, C.byref(p), C.byref(n))
-        return st, (p.value or 0), n.value
+        b, a = _out()
+        st = self.lib.grouter_get(self.h, _fa(f), oid, stream, a, a + 8)
+        return st, b[0], b[1]
 
     def get_into(self, f, oid: int, dst: int, cap: int, stream=0):
-        n = C.c_uint64(0)   # per call: one context serves several client threads
-        st = self.lib.grouter_get_into(self.h, C.byref(f), oid, dst or None, cap, stream or None,
-                                       C.byref(n))
-        return st, n.value
+        b, a = _out()
+        st = self.lib.grouter_get_into(self.h, _fa(f), oid, dst, cap, stream, a)
+        return st, b[0]
 
     def release(self, f, oid: int, ptr: int, stream=0):
-        return self.lib.grouter_release(self.h, C.byref(f), oid, ptr or None, stream or None)
+        return self.lib.grouter_release(self.h, _fa(f), oid, ptr, stream)
 
     def free(self, f, oid: int):
-        return self.lib.grouter_free(self.h, C.byref(f), oid)
+        return self.lib.grouter_free(self.h, _fa(f), oid)
 
     # cross-process handoff
     def export_ipc(self, f, oid):

@@ -64,3 +64,28 @@ for name, f in (("get_into", gi), ("test_memcpy", mc), ("raw ctypes memcpy", raw
     f(0)
     print(f"{name:20s} host {host_cost(f):6.2f} us   dev-timed {dev_cost(f):6.2f} us", flush=True)
 ctx.close()
+
+# blocking cFn put of 4 KiB (fast copy-engine path) vs a bare pinned H2D + wait through the binding
+ctx2 = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED]))
+cf = G.fn(2, 1, G.HOST)
+
+
+def put4k(i):
+    st, o = ctx2.put(cf, host.data_ptr(), n, 0, 0)
+    ctx2.free(cf, o)
+
+
+def put4k_only(i):
+    st, o = ctx2.put(cf, host.data_ptr(), n, 0, 0)
+    frees.append(o)
+
+
+frees = []
+h2d = lambda i: G.test_memcpy(d[0].data_ptr(), host.data_ptr(), n, 0, True)
+for name, f in (("put+free 4 KiB", put4k), ("put 4 KiB", put4k_only), ("bare H2D+wait", h2d)):
+    f(0)
+    print(f"{name:20s} host {host_cost(f):6.2f} us", flush=True)
+    for o in frees:
+        ctx2.free(cf, o)
+    frees.clear()
+ctx2.close()
