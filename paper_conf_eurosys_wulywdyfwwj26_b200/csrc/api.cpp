@@ -216,10 +216,12 @@ bool host_reserve(grouter_ctx *c, uint64_t ch) {
 }
 
 // Physical storage for a reservation already charged; undoes the charge on failure.
-uint8_t *storage(grouter_ctx *c, int loc, uint64_t ch) {
+// lk: the caller's lock, which a pool growth may release (callers that hold no
+// object-table reference across the call: put, alloc)
+uint8_t *storage(grouter_ctx *c, int loc, uint64_t ch, std::unique_lock<std::mutex> *lk = nullptr) {
   if (!ch) return nullptr;
   try {
-    return loc == GROUTER_HOST ? host_alloc(c, ch) : dev_alloc(c, loc, ch);
+    return loc == GROUTER_HOST ? host_alloc(c, ch) : dev_alloc(c, loc, ch, lk);
   } catch (...) {
     if (loc == GROUTER_HOST) c->host_used -= ch;
     else c->dev[loc].used -= ch;
@@ -626,7 +628,7 @@ grouter_status grouter_put(grouter_ctx *c, const grouter_fn *fn, const void *src
   const uint64_t ch = charge(n);
   if (home != GROUTER_HOST && !reserve(c, home, ch)) home = GROUTER_HOST;    // R16
   if (home == GROUTER_HOST && !host_reserve(c, ch)) return fail(GROUTER_ENOMEM, "host store full");
-  uint8_t *ptr = storage(c, home, ch);
+  uint8_t *ptr = storage(c, home, ch, &g.lk);
   if (hp.on) p1 = p2 = now_ns();
   Obj o;
   o.oid = c->next_oid++;
@@ -703,7 +705,7 @@ grouter_status grouter_alloc(grouter_ctx *c, const grouter_fn *fn, uint64_t n, i
   const uint64_t ch = charge(n);
   if (home != GROUTER_HOST ? !reserve(c, home, ch) : !host_reserve(c, ch))
     return fail(GROUTER_ENOMEM, "alloc: does not fit after eviction");
-  uint8_t *ptr = storage(c, home, ch);
+  uint8_t *ptr = storage(c, home, ch, &g.lk);
   Obj o;
   o.oid = c->next_oid++;
   o.wf = fn->workflow_id;

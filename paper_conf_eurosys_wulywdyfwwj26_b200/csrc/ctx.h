@@ -388,7 +388,10 @@ void ded_sweep(grouter_ctx *c, std::unique_lock<std::mutex> *lk, bool wait);
 void ipc_release_all(grouter_ctx *c);
 // pool.cpp
 uint64_t pool_target(grouter_ctx *c, int logical);   // R44 target at the current clock
-uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len);   // may grow the pool
+// may grow the pool; with `lk` (the caller's hold on c->mu, real-time mode)
+// the growth's driver calls run with the lock released -- only for callers
+// that hold no reference into the object table across the call (put, alloc)
+uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len, std::unique_lock<std::mutex> *lk = nullptr);
 void dev_free(grouter_ctx *c, int logical, uint8_t *p, uint64_t len, Fences &&f);
 uint8_t *host_alloc(grouter_ctx *c, uint64_t len);
 void host_free(grouter_ctx *c, uint8_t *p, uint64_t len, Fences &&f);

@@ -385,7 +385,7 @@ static bool all_grounded(const grouter_ctx *c, const Quarantined &q) {
 // Physical pages for `len` bytes (a multiple of 2 MiB) on a logical GPU.
 // Order: free runs; reclaimed quarantine; wait for grounded quarantine (after
 // draining queued work so no wait depends on the caller); grow the mapping.
-uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
+uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len, std::unique_lock<std::mutex> *lk) {
   if (c->cfg.flags & GROUTER_NO_POOL) {  // ablation: no pool (Fig. 16 "ES" off)
     nopool_sweep(c, false);
     DeviceGuard g(c->dev[logical].phys);
@@ -409,6 +409,30 @@ uint8_t *dev_alloc(grouter_ctx *c, int logical, uint64_t len) {
       if (all_grounded(c, q)) host_wait(q.fences);
     P.heap.reclaim();
     if (P.heap.take(len, &off)) return (uint8_t *)(P.base + off);
+  }
+  if (lk && lk->owns_lock() && !c->replay) {
+    // grow by a whole segment of its own without the context lock: cuMemCreate /
+    // cuMemSetAccess took up to ~60 ms while copies streamed (tools/vmmlat.cu),
+    // and meanwhile the dispatch thread and the other callers keep going
+    const uint64_t seg = std::max<uint64_t>(len, 64ull << 20);
+    uint64_t voff = 0;
+    if (P.reserve(seg, voff)) {
+      const CUdeviceptr base = P.base;
+      const int phys = P.phys;
+      const std::vector<int> access = P.access;
+      lk->unlock();
+      DevicePool::Seg sg{};
+      bool ok = true;
+      try {
+        sg = DevicePool::map_seg(base, voff, seg, phys, access, true, len);
+      } catch (const Error &) {
+        ok = false;
+      }
+      lk->lock();
+      if (ok) P.publish(sg);
+      else P.unreserve(voff, seg);
+      if (ok && P.heap.take(len, &off)) return (uint8_t *)(P.base + off);
+    }
   }
   P.grow(len - std::min(len, P.heap.tail_free(P.va_top)));
   if (!P.heap.take(len, &off)) throw Error(GROUTER_ENOMEM, "pool fragmentation");

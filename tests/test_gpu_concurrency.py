@@ -144,3 +144,63 @@ def test_concurrent_clients(flags, rep):
             assert st.restore_count > 0
     finally:
         ctx.close()
+
+
+def test_pool_growth_without_the_lock_under_concurrency():
+    """Puts that must grow the pool (a cold pool, no pre-warm floor) from
+    several threads at once: their segment creation runs with the context
+    lock released (pool.cpp dev_alloc), so other callers and the dispatch
+    thread proceed meanwhile.  Every object reads back its own bytes, the
+    mapping covers what is resident, and the pool drains to zero."""
+    calib = C.b200_hgx(1)
+    calib["device_map"] = [0]
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED],
+                                    pool_floor_bytes=0))
+    errors = []
+    sizes = [3 * MiB + 5, 17 * MiB, 70 * MiB + 1, 130 * MiB]
+
+    def worker(t):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            f = G.fn(40 + t, 1, 0)
+            g = G.fn(40 + t, 2, 0)
+            src = torch.empty(max(sizes), dtype=torch.uint8, device="cuda")
+            dst = torch.empty(max(sizes), dtype=torch.uint8, device="cuda")
+            live = []
+            for i in range(12):
+                n = sizes[(t + i) % len(sizes)]
+                seed = 7000 + 100 * t + i
+                G.check(G.test_fill(src.data_ptr(), n, seed, 0, s.cuda_stream), "fill")
+                st, oid = ctx.put(f, src.data_ptr(), n, G.NOHINT, 0, s.cuda_stream)
+                G.check(st, "put")
+                live.append((oid, n, seed))
+                if len(live) > 3:
+                    oid, n, seed = live.pop(0)
+                    G.check(ctx.get_into(g, oid, dst.data_ptr(), n, s.cuda_stream)[0], "get_into")
+                    s.synchronize()
+                    st, bad, first = G.test_verify(dst.data_ptr(), n, seed, 0, 0)
+                    assert st == 0 and bad == 0, (t, n, bad, first)
+                    G.check(ctx.free(f, oid), "free")
+            for oid, n, seed in live:
+                G.check(ctx.get_into(g, oid, dst.data_ptr(), n, s.cuda_stream)[0], "get_into")
+                s.synchronize()
+                st, bad, first = G.test_verify(dst.data_ptr(), n, seed, 0, 0)
+                assert st == 0 and bad == 0, (t, n, bad, first)
+                G.check(ctx.free(f, oid), "free")
+        except Exception as e:  # pragma: no cover - reported below
+            errors.append(repr(e))
+
+    try:
+        ths = [threading.Thread(target=worker, args=(t,)) for t in range(6)]
+        for th in ths:
+            th.start()
+        for th in ths:
+            th.join()
+        assert not errors, errors
+        G.check(ctx.sync(), "sync")
+        st = ctx.stats()
+        assert st.used[0] == 0 and st.host_used == 0
+        assert st.mapped[0] >= 130 * MiB
+    finally:
+        ctx.close()
