@@ -2,7 +2,8 @@
 // 10 MiB batch copies (the O8 preemption granularity) cost link time, and do
 // two copy-engine streams used alternately hide the per-copy setup?  Per
 // pattern: back-to-back GB/s over 40 puts and the single-put latency.
-//   nvcc -gencode arch=compute_100a,code=sm_100a -O2 tools/ce2.cu -o tools/ce2
+//   nvcc -gencode arch=compute_100a,code=sm_100a -O2 tools/ce2.cu -lcuda -o tools/ce2
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -21,6 +22,13 @@ int main() {
   cudaEventCreate(&a);
   cudaEventCreate(&b);
   cudaEventCreateWithFlags(&j, cudaEventDisableTiming);
+  std::vector<cudaEvent_t> evs(8);
+  for (auto &e : evs) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+  unsigned int *word;
+  cudaHostAlloc(&word, 64, cudaHostAllocMapped);
+  CUdeviceptr dword;
+  cudaHostGetDevicePointer((void **)&dword, word, 0);
+  static unsigned int seq = 0;
   auto put = [&](int mode) {
     if (mode == 0) {
       cudaMemcpyAsync(d, h, n, cudaMemcpyHostToDevice, s[0]);
@@ -29,16 +37,19 @@ int main() {
     int k = 0;
     for (size_t off = 0; off < n; off += batch, ++k) {
       size_t len = std::min(batch, n - off);
-      cudaStream_t st = mode == 1 ? s[0] : s[k & 1];
+      cudaStream_t st = mode == 2 ? s[k & 1] : s[0];
       cudaMemcpyAsync((char *)d + off, (char *)h + off, len, cudaMemcpyHostToDevice, st);
+      if (mode == 3) cudaEventRecord(evs[k & 7], st);           // the library's per-round event
+      if (mode == 4) cuStreamWriteValue32(st, dword, ++seq, 0);  // or a completion word
     }
     if (mode == 2) {  // join the second stream back into the first
       cudaEventRecord(j, s[1]);
       cudaStreamWaitEvent(s[0], j, 0);
     }
   };
-  const char *names[] = {"1 copy of 38.5 MB", "4 x 10 MiB, one stream", "4 x 10 MiB, two streams alternating"};
-  for (int mode = 0; mode < 3; ++mode) {
+  const char *names[] = {"1 copy of 38.5 MB", "4 x 10 MiB, one stream", "4 x 10 MiB, two streams alternating",
+                         "4 x 10 MiB, event after each", "4 x 10 MiB, stream write after each"};
+  for (int mode = 0; mode < 5; ++mode) {
     for (int i = 0; i < 3; ++i) put(mode);
     cudaDeviceSynchronize();
     cudaEventRecord(a, s[0]);
