@@ -150,6 +150,7 @@ struct Server {
   Stride<ChunkItem> sched;
   cudaStream_t stream = nullptr;      // SM-copy stream / CE stream
   cudaStream_t fwd_stream = nullptr;  // H2D: relay forward kernel stream
+  cudaStream_t pub_stream = nullptr;  // CE servers: completion-word writes (publish_ce)
   uint32_t *scratch = nullptr;        // device scratch of the copy kernel on `stream`
   uint32_t *fwd_scratch = nullptr;    // ... on `fwd_stream`
   struct Inflight {

@@ -41,6 +41,12 @@ int main() {
       cudaMemcpyAsync((char *)d + off, (char *)h + off, len, cudaMemcpyHostToDevice, st);
       if (mode == 3) cudaEventRecord(evs[k & 7], st);           // the library's per-round event
       if (mode == 4) cuStreamWriteValue32(st, dword, ++seq, 0);  // or a completion word
+      if (mode == 5) cuStreamWriteValue32(st, dword, ++seq, CU_STREAM_WRITE_VALUE_NO_MEMORY_BARRIER);
+      if (mode == 6) {  // the word written from a side stream after an event (the CE stream runs on)
+        cudaEventRecord(evs[k & 7], st);
+        cudaStreamWaitEvent(s[2], evs[k & 7], 0);
+        cuStreamWriteValue32(s[2], dword, ++seq, 0);
+      }
     }
     if (mode == 2) {  // join the second stream back into the first
       cudaEventRecord(j, s[1]);
@@ -48,8 +54,9 @@ int main() {
     }
   };
   const char *names[] = {"1 copy of 38.5 MB", "4 x 10 MiB, one stream", "4 x 10 MiB, two streams alternating",
-                         "4 x 10 MiB, event after each", "4 x 10 MiB, stream write after each"};
-  for (int mode = 0; mode < 5; ++mode) {
+                         "4 x 10 MiB, event after each", "4 x 10 MiB, stream write after each",
+                         "4 x 10 MiB, write (no barrier) after each", "4 x 10 MiB, event + side-stream write"};
+  for (int mode = 0; mode < 7; ++mode) {
     for (int i = 0; i < 3; ++i) put(mode);
     cudaDeviceSynchronize();
     cudaEventRecord(a, s[0]);
