@@ -86,22 +86,6 @@ void caller_wait(grouter_ctx *c, cudaStream_t s, const Fences &f) {
   }
 }
 
-// A point on a CALLER's stream: the library writes a fresh completion word
-// from that stream (cuStreamWriteValue32) and waits for / polls the word.
-// Caller streams may come from another runtime instance (PyTorch's), so no
-// event handle crosses that boundary.
-Waitable signal(grouter_ctx *c, cudaStream_t s, int phys) {
-  (void)phys;
-  std::vector<grouter_chunk> one(1, grouter_chunk{0, 0, 0, 0});
-  XferRef x = new_xfer_slot(c, one);
-  GR_CU(drv().streamWriteValue32((CUstream)s, (CUdeviceptr)(uintptr_t)&x->words[0], x->target[0], 0));
-  Waitable w;
-  w.word = &x->words[0];
-  w.target = x->target[0];
-  w.epoch = c->epoch;
-  return w;
-}
-
 static Waitable ev_wait(grouter_ctx *c, EventRef e) {
   Waitable w;
   w.ev = std::move(e);
@@ -113,6 +97,20 @@ EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
   EventRef e = c->phys.at(phys)->events.get();
   GR_CUDA(cudaEventRecord(e->ev, s));
   return e;
+}
+
+// A point on a CALLER's stream: an event recorded there (the caller's runtime
+// and this library's share the device's primary context; the fast direct path
+// records its completion on caller streams the same way).  Round 1 wrote a
+// completion word from the caller's stream instead: cuStreamWriteValue32
+// carries a memory barrier that idles the stream ~3.5-5 us (tools/ce2.cu; the
+// launch_round note above), which every seal / release / stream-ordered put
+// of a function would have paid on its own stream.
+Waitable signal(grouter_ctx *c, cudaStream_t s, int phys) {
+  DeviceGuard g(phys);  // a fresh pooled event is created on the current device
+  Waitable w = ev_wait(c, record(c, s, phys));
+  w.origin = s;
+  return w;
 }
 
 void host_wait(const Fences &f, double timeout_s, const std::atomic<bool> *abort) {
