@@ -13,7 +13,9 @@
 //    host-mapped memory, one per path.  Producers publish ABSOLUTE values
 //    (the host knows how many of the transfer's path-p chunks each round
 //    carries): SM kernels with st.release.sys from the round's last CTA, copy
-//    engines with cuStreamWriteValue32 after their memcpys.  Consumers wait
+//    engines with cuStreamWriteValue32 after their memcpys (on the server's
+//    publish stream behind an event, so the write's memory barrier does not
+//    idle the copy engine).  Consumers wait
 //    with cuStreamWaitValue32(GEQ) on their own stream, or poll from the
 //    host -- no host round trip on the data path, no partial visibility.
 //  * Each server (SM-copy egress of a GPU, H2D engine of a route GPU, D2H
