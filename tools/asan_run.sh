@@ -9,6 +9,8 @@ set -x
 D=gpurun_out/asan
 mkdir -p $D
 python paper_conf_eurosys_wulywdyfwwj26_b200/_build.py --asan
+# the product build too, before the preload (nvcc must not run under ASan)
+python -c "from paper_conf_eurosys_wulywdyfwwj26_b200 import _build; _build.build()"
 # libstdc++ preloaded too: the runtime must see it at start (the library throws C++ exceptions)
 export LD_PRELOAD="$(gcc -print-file-name=libasan.so) $(gcc -print-file-name=libstdc++.so)" GROUTER_LIB=asan
 export ASAN_OPTIONS="protect_shadow_gap=0:detect_leaks=0:halt_on_error=0:log_path=$D/asan"

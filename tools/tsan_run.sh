@@ -8,6 +8,7 @@ set -x
 D=gpurun_out/tsan
 mkdir -p $D
 python paper_conf_eurosys_wulywdyfwwj26_b200/_build.py --tsan
+python -c "from paper_conf_eurosys_wulywdyfwwj26_b200 import _build; _build.build()"
 export LD_PRELOAD=$(gcc -print-file-name=libtsan.so) GROUTER_LIB=tsan
 TSAN_OPTIONS="halt_on_error=0 log_path=$D/control" python - <<'PY'
 import ctypes, sys
