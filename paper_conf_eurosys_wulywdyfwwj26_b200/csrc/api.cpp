@@ -362,10 +362,10 @@ XferRef start_transfer(grouter_ctx *c, uint32_t tenant, int src_loc, int dst_loc
   // never a direct launch): the source's copy server pushes, the consumer
   // stream waits on the completion words
   const bool may_direct = !(c->cfg.flags & GROUTER_FORCE_REMOTE) || src_loc == dst_loc;
-  if (caller && direct && n && may_direct && server_kind_for(src_loc, dst_loc) == SK_COPY) {
+  if (caller && direct && n && server_kind_for(src_loc, dst_loc) == SK_COPY) {  // (small pulls: forced too)
     const int server = src_loc == GROUTER_REMOTE ? dst_loc : src_loc;
     XferRef fx = fast_direct(c, tenant, server, dst_loc, (uint64_t)(uintptr_t)src, (uint64_t)(uintptr_t)dst, n,
-                             pool_src && src_loc >= 0, deps, caller, c->dev[caller_logical].phys);
+                             pool_src && src_loc >= 0, deps, caller, caller_logical);
     if (fx) {
       *direct = true;
       if (hprof().on) hprof().t[4] += now_ns() - tst;

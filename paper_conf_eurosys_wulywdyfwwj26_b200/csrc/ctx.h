@@ -354,7 +354,7 @@ XferRef fast_ce(grouter_ctx *c, uint32_t tenant, int kind, const std::vector<gro
                 uint64_t dst, uint64_t n, const Fences &deps);
 XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
-                    int caller_phys);
+                    int caller_logical);
 void stream_wait(grouter_ctx *c, cudaStream_t s, int phys, const Fences &f);  // submitted fences only
 // Waits on a CALLER stream: submitted fences now, the others as soon as their
 // producer transfer is submitted.

@@ -35,6 +35,8 @@
 #include <cstring>
 #include <thread>
 
+#include <sys/prctl.h>
+
 #include "ctx.h"
 #include "kernels.h"
 
@@ -245,6 +247,13 @@ static uint32_t weight_of(grouter_ctx *c, uint32_t t) {
 }
 
 static void retire(Server &s);
+static inline void cpu_relax() {
+#if defined(__x86_64__) || defined(__i386__)
+  __builtin_ia32_pause();
+#else
+  std::this_thread::yield();
+#endif
+}
 
 static void log_batch(grouter_ctx *c, Server &s, uint32_t tenant,
                       const std::vector<ChunkItem> &b, uint64_t bytes) {
@@ -536,14 +545,65 @@ void harvest_profile(grouter_ctx *c, bool wait) {
 
 // SM-copy server: one kernel launch per round segment (D2D push over
 // NVLink, or a same-GPU HBM copy).
+//
+// A transfer that is the ONLY work queued on the server (one tenant, one
+// transfer, no urgent work) goes out WHOLE in one round (R55, the queued
+// counterpart of R53's direct launch): e.g. a GPU -> other-GPU get, whose
+// consumer stream lives on another device and so never takes the direct
+// launch.  A batch per round costs a launch and a dispatch reaction per
+// 10 MiB -- at NVLink rates (~14 us per batch) that, not the link, bounds a
+// large push (tools/peerpath.py).  A tenant arriving later waits behind the
+// <= 2 rounds in flight, as behind a direct launch.  Real-time mode without
+// GROUTER_LOG only (replay and the log keep one batch per round).
+static void complete_by_event(grouter_ctx *c, const std::vector<Xfer *> &xs, const EventRef &e, cudaStream_t st);
+static bool single_transfer(const Server &s) {
+  if (!s.carry.empty() || !s.urgent.empty()) return false;
+  const Xfer *only = nullptr;
+  for (auto &kv : s.sched.tenants) {
+    const auto &q = kv.second.q;
+    if (q.empty()) continue;
+    if (only || q.front().x != q.back().x) return false;
+    only = q.front().x;
+  }
+  return only != nullptr;
+}
+
 static size_t round_copy(grouter_ctx *c, Server &s) {
   NvtxRange nvtx_("round copy");
-  const uint32_t nb = refill_one(c, s);
+  static const bool solo_off = getenv("GR_NO_FAST") != nullptr || getenv("GR_NO_SOLO") != nullptr;
+  const bool solo = !solo_off && !c->replay && !(c->cfg.flags & GROUTER_LOG) && single_transfer(s);
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
-  take(s, batch_budget(c, s), items, cut);
+  uint32_t nb;
+  if (solo) {
+    nb = refill(c, s, UINT32_MAX, kDirectBytes, kDirectItems);
+    take(s, kDirectBytes, items, cut, kDirectItems);
+  } else {
+    nb = refill_one(c, s);
+    take(s, batch_budget(c, s), items, cut);
+  }
   if (items.empty()) return 0;
   DeviceGuard g(s.phys);
+  if (solo) {
+    // one launch moves the whole transfer: complete it by an event, not words
+    Xfer *x = items[0].x;
+    static const bool ev_done = !getenv("GR_NO_EVDONE");
+    const bool whole = ev_done && !x->word_fenced && x->submitted_chunks == 0 && x->waiters.empty() &&
+                       items.size() == x->nchunks && std::count(cut.begin(), cut.end(), 1) <= (cut[0] ? 1 : 0) &&
+                       !(c->cfg.flags & GROUTER_FORCE_REMOTE);  // forced remote: in-kernel publish
+    if (whole) {
+      if (cut[0]) stream_wait(c, s.stream, s.phys, x->deps);
+      bool deferred = false;
+      launch_round(c, s, s.stream, s.scratch, items, nullptr, &deferred);
+      EventRef ev = record(c, s.stream, s.phys);
+      if (deferred) complete_by_event(c, {x}, ev, s.stream);
+      for (auto &it : items) c->stats.link_bytes[0][s.logical] += it.bytes;
+      s.inflight.push_back({ev_wait(c, ev), nullptr, nb});
+      c->stats.rounds++;
+      after_submit(c, items);
+      return items.size();
+    }
+  }
   for (size_t i = 0; i < items.size(); ++i) {
     if (cut[i]) {
       if (!seg.empty()) launch_round(c, s, s.stream, s.scratch, seg, nullptr);
@@ -874,14 +934,33 @@ void flush_all(grouter_ctx *c) {
 // completion slot (~1.5 us of host time per call, tools/libcost.cpp).  Only
 // for static-assignment engines (16 B-aligned addresses: wv8 / tmas4, no
 // device scratch).  Returns null when the queued path must be used.
+//
+// Small GPU -> other-GPU copies (<= kPullMax) run here too, as a PULL on the
+// consumer's stream (R56): the consumer GPU's SMs read the source over
+// NVLink (pool pages and peer buffers are mapped for every GPU), so the
+// consumer's stream needs no cross-device event, no completion words and no
+// wait on the source GPU's server stream -- at these sizes that chain, not
+// the link, is the latency (tools/peerpath.py).  Larger ones are pushed by
+// the source GPU's copy server (R40, R55).  The source's server still does
+// the stride accounting: the bytes use its NVLink egress.
+static const uint64_t kPullMax = 4ull << 20;
+
 XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst_logical, uint64_t src,
                     uint64_t dst, uint64_t n, bool local_src, const Fences &deps, cudaStream_t caller,
-                    int caller_phys) {
+                    int caller_logical) {
   static const bool off = getenv("GR_NO_FAST") != nullptr || getenv("GR_COPY") != nullptr;
-  const uint32_t never = GROUTER_LOG | GROUTER_FORCE_REMOTE | GROUTER_COPY_TMA;
+  static const bool pull_off = getenv("GR_NO_PULL") != nullptr;
+  const uint32_t never = GROUTER_LOG | GROUTER_COPY_TMA;
   if (off || c->replay || !caller || (c->cfg.flags & never) || !n || ((src | dst) & 15)) return nullptr;
+  if (caller_logical < 0) return nullptr;
   Server &s = c->dev[server_logical].copy;
-  if (s.phys != caller_phys || !s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
+  const int caller_phys = c->dev[caller_logical].phys;
+  // forced remote (test): logical GPUs stand for physical ones
+  const bool forced = (c->cfg.flags & GROUTER_FORCE_REMOTE) != 0;
+  const bool cross = forced ? server_logical != caller_logical : s.phys != caller_phys;
+  if (forced && !cross) return nullptr;  // forced remote: same-GPU rounds take the queued path
+  if (cross && (pull_off || n > kPullMax)) return nullptr;
+  if (!s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
   for (auto &f : s.inflight)
     if (f.direct != caller) {
       retire(s);
@@ -901,11 +980,12 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   x->nchunks = x->submitted_chunks = (uint32_t)((n + C - 1) / C);
   x->local_src = local_src;
   c->stats.xfer_count++;
-  DeviceGuard g(s.phys);
-  stream_wait(c, caller, s.phys, deps);  // no-op for completed fences
+  DeviceGuard g(caller_phys);
+  stream_wait(c, caller, caller_phys, deps);  // no-op for completed fences
   if (!c->params) c->params = new CopyParamsHost();
   CopyParams *p = &c->params->p;
-  const bool local = dst_logical >= 0 && c->dev[dst_logical].phys == s.phys;
+  const bool local = !forced && dst_logical >= 0 && c->dev[dst_logical].phys == caller_phys;
+  local_src &= !cross;  // a pull reads the other GPU's memory
   p->flags = (local ? kFlagLocalDst : 0) | (local_src ? kFlagLocalSrc : 0);
   p->n_chunks = 1;
   p->n_pub = 0;
@@ -915,7 +995,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   p->stamp = nullptr;
   p->chunk[0] = {src, dst, n};
   bool host_pub = false;
-  PhysDev &pd = *c->phys.at(s.phys);
+  PhysDev &pd = *c->phys.at(caller_phys);
   // Tiny same-device copies (<= 64 KiB; GR_SMALL_CE overrides for measurement)
   // go to the copy engine: its start latency beats a kernel launch's there
   // (C++ single calls, tools/libcost.cpp: 4 KiB 7.94 -> 7.14 us, 64 KiB
@@ -923,28 +1003,28 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   // kernel is at or below the copy engine
   static const uint64_t small_ce =
       getenv("GR_SMALL_CE") ? strtoull(getenv("GR_SMALL_CE"), nullptr, 0) : (64ull << 10);
-  if (n <= small_ce) {
+  if (n <= small_ce && !cross) {
     GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, n, cudaMemcpyDeviceToDevice, caller));
     host_pub = true;
   } else {
     const bool prof = (c->cfg.flags & GROUTER_PROFILE) != 0;  // the same events and stamps as launch_round
-    ProfRec pr{s.phys, nullptr, nullptr, n};
+    ProfRec pr{caller_phys, nullptr, nullptr, n};
     if (prof) prof_begin(pd, caller, pr, p->stamp);
     int e = launch_copy(*p, pd.sm_count, (int)c->cfg.copy_ctas_per_sm, false, caller, &host_pub);
     if (e != 0) throw Error(GROUTER_ECUDA, std::string("gr_copy launch: ") + cudaGetErrorString((cudaError_t)e));
     if (prof) prof_end(c, caller, pr);
   }
   if (!host_pub) throw Error(GROUTER_ECUDA, "internal: fast direct launch needs a static engine");
-  x->done_ev = record(c, caller, s.phys);
+  x->done_ev = record(c, caller, caller_phys);
   x->done_stream = caller;
   // the bookkeeping a queued dispatch would have done
   s.sched.account_solo(tenant, n, C, weight_of(c, tenant));
   note_dispatch(c, tenant, SK_COPY, n);
   c->stats.link_bytes[0][s.logical] += n;
   c->stats.rounds++;
-  if (n > small_ce) {
+  if (n > small_ce || cross) {
     c->stats.kernel_launches++;
-    if (!local) c->stats.peer_launches++;
+    if (!local || cross) c->stats.peer_launches++;
   }
   Waitable w;
   w.ev = x->done_ev;
@@ -1125,16 +1205,33 @@ static constexpr uint64_t kTrimDelayNs = 1000000000ull;  // 1 s of sustained exc
 // Dispatch thread (L269-L271 I/O daemon): pumps the servers' queues and
 // retires completed rounds.  Nothing here may block in a slow driver call:
 // while a blocking host put waits, this thread alone issues its next batches.
+//
+// Poll period while work is queued.  A copy engine's round (one 10 MiB batch
+// over PCIe) lasts ~190 us, so a 20 us sleep keeps its two-round window
+// full.  An SM-copy round is one 10 MiB batch over NVLink (~14 us) or HBM
+// (~3 us): with two rounds in flight the next launch must follow a
+// completion within a few microseconds, or the link idles between rounds
+// (measured on the forced-remote path, tools/peerpath.py: a 20 us sleep --
+// ~70 us with the default 50 us timer slack -- left 1 GiB pushes at 0.08 of
+// the HBM copy rate).  So while an SM-copy server has backlog the thread
+// spins with the lock released (~1 us between polls; one core, only while
+// such a backlog exists) and only those servers are polled.
 static void daemon_main(grouter_ctx *c) {
+  prctl(PR_SET_TIMERSLACK, 1000UL, 0, 0, 0);  // 1 us: sleeps close to what they ask for
   std::unique_lock<std::mutex> lk(c->mu);
+  uint32_t spins = 0;
   while (!c->stop) {
-    bool backlog = false, busy = false;
+    bool backlog = false, busy = false, sm_backlog = false;
     try {
       if (!c->replay) pump(c, false);
+      for (auto &d : c->dev) sm_backlog |= !c->replay && has_work(d.copy);
+      // full retire sweep (event queries on every server) only when not
+      // spinning, or every 64th spin
+      const bool sweep = !sm_backlog || (++spins & 63) == 0;
       for (auto &d : c->dev) {
         backlog |= has_work(d.copy) || has_work(d.h2d) || has_work(d.d2h);
         busy |= !d.copy.inflight.empty() || !d.h2d.inflight.empty() || !d.d2h.inflight.empty();
-        if (!c->replay) {
+        if (!c->replay && sweep) {
           retire(d.copy);
           retire(d.h2d);
           retire(d.d2h);
@@ -1144,8 +1241,14 @@ static void daemon_main(grouter_ctx *c) {
       set_error(e.what());
       c->sticky_error = true;
       c->submit_cv.notify_all();  // callers blocked in order_after fail with ECUDA
+      sm_backlog = false;
     }
-    if (backlog && !c->replay) {
+    if (sm_backlog) {
+      lk.unlock();
+      const uint64_t t0 = now_ns();
+      while (now_ns() - t0 < 1000) cpu_relax();
+      lk.lock();
+    } else if (backlog && !c->replay) {
       lk.unlock();
       std::this_thread::sleep_for(std::chrono::microseconds(20));
       lk.lock();

@@ -301,6 +301,47 @@ def test_config_traces_forced_remote(replay):
         assert st.peer_launches == st.kernel_launches > 0
 
 
+@pytest.mark.parametrize("n", [4096, 4 * MiB - 16, 4 * MiB + 4096, 64 * MiB + 12288])
+def test_cross_gpu_dispatch_forced_remote(n):
+    """R55 / R56 on the peer branch: a gFn on logical GPU1 get_into's objects
+    of logical GPU0 on its own stream.  A copy of <= 4 MiB on an idle server
+    is ONE pull launch on the consumer's stream; a larger one alone on the
+    source's copy server is ONE push launch (whole transfer, not a round per
+    10 MiB batch).  Every launch takes the peer branch, every delivered byte
+    equals the generator's, and the stride accounting advances as for queued
+    batches (tenant bytes = n per get)."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    pool_floor_bytes=64 * MiB, flags=G.FORCE_REMOTE))
+    try:
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 515, 0, 0))
+        torch.cuda.synchronize()
+        st, oid = ctx.put(G.fn(9, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        assert ctx.where(oid) == (G.OK, 0)
+        ctx.sync()
+        s1 = torch.cuda.Stream()
+        dst = torch.zeros(n + 64, dtype=torch.uint8, device="cuda")
+        f1 = G.fn(9, 2, 1)
+        for rep in range(3):
+            st0 = ctx.stats()
+            dst.zero_()
+            torch.cuda.synchronize()
+            G.check(ctx.get_into(f1, oid, dst.data_ptr(), n, s1.cuda_stream)[0], "get_into")
+            s1.synchronize()
+            st1 = ctx.stats()
+            assert st1.kernel_launches - st0.kernel_launches == 1, (rep, st1.kernel_launches - st0.kernel_launches)
+            assert st1.peer_launches - st0.peer_launches == 1
+            assert st1.link_bytes[0][0] - st0.link_bytes[0][0] == n   # the source GPU's egress
+            st, bad, first = G.test_verify(dst.data_ptr(), n, 515, 0, 0)
+            assert st == 0 and bad == 0, (rep, bad, first)
+            assert not dst[n:].any()
+        assert ctx.tenant_stats(9)[0] >= 3 * n
+    finally:
+        ctx.close()
+
+
 @pytest.mark.parametrize("replay", [True, False])
 def test_ce_relay_parity(replay):
     """GROUTER_CE_RELAY: the route GPUs' copy engines write the destination's
