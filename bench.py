@@ -1023,6 +1023,8 @@ def run_gpu(args, rank, world, local_rank):
     calib = b200_hgx(1 if world == 1 else 2)
     calib["device_map"] = [dev] if world == 1 else [dev, cons_dev]
     flags = G.PROFILE | (G.COPY_TMA if args.tma else 0) | (G.NO_MULTIPATH if world > 1 else 0)
+    if same_gpu and os.environ.get("GR_BENCH_FORCE_REMOTE") == "1":
+        flags |= G.FORCE_REMOTE   # plumbing on one GPU: the dispatch and kernel branch of a physical pair
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 << 20, pool_cap=[G.UNLIMITED] * calib["n_gpus"],
                                     flags=flags, copy_ctas_per_sm=args.ctas))
     cons_logical = 0 if world == 1 else 1

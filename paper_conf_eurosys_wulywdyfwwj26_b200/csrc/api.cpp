@@ -563,6 +563,10 @@ grouter_status grouter_init(const grouter_config *cfg_in, grouter_ctx **out) {
 
 grouter_status grouter_finalize(grouter_ctx *c) {
   if (!c) return fail(GROUTER_EINVAL, "null ctx");
+  if (hprof().on && (hprof().rounds[0] || hprof().rounds[1]))
+    fprintf(stderr, "[grouter host profile] dispatch rounds: SM copy x%llu %.2f us each, copy engine x%llu %.2f us each\n",
+            (unsigned long long)hprof().rounds[0], hprof().t[19] / std::max<uint64_t>(1, hprof().rounds[0]) / 1e3,
+            (unsigned long long)hprof().rounds[1], hprof().t[20] / std::max<uint64_t>(1, hprof().rounds[1]) / 1e3);
   if (hprof().on && (hprof().calls || hprof().put_calls)) {
     HostProf &h = hprof();
     fprintf(stderr, "[grouter host profile] get_into calls %llu: lock+lookup %.2f us, transfer+launch %.2f us, "

@@ -189,7 +189,9 @@ inline void prune(Fences &f) {
 struct HostProf {
   bool on = false;
   uint64_t calls = 0, put_calls = 0;
-  double t[24] = {};  // [0..7] get_into stages, [8..15] blocking put stages, [16..18] put -> H2D copy
+  uint64_t rounds[2] = {};  // SM-copy rounds, copy-engine rounds (H2D and D2H) timed in t[19], t[20]
+  double t[24] = {};  // [0..7] get_into stages, [8..15] blocking put stages, [16..18] put -> H2D copy,
+                     // [19..23] dispatch rounds: host ns / count per server kind (copy, h2d, d2h) and relayed chunks
 };
 HostProf &hprof();
 uint64_t now_ns();

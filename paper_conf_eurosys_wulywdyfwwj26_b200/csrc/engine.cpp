@@ -893,7 +893,14 @@ static size_t pump_server(grouter_ctx *c, Server &s, bool force) {
       --c->inject_round_failures;
       throw Error(GROUTER_ECUDA, "injected dispatch-round failure (grouter_test_inject)");
     }
+    const uint64_t tr = hprof().on ? now_ns() : 0;
     size_t n = s.kind == SK_COPY ? round_copy(c, s) : s.kind == SK_H2D ? round_h2d(c, s) : round_d2h(c, s);
+    if (tr && n) {  // GROUTER_HOST_PROFILE: host time per dispatch round (the dispatch thread's budget)
+      static std::mutex m;
+      std::lock_guard<std::mutex> lk(m);
+      hprof().t[s.kind == SK_COPY ? 19 : 20] += now_ns() - tr;
+      hprof().rounds[s.kind == SK_COPY ? 0 : 1]++;
+    }
     if (!n) break;  // blocked on another server's submission
     total += n;
   }

@@ -10,7 +10,9 @@ Per size: back-to-back GB/s (read + write bytes over HBM, so the per-launch
 overhead shows ~10x larger than it would over NVLink) and single-call p50
 (CUDA events on the consumer stream, host path included)."""
 import json
+import os
 import sys
+import time
 
 sys.path.insert(0, ".")
 import torch  # noqa: E402
@@ -20,8 +22,9 @@ from synth import calib as C  # noqa: E402
 
 G.load()
 out = {}
-modes = [("direct", 0), ("remote", G.FORCE_REMOTE)]
-for name, flags in modes:
+modes = [m for m in [("direct", 0), ("remote", G.FORCE_REMOTE)]
+         if m[0] in os.environ.get("PEERPATH_MODES", "direct,remote").split(",")]
+for name, flags in ([] if os.environ.get("PEERPATH_LEGB") else modes):
     calib = C.virtual(2)
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * 2,
                                     flags=flags, pool_floor_bytes=64 << 20))
@@ -72,4 +75,44 @@ for name, flags in modes:
     res["rounds"] = st.rounds
     out[name] = res
     ctx.close()
-print(json.dumps(out))
+if out:
+    print(json.dumps(out))
+
+# bench.py's N >= 2 leg-B pattern: 20 distinct 38.5 MB objects of logical GPU0
+# get_into'd by GPU1 round robin into 8 bindings on one stream, back to back
+if os.environ.get("PEERPATH_LEGB"):
+    for name, flags in modes:
+        ctx = G.Ctx(G.config_from_calib(C.virtual(2), host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * 2,
+                                        flags=flags, pool_floor_bytes=64 << 20))
+        n = 38_535_168
+        src = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), n, 77, 0, 0))
+        torch.cuda.synchronize()
+        oids = [ctx.put(G.fn(1, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)[1] for _ in range(20)]
+        ctx.sync()
+        binds = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(8)]
+        s1 = torch.cuda.Stream()
+        f1 = G.fn(1, 2, 1)
+
+        def legb():
+            for i, oid in enumerate(oids):
+                G.check(ctx.get_into(f1, oid, binds[i % 8].data_ptr(), n, s1.cuda_stream)[0], "get_into")
+        legb()
+        s1.synchronize()
+        k0 = ctx.stats()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s1)
+        t0 = time.perf_counter()
+        for _ in range(20):
+            legb()
+        th = time.perf_counter() - t0
+        b.record(s1)
+        b.synchronize()
+        k1 = ctx.stats()
+        out[f"legb_{name}"] = {"us_per_get": round(a.elapsed_time(b) * 1e3 / 400, 2),
+                               "host_us_per_call": round(th * 1e6 / 400, 2),
+                               "launches_per_get": (k1.kernel_launches - k0.kernel_launches) / 400}
+        st, bad, _ = G.test_verify(binds[3].data_ptr(), n, 77, 0, 0)
+        assert st == 0 and bad == 0
+        ctx.close()
+    print(json.dumps({k: v for k, v in out.items() if k.startswith("legb")}))
