@@ -1220,9 +1220,9 @@ static constexpr uint64_t kTrimDelayNs = 1000000000ull;  // 1 s of sustained exc
 // completion within a few microseconds, or the link idles between rounds
 // (measured on the forced-remote path, tools/peerpath.py: a 20 us sleep --
 // ~70 us with the default 50 us timer slack -- left 1 GiB pushes at 0.08 of
-// the HBM copy rate).  So while an SM-copy server has backlog the thread
-// spins with the lock released (~1 us between polls; one core, only while
-// such a backlog exists) and only those servers are polled.
+// the HBM copy rate).  So while an SM-copy server's backlog waits for a free
+// slot in its window the thread spins with the lock released (~1 us between
+// polls; one core, only then), with the full retire sweep every 64 polls.
 static void daemon_main(grouter_ctx *c) {
   prctl(PR_SET_TIMERSLACK, 1000UL, 0, 0, 0);  // 1 us: sleeps close to what they ask for
   std::unique_lock<std::mutex> lk(c->mu);
@@ -1231,7 +1231,9 @@ static void daemon_main(grouter_ctx *c) {
     bool backlog = false, busy = false, sm_backlog = false;
     try {
       if (!c->replay) pump(c, false);
-      for (auto &d : c->dev) sm_backlog |= !c->replay && has_work(d.copy);
+      // spin only while a copy server's queued work waits for its in-flight
+      // window (work blocked on another server's submission sleeps as before)
+      for (auto &d : c->dev) sm_backlog |= !c->replay && has_work(d.copy) && d.copy.inflight.size() >= 2;
       // full retire sweep (event queries on every server) only when not
       // spinning, or every 64th spin
       const bool sweep = !sm_backlog || (++spins & 63) == 0;

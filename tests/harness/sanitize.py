@@ -98,4 +98,25 @@ for i in range(6):
     ctx.release(cf, oid, ptr, 0)
     ctx.free(cf, oid)
 ctx.close()
+# cross-GPU dispatch on the peer branch (R55, R56): small pulls on the
+# consumer's stream and whole-transfer pushes from the source's copy server,
+# back to back on one consumer stream (the third get queues behind the window)
+ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                pool_floor_bytes=64 * MiB, flags=G.FORCE_REMOTE))
+s = torch.cuda.Stream()
+for n in (64 * 1024 + 16, 4 * MiB, 12 * MiB + 4096):
+    src = torch.empty(n, dtype=torch.uint8, device="cuda")
+    G.check(G.test_fill(src.data_ptr(), n, 21, 0, 0))
+    torch.cuda.synchronize()
+    st, oid = ctx.put(G.fn(4, 1, 0), src.data_ptr(), n, G.NOHINT, 0, 0)
+    G.check(st, "put")
+    ctx.sync()
+    dsts = [torch.empty(n, dtype=torch.uint8, device="cuda") for _ in range(3)]
+    for i in range(6):
+        G.check(ctx.get_into(G.fn(4, 2, 1), oid, dsts[i % 3].data_ptr(), n, s.cuda_stream)[0])
+    s.synchronize()
+    for d in dsts:
+        assert G.test_verify(d.data_ptr(), n, 21, 0, 0)[1] == 0
+    ctx.free(G.fn(4, 1, 0), oid)
+ctx.close()
 print("sanitize workload OK", os.environ.get("GR_COPY", "default"))
