@@ -1093,12 +1093,12 @@ def run_gpu(args, rank, world, local_rank):
     run_requests(R * args.warmup)
     verify(R * args.warmup, "warm-up")
     total = R * args.steps
-    barrier()
     st0 = ctx.stats()
     clk = ClockSampler(dev)
     clk.start()
     ts = torch.cuda.Stream(device=cons_dev)          # timing stream: every consumer stream joins it
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()                                        # last before the region: ranks start together
     e0.record(ts)
     for qs in qstreams:
         qs.wait_event(e0)

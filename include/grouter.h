@@ -91,10 +91,11 @@ extern "C" {
                                       sources and destinations were on another GPU (the NVLink
                                       branch: system-scope fences, no L2 prefetch, no TMA bulk
                                       engine, completion published in-kernel), and a copy between
-                                      two logical GPUs never runs as a direct launch on the
-                                      consumer's stream (the source's copy server pushes, the
-                                      consumer waits on completion words), so one-GPU test boxes
-                                      execute the code a physical peer transfer runs          */
+                                      two logical GPUs takes the dispatch of a physical pair: the
+                                      source's copy server pushes it (the consumer waits on
+                                      completion words), or, <= 4 MiB on an idle server, the
+                                      consumer's stream pulls it (R55, R56), so one-GPU
+                                      test boxes execute the code a physical peer transfer runs */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;
@@ -254,7 +255,11 @@ grouter_status grouter_seal(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid 
 grouter_status grouter_get(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *stream,
                            const void **ptr, uint64_t *n);
 /* Get into caller memory `dst` (device memory of fn->device, or host memory
- * for a CPU fn); always copies.  EINVAL if dst_cap < n. *n_out may be NULL. */
+ * for a CPU fn); always copies.  EINVAL if dst_cap < n. *n_out may be NULL.
+ * A GPU -> other-GPU copy is pushed by the source GPU's SMs over NVLink
+ * (whole when it is the only work of that copy server, R55), or, <= 4 MiB on
+ * an idle server with a non-NULL `stream`, pulled by the consumer GPU's SMs
+ * on `stream` (R56); either way `stream` sees the bytes in order. */
 grouter_status grouter_get_into(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid oid, void *dst,
                                 uint64_t dst_cap, void *stream, uint64_t *n_out);
 /* Drops a lease (ptr as returned by grouter_get).  Stream-ordered: pages are
