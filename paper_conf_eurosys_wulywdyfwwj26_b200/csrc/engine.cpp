@@ -484,11 +484,23 @@ static void launch_round(grouter_ctx *c, Server &s, cudaStream_t st, uint32_t *s
       part.push_back(it);
       bytes += it.bytes;
     }
-    // publish values after this launch
+    // publish values after this launch -- only for the (transfer, path)
+    // words whose LAST chunk this launch carries: every fence on a word waits
+    // for its final value (done_fences; R5, no partial visibility), and a
+    // path's chunks run in stream order on one stream, so earlier launches
+    // need not publish -- nor pay the in-kernel protocol (a system-scope
+    // fence per CTA on the peer branch: ~12 us per launch measured through
+    // GROUTER_FORCE_REMOTE, tools/peerpath.py)
     std::vector<Pub> pubs = issue(part);
+    uint32_t npub = 0;
     for (uint32_t k = 0; k < p->n_pub; ++k)
       for (auto &pb : pubs)
-        if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path]) p->pub[k].value = pb.x->value_after(pb.path);
+        if (p->pub[k].word == (uint64_t)(uintptr_t)&pb.x->words[pb.path] &&
+            pb.x->issued[pb.path] == pb.x->total[pb.path]) {
+          p->pub[npub] = p->pub[k];
+          p->pub[npub++].value = pb.x->value_after(pb.path);
+        }
+    p->n_pub = npub;
     ProfRec pr{s.phys, nullptr, nullptr, bytes};
     p->stamp = nullptr;
     if (prof) prof_begin(pd, st, pr, p->stamp);
@@ -547,22 +559,30 @@ void harvest_profile(grouter_ctx *c, bool wait) {
 // NVLink, or a same-GPU HBM copy).
 //
 // A transfer that is the ONLY work queued on the server (one tenant, one
-// transfer, no urgent work) goes out WHOLE in one round (R55, the queued
-// counterpart of R53's direct launch): e.g. a GPU -> other-GPU get, whose
-// consumer stream lives on another device and so never takes the direct
-// launch.  A batch per round costs a launch and a dispatch reaction per
-// 10 MiB -- at NVLink rates (~14 us per batch) that, not the link, bounds a
-// large push (tools/peerpath.py).  A tenant arriving later waits behind the
-// <= 2 rounds in flight, as behind a direct launch.  Real-time mode without
-// GROUTER_LOG only (replay and the log keep one batch per round).
+// transfer, no urgent work) goes out in rounds of up to 64 MiB -- whole when
+// it fits (R55): e.g. a GPU -> other-GPU get, whose consumer stream lives on
+// another device and so never takes the direct launch.  A batch per round
+// costs a launch and a dispatch reaction per 10 MiB -- at NVLink rates
+// (~14 us per batch) that, not the link, bounds a large push
+// (tools/peerpath.py).  A tenant arriving later waits behind the <= 2 rounds
+// in flight: <= 128 MiB, ~170 us over NVLink (10 MiB batches: ~28 us).
+// Real-time mode without GROUTER_LOG only (replay and the log keep one batch
+// per round).
 static void complete_by_event(grouter_ctx *c, const std::vector<Xfer *> &xs, const EventRef &e, cudaStream_t st);
+static const uint64_t kSoloBytes = 64ull << 20;  // R55: at most 64 MiB per solo round
 static bool single_transfer(const Server &s) {
-  if (!s.carry.empty() || !s.urgent.empty()) return false;
+  if (!s.urgent.empty()) return false;
   const Xfer *only = nullptr;
+  for (auto &it : s.carry) {  // the rest of a solo round's last batch
+    if (only && it.x != only) return false;
+    only = it.x;
+  }
+  bool queued = false;
   for (auto &kv : s.sched.tenants) {
     const auto &q = kv.second.q;
     if (q.empty()) continue;
-    if (only || q.front().x != q.back().x) return false;
+    if (queued || q.front().x != q.back().x || (only && q.front().x != only)) return false;
+    queued = true;
     only = q.front().x;
   }
   return only != nullptr;
@@ -576,8 +596,8 @@ static size_t round_copy(grouter_ctx *c, Server &s) {
   std::vector<char> cut;
   uint32_t nb;
   if (solo) {
-    nb = refill(c, s, UINT32_MAX, kDirectBytes, kDirectItems);
-    take(s, kDirectBytes, items, cut, kDirectItems);
+    nb = refill(c, s, UINT32_MAX, kSoloBytes, kDirectItems);
+    take(s, kSoloBytes, items, cut, kDirectItems);
   } else {
     nb = refill_one(c, s);
     take(s, batch_budget(c, s), items, cut);

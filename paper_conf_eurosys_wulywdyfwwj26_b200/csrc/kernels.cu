@@ -247,11 +247,11 @@ __device__ __forceinline__ void finish_round(const KP &p) {
   if (threadIdx.x == 0) {
     // local destinations only need GPU-scope ordering before the counter;
     // peer (NVLink) destinations need the system-scope fence
-    if (p.flags & kFlagLocalDst) __threadfence();
+    if ((p.flags & kFlagLocalDst) || p.n_pub == 0) __threadfence();  // n_pub 0: only the scratch reset
     else __threadfence_system();
     unsigned prev = atomicAdd(&p.scratch[1], 1u);
     if (prev == gridDim.x - 1) {
-      __threadfence_system();
+      if (p.n_pub) __threadfence_system();
       for (uint32_t i = 0; i < p.n_pub; ++i) st_release_sys(p.pub[i].word, p.pub[i].value);
       // every CTA has stopped claiming: reset for the next launch on this stream
       p.scratch[0] = 0;
@@ -711,6 +711,8 @@ int launch_copy(CopyParams &p, int sm_count, int ctas_per_sm, bool tma, void *st
   if (host_publish && is_static && !p.counts) {
     p.flags |= kFlagNoPublish;
     *host_publish = true;
+  } else if (p.n_pub == 0 && is_static && !p.counts) {
+    p.flags |= kFlagNoPublish;  // nothing to publish and no ticket scratch to reset
   }
   if (p.n_chunks <= (uint32_t)SmallParams::kChunks && p.n_pub <= (uint32_t)SmallParams::kPubs) {
     SmallParams q;

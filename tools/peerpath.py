@@ -22,7 +22,8 @@ from synth import calib as C  # noqa: E402
 
 G.load()
 out = {}
-modes = [m for m in [("direct", 0), ("remote", G.FORCE_REMOTE)]
+PROF = G.PROFILE if os.environ.get("PEERPATH_PROFILE") else 0   # kernel %globaltimer stamps per launch
+modes = [m for m in [("direct", 0 | PROF), ("remote", G.FORCE_REMOTE | PROF)]
          if m[0] in os.environ.get("PEERPATH_MODES", "direct,remote").split(",")]
 for name, flags in ([] if os.environ.get("PEERPATH_LEGB") else modes):
     calib = C.virtual(2)
@@ -57,6 +58,8 @@ for name, flags in ([] if os.environ.get("PEERPATH_LEGB") else modes):
             b.synchronize()
             lat.append(a.elapsed_time(b) * 1e3)
         lat.sort()
+        ctx.sync()
+        k0 = ctx.stats()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(s1)
         for i in range(reps):
@@ -64,15 +67,20 @@ for name, flags in ([] if os.environ.get("PEERPATH_LEGB") else modes):
         b.record(s1)
         b.synchronize()
         ms = a.elapsed_time(b)
-        st0 = ctx.stats()
+        ctx.sync()
+        k1 = ctx.stats()
         res[n] = {"p50_us": round(lat[len(lat) // 2], 2), "b2b_us": round(ms * 1e3 / reps, 2),
-                  "b2b_GBps_rw": round(2 * n * reps / (ms / 1e3) / 1e9, 1)}
+                  "b2b_GBps_rw": round(2 * n * reps / (ms / 1e3) / 1e9, 1),
+                  "b2b_launches_per_get": (k1.kernel_launches - k0.kernel_launches) / reps}
+        if k1.timed_kernel_launches > k0.timed_kernel_launches:   # PEERPATH_PROFILE: the kernels' own spans
+            res[n]["b2b_kernel_us_per_get"] = round((k1.timed_kernel_ns - k0.timed_kernel_ns) / 1e3 / reps, 2)
         for oid in oids:
             ctx.free(G.fn(9, 1, 0), oid)
         del src, dst
     st = ctx.stats()
     res["kernel_launches"] = st.kernel_launches
     res["rounds"] = st.rounds
+
     out[name] = res
     ctx.close()
 if out:
