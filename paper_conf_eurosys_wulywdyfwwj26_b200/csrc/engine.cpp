@@ -722,6 +722,52 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
                                    p.x->value_after(p.path), 0));
 }
 
+// Copy-engine runs of a round: contiguous chunks become ONE copy, and chunks
+// of equal size at a constant source and destination stride -- a route's
+// share of an interleaved plan (R4: chunk i of route r sits Σ_routes c
+// after chunk i-1), whose source AND destination are strided alike when the
+// route's copy engine writes the destination directly (its own chunks, or
+// GROUTER_CE_RELAY) -- become ONE 2-D copy (cudaMemcpy2DAsync).  Each copy
+// costs the engine ~3 us of setup (tools/ce2.cu, probe), so five 2 MiB
+// chunks per round copied one by one cost a relayed link ~8% of its rate.
+// A 2-D run never spans two transfers: its pitched source and destination
+// ranges must each lie inside one allocation (the transfer's source buffer
+// and its destination object), which chunks of unrelated transfers at equal
+// spacing would not (spills of equal-sized victims, say).
+struct CeRun {
+  static constexpr uint64_t kMaxPitch = (1ull << 31) - 1;  // cudaMemcpy2D pitch limit
+  uint64_t src = 0, dst = 0, width = 0, height = 0, spitch = 0, dpitch = 0;
+  const void *owner = nullptr;  // the transfer of the run's first chunk
+  bool add(uint64_t s, uint64_t d, uint64_t n, const void *x) {  // true: absorbed into this run
+    if (!height) {
+      src = s, dst = d, width = n, height = 1, owner = x;
+      return true;
+    }
+    if (height == 1 && s == src + width && d == dst + width) {
+      width += n;
+      return true;
+    }
+    if (n != width || x != owner) return false;
+    if (height == 1) {
+      if (s <= src || d <= dst) return false;
+      const uint64_t sp = s - src, dp = d - dst;
+      if (sp < width || dp < width || sp > kMaxPitch || dp > kMaxPitch) return false;
+      spitch = sp, dpitch = dp, height = 2;
+      return true;
+    }
+    if (s != src + height * spitch || d != dst + height * dpitch) return false;
+    ++height;
+    return true;
+  }
+  bool empty() const { return height == 0; }
+  void flush(cudaMemcpyKind kind, cudaStream_t st) {
+    if (!height) return;
+    if (height == 1) GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, width, kind, st));
+    else GR_CUDA(cudaMemcpy2DAsync((void *)dst, dpitch, (const void *)src, spitch, width, height, kind, st));
+    height = 0;
+  }
+};
+
 // H2D server of route GPU r: CE copies of up to two batches (L229).  Chunks
 // for r itself land in the lease; relayed chunks go through r's staging ring
 // and a forward round kernel on r pushes them to their destination.
@@ -740,11 +786,11 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   EventRef last_fwd;
   // contiguous direct chunks of a round go to the copy engine as ONE copy
   // (per-copy engine overhead ~3.6 us measured by the probe)
-  uint64_t run_src = 0, run_dst = 0, run_len = 0;
+  CeRun run;
   auto flush_run = [&]() {
-    if (run_len) {
+    if (!run.empty()) {
       const uint64_t tm = tl_put_t0 ? now_ns() : 0;
-      GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyDefault, s.stream));
+      run.flush(cudaMemcpyDefault, s.stream);
       if (tl_put_t0) {  // profiling: put call -> its first H2D copy submitted
         const uint64_t te = now_ns();
         hprof().t[14] += te - tl_put_t0;
@@ -754,7 +800,6 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
         tl_put_t0 = 0;
       }
     }
-    run_len = 0;
   };
   // Relay forward, pipelined per chunk (K4', L182 "chunks are pipelined
   // across GPU streams"): as soon as a relayed chunk's copy into the staging
@@ -811,14 +856,13 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
     // own PCIe link and writes the destination's pages directly (over NVLink
     // on a multi-GPU box): no staging slot, no forward launch
     if (it.dst_logical == s.logical || ce_relay) {
-      if (run_len && !it.x->pageable_src && run_src + run_len == src && run_dst + run_len == it.dst) {
-        run_len += it.bytes;
-      } else {
+      if (it.x->pageable_src) {  // bounce slot: copy now, the slot is reused
         flush_run();
-        run_src = src;
-        run_dst = it.dst;
-        run_len = it.bytes;
-        if (it.x->pageable_src) flush_run();  // bounce slot: copy now, the slot is reused
+        run.add(src, it.dst, it.bytes, it.x);
+        flush_run();
+      } else if (!run.add(src, it.dst, it.bytes, it.x)) {
+        flush_run();
+        run.add(src, it.dst, it.bytes, it.x);
       }
       direct.push_back(it);
     } else {
@@ -858,13 +902,8 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
   if (items.empty()) return 0;
   const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
-  uint64_t run_src = 0, run_dst = 0, run_len = 0;
-  auto flush_run = [&]() {
-    if (run_len)
-      GR_CUDA(cudaMemcpyAsync((void *)run_dst, (const void *)run_src, run_len, cudaMemcpyDeviceToHost,
-                              s.stream));
-    run_len = 0;
-  };
+  CeRun run;
+  auto flush_run = [&]() { run.flush(cudaMemcpyDefault, s.stream); };
   for (size_t i = 0; i < items.size(); ++i) {
     const ChunkItem &it = items[i];
     if (cut[i]) {
@@ -872,13 +911,9 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
       publish_ce(c, s, seg, evented);
       stream_wait(c, s.stream, s.phys, it.x->deps);
     }
-    if (run_len && run_src + run_len == it.src && run_dst + run_len == it.dst) {
-      run_len += it.bytes;
-    } else {
+    if (!run.add(it.src, it.dst, it.bytes, it.x)) {
       flush_run();
-      run_src = it.src;
-      run_dst = it.dst;
-      run_len = it.bytes;
+      run.add(it.src, it.dst, it.bytes, it.x);
     }
     seg.push_back(it);
     c->stats.link_bytes[2][s.logical] += it.bytes;
