@@ -1058,13 +1058,14 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   p->chunk[0] = {src, dst, n};
   bool host_pub = false;
   PhysDev &pd = *c->phys.at(caller_phys);
-  // Tiny same-device copies (<= 64 KiB; GR_SMALL_CE overrides for measurement)
+  // Small same-device copies (<= 1 MiB; GR_SMALL_CE overrides for measurement)
   // go to the copy engine: its start latency beats a kernel launch's there
   // (C++ single calls, tools/libcost.cpp: 4 KiB 7.94 -> 7.14 us, 64 KiB
-  // 8.80 -> 8.58 us; a bare cudaMemcpyAsync 7.04 / 8.03 us); from 1 MiB the
-  // kernel is at or below the copy engine
+  // 8.80 -> 8.58 us; through Python, tools/smallce.py, 256 KiB-1 MiB p50
+  // 9.0-9.9 us by kernel vs 7.7-9.2 us by copy engine; from 1.5 MiB on the
+  // two are within run-to-run noise and the kernel keeps the HBM roofline)
   static const uint64_t small_ce =
-      getenv("GR_SMALL_CE") ? strtoull(getenv("GR_SMALL_CE"), nullptr, 0) : (64ull << 10);
+      getenv("GR_SMALL_CE") ? strtoull(getenv("GR_SMALL_CE"), nullptr, 0) : (1ull << 20);
   if (n <= small_ce && !cross) {
     GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, n, cudaMemcpyDeviceToDevice, caller));
     host_pub = true;
