@@ -783,11 +783,15 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
     finally:
         ctx.close()
     out["d2d_sweep"] = measure_d2d_sweep(world, G, calib, devs)
+    # the same gets pulled by GPU1's SMs at every size (GROUTER_PULL_ALL; default: pulls <= 4 MiB,
+    # R56): the data for the pull/push threshold on NVLink 5
+    out["d2d_sweep_pull"] = measure_d2d_sweep(world, G, calib, devs, sizes=(16 << 20, 38_535_168, 256 << 20, 1 << 30),
+                                              flags=G.PULL_ALL)
     return out
 
 
 def measure_d2d_sweep(world, G, calib, devs, sizes=(4096, 65536, 1 << 20, 16 << 20, 38_535_168, 64 << 20,
-                                                     256 << 20, 1 << 30)):
+                                                     256 << 20, 1 << 30), flags=0):
     """cfg3 (i) at N >= 2 (the metric's "latency & GB/s vs size"): a gFn on
     GPU1 get_into's an object resident on GPU0 (GPU0's SM copy pushes it over
     NVLink), per size: p50/p99 of single calls on an idle pair (CUDA events on
@@ -795,7 +799,7 @@ def measure_d2d_sweep(world, G, calib, devs, sizes=(4096, 65536, 1 << 20, 16 << 
     cudaMemcpyPeerAsync on the same buffers.  Byte-verified per size."""
     import torch
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * world,
-                                    pool_floor_bytes=64 << 20))
+                                    pool_floor_bytes=64 << 20, flags=flags))
     res = []
     try:
         s1 = torch.cuda.Stream(device=f"cuda:{devs[1]}")

@@ -96,6 +96,11 @@ extern "C" {
                                       completion words), or, <= 4 MiB on an idle server, the
                                       consumer's stream pulls it (R55, R56), so one-GPU
                                       test boxes execute the code a physical peer transfer runs */
+#define GROUTER_PULL_ALL      0x4000u/* MEASUREMENT: every GPU -> other-GPU copy requested on a
+                                      consumer stream while the source's copy server is idle is
+                                      pulled by the consumer GPU (R56 without its 4 MiB bound),
+                                      so bench.py can time pull against push per size on a
+                                      multi-GPU box (d2d_sweep_pull)                          */
 
 typedef uint64_t grouter_oid;      /* opaque, 0 never valid: (node << 48) | seq, node 0 */
 typedef struct grouter_ctx grouter_ctx;

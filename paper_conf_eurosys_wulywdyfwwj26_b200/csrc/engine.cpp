@@ -1021,7 +1021,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   const bool forced = (c->cfg.flags & GROUTER_FORCE_REMOTE) != 0;
   const bool cross = forced ? server_logical != caller_logical : s.phys != caller_phys;
   if (forced && !cross) return nullptr;  // forced remote: same-GPU rounds take the queued path
-  if (cross && (pull_off || n > kPullMax)) return nullptr;
+  if (cross && (pull_off || (n > kPullMax && !(c->cfg.flags & GROUTER_PULL_ALL)))) return nullptr;
   if (!s.carry.empty() || !s.urgent.empty() || !s.sched.empty()) return nullptr;
   for (auto &f : s.inflight)
     if (f.direct != caller) {

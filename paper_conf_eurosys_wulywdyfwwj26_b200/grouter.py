@@ -35,6 +35,7 @@ NO_TOPOLOGY = 0x400         # ablation "TA off" (Fig. 16): route sets ignore sha
 HOST_CENTRIC = 0x800        # ablation "UF off" (Fig. 16): GPU -> GPU copies through host memory (R49)
 FORCE_REMOTE = 0x1000       # test only: every copy-kernel round takes the peer (NVLink) branch
 CE_RELAY = 0x2000           # striped H2D: route GPUs' copy engines write the destination directly
+PULL_ALL = 0x4000           # measurement: cross-GPU copies on an idle server are pulled at any size (R56)
 
 OK, EINVAL, ENOENT, EPERM, ENOMEM, EBUSY, ECUDA, ESTATE = range(8)
 STATUS = ["OK", "EINVAL", "ENOENT", "EPERM", "ENOMEM", "EBUSY", "ECUDA", "ESTATE"]
