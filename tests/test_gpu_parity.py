@@ -301,18 +301,22 @@ def test_config_traces_forced_remote(replay):
         assert st.peer_launches == st.kernel_launches > 0
 
 
+@pytest.mark.parametrize("pull_all", [False, True])
 @pytest.mark.parametrize("n", [4096, 4 * MiB - 16, 4 * MiB + 4096, 64 * MiB + 12288])
-def test_cross_gpu_dispatch_forced_remote(n):
+def test_cross_gpu_dispatch_forced_remote(n, pull_all):
     """R55 / R56 on the peer branch: a gFn on logical GPU1 get_into's objects
     of logical GPU0 on its own stream.  A copy of <= 4 MiB on an idle server
     is ONE pull launch on the consumer's stream; a larger one alone on the
     source's copy server is pushed in rounds of up to 64 MiB (one launch when
-    it fits, not a round per 10 MiB batch).  Every launch takes the peer branch, every delivered byte
+    it fits, not a round per 10 MiB batch); GROUTER_PULL_ALL pulls every
+    size in one launch (the bench's pull-vs-push data).  Every launch takes
+    the peer branch, every delivered byte
     equals the generator's, and the stride accounting advances as for queued
     batches (tenant bytes = n per get)."""
     calib = C.virtual(2)
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
-                                    pool_floor_bytes=64 * MiB, flags=G.FORCE_REMOTE))
+                                    pool_floor_bytes=64 * MiB,
+                                    flags=G.FORCE_REMOTE | (G.PULL_ALL if pull_all else 0)))
     try:
         src = torch.empty(n, dtype=torch.uint8, device="cuda")
         G.check(G.test_fill(src.data_ptr(), n, 515, 0, 0))
@@ -331,7 +335,7 @@ def test_cross_gpu_dispatch_forced_remote(n):
             G.check(ctx.get_into(f1, oid, dst.data_ptr(), n, s1.cuda_stream)[0], "get_into")
             s1.synchronize()
             st1 = ctx.stats()
-            launches = 1 if n <= 4 * MiB else -(-n // (64 * MiB))   # a pull, or pushes of <= 64 MiB rounds
+            launches = 1 if n <= 4 * MiB or pull_all else -(-n // (64 * MiB))   # a pull, or <= 64 MiB pushes
             assert st1.kernel_launches - st0.kernel_launches == launches, (rep, st1.kernel_launches - st0.kernel_launches)
             assert st1.peer_launches - st0.peer_launches == launches
             assert st1.link_bytes[0][0] - st0.link_bytes[0][0] == n   # the source GPU's egress
