@@ -787,9 +787,6 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
     # R56): the data for the pull/push threshold on NVLink 5
     out["d2d_sweep_pull"] = measure_d2d_sweep(world, G, calib, devs, sizes=(16 << 20, 38_535_168, 256 << 20, 1 << 30),
                                               flags=G.PULL_ALL)
-    # pushes through the TMA bulk engine (GROUTER_COPY_TMA; default: wv8 LD/ST on peer rounds)
-    out["d2d_sweep_tma"] = measure_d2d_sweep(world, G, calib, devs, sizes=(16 << 20, 38_535_168, 256 << 20, 1 << 30),
-                                             flags=G.COPY_TMA)
     return out
 
 
