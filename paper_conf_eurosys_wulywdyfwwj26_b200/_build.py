@@ -24,7 +24,7 @@ LIB = os.path.join(HERE, "libgrouter.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 SOURCES = ["api.cpp", "engine.cpp", "ipc.cpp", "paths.cpp", "plan.cpp", "pool.cpp", "probe.cpp", "kernels.cu"]
-HEADERS = ["common.h", "ctx.h", "kernels.h", "plan.h", "stride.h"]
+HEADERS = ["ce_run.h", "common.h", "ctx.h", "kernels.h", "plan.h", "stride.h"]
 
 
 def _inputs():

@@ -37,6 +37,7 @@
 
 #include <sys/prctl.h>
 
+#include "ce_run.h"
 #include "ctx.h"
 #include "kernels.h"
 
@@ -722,51 +723,14 @@ static void publish_ce(grouter_ctx *c, Server &s, std::vector<ChunkItem> &seg,
                                    p.x->value_after(p.path), 0));
 }
 
-// Copy-engine runs of a round: contiguous chunks become ONE copy, and chunks
-// of equal size at a constant source and destination stride -- a route's
-// share of an interleaved plan (R4: chunk i of route r sits Σ_routes c
-// after chunk i-1), whose source AND destination are strided alike when the
-// route's copy engine writes the destination directly (its own chunks, or
-// GROUTER_CE_RELAY) -- become ONE 2-D copy (cudaMemcpy2DAsync).  Each copy
-// costs the engine ~3 us of setup (tools/ce2.cu, probe), so five 2 MiB
-// chunks per round copied one by one cost a relayed link ~8% of its rate.
-// A 2-D run never spans two transfers: its pitched source and destination
-// ranges must each lie inside one allocation (the transfer's source buffer
-// and its destination object), which chunks of unrelated transfers at equal
-// spacing would not (spills of equal-sized victims, say).
-struct CeRun {
-  static constexpr uint64_t kMaxPitch = (1ull << 31) - 1;  // cudaMemcpy2D pitch limit
-  uint64_t src = 0, dst = 0, width = 0, height = 0, spitch = 0, dpitch = 0;
-  const void *owner = nullptr;  // the transfer of the run's first chunk
-  bool add(uint64_t s, uint64_t d, uint64_t n, const void *x) {  // true: absorbed into this run
-    if (!height) {
-      src = s, dst = d, width = n, height = 1, owner = x;
-      return true;
-    }
-    if (height == 1 && s == src + width && d == dst + width) {
-      width += n;
-      return true;
-    }
-    if (n != width || x != owner) return false;
-    if (height == 1) {
-      if (s <= src || d <= dst) return false;
-      const uint64_t sp = s - src, dp = d - dst;
-      if (sp < width || dp < width || sp > kMaxPitch || dp > kMaxPitch) return false;
-      spitch = sp, dpitch = dp, height = 2;
-      return true;
-    }
-    if (s != src + height * spitch || d != dst + height * dpitch) return false;
-    ++height;
-    return true;
-  }
-  bool empty() const { return height == 0; }
-  void flush(cudaMemcpyKind kind, cudaStream_t st) {
-    if (!height) return;
-    if (height == 1) GR_CUDA(cudaMemcpyAsync((void *)dst, (const void *)src, width, kind, st));
-    else GR_CUDA(cudaMemcpy2DAsync((void *)dst, dpitch, (const void *)src, spitch, width, height, kind, st));
-    height = 0;
-  }
-};
+// Issues a finished run as one copy (1-D) or one pitched copy (2-D).
+static void flush_ce_run(CeRun &r, cudaMemcpyKind kind, cudaStream_t st) {
+  if (!r.height) return;
+  if (r.height == 1) GR_CUDA(cudaMemcpyAsync((void *)r.dst, (const void *)r.src, r.width, kind, st));
+  else GR_CUDA(cudaMemcpy2DAsync((void *)r.dst, r.dpitch, (const void *)r.src, r.spitch, r.width, r.height, kind, st));
+  r.height = 0;
+}
+
 
 // H2D server of route GPU r: CE copies of up to two batches (L229).  Chunks
 // for r itself land in the lease; relayed chunks go through r's staging ring
@@ -790,7 +754,7 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
   auto flush_run = [&]() {
     if (!run.empty()) {
       const uint64_t tm = tl_put_t0 ? now_ns() : 0;
-      run.flush(cudaMemcpyDefault, s.stream);
+      flush_ce_run(run, cudaMemcpyDefault, s.stream);
       if (tl_put_t0) {  // profiling: put call -> its first H2D copy submitted
         const uint64_t te = now_ns();
         hprof().t[14] += te - tl_put_t0;
@@ -903,7 +867,7 @@ static size_t round_d2h(grouter_ctx *c, Server &s) {
   const std::vector<Xfer *> evented = whole_in_round(c, s, items);
   DeviceGuard g(s.phys);
   CeRun run;
-  auto flush_run = [&]() { run.flush(cudaMemcpyDefault, s.stream); };
+  auto flush_run = [&]() { flush_ce_run(run, cudaMemcpyDefault, s.stream); };
   for (size_t i = 0; i < items.size(); ++i) {
     const ChunkItem &it = items[i];
     if (cut[i]) {

@@ -28,3 +28,19 @@ def test_c99_consumer(tmp_path):
     import torch
     if not torch.cuda.is_available():
         assert "GROUTER_ECUDA" in r.stdout, r.stdout   # no CPU fallback
+
+
+@pytest.mark.skipif(shutil.which("g++") is None, reason="needs g++")
+def test_ce_run_builder(tmp_path):
+    """The copy-engine run builder (csrc/ce_run.h) on hand-written chunk
+    lists: contiguous chunks -> one copy, a route's interleaved chunks of one
+    transfer -> one 2-D copy, never across transfers, breaks on stride,
+    direction or pitch limit (tests/c/ce_run_test.cpp)."""
+    exe = tmp_path / "ce_run_test"
+    r = subprocess.run(["g++", "-std=c++17", "-Wall", "-Wextra", "-Werror", "-O1",
+                        os.path.join(ROOT, "tests", "c", "ce_run_test.cpp"), "-o", str(exe)],
+                       capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
+    r = subprocess.run([str(exe)], capture_output=True, text=True, timeout=60)
+    assert r.returncode == 0, r.stdout
+    assert r.stdout.count(": ok") == 9, r.stdout
