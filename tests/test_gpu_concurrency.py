@@ -120,7 +120,10 @@ def _client(ctx, t, errors, counts, rep=0):
 
 
 @pytest.mark.parametrize("rep", range(2))
-@pytest.mark.parametrize("flags", [0, G.RESTORE | G.STRIPED_MIGRATION, G.D2H_MULTIPATH | G.NO_POOL])
+# FORCE_REMOTE: the cross-GPU gets take a physical pair's dispatch (pulls <= 4 MiB, pushes
+# from the source's copy server, R55 / R56) while other threads evict, spill and copy
+@pytest.mark.parametrize("flags", [0, G.RESTORE | G.STRIPED_MIGRATION, G.D2H_MULTIPATH | G.NO_POOL,
+                                   G.FORCE_REMOTE | G.RESTORE])
 def test_concurrent_clients(flags, rep):
     calib = C.virtual(K)
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=256 * MiB, pool_cap=[24 * MiB] * K,
