@@ -8,7 +8,11 @@ virtual 2-GPU topology (both logical GPUs = device 0).  Modes:
              words / events on the consumer stream).
 Per size: back-to-back GB/s (read + write bytes over HBM, so the per-launch
 overhead shows ~10x larger than it would over NVLink) and single-call p50
-(CUDA events on the consumer stream, host path included)."""
+(CUDA events on the consumer stream, host path included).
+Env: PEERPATH_MODES=direct,remote (which modes), PEERPATH_PROFILE=1 (kernel
+%globaltimer spans per size via GROUTER_PROFILE), PEERPATH_LEGB=1 (only the
+bench's N >= 2 leg-B pattern: 20 objects round robin into 8 bindings).
+Results: profiles/r02_peerpath.txt."""
 import json
 import os
 import sys
