@@ -778,6 +778,12 @@ def measure_d2d_push(world, G, calib, devs, n=N_BYTES, objs=8, reps=10):
         out["d2d_ring"] = {"what": f"all {world} GPUs get_into their ring successor's objects at once",
                            "aggregate_GBps": round(gbps, 1), "per_gpu_GBps": round(gbps / world, 1),
                            "us_per_get": round(us, 2)}
+        if world >= 4:   # cfg3 (ii): the permutation i -> (i + N/2) mod N, all pairs at once
+            gbps, us = run([(c, (c + world // 2) % world) for c in range(world)])
+            out["d2d_perm"] = {"what": f"all {world} GPUs get_into the objects of GPU (i + {world // 2}) mod {world} "
+                                       "at once (cfg3 (ii))",
+                               "aggregate_GBps": round(gbps, 1), "per_gpu_GBps": round(gbps / world, 1),
+                               "frac_per_gpu": round(gbps / world / NVL_PEAK, 3), "us_per_get": round(us, 2)}
     except Exception as e:  # reported, never fatal for the line
         out["d2d_error"] = f"{type(e).__name__}: {e}"[:300]
     finally:
