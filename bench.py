@@ -1363,7 +1363,8 @@ def run_gpu(args, rank, world, local_rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=350,
+                    help="timed steps (20 requests each): 350 = ~5 s of closed loop at one GPU (SURVEY §8(d))")
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="grouter", choices=["grouter", "reference"])
     ap.add_argument("--requests", type=int, default=20)
