@@ -24,11 +24,12 @@
 //    or one memcpy burst (CE).  <= 2 rounds -- so <= 2 batches, SURVEY O8 --
 //    in flight per server in real-time mode; replay mode dispatches only at
 //    grouter_flush().
-//  * Host->GPU relay: CE copies a chunk into a staging slot on route GPU r,
-//    an event hands that chunk's slot to r's forward stream, a forward launch
-//    pushes it over NVLink into the lease on d and publishes the chunk's word
-//    (per chunk: the NVLink hop overlaps the next chunk's PCIe copy); the
-//    slot is reused after that launch's event.
+//  * Host->GPU relay: CE copies a route's chunks of a round into consecutive
+//    staging slots on route GPU r (one 2-D copy), an event hands them to r's
+//    forward stream, one forward launch pushes them over NVLink into the
+//    lease on d (the path's last chunk alone, so the tail is one chunk's
+//    forward) and the launch with the last chunk publishes the word; the
+//    slots are reused after that launch's event.
 #include <algorithm>
 #include <cstdio>
 #include <chrono>
@@ -765,35 +766,92 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
       }
     }
   };
-  // Relay forward, pipelined per chunk (K4', L182 "chunks are pipelined
-  // across GPU streams"): as soon as a relayed chunk's copy into the staging
-  // slot is enqueued, the forward stream waits for exactly that copy and a
-  // forward launch pushes that chunk to its destination and publishes its
-  // completion word -- the NVLink hop of chunk k overlaps the PCIe copy of
-  // chunk k+1, and the relay adds one chunk's forward to the tail instead of
-  // a whole round's.  The forward kernels run only while a chunk is moving
-  // (no SMs parked polling for PCIe arrivals).
-  // GR_SEGMENT_FWD=1 (measurement only, tools/relaytail.py): the round-1
-  // design -- one forward launch per segment after all its CE copies
+  // Relay forward (K4', L182 "chunks are pipelined across GPU streams").  A
+  // route's relayed chunks of one transfer in a round form a GROUP: they are
+  // copied into consecutive staging slots by ONE 2-D copy (equal chunks at
+  // the plan's interleave stride, R4) and pushed to the destination by ONE
+  // forward launch on the route GPU's forward stream, which waits for exactly
+  // that copy; the forward of round j overlaps the copies of round j+1.  In
+  // the round that carries the path's LAST chunk, that chunk is copied and
+  // forwarded on its own after the group, so the relay adds one chunk's
+  // forward to the transfer's tail, not a round's.  Per chunk, a copy costs
+  // the copy engine ~3 us of setup and the dispatch thread ~7 us of host time
+  // (copy, event, stream wait, launch, event; tools/relaycost.py): one copy
+  // and one forward per round instead of five.  The forward kernels run only
+  // while a chunk is moving (no SMs parked polling for PCIe arrivals).
+  // Measurement only: GR_CHUNK_FWD=1 (every relayed chunk copied and
+  // forwarded alone, the previous design), GR_SEGMENT_FWD=1 (the round-1
+  // design: one forward per segment after all of its chunk copies).
   static const bool segment_fwd = getenv("GR_SEGMENT_FWD") != nullptr;
+  static const bool chunk_fwd = getenv("GR_CHUNK_FWD") != nullptr;
   std::vector<ChunkItem> seg_relay;
   std::vector<uint64_t> seg_src;
   std::vector<uint32_t> seg_slots;
-  auto forward_chunk = [&](const ChunkItem &it, uint64_t slot, uint32_t k) {
+  // slots [k0, k0 + g) of the staging ring, consecutive (a group never wraps:
+  // the ring's tail slots are skipped instead); waits for their last readers
+  auto take_slots = [&](uint32_t g) -> uint32_t {
+    if (s.next_slot + g > s.n_slots) s.next_slot = 0;
+    const uint32_t k0 = s.next_slot;
+    s.next_slot = (k0 + g) % s.n_slots;
+    EventRef last;
+    for (uint32_t k = k0; k < k0 + g; ++k)
+      if (s.slot_free[k] && s.slot_free[k] != last) {
+        GR_CUDA(cudaStreamWaitEvent(s.stream, s.slot_free[k]->ev, 0));
+        last = s.slot_free[k];
+      }
+    return k0;
+  };
+  auto forward = [&](const std::vector<ChunkItem> &its, const std::vector<uint64_t> &srcs, uint32_t k0) {
+    EventRef ce = record(c, s.stream, s.phys);
+    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
+    launch_round(c, s, s.fwd_stream, s.fwd_scratch, its, srcs.data());
+    last_fwd = record(c, s.fwd_stream, s.phys);
+    for (uint32_t k = k0; k < k0 + (uint32_t)its.size(); ++k) s.slot_free[k] = last_fwd;
+  };
+  // a chunk on its own: one copy into one slot, one forward
+  auto relay_one = [&](const ChunkItem &it, uint64_t src) {
+    const uint32_t k = take_slots(1);
+    uint8_t *slot = s.staging + (uint64_t)k * s.slot_bytes;
+    GR_CUDA(cudaMemcpyAsync(slot, (const void *)src, it.bytes, cudaMemcpyHostToDevice, s.stream));
     if (segment_fwd) {
       seg_relay.push_back(it);
-      seg_src.push_back(slot);
+      seg_src.push_back((uint64_t)slot);
       seg_slots.push_back(k);
       return;
     }
-    EventRef ce = record(c, s.stream, s.phys);
-    GR_CUDA(cudaStreamWaitEvent(s.fwd_stream, ce->ev, 0));
-    const std::vector<ChunkItem> one(1, it);
-    launch_round(c, s, s.fwd_stream, s.fwd_scratch, one, &slot);
-    last_fwd = record(c, s.fwd_stream, s.phys);
-    s.slot_free[k] = last_fwd;
+    forward(std::vector<ChunkItem>(1, it), std::vector<uint64_t>(1, (uint64_t)slot), k);
+  };
+  std::vector<ChunkItem> grp;  // pending group: same transfer and path, equal chunks, one stride
+  auto flush_group = [&]() {
+    if (grp.empty()) return;
+    const ChunkItem &l = grp.back();
+    const bool has_last = l.x->total[l.path] - l.x->issued[l.path] == grp.size();
+    const size_t g = grp.size() - (has_last && grp.size() > 1 ? 1 : 0);
+    if (g == 1) {
+      relay_one(grp[0], grp[0].src);
+    } else {
+      const uint32_t k0 = take_slots((uint32_t)g);
+      uint8_t *slot0 = s.staging + (uint64_t)k0 * s.slot_bytes;
+      const uint64_t spitch = grp[1].src - grp[0].src;
+      GR_CUDA(cudaMemcpy2DAsync(slot0, s.slot_bytes, (const void *)grp[0].src, spitch, grp[0].bytes, g,
+                                cudaMemcpyHostToDevice, s.stream));
+      std::vector<ChunkItem> its(grp.begin(), grp.begin() + g);
+      std::vector<uint64_t> srcs(g);
+      for (size_t j = 0; j < g; ++j) srcs[j] = (uint64_t)(slot0 + j * s.slot_bytes);
+      forward(its, srcs, k0);
+    }
+    if (g < grp.size()) relay_one(grp.back(), grp.back().src);
+    grp.clear();
+  };
+  auto group_accepts = [&](const ChunkItem &it) {
+    if (grp.empty()) return true;
+    const ChunkItem &a = grp.front();
+    if (it.x != a.x || it.path != a.path || it.bytes != a.bytes || grp.size() >= s.n_slots / 2) return false;
+    if (grp.size() == 1) return it.src > a.src && it.src - a.src >= a.bytes && it.src - a.src <= CeRun::kMaxPitch;
+    return it.src == a.src + grp.size() * (grp[1].src - a.src);
   };
   auto end_segment = [&]() {
+    flush_group();
     flush_run();
     publish_ce(c, s, direct, evented);
     if (!seg_relay.empty()) {
@@ -831,12 +889,13 @@ static size_t round_h2d(grouter_ctx *c, Server &s) {
       direct.push_back(it);
     } else {
       flush_run();
-      uint32_t k = s.next_slot;
-      s.next_slot = (k + 1) % s.n_slots;
-      if (s.slot_free[k]) GR_CUDA(cudaStreamWaitEvent(s.stream, s.slot_free[k]->ev, 0));
-      uint8_t *slot = s.staging + (uint64_t)k * s.slot_bytes;
-      GR_CUDA(cudaMemcpyAsync(slot, (const void *)src, it.bytes, cudaMemcpyHostToDevice, s.stream));
-      forward_chunk(it, (uint64_t)slot, k);
+      if (it.x->pageable_src || chunk_fwd || segment_fwd) {  // bounce slot reused at once; measurement modes
+        flush_group();
+        relay_one(it, src);
+      } else {
+        if (!group_accepts(it)) flush_group();
+        grp.push_back(it);
+      }
     }
     if (it.x->pageable_src) c->bounce_ev[bslot] = record(c, s.stream, s.phys);
     c->stats.link_bytes[1][s.logical] += it.bytes;

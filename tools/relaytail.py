@@ -19,7 +19,7 @@ from paper_conf_eurosys_wulywdyfwwj26_b200 import grouter as G  # noqa: E402
 from synth import calib as C  # noqa: E402
 
 G.load()
-out = {"mode": "segment" if os.environ.get("GR_SEGMENT_FWD") else "per-chunk"}
+out = {"mode": "segment" if os.environ.get("GR_SEGMENT_FWD") else ("per-chunk" if os.environ.get("GR_CHUNK_FWD") else "grouped")}
 for k in (2, 4):
     calib = C.virtual(k)
     for name, flags in (("striped", 0), ("direct", G.NO_MULTIPATH)):
