@@ -1063,6 +1063,7 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   x->epoch = c->epoch;
   x->npath = 1;
   x->nchunks = x->submitted_chunks = (uint32_t)((n + C - 1) / C);
+  local_src &= !cross;  // a pull reads the other GPU's memory
   x->local_src = local_src;
   c->stats.xfer_count++;
   DeviceGuard g(caller_phys);
@@ -1070,7 +1071,6 @@ XferRef fast_direct(grouter_ctx *c, uint32_t tenant, int server_logical, int dst
   if (!c->params) c->params = new CopyParamsHost();
   CopyParams *p = &c->params->p;
   const bool local = !forced && dst_logical >= 0 && c->dev[dst_logical].phys == caller_phys;
-  local_src &= !cross;  // a pull reads the other GPU's memory
   p->flags = (local ? kFlagLocalDst : 0) | (local_src ? kFlagLocalSrc : 0);
   p->n_chunks = 1;
   p->n_pub = 0;
