@@ -347,6 +347,70 @@ def test_cross_gpu_dispatch_forced_remote(n, pull_all):
         ctx.close()
 
 
+def test_solo_rounds_yield_to_a_new_tenant():
+    """R55's bound: a transfer alone on an SM-copy server goes out in rounds of
+    at most 64 MiB, so a tenant that arrives while it moves waits behind the
+    <= 2 rounds in flight, not behind the whole transfer.  On the forced peer
+    branch, tenant 1's 1 GiB get_into (16 rounds) starts from a thread,
+    tenant 2's 4 KiB get_into follows while it moves: from tenant 2's arrival
+    (a device event on its idle stream), its copy completes in less than half
+    of the time tenant 1 still needs (device events), and both are byte-exact.
+    With one round for the whole transfer tenant 2 would finish after it."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    pool_floor_bytes=64 * MiB, flags=G.FORCE_REMOTE))
+    try:
+        big, small = 1 << 30, 4096
+        src = torch.empty(big, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(src.data_ptr(), big, 616, 0, 0))
+        torch.cuda.synchronize()
+        st, oa = ctx.put(G.fn(1, 1, 0), src.data_ptr(), big, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        st, ob = ctx.put(G.fn(2, 1, 0), src.data_ptr(), small, G.NOHINT, 0, 0)
+        G.check(st, "put")
+        ctx.sync()
+        del src
+        sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+        da = torch.empty(big, dtype=torch.uint8, device="cuda")
+        db = torch.empty(small, dtype=torch.uint8, device="cuda")
+        import threading
+        import time
+        valid = 0
+        for rep in range(5):
+            e0, ea, eb, eb0 = (torch.cuda.Event(enable_timing=True) for _ in range(4))
+            e0.record(sa)
+            sb.wait_event(e0)
+            errs = []
+
+            def big_get():   # blocks until its last round is submitted
+                try:
+                    G.check(ctx.get_into(G.fn(1, 2, 1), oa, da.data_ptr(), big, sa.cuda_stream)[0], "get_into big")
+                    ea.record(sa)
+                except Exception as e:   # surfaced below
+                    errs.append(e)
+            th = threading.Thread(target=big_get)
+            th.start()
+            time.sleep(100e-6)          # tenant 2 arrives while tenant 1's rounds move
+            eb0.record(sb)              # its arrival, on its idle stream
+            G.check(ctx.get_into(G.fn(2, 2, 1), ob, db.data_ptr(), small, sb.cuda_stream)[0], "get_into small")
+            eb.record(sb)
+            th.join(timeout=60)
+            assert not errs, errs
+            ea.synchronize()
+            eb.synchronize()
+            left_big, t_small = eb0.elapsed_time(ea), eb0.elapsed_time(eb)
+            if left_big < 0.15:         # the host was late: tenant 1 had (nearly) finished
+                continue
+            valid += 1
+            assert t_small < 0.5 * left_big, (rep, t_small, left_big)
+        assert valid >= 2, valid
+        for buf, n in ((da, big), (db, small)):
+            st, bad, first = G.test_verify(buf.data_ptr(), n, 616, 0, 0)
+            assert st == 0 and bad == 0, (n, bad, first)
+    finally:
+        ctx.close()
+
+
 @pytest.mark.parametrize("replay", [True, False])
 def test_ce_relay_parity(replay):
     """GROUTER_CE_RELAY: the route GPUs' copy engines write the destination's
