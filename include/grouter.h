@@ -262,7 +262,7 @@ grouter_status grouter_get(grouter_ctx *ctx, const grouter_fn *fn, grouter_oid o
 /* Get into caller memory `dst` (device memory of fn->device, or host memory
  * for a CPU fn); always copies.  EINVAL if dst_cap < n. *n_out may be NULL.
  * A GPU -> other-GPU copy is pushed by the source GPU's SMs over NVLink
- * (in rounds of up to 64 MiB when it is the only work of that copy server,
+ * (in rounds of up to 7 batches when it is the only work of that copy server,
  * R55), or, <= 4 MiB on
  * an idle server with a non-NULL `stream`, pulled by the consumer GPU's SMs
  * on `stream` (R56); either way `stream` sees the bytes in order. */

@@ -29,7 +29,13 @@ namespace {
 struct Guard {
   grouter_ctx *c;
   std::unique_lock<std::mutex> lk;
-  explicit Guard(grouter_ctx *c_) : c(c_), lk(c_->mu) {}
+  explicit Guard(grouter_ctx *c_) : c(c_), lk(c_->mu, std::defer_lock) {
+    if (!lk.try_lock()) {
+      c->lock_waiters.fetch_add(1, std::memory_order_relaxed);
+      lk.lock();
+      c->lock_waiters.fetch_sub(1, std::memory_order_relaxed);
+    }
+  }
 };
 
 grouter_status fail(grouter_status st, const char *msg) {

@@ -269,6 +269,9 @@ struct grouter_ctx {
   gr::Planner planner;
   bool plan_only = false, replay = false;
   std::mutex mu;                                       // the big lock
+  // API callers blocked on `mu` (Guard): the dispatch thread's spin leaves the
+  // lock alone while any wait, so a spinning dispatch loop cannot starve them
+  std::atomic<int> lock_waiters{0};
   std::vector<gr::LogicalDev> dev;
   std::map<int, std::unique_ptr<gr::PhysDev>> phys;
   gr::HostStore host;

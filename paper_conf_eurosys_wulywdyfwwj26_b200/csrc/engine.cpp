@@ -561,17 +561,17 @@ void harvest_profile(grouter_ctx *c, bool wait) {
 // NVLink, or a same-GPU HBM copy).
 //
 // A transfer that is the ONLY work queued on the server (one tenant, one
-// transfer, no urgent work) goes out in rounds of up to 64 MiB -- whole when
-// it fits (R55): e.g. a GPU -> other-GPU get, whose consumer stream lives on
+// transfer, no urgent work) goes out in rounds of up to 7 whole batches
+// (70 MiB) -- whole when it fits (R55): e.g. a GPU -> other-GPU get, whose consumer stream lives on
 // another device and so never takes the direct launch.  A batch per round
 // costs a launch and a dispatch reaction per 10 MiB -- at NVLink rates
 // (~14 us per batch) that, not the link, bounds a large push
 // (tools/peerpath.py).  A tenant arriving later waits behind the <= 2 rounds
-// in flight: <= 128 MiB, ~170 us over NVLink (10 MiB batches: ~28 us).
+// in flight: <= 140 MiB, ~190 us over NVLink (10 MiB batches: ~28 us).
 // Real-time mode without GROUTER_LOG only (replay and the log keep one batch
 // per round).
 static void complete_by_event(grouter_ctx *c, const std::vector<Xfer *> &xs, const EventRef &e, cudaStream_t st);
-static const uint64_t kSoloBytes = 64ull << 20;  // R55: at most 64 MiB per solo round
+static const uint32_t kSoloBatches = 7;  // R55: at most 7 batches (70 MiB at 5 x 2 MiB) per solo round
 static bool single_transfer(const Server &s) {
   if (!s.urgent.empty()) return false;
   const Xfer *only = nullptr;
@@ -597,9 +597,9 @@ static size_t round_copy(grouter_ctx *c, Server &s) {
   std::vector<ChunkItem> items, seg;
   std::vector<char> cut;
   uint32_t nb;
-  if (solo) {
-    nb = refill(c, s, UINT32_MAX, kSoloBytes, kDirectItems);
-    take(s, kSoloBytes, items, cut, kDirectItems);
+  if (solo) {  // whole batches only: no leftover in the carry for a newcomer to wait behind
+    nb = refill(c, s, kSoloBatches, UINT64_MAX, kDirectItems);
+    take(s, UINT64_MAX, items, cut, kDirectItems);
   } else {
     nb = refill_one(c, s);
     take(s, batch_budget(c, s), items, cut);
@@ -1333,8 +1333,12 @@ static void daemon_main(grouter_ctx *c) {
     }
     if (sm_backlog) {
       lk.unlock();
+      // ~1 us between polls; longer (up to 100 us) while an API caller waits
+      // for the lock, so the unfair mutex is not re-taken ahead of it
       const uint64_t t0 = now_ns();
-      while (now_ns() - t0 < 1000) cpu_relax();
+      for (uint64_t t = t0; t - t0 < 1000 || (c->lock_waiters.load(std::memory_order_relaxed) > 0 && t - t0 < 100000);
+           t = now_ns())
+        cpu_relax();
       lk.lock();
     } else if (backlog && !c->replay) {
       lk.unlock();
