@@ -23,7 +23,9 @@
 //    (plus urgent unscheduled work), executed by one kernel launch (SM copy)
 //    or one memcpy burst (CE).  <= 2 rounds -- so <= 2 batches, SURVEY O8 --
 //    in flight per server in real-time mode; replay mode dispatches only at
-//    grouter_flush().
+//    grouter_flush().  Exceptions on an SM-copy server with nothing else
+//    queued (R53 direct launches, R55 rounds of up to 7 batches of the one
+//    queued transfer): a newcomer waits behind <= 2 of those.
 //  * Host->GPU relay: CE copies a route's chunks of a round into consecutive
 //    staging slots on route GPU r (one 2-D copy), an event hands them to r's
 //    forward stream, one forward launch pushes them over NVLink into the
