@@ -166,6 +166,7 @@ struct Waitable {
 // Appends w to a fence list, replacing the last entry when both are events of
 // the same stream (the newer completes after the older).
 inline void push_fence(std::vector<Waitable> &f, const Waitable &w) {
+  if (!w.ev && !w.word) return;  // the completed fence (an idle stream's point)
   if (!f.empty() && w.ev && !w.word && f.back().ev && !f.back().word && w.origin && f.back().origin == w.origin)
     f.back() = w;
   else

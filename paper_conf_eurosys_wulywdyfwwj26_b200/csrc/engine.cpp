@@ -114,8 +114,20 @@ EventRef record(grouter_ctx *c, cudaStream_t s, int phys) {
 // carries a memory barrier that idles the stream ~3.5-5 us (tools/ce2.cu; the
 // launch_round note above), which every seal / release / stream-ordered put
 // of a function would have paid on its own stream.
+// A point on a caller's stream: "the work enqueued there so far".  When the
+// stream is idle right now that point has passed, and the fence is the
+// completed (empty) one: no event, and no cross-stream wait for whoever
+// depends on it (a push on the source GPU's server stream would otherwise
+// wait on an event of the consumer's stream, one more hand-off between
+// engines -- between devices on a GPU pair).
 Waitable signal(grouter_ctx *c, cudaStream_t s, int phys) {
+  static const bool no_skip = getenv("GR_NO_IDLE_SKIP") != nullptr;
   DeviceGuard g(phys);  // a fresh pooled event is created on the current device
+  if (!no_skip) {
+    const cudaError_t q = cudaStreamQuery(s);
+    if (q == cudaSuccess) return Waitable{};
+    if (q != cudaErrorNotReady) cudaGetLastError();  // e.g. a stream under graph capture: record below
+  }
   Waitable w = ev_wait(c, record(c, s, phys));
   w.origin = s;
   return w;
