@@ -803,7 +803,19 @@ grouter_status grouter_get(grouter_ctx *c, const grouter_fn *fn, grouter_oid oid
     const uint64_t ch = charge(n);
     if (d == GROUTER_HOST ? !host_reserve(c, ch) : !reserve(c, d, ch))
       return fail(GROUTER_ENOMEM, "get: lease does not fit after eviction");
-    uint8_t *lease = storage(c, d, ch);
+    // a lease that needs a new pool segment grows it without the context lock
+    // (the driver calls take up to ~60 ms while copies stream; dev_alloc), so
+    // the object is looked up again: freed or consumed meanwhile -> ENOENT;
+    // moved (spilled, restored) -> copied from where it is now
+    uint8_t *lease = storage(c, d, ch, d == GROUTER_HOST ? nullptr : &g.lk);
+    if (d != GROUTER_HOST) {
+      auto again = c->objects.find(oid);
+      if (again == c->objects.end() || dead(again->second) || &again->second != op) {
+        c->dev[d].used -= ch;
+        dev_free(c, d, lease, ch, Fences{});
+        return fail(GROUTER_ENOENT, "get: object freed while its lease's pages were mapped");
+      }
+    }
     bool direct = false;
     XferRef x;
     try {

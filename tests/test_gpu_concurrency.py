@@ -207,3 +207,56 @@ def test_pool_growth_without_the_lock_under_concurrency():
         assert st.mapped[0] >= 130 * MiB
     finally:
         ctx.close()
+
+
+def test_lease_growth_without_the_lock_under_concurrency():
+    """Copy leases (a gFn on logical GPU1 gets objects of logical GPU0) that
+    must grow GPU1's cold pool, from several threads at once, while other
+    threads put and free on GPU0: the lease's segment creation runs with the
+    context lock released, and the object is looked up again afterwards.
+    Every lease reads its object's bytes; a get of an object freed meanwhile
+    could only return ENOENT (each thread frees its own objects only after
+    releasing their leases, so here every get succeeds); the pools drain."""
+    calib = C.virtual(2)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * 2,
+                                    pool_floor_bytes=0))
+    errors = []
+    sizes = [5 * MiB + 3, 33 * MiB, 70 * MiB + 1, 97 * MiB]
+
+    def worker(t):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            f = G.fn(60 + t, 1, 0)     # producer on GPU0
+            g = G.fn(60 + t, 2, 1)     # consumer on GPU1: copy leases
+            src = torch.empty(max(sizes), dtype=torch.uint8, device="cuda")
+            for i in range(8):
+                n = sizes[(t + i) % len(sizes)]
+                seed = 9000 + 100 * t + i
+                G.check(G.test_fill(src.data_ptr(), n, seed, 0, s.cuda_stream), "fill")
+                st, oid = ctx.put(f, src.data_ptr(), n, G.NOHINT, 0, s.cuda_stream)
+                G.check(st, "put")
+                st, ptr, nn = ctx.get(g, oid, s.cuda_stream)
+                G.check(st, "get")
+                s.synchronize()
+                st, bad, first = G.test_verify(ptr, n, seed, 0, 0)
+                assert st == 0 and bad == 0, (t, n, bad, first)
+                G.check(ctx.release(g, oid, ptr, s.cuda_stream), "release")
+                G.check(ctx.free(f, oid), "free")
+        except Exception as e:  # pragma: no cover - reported below
+            errors.append(repr(e))
+
+    try:
+        ths = [threading.Thread(target=worker, args=(t,)) for t in range(6)]
+        for th in ths:
+            th.start()
+        for th in ths:
+            th.join(timeout=300)
+        assert not any(th.is_alive() for th in ths), "a client thread hung"
+        assert not errors, errors
+        G.check(ctx.sync(), "sync")
+        st = ctx.stats()
+        assert st.used[0] == 0 and st.used[1] == 0 and st.host_used == 0
+        assert st.mapped[1] >= 97 * MiB
+    finally:
+        ctx.close()
