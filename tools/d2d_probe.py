@@ -18,7 +18,7 @@ G.load()
 calib = b200_hgx(2)
 calib["device_map"] = [0, 1]
 res = {}
-for mode, flags in (("push", 0), ("pull", G.PULL_ALL)):   # R55 pushes vs pulls at every size (R56)
+for mode, flags in (("default", 0), ("pull_all", G.PULL_ALL)):   # default: pulls <= 4 MiB, pushes above (R55, R56)
     ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 << 20, pool_cap=[G.UNLIMITED] * 2,
                                     pool_floor_bytes=64 << 20, flags=flags))
     s1 = torch.cuda.Stream(device=1)
