@@ -412,6 +412,52 @@ def test_solo_rounds_yield_to_a_new_tenant():
         ctx.close()
 
 
+@pytest.mark.parametrize("k", [2, 4])
+def test_grouped_relay_forward(k):
+    """The relay hop of a striped cFn put (K4', L178/L182): a route's relayed
+    chunks of one transfer in a round move as one 2-D copy into consecutive
+    staging slots and ONE forward launch, the path's last chunk alone (a
+    one-chunk tail).  For each relayed route with m chunks in rounds of <= 5:
+    at most two forward launches per round and fewer launches than chunks
+    once a round holds >= 3 of them; the delivered tensor is byte-exact."""
+    calib = C.virtual(k)
+    ctx = G.Ctx(G.config_from_calib(calib, host_store_bytes=64 * MiB, pool_cap=[G.UNLIMITED] * k,
+                                    pool_floor_bytes=64 * MiB))
+    try:
+        n = 38_535_168 * 2
+        st, plan = ctx.plan(G.HOST, 0, n)
+        assert st == G.OK
+        per_route = {}
+        for ch in plan:
+            per_route[ch[3]] = per_route.get(ch[3], 0) + 1
+        relayed = {r: m for r, m in per_route.items() if r != 0}
+        assert relayed, plan
+        tmp = torch.empty(n, dtype=torch.uint8, device="cuda")
+        G.check(G.test_fill(tmp.data_ptr(), n, 717, 0, 0))
+        host = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        host.copy_(tmp)
+        del tmp
+        torch.cuda.synchronize()
+        f = G.fn(3, 1, G.HOST)
+        st0 = ctx.stats()
+        st, oid = ctx.put(f, host.data_ptr(), n, 0, 1)
+        G.check(st, "put")
+        st1 = ctx.stats()
+        launches = st1.kernel_launches - st0.kernel_launches
+        rounds = sum(-(-m // 5) for m in relayed.values())
+        chunks = sum(relayed.values())
+        assert launches <= 2 * rounds, (launches, rounds, relayed)
+        assert launches < chunks, (launches, chunks, relayed)
+        dst = torch.empty(n, dtype=torch.uint8, device="cuda")
+        s = torch.cuda.Stream()
+        G.check(ctx.get_into(G.fn(3, 2, 0), oid, dst.data_ptr(), n, s.cuda_stream)[0], "get_into")
+        s.synchronize()
+        st, bad, first = G.test_verify(dst.data_ptr(), n, 717, 0, 0)
+        assert st == 0 and bad == 0, (bad, first)
+    finally:
+        ctx.close()
+
+
 @pytest.mark.parametrize("replay", [True, False])
 def test_ce_relay_parity(replay):
     """GROUTER_CE_RELAY: the route GPUs' copy engines write the destination's
